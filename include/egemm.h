@@ -1,0 +1,145 @@
+/*
+ * egemm.h -- C ABI of the B200-native EGEMM-TC hot path (libegemm.so, sm_100a).
+ *
+ * Paper: B. Feng et al., "EGEMM-TC: Accelerating Scientific Computing on Tensor Cores with
+ * Extended Precision", PPoPP'21.  "P:a-b" = lines of the paper text; "R<n>" =
+ * the readings of the paper listed in DESIGN.md.
+ *
+ * Conventions (all entry points):
+ *  - Every pointer argument is a DEVICE pointer owned by the caller, unless stated.
+ *  - Calls are asynchronous on `stream` (a cudaStream_t; NULL = legacy default stream), never
+ *    synchronise the device, never allocate device memory, and are re-entrant.
+ *  - Matrices are row-major with an explicit row stride `ld*` in ELEMENTS.
+ *  - fp16 "hi"/"lo" buffers hold IEEE binary16 bit patterns (uint16_t).
+ *  - Return value: an egemm_status_t.  Host-side validation is synchronous; EGEMM_ERR_CUDA
+ *    reports a launch failure; asynchronous device faults surface at the caller's next sync.
+ *    egemm_last_error() gives a thread-local human-readable detail of the last non-OK return.
+ *  - There is no CPU fallback: without a usable sm_100a device every compute call returns
+ *    EGEMM_ERR_CUDA / EGEMM_ERR_UNSUPPORTED.
+ */
+#ifndef EGEMM_H
+#define EGEMM_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum {
+  EGEMM_OK = 0,
+  EGEMM_ERR_INVALID_ARG = 1, /* NULL data, negative size, ld < cols, bad terms / k */
+  EGEMM_ERR_UNSUPPORTED = 2, /* alignment / shape outside what the kernels implement */
+  EGEMM_ERR_CUDA = 3,        /* a CUDA launch or runtime call failed */
+  EGEMM_ERR_WORKSPACE = 4    /* workspace NULL or smaller than the *_workspace_size query */
+} egemm_status_t;
+
+/* Static string for a status code. */
+const char* egemm_status_string(int status);
+/* Thread-local detail message for the last non-OK return of this thread ("" if none). */
+const char* egemm_last_error(void);
+/* Library version (major*10000 + minor*100 + patch). */
+int egemm_version(void);
+
+/*
+ * One logical operand matrix, given in fp32 and/or pre-split.
+ *  f32   : fp32 values (may be NULL when hi/lo are given and the call does not need fp32).
+ *  hi,lo : pre-split fp16 parts from egemm_split, K-MAJOR (rows x K, row stride ld_split);
+ *          both NULL = split on the fly into the workspace.
+ *  ld    : row stride of f32 in elements.
+ *  trans : layout of f32 -- 0: stored as documented for the call; 1: stored transposed.
+ *  ld_split: row stride of hi/lo in elements (must be a multiple of 8, i.e. 16-byte rows).
+ */
+typedef struct {
+  const float* f32;
+  const uint16_t* hi;
+  const uint16_t* lo;
+  int64_t ld;
+  int trans;
+  int64_t ld_split;
+} egemm_operand_t;
+
+/*
+ * Round-split (Alg. 1 lines 2-3; Fig. 4b):
+ *   hi = fp16_RN(x);  lo = fp16_RN(x - (float)hi)
+ * RN = round to nearest, ties to even (reading R1).  x - hi is exact in fp32, so hi + lo
+ * carries >= 21 mantissa bits for 2^-3 <= |x| < 65520 (Table 1).
+ *  x      : rows x cols fp32, row stride ldx (>= cols).
+ *  hi, lo : transpose == 0: rows x cols, row stride ldo (>= cols);
+ *           transpose == 1: cols x rows (the transpose), row stride ldo (>= rows).
+ *  range_flags : nullable device uint32; bits are OR-ed in (never cleared):
+ *           bit0 = some |x| >= 65520 or non-finite (hi becomes +-inf / NaN),
+ *           bit1 = some 0 < |x| < 2^-3 (below the 21-bit zone; lo loses bits, R4).
+ * Out-of-range inputs are not an error (IEEE results), only flagged.
+ */
+int egemm_split(const float* x, int64_t rows, int64_t cols, int64_t ldx, uint16_t* hi,
+                uint16_t* lo, int64_t ldo, int transpose, uint32_t* range_flags, void* stream);
+
+/*
+ * Extended-precision GEMM (Alg. 1 "Emulation(D, A, B, C)"):
+ *   D[M x N] = A[M x K] * B[K x N] (+ C[M x N] if C != NULL)
+ * with A, B round-split into fp16 hi/lo and D accumulated in fp32 on the tensor cores as
+ * A_hi B_hi + A_hi B_lo + A_lo B_hi (+ A_lo B_lo when terms == 4) (Alg. 1 l.5-8).
+ *  A : f32 trans=0 -> M x K (ld >= K); trans=1 -> K x M (ld >= M).  hi/lo: M x K.
+ *  B : f32 trans=0 -> K x N (ld >= N); trans=1 -> N x K (ld >= K).  hi/lo: N x K (K-major).
+ *  C : nullable, M x N fp32, row stride ldc.  D: M x N fp32, row stride ldd.  D may not
+ *      alias A or B; D may equal C only if ldd == ldc.
+ *  terms : 0 (tuning-table default, 3), 3, or 4.
+ *  workspace : device scratch of >= egemm_gemm_workspace_size(...) bytes (256-B aligned),
+ *      used for the on-the-fly split of operands given only in fp32.  May be NULL when
+ *      that size is 0.
+ * M == 0 or N == 0: no-op.  K == 0: D = C (or 0).
+ */
+int egemm_gemm(int64_t M, int64_t N, int64_t K, egemm_operand_t A, egemm_operand_t B,
+               const float* C, int64_t ldc, float* D, int64_t ldd, int terms, void* workspace,
+               size_t workspace_bytes, void* stream);
+size_t egemm_gemm_workspace_size(int64_t M, int64_t N, int64_t K, int a_presplit, int b_presplit);
+
+/*
+ * kNN with the emulated GEMM (the GEMM-based kNN of Garcia et al. [9] with its fp32 GEMM
+ * replaced): for each query row q_i of Q[nq x d]
+ * the k rows x_j of X[nx x d] with the smallest squared distance
+ *   dist_ij = ||q_i||^2 + ||x_j||^2 - 2 q_i . x_j ,
+ * ascending by (dist, j), dist clamped to >= 0; self matches are kept (reading R11).
+ *  X, Q  : f32 required (row norms, fp64-accumulated); trans must be 0; hi/lo optional
+ *          (pre-split X = the "index build").
+ *  k     : 1 <= k <= 16 and k <= nx.
+ *  out_idx  : nq x k int32;  out_dist : nq x k fp32.
+ */
+int egemm_knn(egemm_operand_t X, int64_t nx, egemm_operand_t Q, int64_t nq, int64_t d, int k,
+              int32_t* out_idx, float* out_dist, void* workspace, size_t workspace_bytes,
+              void* stream);
+size_t egemm_knn_workspace_size(int64_t nx, int64_t nq, int64_t d, int k, int x_presplit);
+
+/*
+ * One Lloyd step of kMeans on the caller's shard of points (the GEMM-based kMeans of [2],
+ * P:142-145): assign_i = argmin_j (||c_j||^2 - 2 x_i . c_j) (ties -> lowest j),
+ * then fp64 partial sums sums[j][:] = sum_{a_i = j} x_i (from the fp32 x) and int64 counts.
+ * sums / counts / inertia are OVERWRITTEN.  inertia (nullable) = sum_i dist(x_i, c_{a_i}).
+ *  X : f32 required (n x d, trans 0); hi/lo optional (pre-split points).
+ *  centroids : kc x d fp32 (row stride d).
+ */
+int egemm_kmeans_step(egemm_operand_t X, int64_t n, int64_t d, const float* centroids, int64_t kc,
+                      int32_t* assign, double* sums, int64_t* counts, double* inertia,
+                      void* workspace, size_t workspace_bytes, void* stream);
+size_t egemm_kmeans_workspace_size(int64_t n, int64_t d, int64_t kc, int x_presplit);
+
+/* After the caller's all_reduce of sums / counts across ranks:
+ *   centroids[j] = fp32_RN(sums[j] / counts[j]) for counts[j] > 0; unchanged otherwise (R12). */
+int egemm_kmeans_finalize(const double* sums, const int64_t* counts, int64_t kc, int64_t d,
+                          float* centroids, void* stream);
+
+/* Tile configuration used by the next calls of this thread (the tuning-table override).
+ * cg in {1,2}, bn in {128,256}, sep in {0,1}, kc a multiple of 64 (0 = default).
+ * Pass all zeros to restore the tuning table.  Returns EGEMM_ERR_UNSUPPORTED for a
+ * combination the library was not built with. */
+int egemm_set_config(int cg, int bn, int sep, int kc);
+
+/* Number of SMs of the current device (0 without a device). */
+int egemm_num_sms(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* EGEMM_H */

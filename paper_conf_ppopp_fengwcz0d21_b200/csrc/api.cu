@@ -1,0 +1,435 @@
+// api.cu -- the extern "C" boundary of libegemm.so (declared in include/egemm.h):
+// argument validation, tile/term/promotion selection (the tuning table),
+// workspace carving, and the launch sequence of each call.  No allocation, no sync.
+#include <cuda_runtime.h>
+#include <cstdarg>
+#include <cstdio>
+#include <cstdlib>
+#include <cstring>
+#include "../../include/egemm.h"
+#include "egemm_internal.h"
+
+namespace egemm {
+
+static thread_local char g_err[512] = "";
+void set_last_error(const char* fmt, ...) {
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(g_err, sizeof(g_err), fmt, ap);
+  va_end(ap);
+}
+
+int num_sms() {
+  int dev = 0, n = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) return 0;
+  if (cudaDeviceGetAttribute(&n, cudaDevAttrMultiProcessorCount, dev) != cudaSuccess) return 0;
+  return n;
+}
+
+static bool device_ok() {
+  int dev = 0, major = 0, minor = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess) return false;
+  cudaDeviceGetAttribute(&major, cudaDevAttrComputeCapabilityMajor, dev);
+  cudaDeviceGetAttribute(&minor, cudaDevAttrComputeCapabilityMinor, dev);
+  return major == 10 && minor == 0;
+}
+
+// ------------------------------------------------------------------ tuning table
+// Measured choices (tune/README in DESIGN.md): key = (op, M/N/K buckets).
+struct Override {
+  int cg = 0, bn = 0, sep = 0, kc = 0;
+};
+static thread_local Override g_override;
+
+static int env_int(const char* name, int dflt) {
+  const char* v = getenv(name);
+  return (v && *v) ? atoi(v) : dflt;
+}
+
+static TcConfig choose_config(int epi_kind, int64_t M, int64_t N, int64_t K, int terms) {
+  TcConfig c = {};
+  c.terms = terms;
+  c.max_clusters = 0;
+  // default: CTA pair, 256 x 256 tiles, single accumulator in ping-pong, Kc = 256
+  c.cg = 2;
+  c.bn = 256;
+  c.sep = 0;
+  c.kc = 256;
+  if (epi_kind == EPI_STORE && M <= 128) { c.cg = 1; c.bn = 128; c.sep = 1; }
+  if (epi_kind != EPI_STORE) c.kc = (int)(((K + 63) / 64) * 64);
+  // thread-local API override, then environment (experiments)
+  if (g_override.cg) { c.cg = g_override.cg; c.bn = g_override.bn; c.sep = g_override.sep; }
+  if (g_override.kc && epi_kind == EPI_STORE) c.kc = g_override.kc;
+  c.cg = env_int("EGEMM_CG", c.cg);
+  c.bn = env_int("EGEMM_BN", c.bn);
+  c.sep = env_int("EGEMM_SEP", c.sep);
+  if (epi_kind == EPI_STORE) c.kc = env_int("EGEMM_KC", c.kc);
+  c.max_clusters = env_int("EGEMM_MAX_CLUSTERS", 0);
+  if (c.kc < 64) c.kc = 64;
+  c.kc = (c.kc / 64) * 64;
+  return c;
+}
+
+static size_t align256(size_t x) { return (x + 255) & ~size_t(255); }
+static int64_t ldk_of(int64_t K) { return ((K + 7) / 8) * 8; }
+
+struct Carver {
+  char* base;
+  size_t off = 0;
+  template <class T>
+  T* take(size_t count) {
+    T* p = base ? reinterpret_cast<T*>(base + off) : nullptr;
+    off += align256(count * sizeof(T));
+    return p;
+  }
+};
+
+// Make K-major hi/lo of an operand: pre-split pointers if given, else split into ws.
+// rows x K logical (K-major).  f32 layout: trans==0 -> rows x K (ld), trans==1 -> K x rows.
+static int stage_operand(const egemm_operand_t& op, int64_t rows, int64_t K, Carver& cv,
+                         const uint16_t** hi, const uint16_t** lo, int64_t* ld,
+                         cudaStream_t s) {
+  if (op.hi && op.lo) {
+    *hi = op.hi;
+    *lo = op.lo;
+    *ld = op.ld_split;
+    return 0;
+  }
+  const int64_t ldk = ldk_of(K);
+  uint16_t* h = cv.take<uint16_t>((size_t)(rows * ldk));
+  uint16_t* l = cv.take<uint16_t>((size_t)(rows * ldk));
+  int r = op.trans ? launch_split(op.f32, K, rows, op.ld, h, l, ldk, 1, nullptr, s)
+                   : launch_split(op.f32, rows, K, op.ld, h, l, ldk, 0, nullptr, s);
+  if (r) {
+    set_last_error("split launch failed");
+    return EGEMM_ERR_CUDA;
+  }
+  *hi = h;
+  *lo = l;
+  *ld = ldk;
+  return 0;
+}
+
+static int check_operand(const egemm_operand_t& op, int64_t rows, int64_t K, bool is_b,
+                         const char* name) {
+  bool pre = op.hi && op.lo;
+  if ((op.hi == nullptr) != (op.lo == nullptr)) {
+    set_last_error("%s: give both hi and lo or neither", name);
+    return EGEMM_ERR_INVALID_ARG;
+  }
+  if (pre) {
+    if (op.ld_split < K || (op.ld_split % 8) != 0 || ((uintptr_t)op.hi % 16) ||
+        ((uintptr_t)op.lo % 16)) {
+      set_last_error("%s: pre-split ld_split must be >= K, a multiple of 8, 16-B aligned", name);
+      return op.ld_split < K ? EGEMM_ERR_INVALID_ARG : EGEMM_ERR_UNSUPPORTED;
+    }
+    return 0;
+  }
+  if (!op.f32) {
+    set_last_error("%s: NULL data", name);
+    return EGEMM_ERR_INVALID_ARG;
+  }
+  // logical rows x K; stored (trans xor is_b) ? K x rows : rows x K
+  const bool k_outer = is_b ? !op.trans : op.trans;
+  const int64_t need = k_outer ? rows : K;
+  if (op.ld < need) {
+    set_last_error("%s: ld=%lld < %lld", name, (long long)op.ld, (long long)need);
+    return EGEMM_ERR_INVALID_ARG;
+  }
+  return 0;
+}
+
+}  // namespace egemm
+
+using namespace egemm;
+
+extern "C" {
+
+const char* egemm_status_string(int s) {
+  switch (s) {
+    case EGEMM_OK: return "EGEMM_OK";
+    case EGEMM_ERR_INVALID_ARG: return "EGEMM_ERR_INVALID_ARG";
+    case EGEMM_ERR_UNSUPPORTED: return "EGEMM_ERR_UNSUPPORTED";
+    case EGEMM_ERR_CUDA: return "EGEMM_ERR_CUDA";
+    case EGEMM_ERR_WORKSPACE: return "EGEMM_ERR_WORKSPACE";
+  }
+  return "EGEMM_ERR_UNKNOWN";
+}
+
+const char* egemm_last_error(void) { return g_err; }
+int egemm_version(void) { return 100; }
+int egemm_num_sms(void) { return num_sms(); }
+
+int egemm_set_config(int cg, int bn, int sep, int kc) {
+  if (cg == 0 && bn == 0 && sep == 0 && kc == 0) {
+    g_override = Override();
+    return EGEMM_OK;
+  }
+  bool ok = (cg == 2 && bn == 256 && sep == 0) || (cg == 1 && bn == 128) ||
+            (cg == 2 && bn == 128 && sep == 1);
+  if (!ok || kc < 0 || (kc % 64) != 0) {
+    set_last_error("unsupported config cg=%d bn=%d sep=%d kc=%d", cg, bn, sep, kc);
+    return EGEMM_ERR_UNSUPPORTED;
+  }
+  g_override.cg = cg;
+  g_override.bn = bn;
+  g_override.sep = sep;
+  g_override.kc = kc;
+  return EGEMM_OK;
+}
+
+int egemm_split(const float* x, int64_t rows, int64_t cols, int64_t ldx, uint16_t* hi,
+                uint16_t* lo, int64_t ldo, int transpose, uint32_t* range_flags, void* stream) {
+  if (rows < 0 || cols < 0) {
+    set_last_error("negative size");
+    return EGEMM_ERR_INVALID_ARG;
+  }
+  if (rows == 0 || cols == 0) return EGEMM_OK;
+  if (!x || !hi || !lo) {
+    set_last_error("NULL pointer");
+    return EGEMM_ERR_INVALID_ARG;
+  }
+  if (ldx < cols || ldo < (transpose ? rows : cols)) {
+    set_last_error("ld too small");
+    return EGEMM_ERR_INVALID_ARG;
+  }
+  if (!device_ok()) {
+    set_last_error("no sm_100 device");
+    return EGEMM_ERR_CUDA;
+  }
+  if (launch_split(x, rows, cols, ldx, hi, lo, ldo, transpose, range_flags, (cudaStream_t)stream)) {
+    set_last_error("split launch: %s", cudaGetErrorString(cudaGetLastError()));
+    return EGEMM_ERR_CUDA;
+  }
+  return EGEMM_OK;
+}
+
+size_t egemm_gemm_workspace_size(int64_t M, int64_t N, int64_t K, int a_presplit,
+                                 int b_presplit) {
+  if (M <= 0 || N <= 0 || K <= 0) return 0;
+  Carver cv{nullptr};
+  const int64_t ldk = ldk_of(K);
+  if (!a_presplit) { cv.take<uint16_t>((size_t)(M * ldk)); cv.take<uint16_t>((size_t)(M * ldk)); }
+  if (!b_presplit) { cv.take<uint16_t>((size_t)(N * ldk)); cv.take<uint16_t>((size_t)(N * ldk)); }
+  return cv.off;
+}
+
+int egemm_gemm(int64_t M, int64_t N, int64_t K, egemm_operand_t A, egemm_operand_t B,
+               const float* C, int64_t ldc, float* D, int64_t ldd, int terms, void* workspace,
+               size_t workspace_bytes, void* stream) {
+  cudaStream_t s = (cudaStream_t)stream;
+  if (M < 0 || N < 0 || K < 0) {
+    set_last_error("negative size");
+    return EGEMM_ERR_INVALID_ARG;
+  }
+  if (terms == 0) terms = 3;
+  if (terms != 3 && terms != 4) {
+    set_last_error("terms must be 0, 3 or 4");
+    return EGEMM_ERR_INVALID_ARG;
+  }
+  if (M == 0 || N == 0) return EGEMM_OK;
+  if (!D || ldd < N || (C && ldc < N)) {
+    set_last_error("D NULL or ldd/ldc < N");
+    return EGEMM_ERR_INVALID_ARG;
+  }
+  if (!device_ok()) {
+    set_last_error("no sm_100 device");
+    return EGEMM_ERR_CUDA;
+  }
+  if (K == 0) return launch_fill_c(M, N, C, ldc, D, ldd, s) ? EGEMM_ERR_CUDA : EGEMM_OK;
+  int r;
+  if ((r = check_operand(A, M, K, false, "A"))) return r;
+  if ((r = check_operand(B, N, K, true, "B"))) return r;
+  size_t need = egemm_gemm_workspace_size(M, N, K, A.hi != nullptr, B.hi != nullptr);
+  if (need > 0 && (!workspace || workspace_bytes < need)) {
+    set_last_error("workspace %zu < %zu", workspace_bytes, need);
+    return EGEMM_ERR_WORKSPACE;
+  }
+  Carver cv{reinterpret_cast<char*>(workspace)};
+  TcOperands ops = {};
+  if ((r = stage_operand(A, M, K, cv, &ops.a_hi, &ops.a_lo, &ops.lda, s))) return r;
+  // B logical K x N: as an operand it is N rows x K; f32 trans==0 means stored K x N.
+  egemm_operand_t Bt = B;
+  Bt.trans = !B.trans;
+  if ((r = stage_operand(Bt, N, K, cv, &ops.b_hi, &ops.b_lo, &ops.ldb, s))) return r;
+  TcConfig cfg = choose_config(EPI_STORE, M, N, K, terms);
+  TcEpilogue epi = {};
+  epi.kind = EPI_STORE;
+  epi.D = D;
+  epi.ldd = ldd;
+  epi.C = C;
+  epi.ldc = ldc;
+  r = launch_tc(M, N, K, ops, cfg, epi, s);
+  return r == 0 ? EGEMM_OK : (r == 2 ? EGEMM_ERR_UNSUPPORTED : EGEMM_ERR_CUDA);
+}
+
+static int knn_slices(int64_t nq, int64_t nx, int cg, int bn) {
+  const int64_t m_tiles = (nq + 128 * cg - 1) / (128 * cg);
+  const int64_t n_tiles = (nx + bn - 1) / bn;
+  const int64_t clusters = num_sms() / cg > 0 ? num_sms() / cg : 1;
+  int best = 1;
+  double best_eff = 0.0;
+  for (int s = 1; s <= 8 && s <= n_tiles; s++) {
+    int64_t units = m_tiles * s;
+    int64_t waves = (units + clusters - 1) / clusters;
+    double eff = (double)units / (double)(waves * clusters);
+    if (eff >= 0.97) return s;
+    if (eff > best_eff + 1e-9) { best_eff = eff; best = s; }
+  }
+  return best;
+}
+
+size_t egemm_knn_workspace_size(int64_t nx, int64_t nq, int64_t d, int k, int x_presplit) {
+  if (nx <= 0 || nq <= 0 || d <= 0 || k <= 0) return 0;
+  Carver cv{nullptr};
+  const int64_t ldk = ldk_of(d);
+  if (!x_presplit) { cv.take<uint16_t>((size_t)(nx * ldk)); cv.take<uint16_t>((size_t)(nx * ldk)); }
+  cv.take<uint16_t>((size_t)(nq * ldk));
+  cv.take<uint16_t>((size_t)(nq * ldk));
+  cv.take<float>((size_t)nx);
+  cv.take<float>((size_t)nq);
+  cv.take<float>((size_t)(8 * nq * k));
+  cv.take<int32_t>((size_t)(8 * nq * k));
+  return cv.off;
+}
+
+int egemm_knn(egemm_operand_t X, int64_t nx, egemm_operand_t Q, int64_t nq, int64_t d, int k,
+              int32_t* out_idx, float* out_dist, void* workspace, size_t workspace_bytes,
+              void* stream) {
+  cudaStream_t s = (cudaStream_t)stream;
+  if (nx < 0 || nq < 0 || d <= 0 || k < 1 || k > 16 || k > nx) {
+    set_last_error("need nx, nq >= 0, d > 0, 1 <= k <= min(16, nx)");
+    return EGEMM_ERR_INVALID_ARG;
+  }
+  if (nq == 0) return EGEMM_OK;
+  if (!X.f32 || !Q.f32 || X.trans || Q.trans || X.ld < d || Q.ld < d || !out_idx || !out_dist) {
+    set_last_error("X/Q need fp32 rows (trans 0, ld >= d) and outputs");
+    return EGEMM_ERR_INVALID_ARG;
+  }
+  if (d > 1024) {
+    set_last_error("d > 1024 not supported by the fused epilogue");
+    return EGEMM_ERR_UNSUPPORTED;
+  }
+  if (!device_ok()) {
+    set_last_error("no sm_100 device");
+    return EGEMM_ERR_CUDA;
+  }
+  int r;
+  if ((r = check_operand(X, nx, d, false, "X"))) return r;
+  size_t need = egemm_knn_workspace_size(nx, nq, d, k, X.hi != nullptr);
+  if (!workspace || workspace_bytes < need) {
+    set_last_error("workspace %zu < %zu", workspace_bytes, need);
+    return EGEMM_ERR_WORKSPACE;
+  }
+  TcConfig cfg = choose_config(EPI_KNN, nq, nx, d, 3);
+  Carver cv{reinterpret_cast<char*>(workspace)};
+  TcOperands ops = {};
+  if ((r = stage_operand(X, nx, d, cv, &ops.b_hi, &ops.b_lo, &ops.ldb, s))) return r;
+  egemm_operand_t Qs = Q;
+  Qs.hi = Qs.lo = nullptr;
+  if ((r = stage_operand(Qs, nq, d, cv, &ops.a_hi, &ops.a_lo, &ops.lda, s))) return r;
+  float* xnorm = cv.take<float>((size_t)nx);
+  float* qnorm = cv.take<float>((size_t)nq);
+  float* pkey = cv.take<float>((size_t)(8 * nq * k));
+  int32_t* pidx = cv.take<int32_t>((size_t)(8 * nq * k));
+  if (launch_rownorm(X.f32, nx, d, X.ld, xnorm, s) || launch_rownorm(Q.f32, nq, d, Q.ld, qnorm, s))
+    return EGEMM_ERR_CUDA;
+  TcEpilogue epi = {};
+  epi.kind = EPI_KNN;
+  epi.bnorm = xnorm;
+  epi.knn_k = k;
+  epi.n_slices = knn_slices(nq, nx, cfg.cg, cfg.bn);
+  epi.part_key = pkey;
+  epi.part_idx = pidx;
+  r = launch_tc(nq, nx, d, ops, cfg, epi, s);
+  if (r) return r == 2 ? EGEMM_ERR_UNSUPPORTED : EGEMM_ERR_CUDA;
+  if (launch_knn_merge(pkey, pidx, epi.n_slices, nq, k, qnorm, out_idx, out_dist, s))
+    return EGEMM_ERR_CUDA;
+  return EGEMM_OK;
+}
+
+size_t egemm_kmeans_workspace_size(int64_t n, int64_t d, int64_t kc, int x_presplit) {
+  if (n <= 0 || d <= 0 || kc <= 0) return 0;
+  Carver cv{nullptr};
+  const int64_t ldk = ldk_of(d);
+  if (!x_presplit) { cv.take<uint16_t>((size_t)(n * ldk)); cv.take<uint16_t>((size_t)(n * ldk)); }
+  cv.take<uint16_t>((size_t)(kc * ldk));
+  cv.take<uint16_t>((size_t)(kc * ldk));
+  cv.take<float>((size_t)kc);
+  cv.take<float>((size_t)n);
+  cv.take<float>((size_t)n);
+  return cv.off;
+}
+
+int egemm_kmeans_step(egemm_operand_t X, int64_t n, int64_t d, const float* centroids, int64_t kc,
+                      int32_t* assign, double* sums, int64_t* counts, double* inertia,
+                      void* workspace, size_t workspace_bytes, void* stream) {
+  cudaStream_t s = (cudaStream_t)stream;
+  if (n < 0 || d <= 0 || kc <= 0 || !centroids || !assign || !sums || !counts) {
+    set_last_error("need n >= 0, d > 0, kc > 0 and non-NULL centroids/assign/sums/counts");
+    return EGEMM_ERR_INVALID_ARG;
+  }
+  if (!X.f32 || X.trans || X.ld < d) {
+    set_last_error("X needs fp32 rows (trans 0, ld >= d)");
+    return EGEMM_ERR_INVALID_ARG;
+  }
+  if (d > 1024) {
+    set_last_error("d > 1024 not supported by the fused epilogue");
+    return EGEMM_ERR_UNSUPPORTED;
+  }
+  if (!device_ok()) {
+    set_last_error("no sm_100 device");
+    return EGEMM_ERR_CUDA;
+  }
+  int r;
+  if ((r = check_operand(X, n, d, false, "X"))) return r;
+  size_t need = egemm_kmeans_workspace_size(n, d, kc, X.hi != nullptr);
+  if (n > 0 && (!workspace || workspace_bytes < need)) {
+    set_last_error("workspace %zu < %zu", workspace_bytes, need);
+    return EGEMM_ERR_WORKSPACE;
+  }
+  if (n == 0)
+    return launch_kmeans_accumulate(nullptr, 0, d, d, nullptr, nullptr, nullptr, kc, sums, counts,
+                                    inertia, s)
+               ? EGEMM_ERR_CUDA
+               : EGEMM_OK;
+  TcConfig cfg = choose_config(EPI_KMEANS, n, kc, d, 3);
+  Carver cv{reinterpret_cast<char*>(workspace)};
+  TcOperands ops = {};
+  if ((r = stage_operand(X, n, d, cv, &ops.a_hi, &ops.a_lo, &ops.lda, s))) return r;
+  egemm_operand_t Cop = {centroids, nullptr, nullptr, d, 0, 0};
+  if ((r = stage_operand(Cop, kc, d, cv, &ops.b_hi, &ops.b_lo, &ops.ldb, s))) return r;
+  float* cnorm = cv.take<float>((size_t)kc);
+  float* best = cv.take<float>((size_t)n);
+  float* xnorm = cv.take<float>((size_t)n);
+  if (launch_rownorm(centroids, kc, d, d, cnorm, s)) return EGEMM_ERR_CUDA;
+  if (inertia && launch_rownorm(X.f32, n, d, X.ld, xnorm, s)) return EGEMM_ERR_CUDA;
+  TcEpilogue epi = {};
+  epi.kind = EPI_KMEANS;
+  epi.bnorm = cnorm;
+  epi.assign = assign;
+  epi.best_key = best;
+  r = launch_tc(n, kc, d, ops, cfg, epi, s);
+  if (r) return r == 2 ? EGEMM_ERR_UNSUPPORTED : EGEMM_ERR_CUDA;
+  if (launch_kmeans_accumulate(X.f32, n, d, X.ld, assign, best, xnorm, kc, sums, counts, inertia,
+                               s))
+    return EGEMM_ERR_CUDA;
+  return EGEMM_OK;
+}
+
+int egemm_kmeans_finalize(const double* sums, const int64_t* counts, int64_t kc, int64_t d,
+                          float* centroids, void* stream) {
+  if (kc < 0 || d < 0 || (kc * d > 0 && (!sums || !counts || !centroids))) {
+    set_last_error("bad kmeans_finalize arguments");
+    return EGEMM_ERR_INVALID_ARG;
+  }
+  if (!device_ok()) {
+    set_last_error("no sm_100 device");
+    return EGEMM_ERR_CUDA;
+  }
+  return launch_kmeans_finalize(sums, counts, kc, d, centroids, (cudaStream_t)stream)
+             ? EGEMM_ERR_CUDA
+             : EGEMM_OK;
+}
+
+}  // extern "C"

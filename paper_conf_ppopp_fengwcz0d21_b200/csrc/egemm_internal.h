@@ -1,0 +1,76 @@
+// egemm_internal.h -- declarations shared by the library's translation units (not public).
+#pragma once
+#include <cstdint>
+#include <cuda_runtime.h>
+
+namespace egemm {
+
+int num_sms();
+
+int launch_split(const float* x, int64_t rows, int64_t cols, int64_t ldx, uint16_t* hi,
+                 uint16_t* lo, int64_t ldo, int transpose, uint32_t* range_flags,
+                 cudaStream_t stream);
+
+// Epilogue policies of the tensor-core kernel.
+enum EpiKind : int { EPI_STORE = 0, EPI_KNN = 1, EPI_KMEANS = 2 };
+
+// Operands of one launch of the tcgen05 kernel.  hi/lo are fp16 bit patterns, K-major:
+// A is rows_a x K (row stride lda elements), B is rows_b x K (row stride ldb).
+struct TcOperands {
+  const uint16_t* a_hi;
+  const uint16_t* a_lo;
+  int64_t lda;
+  const uint16_t* b_hi;
+  const uint16_t* b_lo;
+  int64_t ldb;
+};
+
+struct TcConfig {
+  int cg;        // 1 or 2 (cta_group)
+  int bn;        // MMA N per cluster tile
+  int sep;       // separate hh / cross accumulators
+  int kc;        // promotion interval in k elements (multiple of 64)
+  int terms;     // 3 or 4
+  int max_clusters;  // 0 = all SMs
+};
+
+struct TcEpilogue {
+  int kind;
+  // EPI_STORE
+  float* D;
+  int64_t ldd;
+  const float* C;
+  int64_t ldc;
+  // EPI_KNN / EPI_KMEANS: per-B-row squared norms (||x_j||^2 or ||c_j||^2)
+  const float* bnorm;
+  // EPI_KNN
+  int knn_k;
+  int n_slices;
+  float* part_key;     // [n_slices][M][knn_k]
+  int32_t* part_idx;   // [n_slices][M][knn_k]
+  // EPI_KMEANS
+  int32_t* assign;     // [M]
+  float* best_key;     // [M] ||c_a||^2 - 2 x.c_a
+};
+
+int launch_tc(int64_t M, int64_t N, int64_t K, const TcOperands& ops, const TcConfig& cfg,
+              const TcEpilogue& epi, cudaStream_t stream);
+
+// apps.cu
+int launch_rownorm(const float* x, int64_t rows, int64_t d, int64_t ld, float* out,
+                   cudaStream_t stream);
+int launch_knn_merge(const float* part_key, const int32_t* part_idx, int n_slices, int64_t nq,
+                     int k, const float* qnorm, int32_t* out_idx, float* out_dist,
+                     cudaStream_t stream);
+int launch_kmeans_accumulate(const float* X, int64_t n, int64_t d, int64_t ldx,
+                             const int32_t* assign, const float* best_key, const float* xnorm,
+                             int64_t kc, double* sums, int64_t* counts, double* inertia,
+                             cudaStream_t stream);
+int launch_kmeans_finalize(const double* sums, const int64_t* counts, int64_t kc, int64_t d,
+                           float* centroids, cudaStream_t stream);
+int launch_fill_c(int64_t M, int64_t N, const float* C, int64_t ldc, float* D, int64_t ldd,
+                  cudaStream_t stream);
+
+void set_last_error(const char* fmt, ...);
+
+}  // namespace egemm

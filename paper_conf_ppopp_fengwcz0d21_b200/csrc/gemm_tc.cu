@@ -1,0 +1,599 @@
+// gemm_tc.cu -- the EGEMM tensor-core kernel for sm_100a (tcgen05 + TMA + TMEM).
+//
+// Computes, per output element, the emulated extended-precision product of Alg. 1
+// (PAPER.md P:739-757):  sum_k  A_hi*B_hi + A_hi*B_lo + A_lo*B_hi (+ A_lo*B_lo if terms=4)
+// on fp16 tensor cores with fp32 accumulation (Alg. 1 l.5-8; "data combination through the
+// fp32 accumulator"), and hands the fp32 result to an epilogue policy:
+//   EPI_STORE   D = result (+ C)                          (Alg. 1's D = A x B + C)
+//   EPI_KNN     key = ||x_j||^2 - 2 q.x_j, register top-k  (kNN case study)
+//   EPI_KMEANS  key = ||c_j||^2 - 2 x.c_j, running argmin (kMeans case study)
+//
+// B200 design:
+//  * warp-specialised persistent kernel, 12 warps: w0 TMA producer, w1 MMA issuer (one
+//    elected lane; leader CTA only when CG == 2), w2 TMEM allocator, w3 idle, w4..w11
+//    epilogue (two warps per TMEM lane quarter, each owning BN/2 columns).
+//  * operands: pre-split fp16 hi/lo, K-major, loaded by TMA into 128-B-swizzled stages
+//    (BK = 64 fp16 = one swizzle atom row) in a STAGES-deep full/empty mbarrier ring.
+//  * CG == 2: cta_group::2 pair, UMMA M = 256, each CTA stages its 128 A rows and BN/2 B
+//    rows; the leader issues the MMAs, commits multicast to both CTAs.
+//  * accumulation: two TMEM accumulator buffers used in ping-pong per k-chunk of Kc
+//    elements ("promotion"): the MMA warp fills one while the epilogue warps drain the
+//    other into an fp32 register running total with round-to-nearest adds.  This bounds
+//    the error of the tensor core's internal fp32 accumulation (P:729-737 report only 21
+//    matching bits) to Kc-long sums -- the TMEM analogue of the paper's FRAG caching of
+//    C across the k-loop (Table 2).  SEP additionally keeps the
+//    hi*hi and cross products in separate accumulators (needs 4 x BN TMEM columns).
+#include <cuda.h>
+#include <cudaTypedefs.h>
+#include <cuda_runtime.h>
+#include <cstdint>
+#include <cstdio>
+#include <mutex>
+#include "egemm_internal.h"
+#include "ptx.cuh"
+
+namespace egemm {
+
+constexpr int kBM = 128;       // rows per CTA (TMEM lanes)
+constexpr int kBK = 64;        // k elements per stage (128 B of fp16: one SW128 row)
+constexpr int kThreads = 384;  // 12 warps
+constexpr int kEpiWarp0 = 4;
+constexpr int kKnnMax = 16;
+
+struct KParams {
+  int M, N;
+  int num_kb;       // ceil(K / 64)
+  int kb_per_chunk; // Kc / 64
+  int terms;
+  int m_tiles, n_tiles;
+  int num_units;
+  int n_slices, tiles_per_slice;  // EPI_KNN
+  // epilogue
+  float* D;
+  int64_t ldd;
+  const float* C;
+  int64_t ldc;
+  int vec_ok;
+  const float* bnorm;
+  int knn_k;
+  float* part_key;
+  int32_t* part_idx;
+  int32_t* assign;
+  float* best_key;
+};
+
+template <int CG, int BN>
+struct Geo {
+  static constexpr int BNC = BN / CG;                  // B rows staged per CTA
+  static constexpr int A_BYTES = kBM * kBK * 2;        // one of A_hi / A_lo
+  static constexpr int B_BYTES = BNC * kBK * 2;        // one of B_hi / B_lo
+  static constexpr int STAGE_BYTES = 2 * A_BYTES + 2 * B_BYTES;
+  static constexpr int COLS = BN / 2;                  // columns per epilogue warp
+};
+
+struct UnitInfo {
+  int m_tile, n_begin, n_count, slice;
+};
+
+template <int EPI>
+__device__ __forceinline__ UnitInfo decode_unit(const KParams& p, int u) {
+  UnitInfo r;
+  if constexpr (EPI == EPI_STORE) {
+    // bands of up to 8 m-tiles, m fastest inside a band: concurrent clusters share A and B
+    // k-slabs in L2.
+    const int GM = 8;
+    int band = u / (GM * p.n_tiles);
+    int m0 = band * GM;
+    int gm = min(GM, p.m_tiles - m0);
+    int idx = u - band * GM * p.n_tiles;
+    r.m_tile = m0 + idx % gm;
+    r.n_begin = idx / gm;
+    r.n_count = 1;
+    r.slice = 0;
+  } else if constexpr (EPI == EPI_KNN) {
+    // concurrent clusters share the reference slice (B) -> one HBM read per B tile.
+    r.slice = u / p.m_tiles;
+    r.m_tile = u - r.slice * p.m_tiles;
+    r.n_begin = r.slice * p.tiles_per_slice;
+    r.n_count = min(p.tiles_per_slice, p.n_tiles - r.n_begin);
+    if (r.n_count < 0) r.n_count = 0;
+  } else {
+    r.m_tile = u;
+    r.n_begin = 0;
+    r.n_count = p.n_tiles;
+    r.slice = 0;
+  }
+  return r;
+}
+
+// lexicographic (key, idx) insertion into an ascending register list of length KN
+template <int KN>
+__device__ __forceinline__ void topk_insert(float (&kd)[KN], int (&ki)[KN], float key, int idx) {
+  if (key < kd[KN - 1] || (key == kd[KN - 1] && idx < ki[KN - 1])) {
+    kd[KN - 1] = key;
+    ki[KN - 1] = idx;
+#pragma unroll
+    for (int t = KN - 1; t > 0; t--) {
+      bool sw = (kd[t] < kd[t - 1]) || (kd[t] == kd[t - 1] && ki[t] < ki[t - 1]);
+      float a = kd[t], b = kd[t - 1];
+      int ia = ki[t], ib = ki[t - 1];
+      kd[t] = sw ? b : a;
+      kd[t - 1] = sw ? a : b;
+      ki[t] = sw ? ib : ia;
+      ki[t - 1] = sw ? ia : ib;
+    }
+  }
+}
+
+__device__ __forceinline__ void named_bar_sync(int id, int nthreads) {
+  asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
+}
+
+template <int CG, int BN, bool SEP, int EPI, int STAGES>
+__global__ void __launch_bounds__(kThreads, 1)
+    egemm_tc_kernel(const __grid_constant__ CUtensorMap tm_ahi,
+                    const __grid_constant__ CUtensorMap tm_alo,
+                    const __grid_constant__ CUtensorMap tm_bhi,
+                    const __grid_constant__ CUtensorMap tm_blo, const KParams p) {
+  using G = Geo<CG, BN>;
+  constexpr int COLS = G::COLS;
+  constexpr int NACC = SEP ? 4 : 2;
+  constexpr uint32_t TMEM_COLS = (NACC * BN <= 32) ? 32 : (NACC * BN <= 64) ? 64
+                                 : (NACC * BN <= 128) ? 128 : (NACC * BN <= 256) ? 256 : 512;
+  static_assert(NACC * BN <= 512, "TMEM overflow");
+  static_assert(COLS % 32 == 0, "epilogue column split");
+
+  extern __shared__ __align__(1024) uint8_t smem_raw[];
+  uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
+                                             ~uintptr_t(1023));
+  uint8_t* stage_base = smem;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + STAGES * G::STAGE_BYTES);
+  uint64_t* full = bars;
+  uint64_t* empty = bars + STAGES;
+  uint64_t* acc_full = bars + 2 * STAGES;
+  uint64_t* acc_empty = bars + 2 * STAGES + 2;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * STAGES + 4);
+  uint8_t* scratch = reinterpret_cast<uint8_t*>(bars + 2 * STAGES + 8);  // epilogue merges
+
+  const int warp = threadIdx.x >> 5;
+  const int lane = threadIdx.x & 31;
+  const uint32_t rank = (CG == 2) ? ptx::cluster_ctarank() : 0u;
+  const int cluster = (CG == 2) ? (int)ptx::cluster_id_x() : (int)blockIdx.x;
+  const int nclusters = (CG == 2) ? (int)ptx::nclusters_x() : (int)gridDim.x;
+  const bool leader = (rank == 0);
+
+  if (warp == 0 && lane == 0) {
+    ptx::prefetch_tmap(&tm_ahi);
+    ptx::prefetch_tmap(&tm_alo);
+    ptx::prefetch_tmap(&tm_bhi);
+    ptx::prefetch_tmap(&tm_blo);
+  }
+  if (warp == 1 && lane == 0) {
+    for (int s = 0; s < STAGES; s++) {
+      ptx::mbar_init(&full[s], 1);
+      ptx::mbar_init(&empty[s], 1);
+    }
+    for (int b = 0; b < 2; b++) {
+      ptx::mbar_init(&acc_full[b], 1);
+      ptx::mbar_init(&acc_empty[b], 8 * CG);  // one arrive per epilogue warp of the pair
+    }
+    ptx::fence_mbar_init();
+  }
+  if (warp == 2) ptx::tmem_alloc<CG>(tmem_slot, TMEM_COLS);
+  ptx::tc_fence_before();
+  if constexpr (CG == 2) ptx::cluster_sync(); else __syncthreads();
+  ptx::tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+
+  const int nch = (p.num_kb + p.kb_per_chunk - 1) / p.kb_per_chunk;
+
+  if (warp == 0) {
+    // ============================ TMA producer ============================
+    if (lane == 0) {
+      int stage = 0;
+      uint32_t phase = 0;
+      for (int u = cluster; u < p.num_units; u += nclusters) {
+        UnitInfo ui = decode_unit<EPI>(p, u);
+        const int arow = ui.m_tile * (kBM * CG) + (int)rank * kBM;
+        for (int ns = 0; ns < ui.n_count; ns++) {
+          const int brow = (ui.n_begin + ns) * BN + (int)rank * G::BNC;
+          for (int kb = 0; kb < p.num_kb; kb++) {
+            ptx::mbar_wait(&empty[stage], phase ^ 1u);
+            uint8_t* sb = stage_base + stage * G::STAGE_BYTES;
+            if (leader) ptx::mbar_arrive_expect_tx(&full[stage], G::STAGE_BYTES * CG);
+            const int k0 = kb * kBK;
+            if constexpr (CG == 1) {
+              ptx::tma_load_2d(&tm_ahi, &full[stage], sb, k0, arow);
+              ptx::tma_load_2d(&tm_alo, &full[stage], sb + G::A_BYTES, k0, arow);
+              ptx::tma_load_2d(&tm_bhi, &full[stage], sb + 2 * G::A_BYTES, k0, brow);
+              ptx::tma_load_2d(&tm_blo, &full[stage], sb + 2 * G::A_BYTES + G::B_BYTES, k0, brow);
+            } else {
+              ptx::tma_load_2d_pair(&tm_ahi, &full[stage], sb, k0, arow);
+              ptx::tma_load_2d_pair(&tm_alo, &full[stage], sb + G::A_BYTES, k0, arow);
+              ptx::tma_load_2d_pair(&tm_bhi, &full[stage], sb + 2 * G::A_BYTES, k0, brow);
+              ptx::tma_load_2d_pair(&tm_blo, &full[stage], sb + 2 * G::A_BYTES + G::B_BYTES, k0,
+                                    brow);
+            }
+            if (++stage == STAGES) { stage = 0; phase ^= 1u; }
+          }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    // ============================ MMA issuer ============================
+    if (leader && lane == 0) {
+      constexpr uint32_t idesc = ptx::idesc_f16_f32(kBM * CG, BN);
+      const uint32_t sbase = ptx::smem_u32(stage_base);
+      int stage = 0;
+      uint32_t phase = 0;
+      uint32_t chunk_ctr = 0;
+      for (int u = cluster; u < p.num_units; u += nclusters) {
+        UnitInfo ui = decode_unit<EPI>(p, u);
+        for (int ns = 0; ns < ui.n_count; ns++) {
+          for (int ch = 0; ch < nch; ch++) {
+            const uint32_t buf = chunk_ctr & 1u;
+            const uint32_t use = chunk_ctr >> 1;
+            if constexpr (CG == 2) ptx::mbar_wait_cluster(&acc_empty[buf], (use & 1u) ^ 1u);
+            else ptx::mbar_wait(&acc_empty[buf], (use & 1u) ^ 1u);
+            ptx::tc_fence_after();
+            const uint32_t acc_hh = tmem_base + (SEP ? 2 * buf : buf) * BN;
+            const uint32_t acc_x = SEP ? acc_hh + BN : acc_hh;
+            const int kb0 = ch * p.kb_per_chunk;
+            const int kb1 = min(p.num_kb, kb0 + p.kb_per_chunk);
+            for (int kb = kb0; kb < kb1; kb++) {
+              ptx::mbar_wait(&full[stage], phase);
+              ptx::tc_fence_after();
+              const uint32_t sa = sbase + stage * G::STAGE_BYTES;
+              const uint64_t d_ahi = ptx::sdesc_kmajor_sw128(sa);
+              const uint64_t d_alo = ptx::sdesc_kmajor_sw128(sa + G::A_BYTES);
+              const uint64_t d_bhi = ptx::sdesc_kmajor_sw128(sa + 2 * G::A_BYTES);
+              const uint64_t d_blo = ptx::sdesc_kmajor_sw128(sa + 2 * G::A_BYTES + G::B_BYTES);
+#pragma unroll
+              for (int k = 0; k < kBK / 16; k++) {
+                const uint64_t ko = (uint64_t)(k * 2);  // +32 B per 16-wide k step (>>4)
+                const uint32_t first = (kb > kb0 || k > 0) ? 1u : 0u;
+                // Alg. 1 order: products involving lo first, hi*hi last
+                ptx::mma_f16<CG>(acc_x, d_ahi + ko, d_blo + ko, idesc, first);
+                ptx::mma_f16<CG>(acc_x, d_alo + ko, d_bhi + ko, idesc, 1u);
+                if (p.terms == 4) ptx::mma_f16<CG>(acc_x, d_alo + ko, d_blo + ko, idesc, 1u);
+                ptx::mma_f16<CG>(acc_hh, d_ahi + ko, d_bhi + ko, idesc, SEP ? first : 1u);
+              }
+              ptx::mma_commit<CG>(&empty[stage]);
+              if (++stage == STAGES) { stage = 0; phase ^= 1u; }
+            }
+            ptx::mma_commit<CG>(&acc_full[buf]);
+            chunk_ctr++;
+          }
+        }
+      }
+    }
+  } else if (warp >= kEpiWarp0) {
+    // ============================ epilogue ============================
+    const int ew = warp - kEpiWarp0;
+    const int q = warp & 3;         // TMEM lane quarter this warp may access
+    const int cgp = ew >> 2;        // column half
+    const uint32_t lane_off = (uint32_t)(q * 32) << 16;
+    uint32_t chunk_ctr = 0;
+    const int row_in_cta = q * 32 + lane;
+
+    float kd[kKnnMax];
+    int ki[kKnnMax];
+    float best = __int_as_float(0x7f800000);
+    int besti = 0x7fffffff;
+
+    for (int u = cluster; u < p.num_units; u += nclusters) {
+      UnitInfo ui = decode_unit<EPI>(p, u);
+      const int64_t row = (int64_t)ui.m_tile * (kBM * CG) + rank * kBM + row_in_cta;
+      if constexpr (EPI == EPI_KNN) {
+#pragma unroll
+        for (int t = 0; t < kKnnMax; t++) { kd[t] = __int_as_float(0x7f800000); ki[t] = 0x7fffffff; }
+      }
+      if constexpr (EPI == EPI_KMEANS) { best = __int_as_float(0x7f800000); besti = 0x7fffffff; }
+
+      for (int ns = 0; ns < ui.n_count; ns++) {
+        const int col_base = (ui.n_begin + ns) * BN + cgp * COLS;
+        if constexpr (EPI == EPI_STORE) {
+          float tot[COLS];
+          float totx[SEP ? COLS : 1];
+#pragma unroll
+          for (int j = 0; j < COLS; j++) tot[j] = 0.f;
+          if constexpr (SEP) {
+#pragma unroll
+            for (int j = 0; j < COLS; j++) totx[j] = 0.f;
+          }
+          for (int ch = 0; ch < nch; ch++) {
+            const uint32_t buf = chunk_ctr & 1u;
+            const uint32_t use = chunk_ctr >> 1;
+            ptx::mbar_wait(&acc_full[buf], use & 1u);
+            ptx::tc_fence_after();
+            const uint32_t acc_hh = tmem_base + lane_off + (SEP ? 2 * buf : buf) * BN + cgp * COLS;
+#pragma unroll
+            for (int c = 0; c < COLS / 32; c++) {
+              float v[32];
+              ptx::tmem_ld32(acc_hh + c * 32, v);
+              ptx::tmem_wait_ld();
+#pragma unroll
+              for (int i = 0; i < 32; i++) tot[c * 32 + i] = __fadd_rn(tot[c * 32 + i], v[i]);
+              if constexpr (SEP) {
+                ptx::tmem_ld32(acc_hh + BN + c * 32, v);
+                ptx::tmem_wait_ld();
+#pragma unroll
+                for (int i = 0; i < 32; i++) totx[c * 32 + i] = __fadd_rn(totx[c * 32 + i], v[i]);
+              }
+            }
+            ptx::tc_fence_before();
+            __syncwarp();
+            if (lane == 0) {
+              if constexpr (CG == 1) ptx::mbar_arrive(&acc_empty[buf]);
+              else ptx::mbar_arrive_cluster(&acc_empty[buf], 0);
+            }
+            chunk_ctr++;
+          }
+          if constexpr (SEP) {
+#pragma unroll
+            for (int j = 0; j < COLS; j++) tot[j] = __fadd_rn(tot[j], totx[j]);
+          }
+          if (row < p.M) {
+            float* drow = p.D + row * p.ldd;
+            const float* crow = p.C ? p.C + row * p.ldc : nullptr;
+            if (p.vec_ok && col_base + COLS <= p.N) {
+#pragma unroll
+              for (int j = 0; j < COLS; j += 4) {
+                float4 o = make_float4(tot[j], tot[j + 1], tot[j + 2], tot[j + 3]);
+                if (crow) {
+                  float4 cv = *reinterpret_cast<const float4*>(crow + col_base + j);
+                  o.x = __fadd_rn(o.x, cv.x); o.y = __fadd_rn(o.y, cv.y);
+                  o.z = __fadd_rn(o.z, cv.z); o.w = __fadd_rn(o.w, cv.w);
+                }
+                *reinterpret_cast<float4*>(drow + col_base + j) = o;
+              }
+            } else {
+#pragma unroll
+              for (int j = 0; j < COLS; j++) {
+                int col = col_base + j;
+                if (col < p.N) drow[col] = crow ? __fadd_rn(tot[j], crow[col]) : tot[j];
+              }
+            }
+          }
+        } else {
+          // kNN / kMeans: one chunk per n-step (host guarantees Kc >= K)
+          const uint32_t buf = chunk_ctr & 1u;
+          const uint32_t use = chunk_ctr >> 1;
+          ptx::mbar_wait(&acc_full[buf], use & 1u);
+          ptx::tc_fence_after();
+          const uint32_t acc_hh = tmem_base + lane_off + (SEP ? 2 * buf : buf) * BN + cgp * COLS;
+#pragma unroll 1
+          for (int c = 0; c < COLS / 32; c++) {
+            float v[32];
+            ptx::tmem_ld32(acc_hh + c * 32, v);
+            ptx::tmem_wait_ld();
+            if constexpr (SEP) {
+              float w[32];
+              ptx::tmem_ld32(acc_hh + BN + c * 32, w);
+              ptx::tmem_wait_ld();
+#pragma unroll
+              for (int i = 0; i < 32; i++) v[i] = __fadd_rn(v[i], w[i]);
+            }
+            const int c0 = col_base + c * 32;
+            float bn[32];
+            if (c0 + 32 <= p.N) {
+#pragma unroll
+              for (int i = 0; i < 32; i += 4) {
+                float4 t = __ldg(reinterpret_cast<const float4*>(p.bnorm + c0 + i));
+                bn[i] = t.x; bn[i + 1] = t.y; bn[i + 2] = t.z; bn[i + 3] = t.w;
+              }
+            } else {
+#pragma unroll
+              for (int i = 0; i < 32; i++)
+                bn[i] = (c0 + i < p.N) ? __ldg(p.bnorm + c0 + i) : __int_as_float(0x7f800000);
+            }
+#pragma unroll
+            for (int i = 0; i < 32; i++) {
+              const float key = __fmaf_rn(-2.f, v[i], bn[i]);  // ||b||^2 - 2 a.b (exact *2)
+              if constexpr (EPI == EPI_KNN) {
+                topk_insert<kKnnMax>(kd, ki, key, c0 + i);
+              } else {
+                if (key < best) { best = key; besti = c0 + i; }
+              }
+            }
+          }
+          ptx::tc_fence_before();
+          __syncwarp();
+          if (lane == 0) {
+            if constexpr (CG == 1) ptx::mbar_arrive(&acc_empty[buf]);
+            else ptx::mbar_arrive_cluster(&acc_empty[buf], 0);
+          }
+          chunk_ctr++;
+        }
+      }
+
+      // ---- unit end: merge the two column halves of each row, write the unit's result
+      if constexpr (EPI == EPI_KNN) {
+        float* sk = reinterpret_cast<float*>(scratch) + (q * 32 + lane) * kKnnMax;
+        int* si = reinterpret_cast<int*>(scratch + kBM * kKnnMax * 4) + (q * 32 + lane) * kKnnMax;
+        if (cgp == 1) {
+#pragma unroll
+          for (int t = 0; t < kKnnMax; t++) { sk[t] = kd[t]; si[t] = ki[t]; }
+        }
+        named_bar_sync(1 + q, 64);
+        if (cgp == 0) {
+#pragma unroll 1
+          for (int t = 0; t < kKnnMax; t++) topk_insert<kKnnMax>(kd, ki, sk[t], si[t]);
+          if (row < p.M) {
+            const int64_t o = ((int64_t)ui.slice * p.M + row) * p.knn_k;
+#pragma unroll
+            for (int t = 0; t < kKnnMax; t++)
+              if (t < p.knn_k) { p.part_key[o + t] = kd[t]; p.part_idx[o + t] = ki[t]; }
+          }
+        }
+        named_bar_sync(1 + q, 64);
+      } else if constexpr (EPI == EPI_KMEANS) {
+        float* sk = reinterpret_cast<float*>(scratch) + (q * 32 + lane);
+        int* si = reinterpret_cast<int*>(scratch + kBM * 4) + (q * 32 + lane);
+        if (cgp == 1) { *sk = best; *si = besti; }
+        named_bar_sync(1 + q, 64);
+        if (cgp == 0) {
+          float ob = *sk;
+          int oi = *si;
+          if (ob < best || (ob == best && oi < besti)) { best = ob; besti = oi; }
+          if (row < p.M) { p.assign[row] = besti; p.best_key[row] = best; }
+        }
+        named_bar_sync(1 + q, 64);
+      }
+    }
+  }
+
+  // ============================ teardown ============================
+  __syncwarp();
+  ptx::tc_fence_before();
+  if constexpr (CG == 2) ptx::cluster_sync(); else __syncthreads();
+  if (warp == 2) {
+    ptx::tc_fence_after();
+    ptx::tmem_dealloc<CG>(tmem_base, TMEM_COLS);
+  }
+}
+
+// ------------------------------------------------------------------ host side
+static PFN_cuTensorMapEncodeTiled_v12000 get_encode() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    cudaDriverEntryPointQueryResult q;
+    void* ptr = nullptr;
+    if (cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &ptr, cudaEnableDefault, &q) ==
+            cudaSuccess &&
+        q == cudaDriverEntryPointSuccess)
+      fn = reinterpret_cast<PFN_cuTensorMapEncodeTiled_v12000>(ptr);
+  });
+  return fn;
+}
+
+// fp16 [rows x cols] row-major with row stride ld elements; box {64, box_rows}, SW128.
+static bool make_tmap_f16(CUtensorMap* m, const void* base, int64_t rows, int64_t cols, int64_t ld,
+                          int box_rows) {
+  auto enc = get_encode();
+  if (!enc) return false;
+  cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {(cuuint64_t)(ld * 2)};
+  cuuint32_t box[2] = {64u, (cuuint32_t)box_rows};
+  cuuint32_t estr[2] = {1u, 1u};
+  CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT16, 2, const_cast<void*>(base), dims, strides,
+                   box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS;
+}
+
+template <int CG, int BN, bool SEP, int EPI, int STAGES>
+static int launch_variant(const CUtensorMap* maps, const KParams& kp, int max_clusters,
+                          cudaStream_t stream) {
+  using G = Geo<CG, BN>;
+  auto kern = egemm_tc_kernel<CG, BN, SEP, EPI, STAGES>;
+  const int scratch = kBM * kKnnMax * 8;
+  const size_t smem = 1024 + (size_t)STAGES * G::STAGE_BYTES + 8 * (2 * STAGES + 8) + scratch;
+  static bool attr_done = false;  // per instantiation
+  if (!attr_done) {
+    if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
+        cudaSuccess) {
+      set_last_error("cudaFuncSetAttribute(smem=%zu) failed", smem);
+      return 3;
+    }
+    if (CG == 2) cudaFuncSetAttribute(kern, cudaFuncAttributeNonPortableClusterSizeAllowed, 0);
+    attr_done = true;
+  }
+  int clusters = num_sms() / CG;
+  if (max_clusters > 0 && max_clusters < clusters) clusters = max_clusters;
+  if (clusters > kp.num_units) clusters = kp.num_units;
+  if (clusters < 1) clusters = 1;
+  cudaLaunchConfig_t cfg = {};
+  cfg.gridDim = dim3((unsigned)(clusters * CG), 1, 1);
+  cfg.blockDim = dim3(kThreads, 1, 1);
+  cfg.dynamicSmemBytes = smem;
+  cfg.stream = stream;
+  cudaLaunchAttribute attr[1];
+  attr[0].id = cudaLaunchAttributeClusterDimension;
+  attr[0].val.clusterDim.x = CG;
+  attr[0].val.clusterDim.y = 1;
+  attr[0].val.clusterDim.z = 1;
+  cfg.attrs = attr;
+  cfg.numAttrs = 1;
+  cudaError_t e = cudaLaunchKernelEx(&cfg, kern, maps[0], maps[1], maps[2], maps[3], kp);
+  if (e != cudaSuccess) {
+    set_last_error("cudaLaunchKernelEx: %s", cudaGetErrorString(e));
+    return 3;
+  }
+  return 0;
+}
+
+template <int EPI>
+static int dispatch(const CUtensorMap* maps, const KParams& kp, const TcConfig& cfg,
+                    cudaStream_t s) {
+  if (cfg.cg == 2 && cfg.bn == 256 && !cfg.sep)
+    return launch_variant<2, 256, false, EPI, 3>(maps, kp, cfg.max_clusters, s);
+  if (cfg.cg == 1 && cfg.bn == 128 && !cfg.sep)
+    return launch_variant<1, 128, false, EPI, 3>(maps, kp, cfg.max_clusters, s);
+  if (cfg.cg == 1 && cfg.bn == 128 && cfg.sep)
+    return launch_variant<1, 128, true, EPI, 3>(maps, kp, cfg.max_clusters, s);
+  if (cfg.cg == 2 && cfg.bn == 128 && cfg.sep)
+    return launch_variant<2, 128, true, EPI, 3>(maps, kp, cfg.max_clusters, s);
+  set_last_error("unsupported tile config cg=%d bn=%d sep=%d", cfg.cg, cfg.bn, cfg.sep);
+  return 2;
+}
+
+int launch_tc(int64_t M, int64_t N, int64_t K, const TcOperands& ops, const TcConfig& cfg,
+              const TcEpilogue& epi, cudaStream_t stream) {
+  if (M <= 0 || N <= 0) return 0;
+  if (M > INT32_MAX / 2 || N > INT32_MAX / 2) {
+    set_last_error("M, N must be < 2^30");
+    return 2;
+  }
+  CUtensorMap maps[4];
+  const int bnc = cfg.bn / cfg.cg;
+  if (!make_tmap_f16(&maps[0], ops.a_hi, M, K, ops.lda, kBM) ||
+      !make_tmap_f16(&maps[1], ops.a_lo, M, K, ops.lda, kBM) ||
+      !make_tmap_f16(&maps[2], ops.b_hi, N, K, ops.ldb, bnc) ||
+      !make_tmap_f16(&maps[3], ops.b_lo, N, K, ops.ldb, bnc)) {
+    set_last_error("cuTensorMapEncodeTiled failed (alignment: base 16 B, ld %% 8 == 0)");
+    return 2;
+  }
+  KParams kp = {};
+  kp.M = (int)M;
+  kp.N = (int)N;
+  kp.num_kb = (int)((K + kBK - 1) / kBK);
+  kp.kb_per_chunk = cfg.kc / kBK;
+  if (kp.kb_per_chunk < 1) kp.kb_per_chunk = 1;
+  kp.terms = cfg.terms;
+  kp.m_tiles = (int)((M + kBM * cfg.cg - 1) / (kBM * cfg.cg));
+  kp.n_tiles = (int)((N + cfg.bn - 1) / cfg.bn);
+  kp.D = epi.D;
+  kp.ldd = epi.ldd;
+  kp.C = epi.C;
+  kp.ldc = epi.ldc;
+  kp.vec_ok = (epi.D && (epi.ldd % 4 == 0) && ((uintptr_t)epi.D % 16 == 0) &&
+               (!epi.C || ((epi.ldc % 4 == 0) && ((uintptr_t)epi.C % 16 == 0))))
+                  ? 1
+                  : 0;
+  kp.bnorm = epi.bnorm;
+  kp.knn_k = epi.knn_k;
+  kp.part_key = epi.part_key;
+  kp.part_idx = epi.part_idx;
+  kp.assign = epi.assign;
+  kp.best_key = epi.best_key;
+  if (epi.kind == EPI_STORE) {
+    kp.num_units = kp.m_tiles * kp.n_tiles;
+    return dispatch<EPI_STORE>(maps, kp, cfg, stream);
+  }
+  if (kp.num_kb > kp.kb_per_chunk) {
+    set_last_error("fused kNN/kMeans epilogues need Kc >= K");
+    return 2;
+  }
+  if (epi.kind == EPI_KNN) {
+    kp.n_slices = epi.n_slices;
+    kp.tiles_per_slice = (kp.n_tiles + epi.n_slices - 1) / epi.n_slices;
+    kp.num_units = kp.m_tiles * epi.n_slices;
+    return dispatch<EPI_KNN>(maps, kp, cfg, stream);
+  }
+  kp.num_units = kp.m_tiles;
+  return dispatch<EPI_KMEANS>(maps, kp, cfg, stream);
+}
+
+}  // namespace egemm

@@ -1,0 +1,241 @@
+"""Thin Python binding of libegemm.so (include/egemm.h): argument marshalling only.
+
+Every compute step runs in the CUDA kernels behind the C ABI.  PyTorch supplies device
+memory, the current stream and (in ``distributed``) process groups.  There is no CPU
+fallback: if the library is missing or the device is not an sm_100 GPU, calls raise.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+
+import torch
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libegemm.so")
+
+OK, ERR_INVALID_ARG, ERR_UNSUPPORTED, ERR_CUDA, ERR_WORKSPACE = 0, 1, 2, 3, 4
+
+
+class EgemmError(RuntimeError):
+    def __init__(self, status: int, fn: str, detail: str):
+        super().__init__("%s -> %s: %s" % (fn, _STATUS.get(status, status), detail))
+        self.status = status
+
+
+_STATUS = {0: "EGEMM_OK", 1: "EGEMM_ERR_INVALID_ARG", 2: "EGEMM_ERR_UNSUPPORTED",
+           3: "EGEMM_ERR_CUDA", 4: "EGEMM_ERR_WORKSPACE"}
+
+
+class Operand(ctypes.Structure):
+    """egemm_operand_t"""
+    _fields_ = [("f32", ctypes.c_void_p), ("hi", ctypes.c_void_p), ("lo", ctypes.c_void_p),
+                ("ld", ctypes.c_int64), ("trans", ctypes.c_int), ("ld_split", ctypes.c_int64)]
+
+
+EXPORTS = ["egemm_status_string", "egemm_last_error", "egemm_version", "egemm_split", "egemm_gemm",
+           "egemm_gemm_workspace_size", "egemm_knn", "egemm_knn_workspace_size",
+           "egemm_kmeans_step", "egemm_kmeans_workspace_size", "egemm_kmeans_finalize",
+           "egemm_set_config", "egemm_num_sms"]
+
+_lib = None
+
+
+def load(path: str = LIB_PATH):
+    """Load libegemm.so (raises if it was not built: there is no fallback)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(path):
+        raise RuntimeError("libegemm.so not built (run python -m paper_conf_ppopp_fengwcz0d21_b200.build)")
+    L = ctypes.CDLL(path)
+    P, I64, I, SZ = ctypes.c_void_p, ctypes.c_int64, ctypes.c_int, ctypes.c_size_t
+    L.egemm_status_string.argtypes = [I]
+    L.egemm_status_string.restype = ctypes.c_char_p
+    L.egemm_last_error.argtypes = []
+    L.egemm_last_error.restype = ctypes.c_char_p
+    L.egemm_version.restype = I
+    L.egemm_split.argtypes = [P, I64, I64, I64, P, P, I64, I, P, P]
+    L.egemm_split.restype = I
+    L.egemm_gemm.argtypes = [I64, I64, I64, Operand, Operand, P, I64, P, I64, I, P, SZ, P]
+    L.egemm_gemm.restype = I
+    L.egemm_gemm_workspace_size.argtypes = [I64, I64, I64, I, I]
+    L.egemm_gemm_workspace_size.restype = SZ
+    L.egemm_knn.argtypes = [Operand, I64, Operand, I64, I64, I, P, P, P, SZ, P]
+    L.egemm_knn.restype = I
+    L.egemm_knn_workspace_size.argtypes = [I64, I64, I64, I, I]
+    L.egemm_knn_workspace_size.restype = SZ
+    L.egemm_kmeans_step.argtypes = [Operand, I64, I64, P, I64, P, P, P, P, P, SZ, P]
+    L.egemm_kmeans_step.restype = I
+    L.egemm_kmeans_workspace_size.argtypes = [I64, I64, I64, I]
+    L.egemm_kmeans_workspace_size.restype = SZ
+    L.egemm_kmeans_finalize.argtypes = [P, P, I64, I64, P, P]
+    L.egemm_kmeans_finalize.restype = I
+    L.egemm_set_config.argtypes = [I, I, I, I]
+    L.egemm_set_config.restype = I
+    L.egemm_num_sms.restype = I
+    _lib = L
+    return L
+
+
+def _check(status: int, fn: str):
+    if status != OK:
+        raise EgemmError(status, fn, load().egemm_last_error().decode())
+
+
+def _ptr(t):
+    return None if t is None else ctypes.c_void_p(t.data_ptr())
+
+
+def _stream(stream=None):
+    s = stream if stream is not None else torch.cuda.current_stream()
+    return ctypes.c_void_p(s.cuda_stream)
+
+
+def _need_cuda(*ts):
+    for t in ts:
+        if t is not None and not t.is_cuda:
+            raise ValueError("egemm expects CUDA tensors (no CPU path)")
+
+
+def _workspace(nbytes: int, device, ws=None):
+    if nbytes == 0:
+        return None, 0
+    if ws is not None and ws.numel() >= nbytes:
+        return ws, ws.numel()
+    return torch.empty(nbytes, dtype=torch.uint8, device=device), nbytes
+
+
+# ---------------------------------------------------------------------------- split
+def split(x: torch.Tensor, transpose: bool = False, range_flags: torch.Tensor | None = None,
+          out: tuple | None = None, stream=None):
+    """Round-split fp32 x [rows, cols] -> (hi, lo) fp16 bit patterns as int16 tensors
+    (viewable as torch.float16).  transpose=True returns the [cols, rows] transpose."""
+    L = load()
+    _need_cuda(x)
+    assert x.dtype == torch.float32 and x.dim() == 2 and x.stride(1) == 1
+    rows, cols = x.shape
+    oshape = (cols, rows) if transpose else (rows, cols)
+    if out is None:
+        hi = torch.empty(oshape, dtype=torch.int16, device=x.device)
+        lo = torch.empty(oshape, dtype=torch.int16, device=x.device)
+    else:
+        hi, lo = out
+    _check(L.egemm_split(_ptr(x), rows, cols, x.stride(0), _ptr(hi), _ptr(lo), hi.stride(0),
+                         1 if transpose else 0, _ptr(range_flags), _stream(stream)), "egemm_split")
+    return hi, lo
+
+
+def operand(f32: torch.Tensor | None = None, hi=None, lo=None, trans: bool = False) -> Operand:
+    op = Operand()
+    op.f32 = f32.data_ptr() if f32 is not None else None
+    op.hi = hi.data_ptr() if hi is not None else None
+    op.lo = lo.data_ptr() if lo is not None else None
+    op.ld = f32.stride(0) if f32 is not None else 0
+    op.trans = 1 if trans else 0
+    op.ld_split = hi.stride(0) if hi is not None else 0
+    return op
+
+
+# ---------------------------------------------------------------------------- GEMM
+def gemm_workspace_size(M, N, K, a_presplit=False, b_presplit=False) -> int:
+    return int(load().egemm_gemm_workspace_size(M, N, K, int(a_presplit), int(b_presplit)))
+
+
+def gemm(A: torch.Tensor | None, B: torch.Tensor | None, C: torch.Tensor | None = None,
+         terms: int = 0, out: torch.Tensor | None = None, a_split=None, b_split=None,
+         b_trans: bool = False, workspace: torch.Tensor | None = None, stream=None):
+    """D = A @ B (+ C) with the EGEMM-TC emulation (Alg. 1).
+
+    A: [M, K] fp32 (or a_split=(hi, lo) [M, K]); B: [K, N] fp32, or [N, K] with b_trans,
+    or b_split=(hi, lo) [N, K] (K-major, e.g. split(B, transpose=True))."""
+    L = load()
+    if A is not None:
+        M, K = A.shape
+    else:
+        M, K = a_split[0].shape
+    if B is not None:
+        N = B.shape[0] if b_trans else B.shape[1]
+    else:
+        N = b_split[0].shape[0]
+    dev = (A if A is not None else a_split[0]).device
+    _need_cuda(A, B, C, out)
+    D = out if out is not None else torch.empty((M, N), dtype=torch.float32, device=dev)
+    opA = operand(A, *(a_split or (None, None)))
+    opB = operand(B, *(b_split or (None, None)), trans=b_trans)
+    need = gemm_workspace_size(M, N, K, a_split is not None, b_split is not None)
+    ws, wsn = _workspace(need, dev, workspace)
+    _check(L.egemm_gemm(M, N, K, opA, opB, _ptr(C), C.stride(0) if C is not None else 0, _ptr(D),
+                        D.stride(0), int(terms), _ptr(ws), wsn, _stream(stream)), "egemm_gemm")
+    return D
+
+
+# ---------------------------------------------------------------------------- kNN
+def knn_workspace_size(nx, nq, d, k, x_presplit=False) -> int:
+    return int(load().egemm_knn_workspace_size(nx, nq, d, k, int(x_presplit)))
+
+
+def knn(X: torch.Tensor, Q: torch.Tensor, k: int, x_split=None, workspace=None, out=None,
+        stream=None):
+    """k nearest rows of X [nx, d] for each query row of Q [nq, d] (squared L2, ascending).
+    Returns (idx int32 [nq, k], dist fp32 [nq, k])."""
+    L = load()
+    _need_cuda(X, Q)
+    nx, d = X.shape
+    nq = Q.shape[0]
+    if out is None:
+        idx = torch.empty((nq, k), dtype=torch.int32, device=X.device)
+        dist = torch.empty((nq, k), dtype=torch.float32, device=X.device)
+    else:
+        idx, dist = out
+    need = knn_workspace_size(nx, nq, d, k, x_split is not None)
+    ws, wsn = _workspace(need, X.device, workspace)
+    _check(L.egemm_knn(operand(X, *(x_split or (None, None))), nx, operand(Q), nq, d, k, _ptr(idx),
+                       _ptr(dist), _ptr(ws), wsn, _stream(stream)), "egemm_knn")
+    return idx, dist
+
+
+# ---------------------------------------------------------------------------- kMeans
+def kmeans_workspace_size(n, d, kc, x_presplit=False) -> int:
+    return int(load().egemm_kmeans_workspace_size(n, d, kc, int(x_presplit)))
+
+
+def kmeans_step(X: torch.Tensor, centroids: torch.Tensor, x_split=None, want_inertia=True,
+                workspace=None, out=None, stream=None):
+    """One local Lloyd step: (assign int32 [n], sums fp64 [kc, d], counts int64 [kc],
+    inertia fp64 [1] or None)."""
+    L = load()
+    _need_cuda(X, centroids)
+    n, d = X.shape
+    kc = centroids.shape[0]
+    assert centroids.is_contiguous()
+    if out is None:
+        assign = torch.empty(n, dtype=torch.int32, device=X.device)
+        sums = torch.empty((kc, d), dtype=torch.float64, device=X.device)
+        counts = torch.empty(kc, dtype=torch.int64, device=X.device)
+        inertia = torch.empty(1, dtype=torch.float64, device=X.device) if want_inertia else None
+    else:
+        assign, sums, counts, inertia = out
+    need = kmeans_workspace_size(n, d, kc, x_split is not None)
+    ws, wsn = _workspace(need, X.device, workspace)
+    _check(L.egemm_kmeans_step(operand(X, *(x_split or (None, None))), n, d, _ptr(centroids), kc,
+                               _ptr(assign), _ptr(sums), _ptr(counts), _ptr(inertia), _ptr(ws),
+                               wsn, _stream(stream)), "egemm_kmeans_step")
+    return assign, sums, counts, inertia
+
+
+def kmeans_finalize(sums: torch.Tensor, counts: torch.Tensor, centroids: torch.Tensor, stream=None):
+    L = load()
+    kc, d = centroids.shape
+    _check(L.egemm_kmeans_finalize(_ptr(sums), _ptr(counts), kc, d, _ptr(centroids),
+                                   _stream(stream)), "egemm_kmeans_finalize")
+    return centroids
+
+
+def set_config(cg: int = 0, bn: int = 0, sep: int = 0, kc: int = 0):
+    """Per-thread tile-config override (all zeros = tuning table)."""
+    _check(load().egemm_set_config(cg, bn, sep, kc), "egemm_set_config")
+
+
+def num_sms() -> int:
+    return int(load().egemm_num_sms())

@@ -1,0 +1,164 @@
+"""GPU parity of egemm_gemm against the oracle (Alg. 1).
+
+Bars (BASELINE.json north_star):
+  * normwise  e = ||D - C64||_F / || |A||B| ||_F <= 1e-6 (K <= 8192) and <= 2 e_naive
+  * elementwise |D - C64| <= elem_bound (reading R18)
+  * bit-exact on the exact pins: integer inputs, identity / permutation A.
+"""
+import numpy as np
+import pytest
+import torch
+
+from paper_conf_ppopp_fengwcz0d21_b200 import inputs
+from tests.gpu_util import require_gpu, to_dev, to_host
+
+pytestmark = pytest.mark.gpu
+
+CONFIGS = [(2, 256, 0, 256), (1, 128, 0, 256), (1, 128, 1, 256), (2, 128, 1, 256), (2, 256, 0, 64),
+           (2, 256, 0, 1024)]
+
+
+def _run(eg, A, B, C=None, terms=0, cfg=None):
+    if cfg is not None:
+        eg.set_config(*cfg)
+    try:
+        D = eg.gemm(to_dev(A), to_dev(B), to_dev(C) if C is not None else None, terms=terms)
+        return to_host(D)
+    finally:
+        if cfg is not None:
+            eg.set_config(0, 0, 0, 0)
+
+
+def _assert_parity(oracle_lib, A, B, D, C=None, terms=3):
+    C64 = oracle_lib.gemm64(A, B, C)
+    e = oracle_lib.normwise_error(D, A, B, C64)
+    en = oracle_lib.normwise_error(oracle_lib.gemm32_naive(A, B, C), A, B, C64)
+    assert e <= 1e-6, e
+    assert e <= 2 * en, (e, en)
+    bound = oracle_lib.elem_bound(A, B, terms=terms)
+    if C is not None:
+        bound = bound + 2.0 ** -23 * np.abs(C)
+    bad = np.abs(D.astype(np.float64) - C64) > bound
+    assert not bad.any(), "elementwise bound exceeded at %s" % (np.argwhere(bad)[:5],)
+    return e, en
+
+
+@pytest.mark.parametrize("cfg", CONFIGS)
+def test_gemm_256_cube(oracle_lib, cfg):
+    """BASELINE configs[0]: M=N=K=256, U[-1,1], against the fp64 oracle."""
+    eg = require_gpu()
+    A, B = inputs.uniform((256, 256), 1), inputs.uniform((256, 256), 2)
+    D = _run(eg, A, B, cfg=cfg)
+    _assert_parity(oracle_lib, A, B, D)
+
+
+@pytest.mark.parametrize("gen", [inputs.in_zone, inputs.stress])
+@pytest.mark.parametrize("cfg", [CONFIGS[0], CONFIGS[2]])
+def test_gemm_distributions(oracle_lib, gen, cfg):
+    eg = require_gpu()
+    A, B = gen((384, 512), 3), gen((512, 320), 4)
+    D = _run(eg, A, B, cfg=cfg)
+    _assert_parity(oracle_lib, A, B, D)
+
+
+@pytest.mark.parametrize("shape", [(1, 1, 1), (7, 5, 3), (300, 200, 100), (129, 257, 65),
+                                   (513, 384, 1000), (64, 1024, 16), (1000, 16, 48)])
+@pytest.mark.parametrize("cfg", [CONFIGS[0], CONFIGS[1], CONFIGS[2]])
+def test_gemm_ragged(oracle_lib, shape, cfg):
+    """Ragged M/N/K tails span partial tiles, partial k-blocks and partial chunks."""
+    eg = require_gpu()
+    M, N, K = shape
+    A, B = inputs.uniform((M, K), 5 + M), inputs.uniform((K, N), 6 + N)
+    D = _run(eg, A, B, cfg=cfg)
+    _assert_parity(oracle_lib, A, B, D)
+
+
+@pytest.mark.parametrize("terms", [3, 4])
+def test_gemm_with_c_and_terms(oracle_lib, terms):
+    eg = require_gpu()
+    A, B, C = inputs.uniform((300, 700), 7), inputs.uniform((700, 260), 8), inputs.uniform((300, 260), 9)
+    D = _run(eg, A, B, C, terms=terms)
+    _assert_parity(oracle_lib, A, B, D, C, terms=terms)
+
+
+def test_gemm_transposed_and_presplit(oracle_lib):
+    eg = require_gpu()
+    A, B = inputs.uniform((256, 384), 10), inputs.uniform((384, 512), 11)
+    Ad, Bd = to_dev(A), to_dev(B)
+    D1 = to_host(eg.gemm(Ad, Bd))
+    D2 = to_host(eg.gemm(Ad, to_dev(np.ascontiguousarray(B.T)), b_trans=True))
+    a_split = eg.split(Ad)
+    b_split = eg.split(Bd, transpose=True)
+    D3 = to_host(eg.gemm(None, None, a_split=a_split, b_split=b_split))
+    assert np.array_equal(D1, D2) and np.array_equal(D1, D3)
+    _assert_parity(oracle_lib, A, B, D1)
+
+
+@pytest.mark.parametrize("cfg", [CONFIGS[0], CONFIGS[2]])
+def test_gemm_integer_exact(cfg):
+    """|a|, |b| <= 32, K = 4096: every partial sum is an integer < 2^24, so the result is
+    exact whatever the order or rounding -> bitwise equal to the integer GEMM."""
+    eg = require_gpu()
+    A, B = inputs.integers((256, 4096), 12), inputs.integers((4096, 384), 13)
+    D = _run(eg, A, B, cfg=cfg)
+    ref = (A.astype(np.int64) @ B.astype(np.int64)).astype(np.float32)
+    assert np.array_equal(D, ref)
+
+
+def test_gemm_identity_exercises_lo(oracle_lib):
+    """A = signed permutation x powers of two: D_ij = s * 2^p * fl32(hi_b + lo_b), bitwise."""
+    eg = require_gpu()
+    n = 256
+    g = inputs.rng(14)
+    perm = g.permutation(n)
+    A = np.zeros((n, n), np.float32)
+    sc = np.exp2(g.integers(-2, 3, size=n)) * np.where(g.random(n) < 0.5, -1, 1)
+    A[np.arange(n), perm] = sc
+    B = inputs.uniform((n, 320), 15)
+    D = _run(eg, A, B)
+    hi, lo = oracle_lib.split(B)
+    rec = (oracle_lib.h2f(hi) + oracle_lib.h2f(lo)).astype(np.float32).astype(np.float64)
+    ref = (sc[:, None] * rec[perm]).astype(np.float32)
+    assert np.array_equal(D, ref)
+    assert not np.array_equal(D, (sc[:, None] * oracle_lib.h2f(hi)[perm]).astype(np.float32))
+
+
+def test_gemm_k_zero_and_empty():
+    eg = require_gpu()
+    C = torch.randn(5, 6, device="cuda")
+    D = eg.gemm(torch.empty(5, 0, device="cuda"), torch.empty(0, 6, device="cuda"), C)
+    assert torch.equal(D, C)
+    D = eg.gemm(torch.empty(0, 4, device="cuda"), torch.empty(4, 6, device="cuda"))
+    assert D.shape == (0, 6)
+
+
+def test_gemm_invalid_args():
+    eg = require_gpu()
+    with pytest.raises(eg.EgemmError) as ei:
+        eg.gemm(torch.ones(4, 4, device="cuda"), torch.ones(4, 4, device="cuda"), terms=5)
+    assert ei.value.status == eg.ERR_INVALID_ARG
+
+
+def test_probe_tensor_core_accumulation(oracle_lib):
+    """Paper Sec. 3.1 precision profiling on tcgen05: with
+    fp16-exact inputs lo = 0, so D = MMA(a[16:32], b[16:32], MMA(a[:16], b[:16], 0)).
+    Compare bitwise with the candidate models; record which one(s) match 100%."""
+    eg = require_gpu()
+    g = inputs.rng(16)
+    M, N, K = 128, 128, 32
+    A = g.uniform(-1, 1, (M, K)).astype(np.float16).astype(np.float32)
+    B = g.uniform(-1, 1, (K, N)).astype(np.float16).astype(np.float32)
+    A[:, 16:] *= np.float32(2.0 ** -6)  # second MMA adds small products to a larger C
+    D = _run(eg, A, B, cfg=(1, 128, 1, 256))
+    idx = [(i, j) for i in range(0, M, 3) for j in range(0, N, 5)][:1200]
+    results = {}
+    for model, e in [("rn", 0), ("rz", 0), ("align", 0), ("align", 1), ("align", 2), ("align", 3)]:
+        ok = 0
+        for i, j in idx:
+            c = oracle_lib.tc_model(A[i, :16], B[:16, j], 0.0, model, e)
+            c = float(np.float32(c))
+            d = oracle_lib.tc_model(A[i, 16:], B[16:, j], c, model, e)
+            ok += (np.float32(d) == D[i, j])
+        results["%s%d" % (model, e)] = ok / len(idx)
+    print("tcgen05 accumulation model match rates:", results)
+    assert max(results.values()) == 1.0, results

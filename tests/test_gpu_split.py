@@ -1,0 +1,73 @@
+"""GPU parity of egemm_split against the oracle's bit-level round-split (bit-exact)."""
+import numpy as np
+import pytest
+import torch
+
+from paper_conf_ppopp_fengwcz0d21_b200 import inputs
+from tests.gpu_util import require_gpu, to_dev, u16
+
+pytestmark = pytest.mark.gpu
+
+
+def _cmp(x, ghi, glo, ohi, olo):
+    nan = np.isnan(x)
+    same = (ghi == ohi) & (glo == olo)
+    # NaN inputs: compare by class (both NaN) -- cvt.rn may canonicalise the payload
+    hn = lambda h: ((h & 0x7C00) == 0x7C00) & ((h & 0x3FF) != 0)
+    same |= nan & hn(ghi) & hn(glo) & hn(ohi) & hn(olo)
+    # x = +-inf: hi = inf, lo = inf - inf = NaN on both sides
+    return same
+
+
+def test_split_all_fp32_patterns(oracle_lib):
+    """Bit-exact against the oracle over ALL 2^32 fp32 bit patterns (chunks of 2^28)."""
+    eg = require_gpu()
+    chunk = 1 << 28
+    for start in range(0, 1 << 32, chunk):
+        x = inputs.all_f32_patterns(start, chunk)
+        ohi, olo = oracle_lib.split(x)
+        xd = to_dev(x).view(-1, 1 << 14)
+        hi, lo = eg.split(xd)
+        ghi, glo = u16(hi).ravel(), u16(lo).ravel()
+        ok = _cmp(x, ghi, glo, ohi, olo)
+        assert ok.all(), "mismatch at pattern 0x%08x" % (start + int(np.argmin(ok)))
+
+
+@pytest.mark.parametrize("shape", [(1, 1), (3, 7), (257, 129), (1024, 1000)])
+def test_split_transpose_and_ragged(oracle_lib, shape):
+    eg = require_gpu()
+    x = inputs.stress(shape, 11)
+    ohi, olo = oracle_lib.split(x)
+    hi, lo = eg.split(to_dev(x))
+    assert np.array_equal(u16(hi), ohi) and np.array_equal(u16(lo), olo)
+    hiT, loT = eg.split(to_dev(x), transpose=True)
+    assert np.array_equal(u16(hiT), ohi.T) and np.array_equal(u16(loT), olo.T)
+
+
+def test_split_strided_view(oracle_lib):
+    eg = require_gpu()
+    big = inputs.uniform((300, 512), 12)
+    xd = to_dev(big)[:, 3:403]  # ld = 512, unaligned base
+    hi, lo = eg.split(xd)
+    ohi, olo = oracle_lib.split(big[:, 3:403])
+    assert np.array_equal(u16(hi), ohi) and np.array_equal(u16(lo), olo)
+
+
+def test_split_range_flags():
+    eg = require_gpu()
+    f = torch.zeros(1, dtype=torch.int32, device="cuda")
+    eg.split(to_dev(inputs.uniform((64, 64), 13, 0.25, 1.0)), range_flags=f)
+    assert int(f.item()) == 0
+    x = inputs.uniform((64, 64), 13, 0.25, 1.0)
+    x[5, 7] = 70000.0
+    eg.split(to_dev(x), range_flags=f)
+    assert int(f.item()) == 1
+    x[9, 9] = 0.01
+    eg.split(to_dev(x), range_flags=f)
+    assert int(f.item()) == 3
+
+
+def test_split_empty():
+    eg = require_gpu()
+    hi, lo = eg.split(torch.empty((0, 5), dtype=torch.float32, device="cuda"))
+    assert hi.shape == (0, 5)
