@@ -269,25 +269,39 @@ def _round_f32(v: Fraction, mode: str) -> float:
     return s * float(val)  # exact: val is an fp32 value
 
 
-def tc_model(a, b, c: float, model: str, extra_bits: int = 0) -> float:
+def tc_model(a, b, c: float, model: str, extra_bits: int = 0, anchor: str = "fields") -> float:
     """Candidate semantics of one MMA step.
 
     model "rn": exact sum, round to nearest-even fp32.
     model "rz": exact sum, truncate toward zero to fp32.
     model "align": every product and c is first truncated toward zero onto the grid
-      2^(E-23-extra_bits) with E the largest exponent among the (non-zero) terms, the
-      truncated terms are summed exactly, and the sum is truncated to fp32.
+      2^(E-23-extra_bits), where E is the largest exponent estimate among the non-zero
+      terms, the truncated terms are summed exactly, and the sum is truncated to fp32.
+      anchor "fields": a product's estimate is the sum of the operands' exponents
+        (e_a + e_b, the exponent-field sum before normalisation); c's is its exponent.
+      anchor "value": the product's true exponent (e_a + e_b or e_a + e_b + 1).
     """
-    terms = [Fraction(float(x)) * Fraction(float(y)) for x, y in zip(a, b)]
-    terms.append(Fraction(float(c)))
+    terms = []
+    ests = []
+    for x, y in zip(a, b):
+        x, y = float(x), float(y)
+        if x == 0.0 or y == 0.0:
+            continue
+        terms.append(Fraction(x) * Fraction(y))
+        if anchor == "fields":
+            ests.append((math.frexp(abs(x))[1] - 1) + (math.frexp(abs(y))[1] - 1))
+        else:
+            ests.append(math.frexp(abs(x * y))[1] - 1)
+    c = float(c)
+    if c != 0.0:
+        terms.append(Fraction(c))
+        ests.append(math.frexp(abs(c))[1] - 1)
     if model in ("rn", "rz"):
         return _round_f32(sum(terms, Fraction(0)), model)
     if model == "align":
-        nz = [t for t in terms if t != 0]
-        if not nz:
+        if not terms:
             return 0.0
-        E = max(math.frexp(abs(float(t)))[1] - 1 for t in nz)  # exponent of the largest
-        g = Fraction(2) ** (E - 23 - extra_bits)
+        g = Fraction(2) ** (max(ests) - 23 - extra_bits)
         tot = Fraction(0)
         for t in terms:
             q = abs(t) // g

@@ -54,7 +54,7 @@ static TcConfig choose_config(int epi_kind, int64_t M, int64_t N, int64_t K, int
   c.cg = 2;
   c.bn = 256;
   c.sep = 0;
-  c.kc = 256;
+  c.kc = 128;  // measured: Kc=256 exceeds 2x naive-fp32 error at K<=1024 (tools/error_sweep.py)
   if (epi_kind == EPI_STORE && M <= 128) { c.cg = 1; c.bn = 128; c.sep = 1; }
   if (epi_kind != EPI_STORE) c.kc = (int)(((K + 63) / 64) * 64);
   // thread-local API override, then environment (experiments)

@@ -63,7 +63,8 @@ def test_knn_self_match_and_duplicates():
     idx, dist = eg.knn(to_dev(X), to_dev(X[[10, 20]]), 3)
     i = to_host(idx)
     assert list(i[0][:2]) == [10, 500] and i[1][0] == 20
-    assert to_host(dist)[1][0] == 0.0
+    # ||q||^2 + ||x||^2 - 2 q.x of identical rows cancels to within the fp32 rounding (R18)
+    assert 0.0 <= to_host(dist)[1][0] <= 1e-5
 
 
 def _kmeans_check(oracle_lib, X, C, ga, gsums, gcounts):
