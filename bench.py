@@ -1,0 +1,442 @@
+"""EGEMM-TC hot-path benchmark (driver contract: one JSON line on rank 0).
+
+Step = one pass of the hot path over one batch of the headline workload (BASELINE.json
+configs[1] at 8192^3, the metric's configuration): round-split of the rank's A rows and of
+B (egemm_split, CUDA cores) + the tcgen05 emulated GEMM (egemm_gemm on the pre-split
+operands).  Inputs: seeded synthetic U[-1,1] fp32 (the paper's distribution),
+resident in HBM; every operand (256 MiB fp32 each) is larger than the 126 MB L2.
+
+Multi-GPU (torchrun, one process per GPU, NCCL): C rows are sharded (strong scaling of the
+fixed 8192^3 problem, BASELINE configs[1] "row-sharded C"); B is broadcast once before
+timing; no collective in the timed loop.  Time = max over ranks of the device time.
+
+Also reported (informational objects): kNN queries/s (configs[3]) and kMeans ms/iteration
+(configs[4]), the split kernel's HBM roofline, and the CPU oracle (cpu_baseline).
+``--impl reference`` times the CPU oracle itself on the host cores (the reference arm).
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import os
+import subprocess
+import sys
+import threading
+import time
+
+import numpy as np
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "EGEMM FP32-equiv TFLOP/s at 8192^3 (2MNK/t, split included)"
+UNIT = "TFLOP/s"
+
+
+def _peaks():
+    try:
+        return json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        return {}
+
+
+def _profile_summary():
+    try:
+        return json.load(open(os.path.join(ROOT, "profiles", "ncu_summary.json")))
+    except Exception:
+        return {}
+
+
+class ClockSampler:
+    """nvidia-smi clocks / throttle reasons sampled DURING the timed region."""
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index: int):
+        self.index = index
+        self.proc = None
+        self.lines = []
+
+    def __enter__(self):
+        try:
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.index), "--query-gpu=" + self.FIELDS,
+                 "--format=csv,noheader,nounits", "-lms", "20"],
+                stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
+            self.t = threading.Thread(target=self._read, daemon=True)
+            self.t.start()
+            t0 = time.time()
+            while not self.lines and time.time() - t0 < 5.0:  # sampler is live before timing
+                time.sleep(0.01)
+            self.n0 = len(self.lines)
+        except Exception:
+            self.proc = None
+        return self
+
+    def mark(self):
+        """Index of the first sample inside the timed region."""
+        self.n0 = len(self.lines)
+
+    def _read(self):
+        for line in self.proc.stdout:
+            self.lines.append(line.strip())
+
+    def __exit__(self, *a):
+        if self.proc is not None:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        sm, mx, reasons = [], [], set()
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        lines = self.lines[getattr(self, "n0", 0):] or self.lines[-3:]
+        for ln in lines:
+            parts = [p.strip() for p in ln.split(",")]
+            if len(parts) < 8:
+                continue
+            try:
+                sm.append(float(parts[0]))
+                mx.append(float(parts[1]))
+            except ValueError:
+                continue
+            for n, v in zip(names, parts[4:8]):
+                if v.lower().startswith("active"):
+                    reasons.add(n)
+        if not sm:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unsampled"]}
+        return {"sm_mhz": float(np.median(sm)), "sm_max_mhz": max(mx), "reasons": sorted(reasons),
+                "samples": len(sm)}
+
+
+def _dist_setup():
+    import torch
+    import torch.distributed as dist
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl")
+    else:
+        torch.cuda.set_device(0)
+    return world, rank, local
+
+
+def _allmax(x: float, world: int) -> float:
+    if world == 1:
+        return x
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([x], dtype=torch.float64, device="cuda")
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def _barrier(world):
+    import torch
+    if world > 1:
+        import torch.distributed as dist
+        dist.barrier()
+    torch.cuda.synchronize()
+
+
+def run_oracle_sample(n: int, target_s: float, seed_a=101, seed_b=102):
+    """Time the CPU oracle (the method's products in fp64, oracle.gemm_emu64, which
+    round-splits its inputs) on a bounded row sample of the n^3 workload."""
+    import oracle
+    from paper_conf_ppopp_fengwcz0d21_b200 import inputs
+    B = inputs.uniform((n, n), seed_b)
+    rows = 4
+    A = inputs.uniform((rows, n), seed_a)
+    t0 = time.perf_counter()
+    oracle.gemm_emu64(A, B, 3)
+    t_small = time.perf_counter() - t0
+    rows = int(max(4, min(n, rows * target_s / max(t_small, 1e-3))))
+    A = inputs.uniform((rows, n), seed_a)
+    t0 = time.perf_counter()
+    oracle.gemm_emu64(A, B, 3)
+    dt = time.perf_counter() - t0
+    return rows, dt, 2.0 * rows * n * n / dt / 1e12
+
+
+def reference_arm(args):
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    import oracle
+    n = args.n
+    cores = oracle.num_threads()
+    # warm-up + steps, each a bounded row sample (sized to ~args.ref_step_s seconds)
+    vals, rows_used, times = [], 0, []
+    for i in range(args.warmup + args.steps):
+        rows, dt, tf = run_oracle_sample(n, args.ref_step_s)
+        if i >= args.warmup:
+            vals.append(tf)
+            rows_used = rows
+            times.append(dt)
+    v = float(np.median(vals))
+    line = {
+        "impl": "reference", "metric": METRIC, "value": v, "unit": UNIT, "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": float(np.median(times)) * 1e3,
+        "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f64",
+        "data": "synthetic U[-1,1] fp32 (seeded PCG64)",
+        "config": {"workload": "egemm %d^3 (BASELINE configs[1]) -- oracle row sample" % n,
+                   "M": n, "N": n, "K": n, "sample_rows_per_step": rows_used},
+        "cpu_baseline": {"value": v, "unit": UNIT, "cores": cores, "kind": "oracle",
+                         "sample": "oracle.gemm_emu64 (round-split + 3-term products in fp64) on "
+                                   "%d of %d rows per step" % (rows_used, n)},
+        "e2e": {"value": v, "unit": UNIT, "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=30)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--n", type=int, default=8192)
+    ap.add_argument("--no-apps", action="store_true", help="skip the kNN / kMeans objects")
+    ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline oracle timing")
+    ap.add_argument("--cpu-seconds", type=float, default=12.0)
+    ap.add_argument("--ref-step-s", type=float, default=8.0)
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        reference_arm(args)
+        return
+
+    import torch
+    from paper_conf_ppopp_fengwcz0d21_b200 import egemm, inputs
+    from paper_conf_ppopp_fengwcz0d21_b200 import distributed as edist
+
+    world, rank, local = _dist_setup()
+    egemm.load()
+    dev = torch.device("cuda", torch.cuda.current_device())
+    n = args.n
+    M, N, K = n, n, n
+    r0, r1 = edist.shard_bounds(M, world, rank, align=256)
+    m_loc = r1 - r0
+    # ---- inputs: A rows of this rank, B broadcast once from rank 0 (outside timing)
+    A_host = inputs.uniform((M, K), 101)[r0:r1]
+    A = torch.from_numpy(np.ascontiguousarray(A_host)).to(dev)
+    B = torch.from_numpy(inputs.uniform((K, N), 102)).to(dev) if rank == 0 else \
+        torch.empty((K, N), dtype=torch.float32, device=dev)
+    edist.broadcast_(B, world)
+    a_split = (torch.empty((m_loc, K), dtype=torch.int16, device=dev),
+               torch.empty((m_loc, K), dtype=torch.int16, device=dev))
+    b_split = (torch.empty((N, K), dtype=torch.int16, device=dev),
+               torch.empty((N, K), dtype=torch.int16, device=dev))
+    D = torch.empty((m_loc, N), dtype=torch.float32, device=dev)
+    stream = torch.cuda.current_stream()
+    launches_per_step = 3  # split A, split B^T, tcgen05 GEMM
+
+    def step():
+        egemm.split(A, out=a_split)
+        egemm.split(B, transpose=True, out=b_split)
+        egemm.gemm(None, None, a_split=a_split, b_split=b_split, out=D)
+
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True),
+           torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    start, stop = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    with ClockSampler(dev.index) as clk:
+        for _ in range(args.warmup):
+            step()
+        _barrier(world)
+        clk.mark()
+        start.record(stream)
+        for i in range(args.steps):
+            ev[i][0].record(stream)
+            egemm.split(A, out=a_split)
+            egemm.split(B, transpose=True, out=b_split)
+            ev[i][1].record(stream)
+            egemm.gemm(None, None, a_split=a_split, b_split=b_split, out=D)
+            ev[i][2].record(stream)
+        stop.record(stream)
+        _barrier(world)
+    t_ms = start.elapsed_time(stop)
+    t_ms = _allmax(t_ms, world)
+    ms_per_step = t_ms / args.steps
+    flop_total = 2.0 * M * N * K  # whole job (all ranks)
+    value = flop_total / (ms_per_step * 1e-3) / 1e12
+    gemm_ms = float(np.mean([e[1].elapsed_time(e[2]) for e in ev]))
+    split_ms = float(np.mean([e[0].elapsed_time(e[1]) for e in ev]))
+    clocks = clk.summary()
+
+    peaks = _peaks()
+    prof = _profile_summary()
+    terms = 3
+    tensor_flop = terms * 2.0 * m_loc * N * K
+    achieved = tensor_flop / (gemm_ms * 1e-3) / 1e12
+    peak = peaks.get("bf16_tflops_sustained", 1409.0)
+    roofline = {
+        "kernel": "egemm_tc_kernel<2,256,...> (tcgen05 cta_group::2, 256x256 tiles)",
+        "bound": "tensor", "achieved": round(achieved, 1), "peak": peak, "unit": "TFLOP/s",
+        "frac": round(achieved / peak, 4),
+        "peak_kind": "measured fp16/bf16 dense, sustained (MEASURED_PEAKS.json bf16_tflops_sustained)",
+        "frac_of_burst": round(achieved / peaks.get("bf16_tflops", 1667.9), 4),
+        "algorithmic": "3 terms x 2MNK fp16 tensor flops per launch (M=%d N=%d K=%d)" % (m_loc, N, K),
+        "kernel_ms": round(gemm_ms, 4),
+        "share_of_step": round(gemm_ms / ms_per_step, 4),
+        "traffic": prof.get("gemm_dram_bytes_per_launch"),
+        "fp32eq_tflops": round(2.0 * m_loc * N * K / (gemm_ms * 1e-3) / 1e12, 1),
+        "vs_tensor_peak_over_terms": round((2.0 * m_loc * N * K / (gemm_ms * 1e-3) / 1e12)
+                                           / (2250.0 / terms), 4),
+    }
+    split_bytes = 8.0 * (m_loc * K + K * N)
+    split_rl = {"kernel": "split (A rows + B^T)", "bound": "hbm",
+                "achieved": round(split_bytes / (split_ms * 1e-3) / 1e9, 1),
+                "peak": peaks.get("hbm_gbs", 6454.0), "unit": "GB/s",
+                "frac": round(split_bytes / (split_ms * 1e-3) / 1e9 / peaks.get("hbm_gbs", 6454.0), 4),
+                "traffic": prof.get("split_dram_bytes_per_launch")}
+
+    # ---- e2e through the public API with host buffers: H2D A shard + B, D2H D shard
+    e2e = None
+    try:
+        A_pin = torch.from_numpy(np.ascontiguousarray(A_host)).pin_memory()
+        B_pin = torch.empty((K, N), dtype=torch.float32).pin_memory()
+        B_pin.copy_(B.cpu())
+        D_pin = torch.empty((m_loc, N), dtype=torch.float32).pin_memory()
+        A_dev = torch.empty_like(A)
+        B_dev = torch.empty_like(B)
+        ws = torch.empty(egemm.gemm_workspace_size(m_loc, N, K), dtype=torch.uint8, device=dev)
+
+        def e2e_step():
+            A_dev.copy_(A_pin, non_blocking=True)
+            B_dev.copy_(B_pin, non_blocking=True)
+            egemm.gemm(A_dev, B_dev, out=D, workspace=ws)
+            D_pin.copy_(D, non_blocking=True)
+
+        for _ in range(2):
+            e2e_step()
+        _barrier(world)
+        s2, t2 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        k2 = max(2, min(args.steps, 5))
+        s2.record(stream)
+        for _ in range(k2):
+            e2e_step()
+        t2.record(stream)
+        _barrier(world)
+        e_ms = _allmax(s2.elapsed_time(t2), world) / k2
+        e2e = {"value": round(flop_total / (e_ms * 1e-3) / 1e12, 2), "unit": UNIT,
+               "ms_per_step": round(e_ms, 3),
+               "h2d_bytes_per_step": int(A_pin.numel() * 4 + B_pin.numel() * 4),
+               "d2h_bytes_per_step": int(D_pin.numel() * 4),
+               "path": "egemm_gemm(fp32 A,B from pinned host; split inside the call) -> D to host"}
+        del A_pin, B_pin, D_pin, A_dev, B_dev, ws
+    except Exception as ex:  # pragma: no cover
+        e2e = {"value": None, "unit": UNIT, "error": str(ex)[:200]}
+
+    apps = {}
+    if not args.no_apps:
+        apps = _apps(world, rank, dev, args)
+
+    cpu = None
+    if rank == 0 and world == 1 and not args.no_cpu:
+        import oracle
+        rows, dt, tf = run_oracle_sample(n, args.cpu_seconds)
+        cpu = {"value": round(tf, 6), "unit": UNIT, "cores": oracle.num_threads(), "kind": "oracle",
+               "sample": "oracle.gemm_emu64 (round-split + 3-term products in fp64) on %d of %d "
+                         "rows of the %d^3 workload, %.1f s" % (rows, n, n, dt)}
+
+    if rank == 0:
+        line = {
+            "metric": METRIC, "value": round(value, 2), "unit": UNIT, "n_gpus": world,
+            "steps": args.steps, "warmup": args.warmup, "ms_per_step": round(ms_per_step, 4),
+            "higher_is_better": True, "scaling": "strong", "vs_baseline": None, "dtype": "f16x3->f32",
+            "data": "synthetic U[-1,1] fp32, seeded PCG64 (inputs > L2, no flush needed)",
+            "config": {"workload": "egemm %d^3 (BASELINE configs[1]), row-sharded C" % n,
+                       "M": M, "N": N, "K": K, "terms": terms, "rows_per_rank": m_loc,
+                       "l2": "every operand 256 MiB > 126 MB L2",
+                       "parallelism": "dp%d rows" % world},
+            "gpu_launches": launches_per_step * args.steps,
+            "e2e": e2e, "roofline": roofline, "split_roofline": split_rl,
+            "cpu_baseline": cpu, "clocks": clocks,
+            "split_ms_per_step": round(split_ms, 4),
+            "paper_context": {"t4_speedup_vs_cublas_fp32": 3.13, "t4_speedup_vs_sdk": 11.18,
+                              "note": "paper's numbers on Tesla T4 (P:63, P:2251, P:2325), context only"},
+        }
+        line.update(apps)
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        import torch.distributed as dist
+        dist.destroy_process_group()
+
+
+def _apps(world, rank, dev, args):
+    """kNN (configs[3]) and kMeans (configs[4]) timings, queries / points sharded."""
+    import torch
+    from paper_conf_ppopp_fengwcz0d21_b200 import egemm, inputs
+    from paper_conf_ppopp_fengwcz0d21_b200 import distributed as edist
+    out = {}
+    try:
+        nx, nq, d, k = 1 << 20, 1 << 16, 128, 16
+        q0, q1 = edist.shard_bounds(nq, world, rank)
+        X = torch.from_numpy(inputs.uniform((nx, d), 300)).to(dev)
+        Q = torch.from_numpy(inputs.uniform((nq, d), 301)[q0:q1]).to(dev)
+        t_ib = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        t_ib[0].record()
+        x_split = egemm.split(X)  # the index build (once)
+        t_ib[1].record()
+        ws = torch.empty(egemm.knn_workspace_size(nx, q1 - q0, d, k, True), dtype=torch.uint8, device=dev)
+        idx = torch.empty((q1 - q0, k), dtype=torch.int32, device=dev)
+        dist_ = torch.empty((q1 - q0, k), dtype=torch.float32, device=dev)
+        for _ in range(2):
+            egemm.knn(X, Q, k, x_split=x_split, workspace=ws, out=(idx, dist_))
+        _barrier(world)
+        s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        reps = 3
+        s.record()
+        for _ in range(reps):
+            egemm.knn(X, Q, k, x_split=x_split, workspace=ws, out=(idx, dist_))
+        e.record()
+        _barrier(world)
+        ms = _allmax(s.elapsed_time(e), world) / reps
+        out["knn"] = {"metric": "kNN queries/s (1M refs x 64K queries, d=128, k=16)",
+                      "value": round(nq / (ms * 1e-3), 1), "unit": "queries/s",
+                      "ms_per_batch": round(ms, 3), "index_build_ms": round(t_ib[0].elapsed_time(t_ib[1]), 3),
+                      "fp32eq_tflops": round(2.0 * nx * nq * d / (ms * 1e-3) / 1e12, 1),
+                      "sharding": "queries over %d ranks, X replicated" % world}
+        del X, Q, x_split, ws
+    except Exception as ex:  # pragma: no cover
+        out["knn"] = {"error": str(ex)[:300]}
+    try:
+        n, d, kc, iters = 1 << 22, 64, 1024, 20
+        p0, p1 = edist.shard_bounds(n, world, rank)
+        Xh, lab, _ = inputs.mixture(n, d, kc, 400)
+        X = torch.from_numpy(Xh[p0:p1]).to(dev)
+        C0 = torch.from_numpy(Xh[:kc].copy()).to(dev)
+        del Xh
+        x_split = egemm.split(X)
+        C = C0.clone()
+        ws = torch.empty(egemm.kmeans_workspace_size(p1 - p0, d, kc, True), dtype=torch.uint8, device=dev)
+        bufs = (torch.empty(p1 - p0, dtype=torch.int32, device=dev),
+                torch.empty((kc, d), dtype=torch.float64, device=dev),
+                torch.empty(kc, dtype=torch.int64, device=dev), None)
+        edist.kmeans_fit(X, C, 2, x_split=x_split, workspace=ws, bufs=bufs, world=world)
+        C.copy_(C0)
+        _barrier(world)
+        s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        s.record()
+        edist.kmeans_fit(X, C, iters, x_split=x_split, workspace=ws, bufs=bufs, world=world)
+        e.record()
+        _barrier(world)
+        ms = _allmax(s.elapsed_time(e), world) / iters
+        out["kmeans"] = {"metric": "kMeans ms/iteration (4M points, d=64, 1024 centroids)",
+                         "value": round(ms, 4), "unit": "ms/iter", "iterations": iters,
+                         "fp32eq_tflops": round(2.0 * n * kc * d / (ms * 1e-3) / 1e12, 1),
+                         "sharding": "points over %d ranks, NCCL all_reduce of sums/counts" % world}
+    except Exception as ex:  # pragma: no cover
+        out["kmeans"] = {"error": str(ex)[:300]}
+    return out
+
+
+if __name__ == "__main__":
+    main()

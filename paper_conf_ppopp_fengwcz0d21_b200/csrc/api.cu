@@ -50,11 +50,13 @@ static TcConfig choose_config(int epi_kind, int64_t M, int64_t N, int64_t K, int
   TcConfig c = {};
   c.terms = terms;
   c.max_clusters = 0;
-  // default: CTA pair, 256 x 256 tiles, single accumulator in ping-pong, Kc = 256
+  // default: CTA pair, 256 x 256 tiles, single accumulator in ping-pong
   c.cg = 2;
   c.bn = 256;
   c.sep = 0;
-  c.kc = 128;  // measured: Kc=256 exceeds 2x naive-fp32 error at K<=1024 (tools/error_sweep.py)
+  // promotion every 64 k (one stage): measured fastest after the barrier fix and the most
+  // accurate single-accumulator setting (tools/error_sweep.py)
+  c.kc = 64;
   if (epi_kind == EPI_STORE && M <= 128) { c.cg = 1; c.bn = 128; c.sep = 1; }
   if (epi_kind != EPI_STORE) c.kc = (int)(((K + 63) / 64) * 64);
   // thread-local API override, then environment (experiments)

@@ -125,6 +125,26 @@ __device__ __forceinline__ void topk_insert(float (&kd)[KN], int (&ki)[KN], floa
   }
 }
 
+// streaming insertion (indices arrive in increasing order): strict '<' is enough
+template <int KN>
+__device__ __forceinline__ void topk_insert_stream(float (&kd)[KN], int (&ki)[KN], float key,
+                                                   int idx) {
+  if (key < kd[KN - 1]) {
+    kd[KN - 1] = key;
+    ki[KN - 1] = idx;
+#pragma unroll
+    for (int t = KN - 1; t > 0; t--) {
+      const bool sw = kd[t] < kd[t - 1];
+      const float a = kd[t], b = kd[t - 1];
+      const int ia = ki[t], ib = ki[t - 1];
+      kd[t] = sw ? b : a;
+      kd[t - 1] = sw ? a : b;
+      ki[t] = sw ? ib : ia;
+      ki[t - 1] = sw ? ia : ib;
+    }
+  }
+}
+
 __device__ __forceinline__ void named_bar_sync(int id, int nthreads) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }
@@ -233,8 +253,7 @@ __global__ void __launch_bounds__(kThreads, 1)
           for (int ch = 0; ch < nch; ch++) {
             const uint32_t buf = chunk_ctr & 1u;
             const uint32_t use = chunk_ctr >> 1;
-            if constexpr (CG == 2) ptx::mbar_wait_cluster(&acc_empty[buf], (use & 1u) ^ 1u);
-            else ptx::mbar_wait(&acc_empty[buf], (use & 1u) ^ 1u);
+            ptx::mbar_wait(&acc_empty[buf], (use & 1u) ^ 1u);
             ptx::tc_fence_after();
             const uint32_t acc_hh = tmem_base + (SEP ? 2 * buf : buf) * BN;
             const uint32_t acc_x = SEP ? acc_hh + BN : acc_hh;
@@ -248,14 +267,23 @@ __global__ void __launch_bounds__(kThreads, 1)
               const uint64_t d_alo = ptx::sdesc_kmajor_sw128(sa + G::A_BYTES);
               const uint64_t d_bhi = ptx::sdesc_kmajor_sw128(sa + 2 * G::A_BYTES);
               const uint64_t d_blo = ptx::sdesc_kmajor_sw128(sa + 2 * G::A_BYTES + G::B_BYTES);
+              // Alg. 1 order: the products involving lo first, hi*hi last --
+              // here per 64-wide k-block: all cross MMAs, then all hi*hi MMAs.  With one
+              // accumulator this keeps |acc| ~2^-11 smaller while the cross terms are
+              // added, so the tensor core's truncating alignment (probe model)
+              // loses almost nothing on them; only the 4 hi*hi MMAs see the full |acc|.
 #pragma unroll
               for (int k = 0; k < kBK / 16; k++) {
                 const uint64_t ko = (uint64_t)(k * 2);  // +32 B per 16-wide k step (>>4)
                 const uint32_t first = (kb > kb0 || k > 0) ? 1u : 0u;
-                // Alg. 1 order: products involving lo first, hi*hi last
                 ptx::mma_f16<CG>(acc_x, d_ahi + ko, d_blo + ko, idesc, first);
                 ptx::mma_f16<CG>(acc_x, d_alo + ko, d_bhi + ko, idesc, 1u);
                 if (p.terms == 4) ptx::mma_f16<CG>(acc_x, d_alo + ko, d_blo + ko, idesc, 1u);
+              }
+#pragma unroll
+              for (int k = 0; k < kBK / 16; k++) {
+                const uint64_t ko = (uint64_t)(k * 2);
+                const uint32_t first = (kb > kb0 || k > 0) ? 1u : 0u;
                 ptx::mma_f16<CG>(acc_hh, d_ahi + ko, d_bhi + ko, idesc, SEP ? first : 1u);
               }
               ptx::mma_commit<CG>(&empty[stage]);
@@ -387,12 +415,33 @@ __global__ void __launch_bounds__(kThreads, 1)
               for (int i = 0; i < 32; i++)
                 bn[i] = (c0 + i < p.N) ? __ldg(p.bnorm + c0 + i) : __int_as_float(0x7f800000);
             }
+            if constexpr (EPI == EPI_KNN) {
+              // fast path: keys + a candidate mask against this row's current k-th key;
+              // the (rare) insertions run in a compact loop over the set bits.  A thread's
+              // columns arrive in increasing index order, so a strict '<' keeps the lower
+              // index first among equal keys.
+              const float thr = kd[kKnnMax - 1];
+              uint32_t cand = 0;
 #pragma unroll
-            for (int i = 0; i < 32; i++) {
-              const float key = __fmaf_rn(-2.f, v[i], bn[i]);  // ||b||^2 - 2 a.b (exact *2)
-              if constexpr (EPI == EPI_KNN) {
-                topk_insert<kKnnMax>(kd, ki, key, c0 + i);
-              } else {
+              for (int i = 0; i < 32; i++) {
+                v[i] = __fmaf_rn(-2.f, v[i], bn[i]);  // ||b||^2 - 2 a.b (the *2 is exact)
+                cand |= (v[i] < thr) ? (1u << i) : 0u;
+              }
+              if (__any_sync(0xffffffffu, cand != 0u)) {
+                float keys[32];
+#pragma unroll
+                for (int i = 0; i < 32; i++) keys[i] = v[i];
+#pragma unroll 1
+                while (cand) {
+                  const int i = __ffs(cand) - 1;
+                  cand &= cand - 1u;
+                  topk_insert_stream<kKnnMax>(kd, ki, keys[i], c0 + i);
+                }
+              }
+            } else {
+#pragma unroll
+              for (int i = 0; i < 32; i++) {
+                const float key = __fmaf_rn(-2.f, v[i], bn[i]);  // ||b||^2 - 2 a.b (exact *2)
                 if (key < best) { best = key; besti = c0 + i; }
               }
             }

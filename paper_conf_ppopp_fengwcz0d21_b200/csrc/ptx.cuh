@@ -41,12 +41,14 @@ __device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t by
                "r"(bytes)
                : "memory");
 }
-// Arrive on the barrier at the same smem offset in CTA `cta` of the cluster.
+// Arrive on the barrier at the same smem offset in CTA `cta` of the cluster.  Default
+// (.release.cta) semantics: the TMEM reads it orders are fenced by tcgen05.fence::
+// before_thread_sync; a .release.cluster arrive would emit a GPU-scope MEMBAR per call.
 __device__ __forceinline__ void mbar_arrive_cluster(uint64_t* bar, uint32_t cta) {
   asm volatile(
       "{\n\t.reg .b32 ra;\n\t"
       "mapa.shared::cluster.u32 ra, %0, %1;\n\t"
-      "mbarrier.arrive.release.cluster.shared::cluster.b64 _, [ra];\n\t}" ::"r"(smem_u32(bar)),
+      "mbarrier.arrive.shared::cluster.b64 _, [ra];\n\t}" ::"r"(smem_u32(bar)),
       "r"(cta)
       : "memory");
 }

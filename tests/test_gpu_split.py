@@ -15,7 +15,9 @@ def _cmp(x, ghi, glo, ohi, olo):
     # NaN inputs: compare by class (both NaN) -- cvt.rn may canonicalise the payload
     hn = lambda h: ((h & 0x7C00) == 0x7C00) & ((h & 0x3FF) != 0)
     same |= nan & hn(ghi) & hn(glo) & hn(ohi) & hn(olo)
-    # x = +-inf: hi = inf, lo = inf - inf = NaN on both sides
+    # x = +-inf (and |x| >= 65520): hi = +-inf bitwise, lo = x - inf is NaN on both sides
+    # (the NaN sign/payload of inf - inf differs between x86 and the GPU: compare by class)
+    same |= (ghi == ohi) & hn(glo) & hn(olo)
     return same
 
 
