@@ -383,19 +383,19 @@ def _apps(world, rank, dev, args):
         Q = torch.from_numpy(inputs.uniform((nq, d), 301)[q0:q1]).to(dev)
         t_ib = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         t_ib[0].record()
-        x_split = egemm.split(X)  # the index build (once)
+        index = egemm.knn_index(X)  # the index build (once): split + norms of X
         t_ib[1].record()
         ws = torch.empty(egemm.knn_workspace_size(nx, q1 - q0, d, k, True), dtype=torch.uint8, device=dev)
         idx = torch.empty((q1 - q0, k), dtype=torch.int32, device=dev)
         dist_ = torch.empty((q1 - q0, k), dtype=torch.float32, device=dev)
         for _ in range(2):
-            egemm.knn(X, Q, k, x_split=x_split, workspace=ws, out=(idx, dist_))
+            egemm.knn(X, Q, k, index=index, workspace=ws, out=(idx, dist_))
         _barrier(world)
         s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         reps = 3
         s.record()
         for _ in range(reps):
-            egemm.knn(X, Q, k, x_split=x_split, workspace=ws, out=(idx, dist_))
+            egemm.knn(X, Q, k, index=index, workspace=ws, out=(idx, dist_))
         e.record()
         _barrier(world)
         ms = _allmax(s.elapsed_time(e), world) / reps
@@ -404,7 +404,7 @@ def _apps(world, rank, dev, args):
                       "ms_per_batch": round(ms, 3), "index_build_ms": round(t_ib[0].elapsed_time(t_ib[1]), 3),
                       "fp32eq_tflops": round(2.0 * nx * nq * d / (ms * 1e-3) / 1e12, 1),
                       "sharding": "queries over %d ranks, X replicated" % world}
-        del X, Q, x_split, ws
+        del X, Q, index, ws
     except Exception as ex:  # pragma: no cover
         out["knn"] = {"error": str(ex)[:300]}
     try:

@@ -102,15 +102,23 @@ size_t egemm_gemm_workspace_size(int64_t M, int64_t N, int64_t K, int a_presplit
  * the k rows x_j of X[nx x d] with the smallest squared distance
  *   dist_ij = ||q_i||^2 + ||x_j||^2 - 2 q_i . x_j ,
  * ascending by (dist, j), dist clamped to >= 0; self matches are kept (reading R11).
- *  X, Q  : f32 required (row norms, fp64-accumulated); trans must be 0; hi/lo optional
- *          (pre-split X = the "index build").
+ *  X     : the references, trans 0.  Either fp32 rows (then split and normed on the fly)
+ *          or the "index" from egemm_knn_index: pre-split hi/lo + x_norms (f32 may be NULL).
+ *  x_norms : nullable nx fp32 ||x_j||^2 (fp64-accumulated, from egemm_knn_index).
+ *  Q     : fp32 query rows (trans 0, ld >= d), split and normed on the fly.
  *  k     : 1 <= k <= 16 and k <= nx.
  *  out_idx  : nq x k int32;  out_dist : nq x k fp32.
  */
-int egemm_knn(egemm_operand_t X, int64_t nx, egemm_operand_t Q, int64_t nq, int64_t d, int k,
-              int32_t* out_idx, float* out_dist, void* workspace, size_t workspace_bytes,
-              void* stream);
+int egemm_knn(egemm_operand_t X, const float* x_norms, int64_t nx, egemm_operand_t Q, int64_t nq,
+              int64_t d, int k, int32_t* out_idx, float* out_dist, void* workspace,
+              size_t workspace_bytes, void* stream);
 size_t egemm_knn_workspace_size(int64_t nx, int64_t nq, int64_t d, int k, int x_presplit);
+
+/* kNN index build: round-split of the references X[nx x d] (row stride ldx) into K-major
+ * hi/lo (row stride ld_split, a multiple of 8) and their squared norms ||x_j||^2
+ * (fp64-accumulated, rounded once to fp32).  Done once; reused by every egemm_knn call. */
+int egemm_knn_index(const float* X, int64_t nx, int64_t d, int64_t ldx, uint16_t* hi, uint16_t* lo,
+                    int64_t ld_split, float* norms, void* stream);
 
 /*
  * One Lloyd step of kMeans on the caller's shard of points (the GEMM-based kMeans of [2],

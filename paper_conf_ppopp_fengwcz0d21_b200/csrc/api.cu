@@ -295,17 +295,44 @@ size_t egemm_knn_workspace_size(int64_t nx, int64_t nq, int64_t d, int k, int x_
   return cv.off;
 }
 
-int egemm_knn(egemm_operand_t X, int64_t nx, egemm_operand_t Q, int64_t nq, int64_t d, int k,
-              int32_t* out_idx, float* out_dist, void* workspace, size_t workspace_bytes,
-              void* stream) {
+int egemm_knn_index(const float* X, int64_t nx, int64_t d, int64_t ldx, uint16_t* hi, uint16_t* lo,
+                    int64_t ld_split, float* norms, void* stream) {
+  cudaStream_t s = (cudaStream_t)stream;
+  if (nx < 0 || d <= 0 || ldx < d || ld_split < d || (ld_split % 8) != 0) {
+    set_last_error("need nx >= 0, d > 0, ldx >= d, ld_split >= d and a multiple of 8");
+    return EGEMM_ERR_INVALID_ARG;
+  }
+  if (nx == 0) return EGEMM_OK;
+  if (!X || !hi || !lo || !norms) {
+    set_last_error("NULL pointer");
+    return EGEMM_ERR_INVALID_ARG;
+  }
+  if (!device_ok()) {
+    set_last_error("no sm_100 device");
+    return EGEMM_ERR_CUDA;
+  }
+  if (launch_split(X, nx, d, ldx, hi, lo, ld_split, 0, nullptr, s) ||
+      launch_rownorm(X, nx, d, ldx, norms, s))
+    return EGEMM_ERR_CUDA;
+  return EGEMM_OK;
+}
+
+int egemm_knn(egemm_operand_t X, const float* x_norms, int64_t nx, egemm_operand_t Q, int64_t nq,
+              int64_t d, int k, int32_t* out_idx, float* out_dist, void* workspace,
+              size_t workspace_bytes, void* stream) {
   cudaStream_t s = (cudaStream_t)stream;
   if (nx < 0 || nq < 0 || d <= 0 || k < 1 || k > 16 || k > nx) {
     set_last_error("need nx, nq >= 0, d > 0, 1 <= k <= min(16, nx)");
     return EGEMM_ERR_INVALID_ARG;
   }
   if (nq == 0) return EGEMM_OK;
-  if (!X.f32 || !Q.f32 || X.trans || Q.trans || X.ld < d || Q.ld < d || !out_idx || !out_dist) {
-    set_last_error("X/Q need fp32 rows (trans 0, ld >= d) and outputs");
+  if ((!X.f32 && !x_norms) || !Q.f32 || X.trans || Q.trans || (X.f32 && X.ld < d) || Q.ld < d ||
+      !out_idx || !out_dist) {
+    set_last_error("X needs fp32 rows or (hi/lo + x_norms); Q fp32 rows (trans 0, ld >= d)");
+    return EGEMM_ERR_INVALID_ARG;
+  }
+  if (!X.f32 && !(X.hi && X.lo)) {
+    set_last_error("X: no data");
     return EGEMM_ERR_INVALID_ARG;
   }
   if (d > 1024) {
@@ -334,8 +361,9 @@ int egemm_knn(egemm_operand_t X, int64_t nx, egemm_operand_t Q, int64_t nq, int6
   float* qnorm = cv.take<float>((size_t)nq);
   float* pkey = cv.take<float>((size_t)(8 * nq * k));
   int32_t* pidx = cv.take<int32_t>((size_t)(8 * nq * k));
-  if (launch_rownorm(X.f32, nx, d, X.ld, xnorm, s) || launch_rownorm(Q.f32, nq, d, Q.ld, qnorm, s))
-    return EGEMM_ERR_CUDA;
+  if (x_norms) xnorm = const_cast<float*>(x_norms);
+  else if (launch_rownorm(X.f32, nx, d, X.ld, xnorm, s)) return EGEMM_ERR_CUDA;
+  if (launch_rownorm(Q.f32, nq, d, Q.ld, qnorm, s)) return EGEMM_ERR_CUDA;
   TcEpilogue epi = {};
   epi.kind = EPI_KNN;
   epi.bnorm = xnorm;
@@ -359,7 +387,7 @@ size_t egemm_kmeans_workspace_size(int64_t n, int64_t d, int64_t kc, int x_presp
   cv.take<uint16_t>((size_t)(kc * ldk));
   cv.take<float>((size_t)kc);
   cv.take<float>((size_t)n);
-  cv.take<float>((size_t)n);
+  cv.take<char>(kmeans_accumulate_ws(n, kc));
   return cv.off;
 }
 
@@ -375,8 +403,8 @@ int egemm_kmeans_step(egemm_operand_t X, int64_t n, int64_t d, const float* cent
     set_last_error("X needs fp32 rows (trans 0, ld >= d)");
     return EGEMM_ERR_INVALID_ARG;
   }
-  if (d > 1024) {
-    set_last_error("d > 1024 not supported by the fused epilogue");
+  if (d > 1024 || kc > 12288) {
+    set_last_error("d > 1024 or kc > 12288 not supported by the fused epilogue / sums");
     return EGEMM_ERR_UNSUPPORTED;
   }
   if (!device_ok()) {
@@ -391,8 +419,8 @@ int egemm_kmeans_step(egemm_operand_t X, int64_t n, int64_t d, const float* cent
     return EGEMM_ERR_WORKSPACE;
   }
   if (n == 0)
-    return launch_kmeans_accumulate(nullptr, 0, d, d, nullptr, nullptr, nullptr, kc, sums, counts,
-                                    inertia, s)
+    return launch_kmeans_accumulate(nullptr, 0, d, d, nullptr, nullptr, kc, sums, counts, inertia,
+                                    nullptr, s)
                ? EGEMM_ERR_CUDA
                : EGEMM_OK;
   TcConfig cfg = choose_config(EPI_KMEANS, n, kc, d, 3);
@@ -403,9 +431,8 @@ int egemm_kmeans_step(egemm_operand_t X, int64_t n, int64_t d, const float* cent
   if ((r = stage_operand(Cop, kc, d, cv, &ops.b_hi, &ops.b_lo, &ops.ldb, s))) return r;
   float* cnorm = cv.take<float>((size_t)kc);
   float* best = cv.take<float>((size_t)n);
-  float* xnorm = cv.take<float>((size_t)n);
+  void* accws = cv.take<char>(kmeans_accumulate_ws(n, kc));
   if (launch_rownorm(centroids, kc, d, d, cnorm, s)) return EGEMM_ERR_CUDA;
-  if (inertia && launch_rownorm(X.f32, n, d, X.ld, xnorm, s)) return EGEMM_ERR_CUDA;
   TcEpilogue epi = {};
   epi.kind = EPI_KMEANS;
   epi.bnorm = cnorm;
@@ -413,10 +440,8 @@ int egemm_kmeans_step(egemm_operand_t X, int64_t n, int64_t d, const float* cent
   epi.best_key = best;
   r = launch_tc(n, kc, d, ops, cfg, epi, s);
   if (r) return r == 2 ? EGEMM_ERR_UNSUPPORTED : EGEMM_ERR_CUDA;
-  if (launch_kmeans_accumulate(X.f32, n, d, X.ld, assign, best, xnorm, kc, sums, counts, inertia,
-                               s))
-    return EGEMM_ERR_CUDA;
-  return EGEMM_OK;
+  r = launch_kmeans_accumulate(X.f32, n, d, X.ld, assign, best, kc, sums, counts, inertia, accws, s);
+  return r == 0 ? EGEMM_OK : (r == 2 ? EGEMM_ERR_UNSUPPORTED : EGEMM_ERR_CUDA);
 }
 
 int egemm_kmeans_finalize(const double* sums, const int64_t* counts, int64_t kc, int64_t d,

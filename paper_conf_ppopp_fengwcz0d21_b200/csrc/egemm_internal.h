@@ -62,10 +62,10 @@ int launch_rownorm(const float* x, int64_t rows, int64_t d, int64_t ld, float* o
 int launch_knn_merge(const float* part_key, const int32_t* part_idx, int n_slices, int64_t nq,
                      int k, const float* qnorm, int32_t* out_idx, float* out_dist,
                      cudaStream_t stream);
+size_t kmeans_accumulate_ws(int64_t n, int64_t kc);
 int launch_kmeans_accumulate(const float* X, int64_t n, int64_t d, int64_t ldx,
-                             const int32_t* assign, const float* best_key, const float* xnorm,
-                             int64_t kc, double* sums, int64_t* counts, double* inertia,
-                             cudaStream_t stream);
+                             const int32_t* assign, const float* best_key, int64_t kc, double* sums,
+                             int64_t* counts, double* inertia, void* ws, cudaStream_t stream);
 int launch_kmeans_finalize(const double* sums, const int64_t* counts, int64_t kc, int64_t d,
                            float* centroids, cudaStream_t stream);
 int launch_fill_c(int64_t M, int64_t N, const float* C, int64_t ldc, float* D, int64_t ldd,

@@ -34,7 +34,7 @@ class Operand(ctypes.Structure):
 
 
 EXPORTS = ["egemm_status_string", "egemm_last_error", "egemm_version", "egemm_split", "egemm_gemm",
-           "egemm_gemm_workspace_size", "egemm_knn", "egemm_knn_workspace_size",
+           "egemm_gemm_workspace_size", "egemm_knn", "egemm_knn_workspace_size", "egemm_knn_index",
            "egemm_kmeans_step", "egemm_kmeans_workspace_size", "egemm_kmeans_finalize",
            "egemm_set_config", "egemm_num_sms"]
 
@@ -61,10 +61,12 @@ def load(path: str = LIB_PATH):
     L.egemm_gemm.restype = I
     L.egemm_gemm_workspace_size.argtypes = [I64, I64, I64, I, I]
     L.egemm_gemm_workspace_size.restype = SZ
-    L.egemm_knn.argtypes = [Operand, I64, Operand, I64, I64, I, P, P, P, SZ, P]
+    L.egemm_knn.argtypes = [Operand, P, I64, Operand, I64, I64, I, P, P, P, SZ, P]
     L.egemm_knn.restype = I
     L.egemm_knn_workspace_size.argtypes = [I64, I64, I64, I, I]
     L.egemm_knn_workspace_size.restype = SZ
+    L.egemm_knn_index.argtypes = [P, I64, I64, I64, P, P, I64, P, P]
+    L.egemm_knn_index.restype = I
     L.egemm_kmeans_step.argtypes = [Operand, I64, I64, P, I64, P, P, P, P, P, SZ, P]
     L.egemm_kmeans_step.restype = I
     L.egemm_kmeans_workspace_size.argtypes = [I64, I64, I64, I]
@@ -131,7 +133,7 @@ def operand(f32: torch.Tensor | None = None, hi=None, lo=None, trans: bool = Fal
     op.f32 = f32.data_ptr() if f32 is not None else None
     op.hi = hi.data_ptr() if hi is not None else None
     op.lo = lo.data_ptr() if lo is not None else None
-    op.ld = f32.stride(0) if f32 is not None else 0
+    op.ld = f32.stride(0) if f32 is not None else (hi.shape[1] if hi is not None else 0)
     op.trans = 1 if trans else 0
     op.ld_split = hi.stride(0) if hi is not None else 0
     return op
@@ -175,23 +177,45 @@ def knn_workspace_size(nx, nq, d, k, x_presplit=False) -> int:
     return int(load().egemm_knn_workspace_size(nx, nq, d, k, int(x_presplit)))
 
 
-def knn(X: torch.Tensor, Q: torch.Tensor, k: int, x_split=None, workspace=None, out=None,
-        stream=None):
+def knn_index(X: torch.Tensor, stream=None):
+    """Index build for kNN: (hi, lo, norms) of the references X [nx, d] (done once)."""
+    L = load()
+    _need_cuda(X)
+    nx, d = X.shape
+    ld = (d + 7) // 8 * 8
+    hi = torch.empty((nx, ld), dtype=torch.int16, device=X.device)[:, :d]
+    lo = torch.empty((nx, ld), dtype=torch.int16, device=X.device)[:, :d]
+    norms = torch.empty(nx, dtype=torch.float32, device=X.device)
+    _check(L.egemm_knn_index(_ptr(X), nx, d, X.stride(0), _ptr(hi), _ptr(lo), ld, _ptr(norms),
+                             _stream(stream)), "egemm_knn_index")
+    return hi, lo, norms
+
+
+def knn(X: torch.Tensor | None, Q: torch.Tensor, k: int, x_split=None, index=None, workspace=None,
+        out=None, stream=None):
     """k nearest rows of X [nx, d] for each query row of Q [nq, d] (squared L2, ascending).
-    Returns (idx int32 [nq, k], dist fp32 [nq, k])."""
+    Pass ``index=knn_index(X)`` to reuse the split references and their norms (X may then
+    be None).  Returns (idx int32 [nq, k], dist fp32 [nq, k])."""
     L = load()
     _need_cuda(X, Q)
-    nx, d = X.shape
-    nq = Q.shape[0]
+    nq, d = Q.shape
+    if index is not None:
+        hi, lo, norms = index
+        nx = hi.shape[0]
+        opX = operand(X, hi, lo)
+    else:
+        nx = X.shape[0]
+        norms = None
+        opX = operand(X, *(x_split or (None, None)))
     if out is None:
-        idx = torch.empty((nq, k), dtype=torch.int32, device=X.device)
-        dist = torch.empty((nq, k), dtype=torch.float32, device=X.device)
+        idx = torch.empty((nq, k), dtype=torch.int32, device=Q.device)
+        dist = torch.empty((nq, k), dtype=torch.float32, device=Q.device)
     else:
         idx, dist = out
-    need = knn_workspace_size(nx, nq, d, k, x_split is not None)
-    ws, wsn = _workspace(need, X.device, workspace)
-    _check(L.egemm_knn(operand(X, *(x_split or (None, None))), nx, operand(Q), nq, d, k, _ptr(idx),
-                       _ptr(dist), _ptr(ws), wsn, _stream(stream)), "egemm_knn")
+    need = knn_workspace_size(nx, nq, d, k, index is not None or x_split is not None)
+    ws, wsn = _workspace(need, Q.device, workspace)
+    _check(L.egemm_knn(opX, _ptr(norms), nx, operand(Q), nq, d, k, _ptr(idx), _ptr(dist), _ptr(ws),
+                       wsn, _stream(stream)), "egemm_knn")
     return idx, dist
 
 
