@@ -387,7 +387,7 @@ size_t egemm_kmeans_workspace_size(int64_t n, int64_t d, int64_t kc, int x_presp
   cv.take<uint16_t>((size_t)(kc * ldk));
   cv.take<float>((size_t)kc);
   cv.take<float>((size_t)n);
-  cv.take<char>(kmeans_accumulate_ws(n, kc));
+  cv.take<char>(kmeans_accumulate_ws(n, d, kc));
   return cv.off;
 }
 
@@ -431,7 +431,7 @@ int egemm_kmeans_step(egemm_operand_t X, int64_t n, int64_t d, const float* cent
   if ((r = stage_operand(Cop, kc, d, cv, &ops.b_hi, &ops.b_lo, &ops.ldb, s))) return r;
   float* cnorm = cv.take<float>((size_t)kc);
   float* best = cv.take<float>((size_t)n);
-  void* accws = cv.take<char>(kmeans_accumulate_ws(n, kc));
+  void* accws = cv.take<char>(kmeans_accumulate_ws(n, d, kc));
   if (launch_rownorm(centroids, kc, d, d, cnorm, s)) return EGEMM_ERR_CUDA;
   TcEpilogue epi = {};
   epi.kind = EPI_KMEANS;

@@ -62,7 +62,7 @@ int launch_rownorm(const float* x, int64_t rows, int64_t d, int64_t ld, float* o
 int launch_knn_merge(const float* part_key, const int32_t* part_idx, int n_slices, int64_t nq,
                      int k, const float* qnorm, int32_t* out_idx, float* out_dist,
                      cudaStream_t stream);
-size_t kmeans_accumulate_ws(int64_t n, int64_t kc);
+size_t kmeans_accumulate_ws(int64_t n, int64_t d, int64_t kc);
 int launch_kmeans_accumulate(const float* X, int64_t n, int64_t d, int64_t ldx,
                              const int32_t* assign, const float* best_key, int64_t kc, double* sums,
                              int64_t* counts, double* inertia, void* ws, cudaStream_t stream);

@@ -66,6 +66,29 @@ def test_kmeans_integer_sums_exact_and_empty_cluster(oracle_lib):
     assert np.array_equal(newc[1], C[1])  # empty cluster keeps its centroid (R12)
 
 
+def test_kmeans_sums_fixed_order_r20(oracle_lib):
+    """Reading R20: group members in ascending i, chunks of 256 summed sequentially, then
+    the chunk sums sequentially -- checked against a pure-Python rendering of that order
+    and against the exact rational sum (fp64 rounding bound)."""
+    from fractions import Fraction
+    X, lab, cent = inputs.mixture(3000, 3, 2, 9, sigma=0.5)
+    a, sums, counts, _, _ = oracle_lib.kmeans_step(X, cent)
+    for j in range(2):
+        mem = [i for i in range(3000) if a[i] == j]
+        assert counts[j] == len(mem) and len(mem) > 600
+        for t in range(3):
+            tot = 0.0
+            for c0 in range(0, len(mem), 256):
+                part = 0.0
+                for i in mem[c0:c0 + 256]:
+                    part = part + float(X[i, t])
+                tot = tot + part
+            assert sums[j, t] == tot
+            exact = sum(Fraction(float(X[i, t])) for i in mem)
+            mag = sum(abs(float(X[i, t])) for i in mem)
+            assert abs(Fraction(sums[j, t]) - exact) <= Fraction(len(mem) * 2.0 ** -52 * mag)
+
+
 def test_kmeans_ties_lowest_index(oracle_lib):
     X = np.array([[0.0, 0.0]], np.float32)
     C = np.array([[1.0, 0.0], [0.0, 1.0], [-1.0, 0.0]], np.float32)
