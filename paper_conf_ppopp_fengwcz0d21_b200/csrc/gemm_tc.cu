@@ -390,10 +390,14 @@ __global__ void __launch_bounds__(kThreads, 1)
           ptx::mbar_wait(&acc_full[buf], use & 1u);
           ptx::tc_fence_after();
           const uint32_t acc_hh = tmem_base + lane_off + (SEP ? 2 * buf : buf) * BN + cgp * COLS;
-#pragma unroll 1
+          // TMEM -> registers software-pipelined: the load of group c+1 is in flight while
+          // group c is processed; the accumulator buffer is handed back to the MMA warp as
+          // soon as the last group has landed in registers.
+          float vbuf[2][32];
+          ptx::tmem_ld32(acc_hh, vbuf[0]);
+#pragma unroll
           for (int c = 0; c < COLS / 32; c++) {
-            float v[32];
-            ptx::tmem_ld32(acc_hh + c * 32, v);
+            float* v = vbuf[c & 1];
             ptx::tmem_wait_ld();
             if constexpr (SEP) {
               float w[32];
@@ -401,6 +405,16 @@ __global__ void __launch_bounds__(kThreads, 1)
               ptx::tmem_wait_ld();
 #pragma unroll
               for (int i = 0; i < 32; i++) v[i] = __fadd_rn(v[i], w[i]);
+            }
+            if (c + 1 < COLS / 32) {
+              ptx::tmem_ld32(acc_hh + (c + 1) * 32, vbuf[(c + 1) & 1]);
+            } else {
+              ptx::tc_fence_before();
+              __syncwarp();
+              if (lane == 0) {
+                if constexpr (CG == 1) ptx::mbar_arrive(&acc_empty[buf]);
+                else ptx::mbar_arrive_cluster(&acc_empty[buf], 0);
+              }
             }
             const int c0 = col_base + c * 32;
             float bn[32];
@@ -421,16 +435,20 @@ __global__ void __launch_bounds__(kThreads, 1)
               // columns arrive in increasing index order, so a strict '<' keeps the lower
               // index first among equal keys.
               const float thr = kd[kKnnMax - 1];
-              uint32_t cand = 0;
+              float mn = __int_as_float(0x7f800000);
 #pragma unroll
               for (int i = 0; i < 32; i++) {
                 v[i] = __fmaf_rn(-2.f, v[i], bn[i]);  // ||b||^2 - 2 a.b (the *2 is exact)
-                cand |= (v[i] < thr) ? (1u << i) : 0u;
+                mn = fminf(mn, v[i]);
               }
-              if (__any_sync(0xffffffffu, cand != 0u)) {
+              if (__any_sync(0xffffffffu, mn < thr)) {
+                uint32_t cand = 0;
                 float keys[32];
 #pragma unroll
-                for (int i = 0; i < 32; i++) keys[i] = v[i];
+                for (int i = 0; i < 32; i++) {
+                  keys[i] = v[i];
+                  cand |= (v[i] < thr) ? (1u << i) : 0u;
+                }
 #pragma unroll 1
                 while (cand) {
                   const int i = __ffs(cand) - 1;
@@ -445,12 +463,6 @@ __global__ void __launch_bounds__(kThreads, 1)
                 if (key < best) { best = key; besti = c0 + i; }
               }
             }
-          }
-          ptx::tc_fence_before();
-          __syncwarp();
-          if (lane == 0) {
-            if constexpr (CG == 1) ptx::mbar_arrive(&acc_empty[buf]);
-            else ptx::mbar_arrive_cluster(&acc_empty[buf], 0);
           }
           chunk_ctr++;
         }
