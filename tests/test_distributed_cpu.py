@@ -1,0 +1,123 @@
+"""World-size-2 gloo tests (CPU) of the data-parallel composition in
+paper_conf_ppopp_fengwcz0d21_b200/distributed.py: shard bounds, broadcast, row gather,
+kNN candidate merge and the kMeans loop (local step -> all_reduce -> finalize).  The
+per-rank compute is injected (the CPU oracle, test-only): on the GPU box it is the C ABI."""
+import os
+import socket
+
+import numpy as np
+import pytest
+import torch
+import torch.distributed as dist
+import torch.multiprocessing as mp
+
+from paper_conf_ppopp_fengwcz0d21_b200 import distributed as edist
+from paper_conf_ppopp_fengwcz0d21_b200 import inputs
+
+
+def _free_port():
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    p = s.getsockname()[1]
+    s.close()
+    return p
+
+
+def _worker(rank, world, port, fn, q):
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        q.put((rank, fn(rank, world)))
+    except Exception as ex:  # pragma: no cover
+        q.put((rank, ex))
+    finally:
+        dist.destroy_process_group()
+
+
+def _run(fn, world=2):
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_worker, args=(r, world, port, fn, q)) for r in range(world)]
+    for p in ps:
+        p.start()
+    out = dict(q.get(timeout=120) for _ in ps)
+    for p in ps:
+        p.join(timeout=60)
+    for r, v in out.items():
+        if isinstance(v, Exception):
+            raise v
+    return out
+
+
+def test_shard_bounds_cover_and_align():
+    for n in (0, 1, 7, 256, 1000, 8192, 8193):
+        for world in (1, 2, 3, 8):
+            for align in (1, 256):
+                b = [edist.shard_bounds(n, world, r, align) for r in range(world)]
+                assert b[0][0] == 0 and b[-1][1] == n
+                assert all(b[i][1] == b[i + 1][0] for i in range(world - 1))
+                if n % align == 0:
+                    assert all(lo % align == 0 for lo, _ in b)
+    assert edist.shard_bounds(8192, 8, 3, 256) == (3072, 4096)
+
+
+def _bcast_gather(rank, world):
+    t = torch.arange(12, dtype=torch.float32).reshape(3, 4) if rank == 0 else torch.zeros(3, 4)
+    edist.broadcast_(t, world)
+    lo, hi = edist.shard_bounds(11, world, rank)
+    local = torch.arange(lo, hi, dtype=torch.float32)[:, None].repeat(1, 2)
+    full = edist.gather_rows(local, 11, world)
+    return t.numpy(), full.numpy()
+
+
+def test_broadcast_and_gather_rows():
+    out = _run(_bcast_gather)
+    for r in range(2):
+        t, full = out[r]
+        assert np.array_equal(t, np.arange(12).reshape(3, 4))
+        assert np.array_equal(full[:, 0], np.arange(11))
+
+
+def test_merge_topk_matches_sort():
+    g = torch.Generator().manual_seed(0)
+    keys = torch.rand(3, 5, 4, generator=g)
+    keys[1, 2, 0] = keys[0, 2, 1]  # a tie across parts -> lower index first
+    idx = torch.randint(0, 1000, (3, 5, 4), generator=g, dtype=torch.int32)
+    idx[1, 2, 0] = 3
+    idx[0, 2, 1] = 9
+    mk, mi = edist.merge_topk(keys, idx, 4)
+    for q in range(5):
+        pairs = sorted(zip(keys[:, q].flatten().tolist(), idx[:, q].flatten().tolist()))[:4]
+        assert mk[q].tolist() == [p[0] for p in pairs] and mi[q].tolist() == [p[1] for p in pairs]
+
+
+def _kmeans_ranks(rank, world):
+    import oracle
+    X, _, _ = inputs.mixture(6000, 8, 16, 3, sigma=0.1)
+    C = torch.from_numpy(X[:16].copy())
+    lo, hi = edist.shard_bounds(6000, world, rank)
+    Xl = torch.from_numpy(X[lo:hi].copy())
+
+    def step(X_, C_, out):
+        a, s, c, _, _ = oracle.kmeans_step(X_.numpy(), C_.numpy())
+        return torch.from_numpy(a), torch.from_numpy(s), torch.from_numpy(c), None
+
+    def finalize(s, c, C_):
+        C_.copy_(torch.from_numpy(oracle.kmeans_finalize(s.numpy(), c.numpy(), C_.numpy())))
+
+    edist.kmeans_fit(Xl, C, 3, world=world, step=step, finalize=finalize)
+    return C.numpy()
+
+
+def test_kmeans_fit_allreduce_equals_single_process(oracle_lib):
+    out = _run(_kmeans_ranks)
+    assert np.array_equal(out[0], out[1])  # every rank runs the same finalize
+    X, _, _ = inputs.mixture(6000, 8, 16, 3, sigma=0.1)
+    C = X[:16].copy()
+    for _ in range(3):
+        a, s, c, _, _ = oracle_lib.kmeans_step(X, C)
+        C = oracle_lib.kmeans_finalize(s, c, C)
+    # sums were reduced across ranks in another fp64 order: <= 1 ulp of fp32 (R20 note)
+    assert np.allclose(out[0], C, rtol=2.0 ** -23, atol=2.0 ** -30)

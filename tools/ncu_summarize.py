@@ -1,0 +1,117 @@
+"""Summarise ncu reports / launch lists into profiles/ (markdown + JSON).  Tool code.
+
+usage: python tools/ncu_summarize.py OUT_PREFIX report1.ncu-rep [report2 ...] [--launch list.csv]
+"""
+import csv
+import io
+import json
+import os
+import subprocess
+import sys
+
+KEYS = [
+    "gpu__time_duration.sum",
+    "gpc__cycles_elapsed.max",
+    "gpc__cycles_elapsed.avg.per_second",
+    "sm__pipe_tensor_cycles_active_realtime.avg.pct_of_peak_sustained_elapsed",
+    "sm__throughput.avg.pct_of_peak_sustained_elapsed",
+    "dram__bytes_read.sum",
+    "dram__bytes_write.sum",
+    "dram__throughput.avg.pct_of_peak_sustained_elapsed",
+    "gpu__dram_throughput.avg.pct_of_peak_sustained_elapsed",
+    "lts__t_sector_hit_rate.pct",
+    "l1tex__data_pipe_tc_wavefronts_mem_shared.sum.pct_of_peak_sustained_elapsed",
+    "launch__registers_per_thread",
+    "launch__grid_size",
+    "launch__block_size",
+    "launch__cluster_dim_x",
+    "smsp__inst_executed.sum",
+    "sm__warps_active.avg.pct_of_peak_sustained_active",
+]
+
+
+def raw(rep):
+    out = subprocess.check_output(["ncu", "-i", rep, "--page", "raw", "--csv"], stderr=subprocess.DEVNULL).decode()
+    rows = list(csv.reader(io.StringIO(out)))
+    hdr, units = rows[0], rows[1]
+    res = []
+    for r in rows[2:]:
+        d = {}
+        for h, u, v in zip(hdr, units, r):
+            d[h] = (v, u)
+        res.append(d)
+    return res
+
+
+def to_bytes(v, u):
+    try:
+        x = float(v.replace(",", ""))
+    except ValueError:
+        return None
+    mult = {"byte": 1, "Kbyte": 1e3, "Mbyte": 1e6, "Gbyte": 1e9, "Tbyte": 1e12}.get(u, None)
+    return x * mult if mult else x
+
+
+def summarize(rep):
+    out = []
+    for d in raw(rep):
+        name = d.get("Kernel Name", ("?", ""))[0]
+        s = {"kernel": name[:140], "report": os.path.basename(rep)}
+        for k in KEYS:
+            if k in d:
+                s[k] = d[k][0] + (" " + d[k][1] if d[k][1] else "")
+        rb = to_bytes(*d["dram__bytes_read.sum"]) if "dram__bytes_read.sum" in d else None
+        wb = to_bytes(*d["dram__bytes_write.sum"]) if "dram__bytes_write.sum" in d else None
+        if rb is not None and wb is not None:
+            s["dram_bytes_total"] = rb + wb
+        out.append(s)
+    return out
+
+
+def launch_list(path):
+    rows = [r for r in csv.reader(open(path)) if len(r) > 10]
+    hdr = rows[0]
+    ik, iv, iu = hdr.index("Kernel Name"), hdr.index("Metric Value"), hdr.index("Metric Unit")
+    agg = {}
+    for r in rows[1:]:
+        k = r[ik].split("(")[0][:80]
+        ns = float(r[iv].replace(",", "")) * (1e3 if r[iu] == "usecond" else 1e6 if r[iu] == "msecond" else 1)
+        a = agg.setdefault(k, [0, 0.0])
+        a[0] += 1
+        a[1] += ns
+    tot = sum(v[1] for v in agg.values())
+    return [{"kernel": k, "launches": v[0], "total_ms": v[1] / 1e6, "share": v[1] / tot}
+            for k, v in sorted(agg.items(), key=lambda kv: -kv[1][1])]
+
+
+def main():
+    args = sys.argv[1:]
+    prefix = args.pop(0)
+    launch = None
+    if "--launch" in args:
+        i = args.index("--launch")
+        launch = args[i + 1]
+        del args[i:i + 2]
+    res = {"kernels": []}
+    for rep in args:
+        res["kernels"] += summarize(rep)
+    if launch:
+        res["launch_list"] = launch_list(launch)
+    json.dump(res, open(prefix + ".json", "w"), indent=1)
+    with open(prefix + ".md", "w") as f:
+        for s in res["kernels"]:
+            f.write("### %s (%s)\n\n| metric | value |\n|---|---|\n" % (s["kernel"], s["report"]))
+            for k, v in s.items():
+                if k not in ("kernel", "report"):
+                    f.write("| %s | %s |\n" % (k, v))
+            f.write("\n")
+        if launch:
+            f.write("### launch list (ncu gpu__time_duration, cold-cache, serialised)\n\n")
+            f.write("| kernel | launches | total ms | share |\n|---|---|---|---|\n")
+            for r in res["launch_list"]:
+                f.write("| %s | %d | %.3f | %.3f |\n" % (r["kernel"], r["launches"], r["total_ms"], r["share"]))
+    print("wrote", prefix + ".json", prefix + ".md")
+
+
+if __name__ == "__main__":
+    main()
