@@ -269,6 +269,10 @@ def main():
     gemm_ms = float(np.mean([e[1].elapsed_time(e[2]) for e in ev]))
     split_ms = float(np.mean([e[0].elapsed_time(e[1]) for e in ev]))
     clocks = clk.summary()
+    try:  # effective SM clock inside the last timed GEMM launch (clock64 / globaltimer)
+        kernel_mhz = egemm.debug_last_clock()
+    except Exception:  # pragma: no cover
+        kernel_mhz = None
 
     peaks = _peaks()
     prof = _profile_summary()
@@ -289,6 +293,9 @@ def main():
         "fp32eq_tflops": round(2.0 * m_loc * N * K / (gemm_ms * 1e-3) / 1e12, 1),
         "vs_tensor_peak_over_terms": round((2.0 * m_loc * N * K / (gemm_ms * 1e-3) / 1e12)
                                            / (2250.0 / terms), 4),
+        "kernel_sm_mhz": round(kernel_mhz, 1) if kernel_mhz else None,
+        "frac_of_clock_adjusted_peak": round(achieved / (148 * 8192 * kernel_mhz * 1e-6), 4)
+        if kernel_mhz else None,
     }
     split_bytes = 8.0 * (m_loc * K + K * N)
     split_rl = {"kernel": "split (A rows + B^T)", "bound": "hbm",

@@ -147,6 +147,10 @@ int egemm_set_config(int cg, int bn, int sep, int kc);
 /* Number of SMs of the current device (0 without a device). */
 int egemm_num_sms(void);
 
+/* Debug: effective SM clock (MHz) of CTA 0 over the last tensor-core kernel launch,
+ * from clock64 / %globaltimer.  Synchronous (copies a device symbol). */
+int egemm_debug_last_clock(double* mhz);
+
 #ifdef __cplusplus
 }
 #endif

@@ -162,6 +162,11 @@ const char* egemm_last_error(void) { return g_err; }
 int egemm_version(void) { return 100; }
 int egemm_num_sms(void) { return num_sms(); }
 
+int egemm_debug_last_clock(double* mhz) {
+  if (!mhz) return EGEMM_ERR_INVALID_ARG;
+  return read_clock_probe(mhz) ? EGEMM_ERR_CUDA : EGEMM_OK;
+}
+
 int egemm_set_config(int cg, int bn, int sep, int kc) {
   if (cg == 0 && bn == 0 && sep == 0 && kc == 0) {
     g_override = Override();

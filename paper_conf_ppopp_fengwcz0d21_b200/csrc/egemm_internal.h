@@ -72,5 +72,6 @@ int launch_fill_c(int64_t M, int64_t N, const float* C, int64_t ldc, float* D, i
                   cudaStream_t stream);
 
 void set_last_error(const char* fmt, ...);
+int read_clock_probe(double* mhz);
 
 }  // namespace egemm

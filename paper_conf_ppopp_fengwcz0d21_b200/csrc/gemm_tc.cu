@@ -34,6 +34,14 @@
 
 namespace egemm {
 
+__device__ unsigned long long g_clock_probe[4];
+
+__device__ __forceinline__ unsigned long long globaltimer_ns() {
+  unsigned long long t;
+  asm volatile("mov.u64 %0, %%globaltimer;" : "=l"(t));
+  return t;
+}
+
 constexpr int kBM = 128;       // rows per CTA (TMEM lanes)
 constexpr int kBK = 64;        // k elements per stage (128 B of fp16: one SW128 row)
 constexpr int kThreads = 384;  // 12 warps
@@ -204,6 +212,10 @@ __global__ void __launch_bounds__(kThreads, 1)
   if constexpr (CG == 2) ptx::cluster_sync(); else __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  if (blockIdx.x == 0 && threadIdx.x == 0) {  // SM-clock probe (egemm_debug_last_clock)
+    g_clock_probe[0] = clock64();
+    g_clock_probe[1] = globaltimer_ns();
+  }
 
   const int nch = (p.num_kb + p.kb_per_chunk - 1) / p.kb_per_chunk;
 
@@ -241,7 +253,9 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
   } else if (warp == 1) {
     // ============================ MMA issuer ============================
-    if (leader && lane == 0) {
+    // The whole warp runs the loop (so stage / descriptor arithmetic stays in uniform
+    // registers); one elected lane -- always the same one -- issues MMAs and commits.
+    if (leader) {
       constexpr uint32_t idesc = ptx::idesc_f16_f32(kBM * CG, BN);
       const uint32_t sbase = ptx::smem_u32(stage_base);
       int stage = 0;
@@ -272,24 +286,29 @@ __global__ void __launch_bounds__(kThreads, 1)
               // accumulator this keeps |acc| ~2^-11 smaller while the cross terms are
               // added, so the tensor core's truncating alignment (probe model)
               // loses almost nothing on them; only the 4 hi*hi MMAs see the full |acc|.
+              const uint32_t acc0 = (kb > kb0) ? 1u : 0u;
+              if (ptx::elect_one()) {
 #pragma unroll
-              for (int k = 0; k < kBK / 16; k++) {
-                const uint64_t ko = (uint64_t)(k * 2);  // +32 B per 16-wide k step (>>4)
-                const uint32_t first = (kb > kb0 || k > 0) ? 1u : 0u;
-                ptx::mma_f16<CG>(acc_x, d_ahi + ko, d_blo + ko, idesc, first);
-                ptx::mma_f16<CG>(acc_x, d_alo + ko, d_bhi + ko, idesc, 1u);
-                if (p.terms == 4) ptx::mma_f16<CG>(acc_x, d_alo + ko, d_blo + ko, idesc, 1u);
-              }
+                for (int k = 0; k < kBK / 16; k++) {
+                  const uint64_t ko = (uint64_t)(k * 2);  // +32 B per 16-wide k step (>>4)
+                  const uint32_t first = k > 0 ? 1u : acc0;
+                  ptx::mma_f16<CG>(acc_x, d_ahi + ko, d_blo + ko, idesc, first);
+                  ptx::mma_f16<CG>(acc_x, d_alo + ko, d_bhi + ko, idesc, 1u);
+                  if (p.terms == 4) ptx::mma_f16<CG>(acc_x, d_alo + ko, d_blo + ko, idesc, 1u);
+                }
 #pragma unroll
-              for (int k = 0; k < kBK / 16; k++) {
-                const uint64_t ko = (uint64_t)(k * 2);
-                const uint32_t first = (kb > kb0 || k > 0) ? 1u : 0u;
-                ptx::mma_f16<CG>(acc_hh, d_ahi + ko, d_bhi + ko, idesc, SEP ? first : 1u);
+                for (int k = 0; k < kBK / 16; k++) {
+                  const uint64_t ko = (uint64_t)(k * 2);
+                  const uint32_t first = k > 0 ? 1u : acc0;
+                  ptx::mma_f16<CG>(acc_hh, d_ahi + ko, d_bhi + ko, idesc, SEP ? first : 1u);
+                }
+                ptx::mma_commit<CG>(&empty[stage]);
               }
-              ptx::mma_commit<CG>(&empty[stage]);
+              __syncwarp();
               if (++stage == STAGES) { stage = 0; phase ^= 1u; }
             }
-            ptx::mma_commit<CG>(&acc_full[buf]);
+            if (ptx::elect_one()) ptx::mma_commit<CG>(&acc_full[buf]);
+            __syncwarp();
             chunk_ctr++;
           }
         }
@@ -512,6 +531,18 @@ __global__ void __launch_bounds__(kThreads, 1)
     ptx::tc_fence_after();
     ptx::tmem_dealloc<CG>(tmem_base, TMEM_COLS);
   }
+  if (blockIdx.x == 0 && threadIdx.x == 0) {
+    g_clock_probe[2] = clock64();
+    g_clock_probe[3] = globaltimer_ns();
+  }
+}
+
+// SM cycles / wall ns of CTA 0 over the last launch (debug: effective SM clock).
+int read_clock_probe(double* mhz) {
+  unsigned long long h[4];
+  if (cudaMemcpyFromSymbol(h, g_clock_probe, sizeof(h)) != cudaSuccess) return 3;
+  *mhz = (h[3] > h[1]) ? (double)(h[2] - h[0]) * 1e3 / (double)(h[3] - h[1]) : 0.0;
+  return 0;
 }
 
 // ------------------------------------------------------------------ host side

@@ -36,7 +36,7 @@ class Operand(ctypes.Structure):
 EXPORTS = ["egemm_status_string", "egemm_last_error", "egemm_version", "egemm_split", "egemm_gemm",
            "egemm_gemm_workspace_size", "egemm_knn", "egemm_knn_workspace_size", "egemm_knn_index",
            "egemm_kmeans_step", "egemm_kmeans_workspace_size", "egemm_kmeans_finalize",
-           "egemm_set_config", "egemm_num_sms"]
+           "egemm_set_config", "egemm_num_sms", "egemm_debug_last_clock"]
 
 _lib = None
 
@@ -76,8 +76,17 @@ def load(path: str = LIB_PATH):
     L.egemm_set_config.argtypes = [I, I, I, I]
     L.egemm_set_config.restype = I
     L.egemm_num_sms.restype = I
+    L.egemm_debug_last_clock.argtypes = [ctypes.POINTER(ctypes.c_double)]
+    L.egemm_debug_last_clock.restype = I
     _lib = L
     return L
+
+
+def debug_last_clock() -> float:
+    """Effective SM clock (MHz) of CTA 0 over the last tensor-core kernel (synchronous)."""
+    v = ctypes.c_double(0.0)
+    _check(load().egemm_debug_last_clock(ctypes.byref(v)), "egemm_debug_last_clock")
+    return v.value
 
 
 def _check(status: int, fn: str):

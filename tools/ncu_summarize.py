@@ -58,8 +58,9 @@ def summarize(rep):
         name = d.get("Kernel Name", ("?", ""))[0]
         s = {"kernel": name[:140], "report": os.path.basename(rep)}
         for k in KEYS:
-            if k in d:
-                s[k] = d[k][0] + (" " + d[k][1] if d[k][1] else "")
+            h = k if k in d else next((x for x in d if x.endswith("." + k)), None)
+            if h is not None:
+                s[k] = d[h][0] + (" " + d[h][1] if d[h][1] else "")
         rb = to_bytes(*d["dram__bytes_read.sum"]) if "dram__bytes_read.sum" in d else None
         wb = to_bytes(*d["dram__bytes_write.sum"]) if "dram__bytes_write.sum" in d else None
         if rb is not None and wb is not None:

@@ -44,8 +44,13 @@ def main():
         egemm.set_config(*cfg)
         t = timeit(lambda: egemm.gemm(None, None, a_split=a_split, b_split=b_split, out=D))
         t2 = timeit(lambda: egemm.gemm(A, B, out=D, workspace=ws))
-        print("cfg %-16s gemm(presplit) %.3f ms = %.1f TF (x3 = %.0f TF fp16)   full %.3f ms = %.1f TF"
-              % (cfg, t, flop / t / 1e9, 3 * flop / t / 1e9, t2, flop / t2 / 1e9), flush=True)
+        egemm.gemm(None, None, a_split=a_split, b_split=b_split, out=D)
+        mhz = egemm.debug_last_clock()
+        peak_at_clk = 148 * 8192 * mhz * 1e6 / 1e12
+        print("cfg %-16s gemm(presplit) %.3f ms = %.1f TF (x3 = %.0f TF fp16, SM %.0f MHz -> "
+              "%.0f%% of tensor peak at that clock)   full %.3f ms = %.1f TF"
+              % (cfg, t, flop / t / 1e9, 3 * flop / t / 1e9, mhz,
+                 100 * 3 * flop / t / 1e9 / peak_at_clk, t2, flop / t2 / 1e9), flush=True)
     egemm.set_config(0, 0, 0, 0)
     # cuBLAS context (library, not our path)
     t = timeit(lambda: torch.matmul(A, B))
