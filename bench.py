@@ -198,7 +198,7 @@ def reference_arm(args):
 def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--gpus", type=int, default=1)
-    ap.add_argument("--steps", type=int, default=30)
+    ap.add_argument("--steps", type=int, default=200)  # ~0.5 s timed: clocks settle, sampler sees it
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--n", type=int, default=8192)
@@ -365,7 +365,8 @@ def main():
                        "parallelism": "dp%d rows" % world},
             "gpu_launches": launches_per_step * args.steps,
             "e2e": e2e, "roofline": roofline, "split_roofline": split_rl,
-            "cpu_baseline": cpu, "clocks": clocks,
+            "cpu_baseline": cpu, "clocks": dict(clocks, sm_mhz_in_kernel=round(kernel_mhz, 1)
+                                                if kernel_mhz else None),
             "split_ms_per_step": round(split_ms, 4),
             "paper_context": {"t4_speedup_vs_cublas_fp32": 3.13, "t4_speedup_vs_sdk": 11.18,
                               "note": "paper's numbers on Tesla T4 (P:63, P:2251, P:2325), context only"},

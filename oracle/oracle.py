@@ -58,6 +58,8 @@ def lib():
         L.oracle_kmeans_step.restype = None
         L.oracle_kmeans_finalize.argtypes = [P, P, I64, I64, P]
         L.oracle_kmeans_finalize.restype = None
+        L.oracle_group_sums.argtypes = [P, I64, I64, P, I64, P, P]
+        L.oracle_group_sums.restype = None
         L.oracle_num_threads.argtypes = []
         L.oracle_num_threads.restype = I
         _lib = L
@@ -225,6 +227,17 @@ def kmeans_finalize(sums, counts, C):
     out = _f32(C).copy()
     lib().oracle_kmeans_finalize(_p(sums), _p(counts), out.shape[0], out.shape[1], _p(out))
     return out
+
+
+def group_sums(X, assign, kc: int):
+    """R20-ordered fp64 sums and int64 counts of X's rows grouped by a given assignment."""
+    X = _f32(X)
+    a = np.ascontiguousarray(assign, np.int32)
+    n, d = X.shape
+    sums = np.empty((kc, d), np.float64)
+    counts = np.empty(kc, np.int64)
+    lib().oracle_group_sums(_p(X), n, d, _p(a), kc, _p(sums), _p(counts))
+    return sums, counts
 
 
 def dist_tolerance(Q, X, mma_ulps: float = 4.0):

@@ -85,11 +85,10 @@ def _kmeans_check(oracle_lib, X, C, ga, gsums, gcounts):
     kc, d = C.shape
     cnt = np.bincount(ga, minlength=kc)
     assert np.array_equal(gcounts, cnt)
-    # the GPU adds each group sequentially in ascending point index, like the oracle
-    # (R20): the fp64 sums are bitwise equal to the oracle's for the same assignment
-    ref = np.zeros((kc, d))
-    np.add.at(ref, ga, X.astype(np.float64))  # unbuffered, element order = ascending i
-    assert np.array_equal(gsums, ref)
+    # the GPU sums each group in the fixed order of reading R20, like the oracle: the fp64
+    # sums are bitwise equal to the oracle's for the same assignment
+    ref, rcnt = oracle_lib.group_sums(X, ga, kc)
+    assert np.array_equal(gsums, ref) and np.array_equal(gcounts, rcnt)
     if np.array_equal(ga, oa):
         assert np.array_equal(gsums, osums) and np.array_equal(gcounts, ocounts)
     return int(ne.sum())

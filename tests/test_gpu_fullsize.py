@@ -1,0 +1,101 @@
+"""Parity at BASELINE.json's full sizes, in the launch configuration bench.py times
+(default tuning table), on outputs the oracle can compute one by one (sampled rows /
+queries / points).  Inputs are the bench's seeded recipes."""
+import numpy as np
+import pytest
+import torch
+
+from paper_conf_ppopp_fengwcz0d21_b200 import inputs
+from tests.gpu_util import require_gpu, to_dev, to_host
+
+pytestmark = pytest.mark.gpu
+
+
+def _gemm_sampled(oracle_lib, M, N, K, seed_a, seed_b, n_rows, presplit=False):
+    eg = require_gpu()
+    A, B = inputs.uniform((M, K), seed_a), inputs.uniform((K, N), seed_b)
+    Ad, Bd = to_dev(A), to_dev(B)
+    if presplit:  # the bench's step: split(A), split(B^T), GEMM on the pre-split operands
+        D = eg.gemm(None, None, a_split=eg.split(Ad), b_split=eg.split(Bd, transpose=True))
+    else:
+        D = eg.gemm(Ad, Bd)
+    D = to_host(D)
+    rows = np.sort(inputs.rng(seed_a + 7).choice(M, size=min(n_rows, M), replace=False))
+    As = A[rows]
+    C64 = oracle_lib.gemm64(As, B)
+    e = oracle_lib.normwise_error(D[rows], As, B, C64)
+    en = oracle_lib.normwise_error(oracle_lib.gemm32_naive(As, B), As, B, C64)
+    assert e <= 1e-6 and e <= 2 * en, (e, en)
+    bound = oracle_lib.elem_bound(As, B)
+    assert np.all(np.abs(D[rows].astype(np.float64) - C64) <= bound)
+    return e, en
+
+
+@pytest.mark.parametrize("n", [1024, 4096])
+def test_square_sweep_sampled(oracle_lib, n):
+    """configs[1] square sweep points (full rows sampled)."""
+    _gemm_sampled(oracle_lib, n, n, n, 100 + n.bit_length(), 200 + n.bit_length(), 128)
+
+
+def test_8192_cube_bench_launch(oracle_lib):
+    """configs[1] at 8192^3, exactly the bench step (pre-split operands), 48 sampled rows."""
+    e, en = _gemm_sampled(oracle_lib, 8192, 8192, 8192, 101, 102, 48, presplit=True)
+    print("8192^3 sampled normwise error %.3e (naive fp32 %.3e)" % (e, en))
+
+
+def test_16384_cube_sampled(oracle_lib):
+    _gemm_sampled(oracle_lib, 16384, 16384, 16384, 115, 215, 16)
+
+
+def test_tall_skinny_full(oracle_lib):
+    """configs[2]: M=65536 N=256 K=1024, all rows against the fp64 oracle."""
+    _gemm_sampled(oracle_lib, 65536, 256, 1024, 200, 201, 65536)
+
+
+def test_knn_full_size_sampled_queries(oracle_lib):
+    """configs[3]: 1M references x 64K queries, d=128, k=16 (the bench's index path);
+    48 sampled queries checked against the exact fp64 kNN under the gap rule (R18)."""
+    eg = require_gpu()
+    nx, nq, d, k = 1 << 20, 1 << 16, 128, 16
+    X, Q = inputs.uniform((nx, d), 300), inputs.uniform((nq, d), 301)
+    Xd, Qd = to_dev(X), to_dev(Q)
+    idx, dist = eg.knn(Xd, Qd, k, index=eg.knn_index(Xd))
+    idx, dist = to_host(idx), to_host(dist)
+    qs = np.sort(inputs.rng(302).choice(nq, size=48, replace=False))
+    oidx, odist = oracle_lib.knn(X, Q[qs], k + 1)
+    exempt = 0
+    for t, i in enumerate(qs):
+        cand = np.unique(np.concatenate([oidx[t], idx[i]]))
+        tau = oracle_lib.dist_tolerance(Q[i:i + 1], X[cand])[0]
+        tau_of = dict(zip(cand.tolist(), tau.tolist()))
+        gap = odist[t, k] - odist[t, k - 1]
+        if gap > tau_of[int(oidx[t, k - 1])] + tau_of[int(oidx[t, k])]:
+            assert set(idx[i].tolist()) == set(oidx[t, :k].tolist()), i
+        else:
+            exempt += 1
+        dd = oracle_lib.sqdist(X[idx[i]], Q[i:i + 1])[0]
+        assert np.all(np.abs(dist[i] - dd) <= np.array([tau_of[int(j)] for j in idx[i]]) + 1e-6)
+    assert exempt <= 2
+
+
+def test_kmeans_full_size_step_sampled(oracle_lib):
+    """configs[4]: 4M points, d=64, 1024 centroids (Forgy init): one step; 32768 sampled
+    points checked against the fp64 argmin under the gap rule; the fp64 sums / counts are
+    bitwise equal to the oracle's R20-ordered sums of the GPU's assignment."""
+    eg = require_gpu()
+    n, d, kc = 1 << 22, 64, 1024
+    X, _, _ = inputs.mixture(n, d, kc, 400)
+    C = X[:kc].copy()
+    Xd = to_dev(X)
+    a, sums, counts, inertia = eg.kmeans_step(Xd, to_dev(C), x_split=eg.split(Xd))
+    a, sums, counts = to_host(a), to_host(sums), to_host(counts)
+    ps = np.sort(inputs.rng(401).choice(n, size=32768, replace=False))
+    oa, _, _, _, _ = oracle_lib.kmeans_step(X[ps], C)
+    D = oracle_lib.sqdist(C, X[ps])
+    tau = oracle_lib.dist_tolerance(X[ps], C)
+    part = np.partition(D, 1, axis=1)
+    strict = (part[:, 1] - part[:, 0]) > 2 * tau.max(axis=1)
+    assert np.array_equal(a[ps][strict], oa[strict])
+    assert (~strict).sum() <= 0.01 * len(ps)
+    ref, rcnt = oracle_lib.group_sums(X, a, kc)
+    assert np.array_equal(counts, rcnt) and np.array_equal(sums, ref)

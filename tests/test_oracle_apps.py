@@ -89,6 +89,13 @@ def test_kmeans_sums_fixed_order_r20(oracle_lib):
             assert abs(Fraction(sums[j, t]) - exact) <= Fraction(len(mem) * 2.0 ** -52 * mag)
 
 
+def test_group_sums_equals_step_sums(oracle_lib):
+    X, _, cent = inputs.mixture(5000, 6, 3, 10, sigma=0.3)
+    a, sums, counts, _, _ = oracle_lib.kmeans_step(X, cent)
+    s2, c2 = oracle_lib.group_sums(X, a, 3)
+    assert np.array_equal(s2, sums) and np.array_equal(c2, counts)
+
+
 def test_kmeans_ties_lowest_index(oracle_lib):
     X = np.array([[0.0, 0.0]], np.float32)
     C = np.array([[1.0, 0.0], [0.0, 1.0], [-1.0, 0.0]], np.float32)
