@@ -150,12 +150,16 @@ def run_oracle_sample(n: int, target_s: float, seed_a=101, seed_b=102):
     import oracle
     from paper_conf_ppopp_fengwcz0d21_b200 import inputs
     B = inputs.uniform((n, n), seed_b)
-    rows = 4
-    A = inputs.uniform((rows, n), seed_a)
-    t0 = time.perf_counter()
-    oracle.gemm_emu64(A, B, 3)
-    t_small = time.perf_counter() - t0
-    rows = int(max(4, min(n, rows * target_s / max(t_small, 1e-3))))
+    # calibrate: the call has a fixed cost (it round-splits all of B) plus a per-row cost
+    ts = {}
+    for r in (4, 20):
+        A = inputs.uniform((r, n), seed_a)
+        t0 = time.perf_counter()
+        oracle.gemm_emu64(A, B, 3)
+        ts[r] = time.perf_counter() - t0
+    per_row = max((ts[20] - ts[4]) / 16, 1e-6)
+    fixed = max(ts[4] - 4 * per_row, 0.0)
+    rows = int(max(4, min(n, (target_s - fixed) / per_row)))
     A = inputs.uniform((rows, n), seed_a)
     t0 = time.perf_counter()
     oracle.gemm_emu64(A, B, 3)

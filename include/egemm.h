@@ -144,6 +144,15 @@ int egemm_kmeans_finalize(const double* sums, const int64_t* counts, int64_t kc,
  * combination the library was not built with. */
 int egemm_set_config(int cg, int bn, int sep, int kc);
 
+/* The measured configuration table (replaces the paper's analytic model,
+ * Sec. 6): path of the loaded tune_table.json ("" = built-in defaults) and,
+ * through *entries (nullable), its number of entries.  Host-only. */
+const char* egemm_tune_table(int* entries);
+/* The configuration the library would use for op (0 gemm, 1 knn, 2 kmeans) at M, N, K
+ * (after table, egemm_set_config and EGEMM_* overrides).  Host-only. */
+int egemm_query_config(int op, int64_t M, int64_t N, int64_t K, int* cg, int* bn, int* sep,
+                       int* kc);
+
 /* Number of SMs of the current device (0 without a device). */
 int egemm_num_sms(void);
 

@@ -46,6 +46,11 @@ static int env_int(const char* name, int dflt) {
   return (v && *v) ? atoi(v) : dflt;
 }
 
+static bool valid_config(int cg, int bn, int sep) {
+  return (cg == 2 && bn == 256 && sep == 0) || (cg == 1 && bn == 128) ||
+         (cg == 2 && bn == 128 && sep == 1);
+}
+
 static TcConfig choose_config(int epi_kind, int64_t M, int64_t N, int64_t K, int terms) {
   TcConfig c = {};
   c.terms = terms;
@@ -58,6 +63,15 @@ static TcConfig choose_config(int epi_kind, int64_t M, int64_t N, int64_t K, int
   // accurate single-accumulator setting (tools/error_sweep.py)
   c.kc = 64;
   if (epi_kind == EPI_STORE && M <= 128) { c.cg = 1; c.bn = 128; c.sep = 1; }
+  {  // the measured table (tools/tune_sweep.py -> tune_table.json) overrides the defaults
+    int cg, bn, sep, kc;
+    if (tune_lookup(epi_kind, M, N, K, &cg, &bn, &sep, &kc) && valid_config(cg, bn, sep)) {
+      c.cg = cg;
+      c.bn = bn;
+      c.sep = sep;
+      if (kc > 0) c.kc = kc;
+    }
+  }
   if (epi_kind != EPI_STORE) c.kc = (int)(((K + 63) / 64) * 64);
   // thread-local API override, then environment (experiments)
   if (g_override.cg) { c.cg = g_override.cg; c.bn = g_override.bn; c.sep = g_override.sep; }
@@ -162,6 +176,22 @@ const char* egemm_last_error(void) { return g_err; }
 int egemm_version(void) { return 100; }
 int egemm_num_sms(void) { return num_sms(); }
 
+const char* egemm_tune_table(int* entries) {
+  if (entries) *entries = tune_table_size();
+  return tune_table_path();
+}
+
+int egemm_query_config(int op, int64_t M, int64_t N, int64_t K, int* cg, int* bn, int* sep,
+                       int* kc) {
+  if (op < 0 || op > 2 || !cg || !bn || !sep || !kc) return EGEMM_ERR_INVALID_ARG;
+  TcConfig c = choose_config(op, M, N, K, 3);
+  *cg = c.cg;
+  *bn = c.bn;
+  *sep = c.sep;
+  *kc = c.kc;
+  return EGEMM_OK;
+}
+
 int egemm_debug_last_clock(double* mhz) {
   if (!mhz) return EGEMM_ERR_INVALID_ARG;
   return read_clock_probe(mhz) ? EGEMM_ERR_CUDA : EGEMM_OK;
@@ -172,9 +202,7 @@ int egemm_set_config(int cg, int bn, int sep, int kc) {
     g_override = Override();
     return EGEMM_OK;
   }
-  bool ok = (cg == 2 && bn == 256 && sep == 0) || (cg == 1 && bn == 128) ||
-            (cg == 2 && bn == 128 && sep == 1);
-  if (!ok || kc < 0 || (kc % 64) != 0) {
+  if (!valid_config(cg, bn, sep) || kc < 0 || (kc % 64) != 0) {
     set_last_error("unsupported config cg=%d bn=%d sep=%d kc=%d", cg, bn, sep, kc);
     return EGEMM_ERR_UNSUPPORTED;
   }

@@ -74,4 +74,10 @@ int launch_fill_c(int64_t M, int64_t N, const float* C, int64_t ldc, float* D, i
 void set_last_error(const char* fmt, ...);
 int read_clock_probe(double* mhz);
 
+// tune.cu: the measured configuration table
+bool tune_lookup(int op, long long M, long long N, long long K, int* cg, int* bn, int* sep,
+                 int* kc);
+const char* tune_table_path();
+int tune_table_size();
+
 }  // namespace egemm

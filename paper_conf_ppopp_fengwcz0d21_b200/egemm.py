@@ -36,7 +36,8 @@ class Operand(ctypes.Structure):
 EXPORTS = ["egemm_status_string", "egemm_last_error", "egemm_version", "egemm_split", "egemm_gemm",
            "egemm_gemm_workspace_size", "egemm_knn", "egemm_knn_workspace_size", "egemm_knn_index",
            "egemm_kmeans_step", "egemm_kmeans_workspace_size", "egemm_kmeans_finalize",
-           "egemm_set_config", "egemm_num_sms", "egemm_debug_last_clock"]
+           "egemm_set_config", "egemm_num_sms", "egemm_debug_last_clock", "egemm_tune_table",
+           "egemm_query_config"]
 
 _lib = None
 
@@ -78,8 +79,28 @@ def load(path: str = LIB_PATH):
     L.egemm_num_sms.restype = I
     L.egemm_debug_last_clock.argtypes = [ctypes.POINTER(ctypes.c_double)]
     L.egemm_debug_last_clock.restype = I
+    L.egemm_tune_table.argtypes = [ctypes.POINTER(ctypes.c_int)]
+    L.egemm_tune_table.restype = ctypes.c_char_p
+    IP = ctypes.POINTER(ctypes.c_int)
+    L.egemm_query_config.argtypes = [I, I64, I64, I64, IP, IP, IP, IP]
+    L.egemm_query_config.restype = I
     _lib = L
     return L
+
+
+def tune_table():
+    """(path of the loaded tune_table.json or '', number of entries)."""
+    n = ctypes.c_int(0)
+    p = load().egemm_tune_table(ctypes.byref(n))
+    return p.decode(), n.value
+
+
+def query_config(op: str, M: int, N: int, K: int):
+    """The (cg, bn, sep, kc) the library picks for op in {'gemm','knn','kmeans'}."""
+    v = [ctypes.c_int(0) for _ in range(4)]
+    _check(load().egemm_query_config({"gemm": 0, "knn": 1, "kmeans": 2}[op], M, N, K,
+                                     *[ctypes.byref(x) for x in v]), "egemm_query_config")
+    return tuple(x.value for x in v)
 
 
 def debug_last_clock() -> float:

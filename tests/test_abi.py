@@ -72,6 +72,28 @@ def test_workspace_queries(lib):
     assert egemm.kmeans_workspace_size(1000, 64, 10) > 0
 
 
+def test_tune_table_lookup(tmp_path):
+    """The measured table (a-8) is parsed and consulted (first matching bucket wins);
+    host-only, so it runs without a GPU (fresh process: the table is loaded once)."""
+    import json
+    import subprocess
+    import sys
+    t = {"entries": [
+        {"op": "gemm", "m_max": 128, "n_max": 1 << 40, "k_max": 1 << 40, "cg": 1, "bn": 128,
+         "sep": 1, "kc": 128, "note": {"nested": [1, 2]}},
+        {"op": "gemm", "m_max": 1 << 40, "n_max": 1 << 40, "k_max": 1 << 40, "cg": 2, "bn": 256,
+         "sep": 0, "kc": 128}]}
+    p = tmp_path / "t.json"
+    p.write_text(json.dumps(t))
+    code = ("import sys; sys.path.insert(0, %r); from paper_conf_ppopp_fengwcz0d21_b200 import egemm;"
+            "print(egemm.tune_table()[1], egemm.query_config('gemm', 100, 5000, 64),"
+            " egemm.query_config('gemm', 9000, 9000, 9000), egemm.query_config('knn', 10, 10, 100))"
+            % ROOT)
+    out = subprocess.check_output([sys.executable, "-c", code],
+                                  env=dict(os.environ, EGEMM_TUNE_TABLE=str(p))).decode().strip()
+    assert out == "2 (1, 128, 1, 128) (2, 256, 0, 128) (2, 256, 0, 128)", out
+
+
 def test_no_gpu_means_loud_failure(lib):
     """Without a device the compute entry points fail loudly (no CPU fallback)."""
     import torch
