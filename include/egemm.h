@@ -97,6 +97,20 @@ int egemm_gemm(int64_t M, int64_t N, int64_t K, egemm_operand_t A, egemm_operand
 size_t egemm_gemm_workspace_size(int64_t M, int64_t N, int64_t K, int a_presplit, int b_presplit);
 
 /*
+ * The same GEMM on HOST buffers (end-to-end use): D_host[M x N] = A_host[M x K] * B_host[K x N]
+ * (row-major, strides lda / ldb / ldd in elements; host memory should be pinned for the
+ * copies to be asynchronous).  B is copied and split once; row chunks of A are then copied
+ * in, split, multiplied and copied out double-buffered, so both PCIe directions overlap the
+ * tensor-core work.  Uses two internal copy streams created once per device (the only
+ * resources the library creates).  Asynchronous w.r.t. the host like the other calls:
+ * D_host is complete when `stream` has completed.  K must be > 0.
+ */
+int egemm_gemm_host(int64_t M, int64_t N, int64_t K, const float* A_host, int64_t lda,
+                    const float* B_host, int64_t ldb, float* D_host, int64_t ldd, int terms,
+                    void* workspace, size_t workspace_bytes, void* stream);
+size_t egemm_gemm_host_workspace_size(int64_t M, int64_t N, int64_t K);
+
+/*
  * kNN with the emulated GEMM (the GEMM-based kNN of Garcia et al. [9] with its fp32 GEMM
  * replaced): for each query row q_i of Q[nq x d]
  * the k rows x_j of X[nx x d] with the smallest squared distance

@@ -6,6 +6,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <mutex>
 #include "../../include/egemm.h"
 #include "egemm_internal.h"
 
@@ -296,6 +297,158 @@ int egemm_gemm(int64_t M, int64_t N, int64_t K, egemm_operand_t A, egemm_operand
   epi.ldc = ldc;
   r = launch_tc(M, N, K, ops, cfg, epi, s);
   return r == 0 ? EGEMM_OK : (r == 2 ? EGEMM_ERR_UNSUPPORTED : EGEMM_ERR_CUDA);
+}
+
+// ------------------------------------------------------------------ host-buffer GEMM
+// D_host = A_host * B_host with the host<->device traffic pipelined against the compute:
+// B is copied and split once, then row chunks of A flow H2D (copy stream) -> split ->
+// tcgen05 GEMM (caller stream) -> D2H (second copy stream), double-buffered, so the two
+// PCIe directions and the GPU work overlap.  Streams/events are created once per device.
+static int64_t host_chunk_rows(int64_t M) {
+  int64_t c = ((M / 8 + 255) / 256) * 256;
+  if (c < 256) c = 256;
+  if (c > 4096) c = 4096;
+  return c > M ? M : c;
+}
+
+struct HostPipe {
+  bool init = false;
+  cudaStream_t s_in = nullptr, s_out = nullptr;
+  cudaEvent_t ev_start, ev_b, ev_in[2], ev_split[2], ev_comp[2], ev_out[2];
+};
+static HostPipe g_pipe[64];
+static std::mutex g_pipe_mu;
+
+static HostPipe* host_pipe() {
+  int dev = 0;
+  if (cudaGetDevice(&dev) != cudaSuccess || dev < 0 || dev >= 64) return nullptr;
+  std::lock_guard<std::mutex> lk(g_pipe_mu);
+  HostPipe& p = g_pipe[dev];
+  if (!p.init) {
+    if (cudaStreamCreateWithFlags(&p.s_in, cudaStreamNonBlocking) != cudaSuccess ||
+        cudaStreamCreateWithFlags(&p.s_out, cudaStreamNonBlocking) != cudaSuccess)
+      return nullptr;
+    cudaEvent_t* evs[] = {&p.ev_start, &p.ev_b, &p.ev_in[0], &p.ev_in[1], &p.ev_split[0],
+                          &p.ev_split[1], &p.ev_comp[0], &p.ev_comp[1], &p.ev_out[0], &p.ev_out[1]};
+    for (cudaEvent_t* e : evs)
+      if (cudaEventCreateWithFlags(e, cudaEventDisableTiming) != cudaSuccess) return nullptr;
+    p.init = true;
+  }
+  return &p;
+}
+
+size_t egemm_gemm_host_workspace_size(int64_t M, int64_t N, int64_t K) {
+  if (M <= 0 || N <= 0 || K <= 0) return 0;
+  const int64_t ldk = ldk_of(K), mc = host_chunk_rows(M);
+  Carver cv{nullptr};
+  cv.take<float>((size_t)(K * N));
+  cv.take<uint16_t>((size_t)(N * ldk));
+  cv.take<uint16_t>((size_t)(N * ldk));
+  for (int b = 0; b < 2; b++) {
+    cv.take<float>((size_t)(mc * K));
+    cv.take<uint16_t>((size_t)(mc * ldk));
+    cv.take<uint16_t>((size_t)(mc * ldk));
+    cv.take<float>((size_t)(mc * N));
+  }
+  return cv.off;
+}
+
+int egemm_gemm_host(int64_t M, int64_t N, int64_t K, const float* A_host, int64_t lda,
+                    const float* B_host, int64_t ldb, float* D_host, int64_t ldd, int terms,
+                    void* workspace, size_t workspace_bytes, void* stream) {
+  cudaStream_t s = (cudaStream_t)stream;
+  if (M < 0 || N < 0 || K < 0 || lda < K || ldb < N || ldd < N) {
+    set_last_error("negative size or ld too small");
+    return EGEMM_ERR_INVALID_ARG;
+  }
+  if (terms == 0) terms = 3;
+  if (terms != 3 && terms != 4) {
+    set_last_error("terms must be 0, 3 or 4");
+    return EGEMM_ERR_INVALID_ARG;
+  }
+  if (M == 0 || N == 0) return EGEMM_OK;
+  if (!A_host || !B_host || !D_host) {
+    set_last_error("NULL host pointer");
+    return EGEMM_ERR_INVALID_ARG;
+  }
+  if (K == 0) {
+    set_last_error("K == 0: use egemm_gemm (nothing to stream)");
+    return EGEMM_ERR_UNSUPPORTED;
+  }
+  if (!device_ok()) {
+    set_last_error("no sm_100 device");
+    return EGEMM_ERR_CUDA;
+  }
+  const size_t need = egemm_gemm_host_workspace_size(M, N, K);
+  if (!workspace || workspace_bytes < need) {
+    set_last_error("workspace %zu < %zu", workspace_bytes, need);
+    return EGEMM_ERR_WORKSPACE;
+  }
+  HostPipe* hp = host_pipe();
+  if (!hp) {
+    set_last_error("stream/event creation failed");
+    return EGEMM_ERR_CUDA;
+  }
+  const int64_t ldk = ldk_of(K), mc = host_chunk_rows(M);
+  Carver cv{reinterpret_cast<char*>(workspace)};
+  float* Bd = cv.take<float>((size_t)(K * N));
+  uint16_t* bhi = cv.take<uint16_t>((size_t)(N * ldk));
+  uint16_t* blo = cv.take<uint16_t>((size_t)(N * ldk));
+  float* Ad[2];
+  uint16_t *ahi[2], *alo[2];
+  float* Dd[2];
+  for (int b = 0; b < 2; b++) {
+    Ad[b] = cv.take<float>((size_t)(mc * K));
+    ahi[b] = cv.take<uint16_t>((size_t)(mc * ldk));
+    alo[b] = cv.take<uint16_t>((size_t)(mc * ldk));
+    Dd[b] = cv.take<float>((size_t)(mc * N));
+  }
+  TcConfig cfg = choose_config(EPI_STORE, mc, N, K, terms);
+  bool ok = true;
+  auto chk = [&](cudaError_t e) { ok = ok && (e == cudaSuccess); };
+  chk(cudaEventRecord(hp->ev_start, s));
+  chk(cudaStreamWaitEvent(hp->s_in, hp->ev_start, 0));
+  chk(cudaStreamWaitEvent(hp->s_out, hp->ev_start, 0));
+  chk(cudaMemcpy2DAsync(Bd, N * sizeof(float), B_host, ldb * sizeof(float), N * sizeof(float), K,
+                        cudaMemcpyHostToDevice, hp->s_in));
+  chk(cudaEventRecord(hp->ev_b, hp->s_in));
+  chk(cudaStreamWaitEvent(s, hp->ev_b, 0));
+  if (!ok || launch_split(Bd, K, N, N, bhi, blo, ldk, 1, nullptr, s)) {
+    set_last_error("B staging failed");
+    return EGEMM_ERR_CUDA;
+  }
+  const int64_t nchunks = (M + mc - 1) / mc;
+  for (int64_t c = 0; c < nchunks && ok; c++) {
+    const int b = (int)(c & 1);
+    const int64_t r0 = c * mc, rows = (M - r0 < mc) ? M - r0 : mc;
+    if (c >= 2) chk(cudaStreamWaitEvent(hp->s_in, hp->ev_split[b], 0));  // Ad[b] free
+    chk(cudaMemcpy2DAsync(Ad[b], K * sizeof(float), A_host + r0 * lda, lda * sizeof(float),
+                          K * sizeof(float), rows, cudaMemcpyHostToDevice, hp->s_in));
+    chk(cudaEventRecord(hp->ev_in[b], hp->s_in));
+    chk(cudaStreamWaitEvent(s, hp->ev_in[b], 0));
+    if (launch_split(Ad[b], rows, K, K, ahi[b], alo[b], ldk, 0, nullptr, s)) ok = false;
+    chk(cudaEventRecord(hp->ev_split[b], s));
+    if (c >= 2) chk(cudaStreamWaitEvent(s, hp->ev_out[b], 0));  // Dd[b] drained
+    TcOperands ops = {ahi[b], alo[b], ldk, bhi, blo, ldk};
+    TcEpilogue epi = {};
+    epi.kind = EPI_STORE;
+    epi.D = Dd[b];
+    epi.ldd = N;
+    if (ok && launch_tc(rows, N, K, ops, cfg, epi, s)) ok = false;
+    chk(cudaEventRecord(hp->ev_comp[b], s));
+    chk(cudaStreamWaitEvent(hp->s_out, hp->ev_comp[b], 0));
+    chk(cudaMemcpy2DAsync(D_host + r0 * ldd, ldd * sizeof(float), Dd[b], N * sizeof(float),
+                          N * sizeof(float), rows, cudaMemcpyDeviceToHost, hp->s_out));
+    chk(cudaEventRecord(hp->ev_out[b], hp->s_out));
+  }
+  // the caller's stream completes only after the last D2H
+  chk(cudaStreamWaitEvent(s, hp->ev_out[(nchunks - 1) & 1], 0));
+  if (nchunks >= 2) chk(cudaStreamWaitEvent(s, hp->ev_out[(nchunks - 2) & 1], 0));
+  if (!ok) {
+    set_last_error("host pipeline: %s", cudaGetErrorString(cudaGetLastError()));
+    return EGEMM_ERR_CUDA;
+  }
+  return EGEMM_OK;
 }
 
 static int knn_slices(int64_t nq, int64_t nx, int cg, int bn) {

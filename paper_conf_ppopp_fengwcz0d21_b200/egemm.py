@@ -37,7 +37,7 @@ EXPORTS = ["egemm_status_string", "egemm_last_error", "egemm_version", "egemm_sp
            "egemm_gemm_workspace_size", "egemm_knn", "egemm_knn_workspace_size", "egemm_knn_index",
            "egemm_kmeans_step", "egemm_kmeans_workspace_size", "egemm_kmeans_finalize",
            "egemm_set_config", "egemm_num_sms", "egemm_debug_last_clock", "egemm_tune_table",
-           "egemm_query_config"]
+           "egemm_query_config", "egemm_gemm_host", "egemm_gemm_host_workspace_size"]
 
 _lib = None
 
@@ -79,6 +79,10 @@ def load(path: str = LIB_PATH):
     L.egemm_num_sms.restype = I
     L.egemm_debug_last_clock.argtypes = [ctypes.POINTER(ctypes.c_double)]
     L.egemm_debug_last_clock.restype = I
+    L.egemm_gemm_host.argtypes = [I64, I64, I64, P, I64, P, I64, P, I64, I, P, SZ, P]
+    L.egemm_gemm_host.restype = I
+    L.egemm_gemm_host_workspace_size.argtypes = [I64, I64, I64]
+    L.egemm_gemm_host_workspace_size.restype = SZ
     L.egemm_tune_table.argtypes = [ctypes.POINTER(ctypes.c_int)]
     L.egemm_tune_table.restype = ctypes.c_char_p
     IP = ctypes.POINTER(ctypes.c_int)
@@ -199,6 +203,28 @@ def gemm(A: torch.Tensor | None, B: torch.Tensor | None, C: torch.Tensor | None 
     ws, wsn = _workspace(need, dev, workspace)
     _check(L.egemm_gemm(M, N, K, opA, opB, _ptr(C), C.stride(0) if C is not None else 0, _ptr(D),
                         D.stride(0), int(terms), _ptr(ws), wsn, _stream(stream)), "egemm_gemm")
+    return D
+
+
+def gemm_host_workspace_size(M, N, K) -> int:
+    return int(load().egemm_gemm_host_workspace_size(M, N, K))
+
+
+def gemm_host(A: torch.Tensor, B: torch.Tensor, out: torch.Tensor | None = None, terms: int = 0,
+              workspace: torch.Tensor | None = None, device=None, stream=None):
+    """D = A @ B on HOST (preferably pinned) fp32 tensors through egemm_gemm_host: the copies
+    are pipelined against the GPU work inside the library.  Asynchronous: synchronise the
+    stream before reading ``out``."""
+    L = load()
+    assert not A.is_cuda and not B.is_cuda and A.dtype == torch.float32 and B.dtype == torch.float32
+    M, K = A.shape
+    N = B.shape[1]
+    D = out if out is not None else torch.empty((M, N), dtype=torch.float32, pin_memory=True)
+    dev = device or torch.device("cuda", torch.cuda.current_device())
+    ws, wsn = _workspace(gemm_host_workspace_size(M, N, K), dev, workspace)
+    _check(L.egemm_gemm_host(M, N, K, _ptr(A), A.stride(0), _ptr(B), B.stride(0), _ptr(D),
+                             D.stride(0), int(terms), _ptr(ws), wsn, _stream(stream)),
+           "egemm_gemm_host")
     return D
 
 
