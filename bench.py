@@ -384,6 +384,31 @@ def _apps(world, rank, dev, args):
     from paper_conf_ppopp_fengwcz0d21_b200 import egemm, inputs
     from paper_conf_ppopp_fengwcz0d21_b200 import distributed as edist
     out = {}
+    try:  # configs[2]: tall-skinny M=65536 N=256 K=1024 (rows sharded), fp32 in -> fp32 out
+        M2, N2, K2 = 65536, 256, 1024
+        r0, r1 = edist.shard_bounds(M2, world, rank, align=256)
+        A2 = torch.from_numpy(inputs.uniform((M2, K2), 200)[r0:r1]).to(dev)
+        B2 = torch.from_numpy(inputs.uniform((K2, N2), 201)).to(dev)
+        ws2 = torch.empty(egemm.gemm_workspace_size(r1 - r0, N2, K2), dtype=torch.uint8, device=dev)
+        D2 = torch.empty((r1 - r0, N2), device=dev)
+        for _ in range(3):
+            egemm.gemm(A2, B2, out=D2, workspace=ws2)
+        _barrier(world)
+        s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        reps = 20
+        s.record()
+        for _ in range(reps):
+            egemm.gemm(A2, B2, out=D2, workspace=ws2)
+        e.record()
+        _barrier(world)
+        ms = _allmax(s.elapsed_time(e), world) / reps
+        out["tall_skinny"] = {"metric": "EGEMM FP32-equiv TFLOP/s, M=65536 N=256 K=1024 (split included)",
+                              "value": round(2.0 * M2 * N2 * K2 / (ms * 1e-3) / 1e12, 1),
+                              "unit": "TFLOP/s", "ms": round(ms, 4),
+                              "config": list(egemm.query_config("gemm", r1 - r0, N2, K2))}
+        del A2, B2, ws2, D2
+    except Exception as ex:  # pragma: no cover
+        out["tall_skinny"] = {"error": str(ex)[:300]}
     try:
         nx, nq, d, k = 1 << 20, 1 << 16, 128, 16
         q0, q1 = edist.shard_bounds(nq, world, rank)
@@ -411,6 +436,7 @@ def _apps(world, rank, dev, args):
                       "value": round(nq / (ms * 1e-3), 1), "unit": "queries/s",
                       "ms_per_batch": round(ms, 3), "index_build_ms": round(t_ib[0].elapsed_time(t_ib[1]), 3),
                       "fp32eq_tflops": round(2.0 * nx * nq * d / (ms * 1e-3) / 1e12, 1),
+                      "kernel_sm_mhz": round(egemm.debug_last_clock(), 1),
                       "sharding": "queries over %d ranks, X replicated" % world}
         del X, Q, index, ws
     except Exception as ex:  # pragma: no cover
@@ -440,6 +466,7 @@ def _apps(world, rank, dev, args):
         out["kmeans"] = {"metric": "kMeans ms/iteration (4M points, d=64, 1024 centroids)",
                          "value": round(ms, 4), "unit": "ms/iter", "iterations": iters,
                          "fp32eq_tflops": round(2.0 * n * kc * d / (ms * 1e-3) / 1e12, 1),
+                         "kernel_sm_mhz": round(egemm.debug_last_clock(), 1),
                          "sharding": "points over %d ranks, NCCL all_reduce of sums/counts" % world}
     except Exception as ex:  # pragma: no cover
         out["kmeans"] = {"error": str(ex)[:300]}

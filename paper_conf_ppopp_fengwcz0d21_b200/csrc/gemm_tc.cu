@@ -44,7 +44,6 @@ __device__ __forceinline__ unsigned long long globaltimer_ns() {
 
 constexpr int kBM = 128;       // rows per CTA (TMEM lanes)
 constexpr int kBK = 64;        // k elements per stage (128 B of fp16: one SW128 row)
-constexpr int kThreads = 384;  // 12 warps
 constexpr int kEpiWarp0 = 4;
 constexpr int kKnnMax = 16;
 
@@ -76,7 +75,14 @@ struct Geo {
   static constexpr int A_BYTES = kBM * kBK * 2;        // one of A_hi / A_lo
   static constexpr int B_BYTES = BNC * kBK * 2;        // one of B_hi / B_lo
   static constexpr int STAGE_BYTES = 2 * A_BYTES + 2 * B_BYTES;
-  static constexpr int COLS = BN / 2;                  // columns per epilogue warp
+};
+
+// epilogue warps: NEPI in {8, 16}; NEPI/4 warps share each TMEM lane quarter and split
+// its BN columns.  Kernel block = 4 control warps + NEPI epilogue warps.
+template <int NEPI>
+struct EpiGeo {
+  static constexpr int GPQ = NEPI / 4;            // column groups per lane quarter
+  static constexpr int THREADS = 128 + 32 * NEPI;
 };
 
 struct UnitInfo {
@@ -157,14 +163,15 @@ __device__ __forceinline__ void named_bar_sync(int id, int nthreads) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }
 
-template <int CG, int BN, bool SEP, int EPI, int STAGES>
-__global__ void __launch_bounds__(kThreads, 1)
+template <int CG, int BN, bool SEP, int EPI, int STAGES, int NEPI>
+__global__ void __launch_bounds__(EpiGeo<NEPI>::THREADS, 1)
     egemm_tc_kernel(const __grid_constant__ CUtensorMap tm_ahi,
                     const __grid_constant__ CUtensorMap tm_alo,
                     const __grid_constant__ CUtensorMap tm_bhi,
                     const __grid_constant__ CUtensorMap tm_blo, const KParams p) {
   using G = Geo<CG, BN>;
-  constexpr int COLS = G::COLS;
+  constexpr int GPQ = EpiGeo<NEPI>::GPQ;
+  constexpr int COLS = BN / GPQ;  // columns per epilogue warp
   constexpr int NACC = SEP ? 4 : 2;
   constexpr uint32_t TMEM_COLS = (NACC * BN <= 32) ? 32 : (NACC * BN <= 64) ? 64
                                  : (NACC * BN <= 128) ? 128 : (NACC * BN <= 256) ? 256 : 512;
@@ -203,7 +210,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     }
     for (int b = 0; b < 2; b++) {
       ptx::mbar_init(&acc_full[b], 1);
-      ptx::mbar_init(&acc_empty[b], 8 * CG);  // one arrive per epilogue warp of the pair
+      ptx::mbar_init(&acc_empty[b], NEPI * CG);  // one arrive per epilogue warp of the pair
     }
     ptx::fence_mbar_init();
   }
@@ -318,7 +325,7 @@ __global__ void __launch_bounds__(kThreads, 1)
     // ============================ epilogue ============================
     const int ew = warp - kEpiWarp0;
     const int q = warp & 3;         // TMEM lane quarter this warp may access
-    const int cgp = ew >> 2;        // column half
+    const int cgp = ew >> 2;        // column group (0 .. GPQ-1) within the lane quarter
     const uint32_t lane_off = (uint32_t)(q * 32) << 16;
     uint32_t chunk_ctr = 0;
     const int row_in_cta = q * 32 + lane;
@@ -412,11 +419,14 @@ __global__ void __launch_bounds__(kThreads, 1)
           // TMEM -> registers software-pipelined: the load of group c+1 is in flight while
           // group c is processed; the accumulator buffer is handed back to the MMA warp as
           // soon as the last group has landed in registers.
-          float vbuf[2][32];
-          ptx::tmem_ld32(acc_hh, vbuf[0]);
+          // (with 16 epilogue warps the extra warps hide the latency instead of registers)
+          constexpr bool PIPE = (NEPI == 8);
+          float vbuf[PIPE ? 2 : 1][32];
+          if (PIPE) ptx::tmem_ld32(acc_hh, vbuf[0]);
 #pragma unroll
           for (int c = 0; c < COLS / 32; c++) {
-            float* v = vbuf[c & 1];
+            float* v = vbuf[PIPE ? (c & 1) : 0];
+            if (!PIPE) ptx::tmem_ld32(acc_hh + c * 32, v);
             ptx::tmem_wait_ld();
             if constexpr (SEP) {
               float w[32];
@@ -426,7 +436,7 @@ __global__ void __launch_bounds__(kThreads, 1)
               for (int i = 0; i < 32; i++) v[i] = __fadd_rn(v[i], w[i]);
             }
             if (c + 1 < COLS / 32) {
-              ptx::tmem_ld32(acc_hh + (c + 1) * 32, vbuf[(c + 1) & 1]);
+              if (PIPE) ptx::tmem_ld32(acc_hh + (c + 1) * 32, vbuf[(c + 1) & 1]);
             } else {
               ptx::tc_fence_before();
               __syncwarp();
@@ -456,10 +466,10 @@ __global__ void __launch_bounds__(kThreads, 1)
               const float thr = kd[kKnnMax - 1];
               float mn = __int_as_float(0x7f800000);
 #pragma unroll
-              for (int i = 0; i < 32; i++) {
-                v[i] = __fmaf_rn(-2.f, v[i], bn[i]);  // ||b||^2 - 2 a.b (the *2 is exact)
-                mn = fminf(mn, v[i]);
-              }
+              for (int i = 0; i < 32; i += 2)  // key = ||b||^2 - 2 a.b (the *2 is exact)
+                ptx::fma2_m2(v[i], v[i + 1], bn[i], bn[i + 1]);
+#pragma unroll
+              for (int i = 0; i < 32; i++) mn = fminf(mn, v[i]);
               if (__any_sync(0xffffffffu, mn < thr)) {
                 uint32_t cand = 0;
                 float keys[32];
@@ -476,10 +486,19 @@ __global__ void __launch_bounds__(kThreads, 1)
                 }
               }
             } else {
+              // group min first (FFMA2 + 3-input FMNMX), the index only when it improves
+              float mn = __int_as_float(0x7f800000);
 #pragma unroll
-              for (int i = 0; i < 32; i++) {
-                const float key = __fmaf_rn(-2.f, v[i], bn[i]);  // ||b||^2 - 2 a.b (exact *2)
-                if (key < best) { best = key; besti = c0 + i; }
+              for (int i = 0; i < 32; i += 2)  // key = ||b||^2 - 2 a.b (the *2 is exact)
+                ptx::fma2_m2(v[i], v[i + 1], bn[i], bn[i + 1]);
+#pragma unroll
+              for (int i = 0; i < 32; i++) mn = fminf(mn, v[i]);
+              if (mn < best) {  // strict: an equal key from a later column never wins
+                int idx = 31;
+#pragma unroll
+                for (int i = 30; i >= 0; i--) idx = (v[i] == mn) ? i : idx;  // lowest index
+                best = mn;
+                besti = c0 + idx;
               }
             }
           }
@@ -489,36 +508,44 @@ __global__ void __launch_bounds__(kThreads, 1)
 
       // ---- unit end: merge the two column halves of each row, write the unit's result
       if constexpr (EPI == EPI_KNN) {
+        // column groups 1..GPQ-1 hand their lists to group 0 one at a time (16 KiB scratch)
         float* sk = reinterpret_cast<float*>(scratch) + (q * 32 + lane) * kKnnMax;
         int* si = reinterpret_cast<int*>(scratch + kBM * kKnnMax * 4) + (q * 32 + lane) * kKnnMax;
-        if (cgp == 1) {
-#pragma unroll
-          for (int t = 0; t < kKnnMax; t++) { sk[t] = kd[t]; si[t] = ki[t]; }
-        }
-        named_bar_sync(1 + q, 64);
-        if (cgp == 0) {
 #pragma unroll 1
-          for (int t = 0; t < kKnnMax; t++) topk_insert<kKnnMax>(kd, ki, sk[t], si[t]);
-          if (row < p.M) {
-            const int64_t o = ((int64_t)ui.slice * p.M + row) * p.knn_k;
+        for (int g = 1; g < GPQ; g++) {
+          if (cgp == g) {
 #pragma unroll
-            for (int t = 0; t < kKnnMax; t++)
-              if (t < p.knn_k) { p.part_key[o + t] = kd[t]; p.part_idx[o + t] = ki[t]; }
+            for (int t = 0; t < kKnnMax; t++) { sk[t] = kd[t]; si[t] = ki[t]; }
           }
+          named_bar_sync(1 + q, 32 * GPQ);
+          if (cgp == 0) {
+#pragma unroll 1
+            for (int t = 0; t < kKnnMax; t++) topk_insert<kKnnMax>(kd, ki, sk[t], si[t]);
+          }
+          named_bar_sync(1 + q, 32 * GPQ);
         }
-        named_bar_sync(1 + q, 64);
+        if (cgp == 0 && row < p.M) {
+          const int64_t o = ((int64_t)ui.slice * p.M + row) * p.knn_k;
+#pragma unroll
+          for (int t = 0; t < kKnnMax; t++)
+            if (t < p.knn_k) { p.part_key[o + t] = kd[t]; p.part_idx[o + t] = ki[t]; }
+        }
       } else if constexpr (EPI == EPI_KMEANS) {
-        float* sk = reinterpret_cast<float*>(scratch) + (q * 32 + lane);
-        int* si = reinterpret_cast<int*>(scratch + kBM * 4) + (q * 32 + lane);
-        if (cgp == 1) { *sk = best; *si = besti; }
-        named_bar_sync(1 + q, 64);
+        float* sk = reinterpret_cast<float*>(scratch);
+        int* si = reinterpret_cast<int*>(scratch + GPQ * kBM * 4);
+        const int r = q * 32 + lane;
+        if (cgp > 0) { sk[(cgp - 1) * kBM + r] = best; si[(cgp - 1) * kBM + r] = besti; }
+        named_bar_sync(1 + q, 32 * GPQ);
         if (cgp == 0) {
-          float ob = *sk;
-          int oi = *si;
-          if (ob < best || (ob == best && oi < besti)) { best = ob; besti = oi; }
+#pragma unroll
+          for (int g = 1; g < GPQ; g++) {
+            const float ob = sk[(g - 1) * kBM + r];
+            const int oi = si[(g - 1) * kBM + r];
+            if (ob < best || (ob == best && oi < besti)) { best = ob; besti = oi; }
+          }
           if (row < p.M) { p.assign[row] = besti; p.best_key[row] = best; }
         }
-        named_bar_sync(1 + q, 64);
+        named_bar_sync(1 + q, 32 * GPQ);
       }
     }
   }
@@ -579,8 +606,10 @@ template <int CG, int BN, bool SEP, int EPI, int STAGES>
 static int launch_variant(const CUtensorMap* maps, const KParams& kp, int max_clusters,
                           cudaStream_t stream) {
   using G = Geo<CG, BN>;
-  auto kern = egemm_tc_kernel<CG, BN, SEP, EPI, STAGES>;
-  const int scratch = kBM * kKnnMax * 8;
+  // kMeans' argmin epilogue is issue-bound next to a 64-deep k-loop: 16 epilogue warps
+  constexpr int NEPI = (EPI == EPI_KMEANS) ? 16 : 8;
+  auto kern = egemm_tc_kernel<CG, BN, SEP, EPI, STAGES, NEPI>;
+  const int scratch = EPI == EPI_KNN ? kBM * kKnnMax * 8 : EPI == EPI_KMEANS ? 2 * 4 * kBM * 4 : 0;
   const size_t smem = 1024 + (size_t)STAGES * G::STAGE_BYTES + 8 * (2 * STAGES + 8) + scratch;
   static bool attr_done = false;  // per instantiation
   if (!attr_done) {
@@ -598,7 +627,7 @@ static int launch_variant(const CUtensorMap* maps, const KParams& kp, int max_cl
   if (clusters < 1) clusters = 1;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)(clusters * CG), 1, 1);
-  cfg.blockDim = dim3(kThreads, 1, 1);
+  cfg.blockDim = dim3(EpiGeo<NEPI>::THREADS, 1, 1);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = stream;
   cudaLaunchAttribute attr[1];

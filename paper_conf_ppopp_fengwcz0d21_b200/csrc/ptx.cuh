@@ -233,6 +233,30 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, float* v) {
       : "memory");
 }
 
+// ------------------------------------------------------------------ packed fp32x2 math
+// (d0, d1) = (b0 - 2 v0, b1 - 2 v1), one FFMA2 (fma.rn.f32x2, sm_100a); each lane is an
+// ordinary round-to-nearest fma, so results equal __fmaf_rn(-2, v, b) bitwise.
+__device__ __forceinline__ void fma2_m2(float& v0, float& v1, float b0, float b1) {
+  asm("{\n\t.reg .b64 a, b, c, d;\n\t"
+      "mov.b64 a, {%0, %1};\n\t"
+      "mov.b64 b, {%2, %3};\n\t"
+      "mov.b64 c, 0xC0000000C0000000;\n\t"
+      "fma.rn.f32x2 d, a, c, b;\n\t"
+      "mov.b64 {%0, %1}, d;\n\t}"
+      : "+f"(v0), "+f"(v1)
+      : "f"(b0), "f"(b1));
+}
+// (a0, a1) += (b0, b1) with round-to-nearest (add.rn.f32x2)
+__device__ __forceinline__ void add2(float& a0, float& a1, float b0, float b1) {
+  asm("{\n\t.reg .b64 a, b;\n\t"
+      "mov.b64 a, {%0, %1};\n\t"
+      "mov.b64 b, {%2, %3};\n\t"
+      "add.rn.f32x2 a, a, b;\n\t"
+      "mov.b64 {%0, %1}, a;\n\t}"
+      : "+f"(a0), "+f"(a1)
+      : "f"(b0), "f"(b1));
+}
+
 // ------------------------------------------------------------------ UMMA descriptors
 // Shared-memory matrix descriptor, K-major operand in the 128-byte-swizzle canonical
 // layout written by a TMA box of {64 fp16, rows} with CU_TENSOR_MAP_SWIZZLE_128B:
