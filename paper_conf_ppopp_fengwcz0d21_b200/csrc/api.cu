@@ -47,6 +47,11 @@ static int env_int(const char* name, int dflt) {
   return (v && *v) ? atoi(v) : dflt;
 }
 
+static bool fused_a_supported(const TcConfig& c) {
+  return (c.cg == 2 && c.bn == 256 && !c.sep) || (c.cg == 2 && c.bn == 128 && c.sep) ||
+         (c.cg == 1 && c.bn == 128 && c.sep);
+}
+
 static bool valid_config(int cg, int bn, int sep) {
   return (cg == 2 && bn == 256 && sep == 0) || (cg == 1 && bn == 128) ||
          (cg == 2 && bn == 128 && sep == 1);
@@ -82,6 +87,7 @@ static TcConfig choose_config(int epi_kind, int64_t M, int64_t N, int64_t K, int
   c.sep = env_int("EGEMM_SEP", c.sep);
   if (epi_kind == EPI_STORE) c.kc = env_int("EGEMM_KC", c.kc);
   c.max_clusters = env_int("EGEMM_MAX_CLUSTERS", 0);
+  c.fa = env_int("EGEMM_FUSED_A", c.fa);
   if (c.kc < 64) c.kc = 64;
   c.kc = (c.kc / 64) * 64;
   return c;
@@ -283,12 +289,21 @@ int egemm_gemm(int64_t M, int64_t N, int64_t K, egemm_operand_t A, egemm_operand
   }
   Carver cv{reinterpret_cast<char*>(workspace)};
   TcOperands ops = {};
-  if ((r = stage_operand(A, M, K, cv, &ops.a_hi, &ops.a_lo, &ops.lda, s))) return r;
+  TcConfig cfg = choose_config(EPI_STORE, M, N, K, terms);
+  // fp32 row-major A can be round-split inside the GEMM (converter warps, a-2 fused mode)
+  const bool fuse_a = cfg.fa && !A.hi && !A.trans && fused_a_supported(cfg);
+  if (fuse_a) {
+    ops.a_f32 = A.f32;
+    ops.lda_f32 = A.ld;
+    cv.take<uint16_t>((size_t)(M * ldk_of(K)));  // keep B's workspace offset unchanged
+    cv.take<uint16_t>((size_t)(M * ldk_of(K)));
+  } else if ((r = stage_operand(A, M, K, cv, &ops.a_hi, &ops.a_lo, &ops.lda, s))) {
+    return r;
+  }
   // B logical K x N: as an operand it is N rows x K; f32 trans==0 means stored K x N.
   egemm_operand_t Bt = B;
   Bt.trans = !B.trans;
   if ((r = stage_operand(Bt, N, K, cv, &ops.b_hi, &ops.b_lo, &ops.ldb, s))) return r;
-  TcConfig cfg = choose_config(EPI_STORE, M, N, K, terms);
   TcEpilogue epi = {};
   epi.kind = EPI_STORE;
   epi.D = D;

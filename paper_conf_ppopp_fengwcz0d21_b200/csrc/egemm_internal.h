@@ -23,6 +23,9 @@ struct TcOperands {
   const uint16_t* b_hi;
   const uint16_t* b_lo;
   int64_t ldb;
+  // fused A split: fp32 A (rows_a x K, row stride lda_f32); a_hi / a_lo then unused
+  const float* a_f32;
+  int64_t lda_f32;
 };
 
 struct TcConfig {
@@ -32,6 +35,7 @@ struct TcConfig {
   int kc;        // promotion interval in k elements (multiple of 64)
   int terms;     // 3 or 4
   int max_clusters;  // 0 = all SMs
+  int fa;        // fused A split allowed (fp32 A converted by in-kernel converter warps)
 };
 
 struct TcEpilogue {

@@ -44,7 +44,6 @@ __device__ __forceinline__ unsigned long long globaltimer_ns() {
 
 constexpr int kBM = 128;       // rows per CTA (TMEM lanes)
 constexpr int kBK = 64;        // k elements per stage (128 B of fp16: one SW128 row)
-constexpr int kEpiWarp0 = 4;
 constexpr int kKnnMax = 16;
 
 struct KParams {
@@ -67,6 +66,11 @@ struct KParams {
   int32_t* part_idx;
   int32_t* assign;
   float* best_key;
+  // fused A split (FA): fp32 A, row stride lda_f32; vec_a = 16-B aligned rows
+  const float* a_f32;
+  int64_t lda_f32;
+  int vec_a;
+  int K;
 };
 
 template <int CG, int BN>
@@ -79,10 +83,15 @@ struct Geo {
 
 // epilogue warps: NEPI in {8, 16}; NEPI/4 warps share each TMEM lane quarter and split
 // its BN columns.  Kernel block = 4 control warps + NEPI epilogue warps.
-template <int NEPI>
+template <int NEPI, bool FA = false>
 struct EpiGeo {
   static constexpr int GPQ = NEPI / 4;            // column groups per lane quarter
-  static constexpr int THREADS = 128 + 32 * NEPI;
+  // FA (fused A split): one extra warpgroup of converter warps in front
+  static constexpr int THREADS = (FA ? 256 : 128) + 32 * NEPI;
+  static constexpr int W_PROD = FA ? 4 : 0;       // TMA producer
+  static constexpr int W_MMA = FA ? 5 : 1;        // MMA issuer
+  static constexpr int W_ALLOC = FA ? 6 : 2;      // TMEM allocator
+  static constexpr int EPI0 = FA ? 8 : 4;         // first epilogue warp
 };
 
 struct UnitInfo {
@@ -163,14 +172,15 @@ __device__ __forceinline__ void named_bar_sync(int id, int nthreads) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }
 
-template <int CG, int BN, bool SEP, int EPI, int STAGES, int NEPI>
-__global__ void __launch_bounds__(EpiGeo<NEPI>::THREADS, 1)
+template <int CG, int BN, bool SEP, int EPI, int STAGES, int NEPI, bool FA>
+__global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
     egemm_tc_kernel(const __grid_constant__ CUtensorMap tm_ahi,
                     const __grid_constant__ CUtensorMap tm_alo,
                     const __grid_constant__ CUtensorMap tm_bhi,
                     const __grid_constant__ CUtensorMap tm_blo, const KParams p) {
   using G = Geo<CG, BN>;
-  constexpr int GPQ = EpiGeo<NEPI>::GPQ;
+  using EG = EpiGeo<NEPI, FA>;
+  constexpr int GPQ = EG::GPQ;
   constexpr int COLS = BN / GPQ;  // columns per epilogue warp
   constexpr int NACC = SEP ? 4 : 2;
   constexpr uint32_t TMEM_COLS = (NACC * BN <= 32) ? 32 : (NACC * BN <= 64) ? 64
@@ -197,15 +207,18 @@ __global__ void __launch_bounds__(EpiGeo<NEPI>::THREADS, 1)
   const int nclusters = (CG == 2) ? (int)ptx::nclusters_x() : (int)gridDim.x;
   const bool leader = (rank == 0);
 
-  if (warp == 0 && lane == 0) {
-    ptx::prefetch_tmap(&tm_ahi);
-    ptx::prefetch_tmap(&tm_alo);
+  if (warp == EG::W_PROD && lane == 0) {
+    if (!FA) {
+      ptx::prefetch_tmap(&tm_ahi);
+      ptx::prefetch_tmap(&tm_alo);
+    }
     ptx::prefetch_tmap(&tm_bhi);
     ptx::prefetch_tmap(&tm_blo);
   }
-  if (warp == 1 && lane == 0) {
+  if (warp == EG::W_MMA && lane == 0) {
     for (int s = 0; s < STAGES; s++) {
-      ptx::mbar_init(&full[s], 1);
+      // FA: the producer's expect_tx arrive plus one arrive per converter warp of the pair
+      ptx::mbar_init(&full[s], FA ? 1 + 4 * CG : 1);
       ptx::mbar_init(&empty[s], 1);
     }
     for (int b = 0; b < 2; b++) {
@@ -214,7 +227,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI>::THREADS, 1)
     }
     ptx::fence_mbar_init();
   }
-  if (warp == 2) ptx::tmem_alloc<CG>(tmem_slot, TMEM_COLS);
+  if (warp == EG::W_ALLOC) ptx::tmem_alloc<CG>(tmem_slot, TMEM_COLS);
   ptx::tc_fence_before();
   if constexpr (CG == 2) ptx::cluster_sync(); else __syncthreads();
   ptx::tc_fence_after();
@@ -226,11 +239,77 @@ __global__ void __launch_bounds__(EpiGeo<NEPI>::THREADS, 1)
 
   const int nch = (p.num_kb + p.kb_per_chunk - 1) / p.kb_per_chunk;
 
-  if (warp == 0) {
+  // FA register budget per warpgroup (512 threads share 64K registers): converters 96,
+  // producer / MMA / allocator 56, the two epilogue warpgroups 176 (running totals).  Each
+  // setmaxnreg sits at the top of its warpgroup's branch so it dominates that role's code.
+  if (FA && warp < 4) {
+    if constexpr (FA) asm volatile("setmaxnreg.dec.sync.aligned.u32 96;");
+    // ================= fused round-split of A (converter warpgroup) =================
+    // Alg. 1 l.2 inside the GEMM: each thread loads 8 consecutive fp32 of one
+    // A row (2 x 16 B), splits them (cvt.rn) and stores the 16 B hi / lo chunks straight
+    // into the 128-B-swizzled K-major stage layout the MMA descriptors expect -- the
+    // paper's LDG -> register -> STS staging with the split folded in.
+    if constexpr (FA) {
+      int stage = 0;
+      uint32_t phase = 0;
+      const int c = lane & 7;         // 16-B chunk (8 fp16) of the 128-B row
+      const int rsub = lane >> 3;     // 4 rows per warp instruction
+      for (int u = cluster; u < p.num_units; u += nclusters) {
+        UnitInfo ui = decode_unit<EPI>(p, u);
+        const int64_t arow0 = (int64_t)ui.m_tile * (kBM * CG) + rank * kBM;
+        for (int ns = 0; ns < ui.n_count; ns++) {
+          for (int kb = 0; kb < p.num_kb; kb++) {
+            ptx::mbar_wait(&empty[stage], phase ^ 1u);
+            const uint32_t sb = ptx::smem_u32(stage_base + stage * G::STAGE_BYTES);
+            const int k = kb * kBK + c * 8;
+            float4 x[16];
+#pragma unroll
+            for (int it = 0; it < 8; it++) {
+              const int r = warp * 32 + it * 4 + rsub;
+              const int64_t row = arow0 + r;
+              const float* src = p.a_f32 + row * p.lda_f32 + k;
+              if (row < p.M && k + 8 <= p.K && p.vec_a) {
+                x[2 * it] = __ldg(reinterpret_cast<const float4*>(src));
+                x[2 * it + 1] = __ldg(reinterpret_cast<const float4*>(src + 4));
+              } else {
+                float t[8];
+#pragma unroll
+                for (int e = 0; e < 8; e++) t[e] = (row < p.M && k + e < p.K) ? __ldg(src + e) : 0.f;
+                x[2 * it] = make_float4(t[0], t[1], t[2], t[3]);
+                x[2 * it + 1] = make_float4(t[4], t[5], t[6], t[7]);
+              }
+            }
+#pragma unroll
+            for (int it = 0; it < 8; it++) {
+              const int r = warp * 32 + it * 4 + rsub;
+              uint32_t hi[4], lo[4];
+              const float* f = reinterpret_cast<const float*>(&x[2 * it]);
+#pragma unroll
+              for (int e = 0; e < 4; e++) ptx::split2(f[2 * e], f[2 * e + 1], hi[e], lo[e]);
+              const uint32_t off = (uint32_t)(r * 128 + ((c ^ (r & 7)) << 4));
+              ptx::sts128(sb + off, hi[0], hi[1], hi[2], hi[3]);
+              ptx::sts128(sb + G::A_BYTES + off, lo[0], lo[1], lo[2], lo[3]);
+            }
+            ptx::fence_proxy_async_smem();  // generic-proxy stores -> visible to tcgen05.mma
+            __syncwarp();
+            if (lane == 0) {
+              if constexpr (CG == 1) ptx::mbar_arrive(&full[stage]);
+              else ptx::mbar_arrive_cluster(&full[stage], 0);
+            }
+            if (++stage == STAGES) { stage = 0; phase ^= 1u; }
+          }
+        }
+      }
+    }
+  } else if (warp < EG::EPI0) {
+   if constexpr (FA) asm volatile("setmaxnreg.dec.sync.aligned.u32 56;");
+   if (warp == EG::W_PROD) {
     // ============================ TMA producer ============================
     if (lane == 0) {
       int stage = 0;
       uint32_t phase = 0;
+      // FA: only B comes through TMA (A is written by the converter warps)
+      constexpr uint32_t TX = FA ? 2 * G::B_BYTES : G::STAGE_BYTES;
       for (int u = cluster; u < p.num_units; u += nclusters) {
         UnitInfo ui = decode_unit<EPI>(p, u);
         const int arow = ui.m_tile * (kBM * CG) + (int)rank * kBM;
@@ -239,16 +318,20 @@ __global__ void __launch_bounds__(EpiGeo<NEPI>::THREADS, 1)
           for (int kb = 0; kb < p.num_kb; kb++) {
             ptx::mbar_wait(&empty[stage], phase ^ 1u);
             uint8_t* sb = stage_base + stage * G::STAGE_BYTES;
-            if (leader) ptx::mbar_arrive_expect_tx(&full[stage], G::STAGE_BYTES * CG);
+            if (leader) ptx::mbar_arrive_expect_tx(&full[stage], TX * CG);
             const int k0 = kb * kBK;
             if constexpr (CG == 1) {
-              ptx::tma_load_2d(&tm_ahi, &full[stage], sb, k0, arow);
-              ptx::tma_load_2d(&tm_alo, &full[stage], sb + G::A_BYTES, k0, arow);
+              if (!FA) {
+                ptx::tma_load_2d(&tm_ahi, &full[stage], sb, k0, arow);
+                ptx::tma_load_2d(&tm_alo, &full[stage], sb + G::A_BYTES, k0, arow);
+              }
               ptx::tma_load_2d(&tm_bhi, &full[stage], sb + 2 * G::A_BYTES, k0, brow);
               ptx::tma_load_2d(&tm_blo, &full[stage], sb + 2 * G::A_BYTES + G::B_BYTES, k0, brow);
             } else {
-              ptx::tma_load_2d_pair(&tm_ahi, &full[stage], sb, k0, arow);
-              ptx::tma_load_2d_pair(&tm_alo, &full[stage], sb + G::A_BYTES, k0, arow);
+              if (!FA) {
+                ptx::tma_load_2d_pair(&tm_ahi, &full[stage], sb, k0, arow);
+                ptx::tma_load_2d_pair(&tm_alo, &full[stage], sb + G::A_BYTES, k0, arow);
+              }
               ptx::tma_load_2d_pair(&tm_bhi, &full[stage], sb + 2 * G::A_BYTES, k0, brow);
               ptx::tma_load_2d_pair(&tm_blo, &full[stage], sb + 2 * G::A_BYTES + G::B_BYTES, k0,
                                     brow);
@@ -258,7 +341,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI>::THREADS, 1)
         }
       }
     }
-  } else if (warp == 1) {
+  } else if (warp == EG::W_MMA) {
     // ============================ MMA issuer ============================
     // The whole warp runs the loop (so stage / descriptor arithmetic stays in uniform
     // registers); one elected lane -- always the same one -- issues MMAs and commits.
@@ -321,9 +404,11 @@ __global__ void __launch_bounds__(EpiGeo<NEPI>::THREADS, 1)
         }
       }
     }
-  } else if (warp >= kEpiWarp0) {
+   }
+  } else {
+    if constexpr (FA) asm volatile("setmaxnreg.inc.sync.aligned.u32 176;");
     // ============================ epilogue ============================
-    const int ew = warp - kEpiWarp0;
+    const int ew = warp - EG::EPI0;
     const int q = warp & 3;         // TMEM lane quarter this warp may access
     const int cgp = ew >> 2;        // column group (0 .. GPQ-1) within the lane quarter
     const uint32_t lane_off = (uint32_t)(q * 32) << 16;
@@ -554,7 +639,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI>::THREADS, 1)
   __syncwarp();
   ptx::tc_fence_before();
   if constexpr (CG == 2) ptx::cluster_sync(); else __syncthreads();
-  if (warp == 2) {
+  if (warp == EG::W_ALLOC) {
     ptx::tc_fence_after();
     ptx::tmem_dealloc<CG>(tmem_base, TMEM_COLS);
   }
@@ -602,13 +687,13 @@ static bool make_tmap_f16(CUtensorMap* m, const void* base, int64_t rows, int64_
   return r == CUDA_SUCCESS;
 }
 
-template <int CG, int BN, bool SEP, int EPI, int STAGES>
+template <int CG, int BN, bool SEP, int EPI, int STAGES, bool FA = false>
 static int launch_variant(const CUtensorMap* maps, const KParams& kp, int max_clusters,
                           cudaStream_t stream) {
   using G = Geo<CG, BN>;
   // kMeans' argmin epilogue is issue-bound next to a 64-deep k-loop: 16 epilogue warps
   constexpr int NEPI = (EPI == EPI_KMEANS) ? 16 : 8;
-  auto kern = egemm_tc_kernel<CG, BN, SEP, EPI, STAGES, NEPI>;
+  auto kern = egemm_tc_kernel<CG, BN, SEP, EPI, STAGES, NEPI, FA>;
   const int scratch = EPI == EPI_KNN ? kBM * kKnnMax * 8 : EPI == EPI_KMEANS ? 2 * 4 * kBM * 4 : 0;
   const size_t smem = 1024 + (size_t)STAGES * G::STAGE_BYTES + 8 * (2 * STAGES + 8) + scratch;
   static bool attr_done = false;  // per instantiation
@@ -627,7 +712,7 @@ static int launch_variant(const CUtensorMap* maps, const KParams& kp, int max_cl
   if (clusters < 1) clusters = 1;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)(clusters * CG), 1, 1);
-  cfg.blockDim = dim3(EpiGeo<NEPI>::THREADS, 1, 1);
+  cfg.blockDim = dim3(EpiGeo<NEPI, FA>::THREADS, 1, 1);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = stream;
   cudaLaunchAttribute attr[1];
@@ -648,6 +733,19 @@ static int launch_variant(const CUtensorMap* maps, const KParams& kp, int max_cl
 template <int EPI>
 static int dispatch(const CUtensorMap* maps, const KParams& kp, const TcConfig& cfg,
                     cudaStream_t s) {
+  if constexpr (EPI == EPI_STORE) {
+    if (kp.a_f32) {  // fused A split (converter warpgroup)
+      if (cfg.cg == 2 && cfg.bn == 256 && !cfg.sep)
+        return launch_variant<2, 256, false, EPI, 3, true>(maps, kp, cfg.max_clusters, s);
+      if (cfg.cg == 2 && cfg.bn == 128 && cfg.sep)
+        return launch_variant<2, 128, true, EPI, 3, true>(maps, kp, cfg.max_clusters, s);
+      if (cfg.cg == 1 && cfg.bn == 128 && cfg.sep)
+        return launch_variant<1, 128, true, EPI, 3, true>(maps, kp, cfg.max_clusters, s);
+      set_last_error("fused A split: unsupported tile config cg=%d bn=%d sep=%d", cfg.cg, cfg.bn,
+                     cfg.sep);
+      return 2;
+    }
+  }
   if (cfg.cg == 2 && cfg.bn == 256 && !cfg.sep)
     return launch_variant<2, 256, false, EPI, 3>(maps, kp, cfg.max_clusters, s);
   if (cfg.cg == 1 && cfg.bn == 128 && !cfg.sep)
@@ -669,14 +767,25 @@ int launch_tc(int64_t M, int64_t N, int64_t K, const TcOperands& ops, const TcCo
   }
   CUtensorMap maps[4];
   const int bnc = cfg.bn / cfg.cg;
-  if (!make_tmap_f16(&maps[0], ops.a_hi, M, K, ops.lda, kBM) ||
-      !make_tmap_f16(&maps[1], ops.a_lo, M, K, ops.lda, kBM) ||
+  const bool fa = ops.a_f32 != nullptr && epi.kind == EPI_STORE;
+  if ((!fa && (!make_tmap_f16(&maps[0], ops.a_hi, M, K, ops.lda, kBM) ||
+               !make_tmap_f16(&maps[1], ops.a_lo, M, K, ops.lda, kBM))) ||
       !make_tmap_f16(&maps[2], ops.b_hi, N, K, ops.ldb, bnc) ||
       !make_tmap_f16(&maps[3], ops.b_lo, N, K, ops.ldb, bnc)) {
     set_last_error("cuTensorMapEncodeTiled failed (alignment: base 16 B, ld %% 8 == 0)");
     return 2;
   }
+  if (fa) {  // A is converted in-kernel; its maps are unused (pass B's as placeholders)
+    maps[0] = maps[2];
+    maps[1] = maps[3];
+  }
   KParams kp = {};
+  kp.K = (int)K;
+  if (fa) {
+    kp.a_f32 = ops.a_f32;
+    kp.lda_f32 = ops.lda_f32;
+    kp.vec_a = ((ops.lda_f32 % 4) == 0 && ((uintptr_t)ops.a_f32 % 16) == 0) ? 1 : 0;
+  }
   kp.M = (int)M;
   kp.N = (int)N;
   kp.num_kb = (int)((K + kBK - 1) / kBK);

@@ -233,6 +233,28 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, float* v) {
       : "memory");
 }
 
+// ------------------------------------------------------------------ round-split helpers
+// Alg. 1 l.2 on two values: hi = fp16_RN(x) (cvt.rn.f16x2.f32, ties to even),
+// lo = fp16_RN(x - hi) with the residual exact in fp32.  Packed fp16x2 bit patterns out.
+__device__ __forceinline__ void split2(float a, float b, uint32_t& hi, uint32_t& lo) {
+  uint32_t h, l;
+  asm("cvt.rn.f16x2.f32 %0, %1, %2;" : "=r"(h) : "f"(b), "f"(a));  // hi half <- b, lo half <- a
+  float ha, hb;
+  asm("{\n\t.reg .f16 x, y;\n\tmov.b32 {x, y}, %2;\n\tcvt.f32.f16 %0, x;\n\tcvt.f32.f16 %1, y;\n\t}"
+      : "=f"(ha), "=f"(hb)
+      : "r"(h));
+  const float ra = __fsub_rn(a, ha), rb = __fsub_rn(b, hb);
+  asm("cvt.rn.f16x2.f32 %0, %1, %2;" : "=r"(l) : "f"(rb), "f"(ra));
+  hi = h;
+  lo = l;
+}
+__device__ __forceinline__ void sts128(uint32_t addr, uint32_t a, uint32_t b, uint32_t c,
+                                       uint32_t d) {
+  asm volatile("st.shared.v4.b32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "r"(a), "r"(b), "r"(c),
+               "r"(d)
+               : "memory");
+}
+
 // ------------------------------------------------------------------ packed fp32x2 math
 // (d0, d1) = (b0 - 2 v0, b1 - 2 v1), one FFMA2 (fma.rn.f32x2, sm_100a); each lane is an
 // ordinary round-to-nearest fma, so results equal __fmaf_rn(-2, v, b) bitwise.

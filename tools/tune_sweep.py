@@ -83,14 +83,13 @@ def main():
                 print("M=%5d N=%5d K=%5d best=%s %s" % (M, N, K, best and best["cfg"],
                       " ".join("%s:%.3fms%s" % (r["cfg"], r["ms"], "" if r["ok"] else "x") for r in res)),
                       flush=True)
-    # bucket order: smallest first so the library's first-match lookup picks the tightest
+    # the largest measured bucket in each dimension is open-ended, then bucket order:
+    # smallest first so the library's first-match lookup picks the tightest bucket
+    for e in entries:
+        for key, top in (("m_max", max(Ms)), ("n_max", max(Ns)), ("k_max", max(Ks))):
+            if e[key] == top:
+                e[key] = 1 << 40
     entries.sort(key=lambda e: (e["m_max"], e["n_max"], e["k_max"]))
-    # catch-all rows: larger shapes use the largest measured bucket's choice
-    big = [e for e in entries if e["m_max"] == max(Ms) and e["n_max"] == max(Ns) and e["k_max"] == max(Ks)]
-    if big:
-        e = dict(big[0])
-        e.update({"m_max": 1 << 40, "n_max": 1 << 40, "k_max": 1 << 40})
-        entries.append(e)
     doc = {"generated_by": "tools/tune_sweep.py", "device": torch.cuda.get_device_name(),
            "when": time.strftime("%Y-%m-%dT%H:%M:%SZ", time.gmtime()),
            "rule": "fastest config with normwise error <= 1e-6 and <= 2x naive fp32 (64 sampled rows)",
