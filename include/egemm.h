@@ -163,9 +163,10 @@ int egemm_set_config(int cg, int bn, int sep, int kc);
  * through *entries (nullable), its number of entries.  Host-only. */
 const char* egemm_tune_table(int* entries);
 /* The configuration the library would use for op (0 gemm, 1 knn, 2 kmeans) at M, N, K
- * (after table, egemm_set_config and EGEMM_* overrides).  Host-only. */
+ * (after table, egemm_set_config and EGEMM_* overrides).  *fused_a (nullable) = 1 when an
+ * fp32 row-major A would be round-split inside the GEMM kernel (a-2 fused mode). */
 int egemm_query_config(int op, int64_t M, int64_t N, int64_t K, int* cg, int* bn, int* sep,
-                       int* kc);
+                       int* kc, int* fused_a);
 
 /* Number of SMs of the current device (0 without a device). */
 int egemm_num_sms(void);

@@ -70,17 +70,23 @@ static TcConfig choose_config(int epi_kind, int64_t M, int64_t N, int64_t K, int
   c.kc = 64;
   if (epi_kind == EPI_STORE && M <= 128) { c.cg = 1; c.bn = 128; c.sep = 1; }
   {  // the measured table (tools/tune_sweep.py -> tune_table.json) overrides the defaults
-    int cg, bn, sep, kc;
-    if (tune_lookup(epi_kind, M, N, K, &cg, &bn, &sep, &kc) && valid_config(cg, bn, sep)) {
+    int cg, bn, sep, kc, fa;
+    if (tune_lookup(epi_kind, M, N, K, &cg, &bn, &sep, &kc, &fa) && valid_config(cg, bn, sep)) {
       c.cg = cg;
       c.bn = bn;
       c.sep = sep;
+      c.fa = fa;
       if (kc > 0) c.kc = kc;
     }
   }
   if (epi_kind != EPI_STORE) c.kc = (int)(((K + 63) / 64) * 64);
   // thread-local API override, then environment (experiments)
-  if (g_override.cg) { c.cg = g_override.cg; c.bn = g_override.bn; c.sep = g_override.sep; }
+  if (g_override.cg) {
+    c.cg = g_override.cg;
+    c.bn = g_override.bn;
+    c.sep = g_override.sep;
+    c.fa = 0;  // an explicit tile override measures the pre-split path unless EGEMM_FUSED_A
+  }
   if (g_override.kc && epi_kind == EPI_STORE) c.kc = g_override.kc;
   c.cg = env_int("EGEMM_CG", c.cg);
   c.bn = env_int("EGEMM_BN", c.bn);
@@ -189,13 +195,14 @@ const char* egemm_tune_table(int* entries) {
 }
 
 int egemm_query_config(int op, int64_t M, int64_t N, int64_t K, int* cg, int* bn, int* sep,
-                       int* kc) {
+                       int* kc, int* fused_a) {
   if (op < 0 || op > 2 || !cg || !bn || !sep || !kc) return EGEMM_ERR_INVALID_ARG;
   TcConfig c = choose_config(op, M, N, K, 3);
   *cg = c.cg;
   *bn = c.bn;
   *sep = c.sep;
   *kc = c.kc;
+  if (fused_a) *fused_a = (op == EPI_STORE && c.fa && fused_a_supported(c)) ? 1 : 0;
   return EGEMM_OK;
 }
 
@@ -441,15 +448,23 @@ int egemm_gemm_host(int64_t M, int64_t N, int64_t K, const float* A_host, int64_
                           K * sizeof(float), rows, cudaMemcpyHostToDevice, hp->s_in));
     chk(cudaEventRecord(hp->ev_in[b], hp->s_in));
     chk(cudaStreamWaitEvent(s, hp->ev_in[b], 0));
-    if (launch_split(Ad[b], rows, K, K, ahi[b], alo[b], ldk, 0, nullptr, s)) ok = false;
-    chk(cudaEventRecord(hp->ev_split[b], s));
+    const bool fuse_a = cfg.fa && fused_a_supported(cfg);
+    if (!fuse_a) {
+      if (launch_split(Ad[b], rows, K, K, ahi[b], alo[b], ldk, 0, nullptr, s)) ok = false;
+      chk(cudaEventRecord(hp->ev_split[b], s));
+    }
     if (c >= 2) chk(cudaStreamWaitEvent(s, hp->ev_out[b], 0));  // Dd[b] drained
     TcOperands ops = {ahi[b], alo[b], ldk, bhi, blo, ldk};
+    if (fuse_a) {  // the GEMM's converter warps split A straight from Ad[b]
+      ops.a_f32 = Ad[b];
+      ops.lda_f32 = K;
+    }
     TcEpilogue epi = {};
     epi.kind = EPI_STORE;
     epi.D = Dd[b];
     epi.ldd = N;
     if (ok && launch_tc(rows, N, K, ops, cfg, epi, s)) ok = false;
+    if (fuse_a) chk(cudaEventRecord(hp->ev_split[b], s));  // Ad[b] consumed by the GEMM
     chk(cudaEventRecord(hp->ev_comp[b], s));
     chk(cudaStreamWaitEvent(hp->s_out, hp->ev_comp[b], 0));
     chk(cudaMemcpy2DAsync(D_host + r0 * ldd, ldd * sizeof(float), Dd[b], N * sizeof(float),

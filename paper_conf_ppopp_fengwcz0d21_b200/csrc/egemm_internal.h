@@ -80,7 +80,7 @@ int read_clock_probe(double* mhz);
 
 // tune.cu: the measured configuration table
 bool tune_lookup(int op, long long M, long long N, long long K, int* cg, int* bn, int* sep,
-                 int* kc);
+                 int* kc, int* fa);
 const char* tune_table_path();
 int tune_table_size();
 

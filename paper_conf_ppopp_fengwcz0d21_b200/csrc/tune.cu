@@ -23,7 +23,7 @@ namespace egemm {
 struct TuneEntry {
   int op = -1;  // EpiKind
   long long m_max = 0, n_max = 0, k_max = 0;
-  int cg = 0, bn = 0, sep = 0, kc = 0;
+  int cg = 0, bn = 0, sep = 0, kc = 0, fa = 0;
 };
 
 static std::vector<TuneEntry> g_table;
@@ -101,7 +101,7 @@ static bool parse_entry(const char*& p, TuneEntry* e) {
       if (!parse_string(p, &v)) return false;
       e->op = v == "gemm" ? EPI_STORE : v == "knn" ? EPI_KNN : v == "kmeans" ? EPI_KMEANS : -1;
     } else if (key == "m_max" || key == "n_max" || key == "k_max" || key == "cg" || key == "bn" ||
-               key == "sep" || key == "kc") {
+               key == "sep" || key == "kc" || key == "fa") {
       char* end = nullptr;
       long long v = strtoll(p, &end, 10);
       if (end == p) return false;
@@ -112,6 +112,7 @@ static bool parse_entry(const char*& p, TuneEntry* e) {
       else if (key == "cg") e->cg = (int)v;
       else if (key == "bn") e->bn = (int)v;
       else if (key == "sep") e->sep = (int)v;
+      else if (key == "fa") e->fa = (int)v;
       else e->kc = (int)v;
     } else if (!skip_value(p)) {
       return false;
@@ -171,7 +172,7 @@ static void load_table() {
 }
 
 bool tune_lookup(int op, long long M, long long N, long long K, int* cg, int* bn, int* sep,
-                 int* kc) {
+                 int* kc, int* fa) {
   std::call_once(g_table_once, load_table);
   for (const TuneEntry& e : g_table) {
     if (e.op != op || M > e.m_max || N > e.n_max || K > e.k_max) continue;
@@ -179,6 +180,7 @@ bool tune_lookup(int op, long long M, long long N, long long K, int* cg, int* bn
     *bn = e.bn;
     *sep = e.sep;
     *kc = e.kc;
+    *fa = e.fa;
     return true;
   }
   return false;

@@ -86,7 +86,7 @@ def load(path: str = LIB_PATH):
     L.egemm_tune_table.argtypes = [ctypes.POINTER(ctypes.c_int)]
     L.egemm_tune_table.restype = ctypes.c_char_p
     IP = ctypes.POINTER(ctypes.c_int)
-    L.egemm_query_config.argtypes = [I, I64, I64, I64, IP, IP, IP, IP]
+    L.egemm_query_config.argtypes = [I, I64, I64, I64, IP, IP, IP, IP, IP]
     L.egemm_query_config.restype = I
     _lib = L
     return L
@@ -99,12 +99,14 @@ def tune_table():
     return p.decode(), n.value
 
 
-def query_config(op: str, M: int, N: int, K: int):
-    """The (cg, bn, sep, kc) the library picks for op in {'gemm','knn','kmeans'}."""
-    v = [ctypes.c_int(0) for _ in range(4)]
+def query_config(op: str, M: int, N: int, K: int, with_fused: bool = False):
+    """The (cg, bn, sep, kc) the library picks for op in {'gemm','knn','kmeans'}
+    (+ fused_a flag when with_fused)."""
+    v = [ctypes.c_int(0) for _ in range(5)]
     _check(load().egemm_query_config({"gemm": 0, "knn": 1, "kmeans": 2}[op], M, N, K,
                                      *[ctypes.byref(x) for x in v]), "egemm_query_config")
-    return tuple(x.value for x in v)
+    out = tuple(x.value for x in v)
+    return out if with_fused else out[:4]
 
 
 def debug_last_clock() -> float:

@@ -22,8 +22,10 @@ import oracle  # noqa: E402
 from paper_conf_ppopp_fengwcz0d21_b200 import egemm, inputs  # noqa: E402
 
 OUT = os.path.join(ROOT, "paper_conf_ppopp_fengwcz0d21_b200", "tune_table.json")
-CONFIGS = [(2, 256, 0, 64), (2, 256, 0, 128), (2, 128, 1, 128), (2, 128, 1, 256),
-           (1, 128, 1, 128), (1, 128, 1, 256), (1, 128, 0, 64)]
+# (cg, bn, sep, kc, fa): fa = the fused in-kernel A split (converter warpgroup)
+CONFIGS = [(2, 256, 0, 64, 0), (2, 256, 0, 128, 0), (2, 128, 1, 128, 0), (2, 128, 1, 256, 0),
+           (1, 128, 1, 128, 0), (1, 128, 1, 256, 0), (1, 128, 0, 64, 0),
+           (2, 256, 0, 64, 1), (2, 256, 0, 128, 1), (2, 128, 1, 256, 1), (1, 128, 1, 256, 1)]
 
 
 def timeit(fn, reps=7):
@@ -43,25 +45,30 @@ def timeit(fn, reps=7):
 def gemm_bucket(M, N, K, rows=64):
     A, B = inputs.uniform((M, K), 11 + M), inputs.uniform((K, N), 13 + N)
     Ad, Bd = torch.from_numpy(A).cuda(), torch.from_numpy(B).cuda()
-    a_split, b_split = egemm.split(Ad), egemm.split(Bd, transpose=True)
+    b_split = egemm.split(Bd, transpose=True)
     D = torch.empty((M, N), device="cuda")
     rs = np.sort(inputs.rng(M + N + K).choice(M, size=min(rows, M), replace=False))
     C64 = oracle.gemm64(A[rs], B)
     en = oracle.normwise_error(oracle.gemm32_naive(A[rs], B), A[rs], B, C64)
+    ws = torch.empty(egemm.gemm_workspace_size(M, N, K, False, True), dtype=torch.uint8, device="cuda")
     res = []
     for cfg in CONFIGS:
-        egemm.set_config(*cfg)
-        t = timeit(lambda: egemm.gemm(None, None, a_split=a_split, b_split=b_split, out=D))
+        egemm.set_config(*cfg[:4])
+        os.environ["EGEMM_FUSED_A"] = str(cfg[4])
+        # the user call with an fp32 A (split separately, or fused into the GEMM) and a
+        # pre-split B: the A split is part of every timed call
+        t = timeit(lambda: egemm.gemm(Ad, None, b_split=b_split, out=D, workspace=ws))
         e = oracle.normwise_error(D.cpu().numpy()[rs], A[rs], B, C64)
         res.append({"cfg": cfg, "ms": t, "err": e, "err_naive": en,
                     "ok": bool(e <= 1e-6 and e <= 2 * en)})
     egemm.set_config(0, 0, 0, 0)
+    os.environ.pop("EGEMM_FUSED_A", None)
     return res
 
 
 def main():
     quick = "--quick" in sys.argv
-    Ms = [128, 256, 1024, 4096, 8192] if not quick else [128, 1024, 8192]
+    Ms = [128, 256, 1024, 4096, 8192, 65536] if not quick else [128, 1024, 8192]
     Ns = [256, 1024, 8192] if not quick else [256, 8192]
     Ks = [256, 1024, 8192] if not quick else [1024, 8192]
     entries, log = [], []
@@ -69,14 +76,16 @@ def main():
     for M in Ms:
         for N in Ns:
             for K in Ks:
+                if M > 8192 and N > 1024:  # the tall bucket is for skinny N (configs[2])
+                    continue
                 res = gemm_bucket(M, N, K)
                 ok = [r for r in res if r["ok"]]
                 best = min(ok, key=lambda r: r["ms"]) if ok else None
                 log.append({"M": M, "N": N, "K": K, "results": res})
                 if best:
-                    cg, bn, sep, kc = best["cfg"]
+                    cg, bn, sep, kc, fa = best["cfg"]
                     entries.append({"op": "gemm", "m_max": M, "n_max": N, "k_max": K, "cg": cg,
-                                    "bn": bn, "sep": sep, "kc": kc,
+                                    "bn": bn, "sep": sep, "kc": kc, "fa": fa,
                                     "ms": round(best["ms"], 4),
                                     "tflops_fp32eq": round(2.0 * M * N * K / best["ms"] / 1e9, 1),
                                     "err_ratio": round(best["err"] / best["err_naive"], 3)})
