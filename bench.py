@@ -361,6 +361,42 @@ def main():
     if not args.no_apps:
         apps = _apps(world, rank, dev, args)
 
+    # context on the same B200 (library GEMMs, not our path): cuBLAS SGEMM (fp32 CUDA
+    # cores, Table 5's cuBLAS-CUDA-FP32) and cuBLAS fp16 (cuBLAS-TC-Half)
+    context = {}
+    if rank == 0 and not args.no_apps:
+        try:
+            prev = torch.backends.cuda.matmul.allow_tf32
+            torch.backends.cuda.matmul.allow_tf32 = False
+            Ac, Bc = A[:min(m_loc, 8192)], B
+            for _ in range(2):
+                torch.matmul(Ac, Bc)
+            s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            s.record()
+            for _ in range(5):
+                torch.matmul(Ac, Bc)
+            e.record()
+            e.synchronize()
+            t_sg = s.elapsed_time(e) / 5
+            torch.backends.cuda.matmul.allow_tf32 = prev
+            Ah, Bh = Ac.half(), Bc.half()
+            for _ in range(2):
+                torch.matmul(Ah, Bh)
+            s.record()
+            for _ in range(10):
+                torch.matmul(Ah, Bh)
+            e.record()
+            e.synchronize()
+            t_h = s.elapsed_time(e) / 10
+            fl = 2.0 * Ac.shape[0] * N * K
+            context = {"cublas_sgemm_tflops": round(fl / (t_sg * 1e-3) / 1e12, 2),
+                       "cublas_fp16_tflops": round(fl / (t_h * 1e-3) / 1e12, 1),
+                       "egemm_vs_cublas_sgemm": round(value / (fl / (t_sg * 1e-3) / 1e12), 2),
+                       "note": "torch.matmul fp32 with TF32 off (cublasSgemm) and fp16, same "
+                               "B200, %d x %d x %d" % (Ac.shape[0], N, K)}
+        except Exception as ex:  # pragma: no cover
+            context = {"error": str(ex)[:200]}
+
     cpu = None
     if rank == 0 and world == 1 and not args.no_cpu:
         import oracle
@@ -386,6 +422,7 @@ def main():
             "split_ms_per_step": round(split_ms, 4),
             "paper_context": {"t4_speedup_vs_cublas_fp32": 3.13, "t4_speedup_vs_sdk": 11.18,
                               "note": "paper's numbers on Tesla T4 (P:63, P:2251, P:2325), context only"},
+            "b200_context": context,
         }
         line.update(apps)
         print(json.dumps(line), flush=True)

@@ -165,3 +165,34 @@ def test_probe_tensor_core_accumulation(oracle_lib):
     print("tcgen05 accumulation model match rates:", results)
     # the model the B200 probe selected
     assert results["align2_fields"] == 1.0, results
+
+
+@pytest.mark.parametrize("cfg", [(2, 256, 0, 128), (2, 128, 1, 256), (1, 128, 1, 256)])
+@pytest.mark.parametrize("shape", [(300, 200, 100), (1000, 256, 1030), (257, 384, 64), (5, 7, 9)])
+def test_gemm_fused_a_split(oracle_lib, monkeypatch, cfg, shape):
+    """a-2 fused mode: fp32 A is round-split by the kernel's converter warps (ragged rows,
+    partial k-blocks, unaligned K) -- same bars as the pre-split path, and bitwise equal
+    to it (same products, same accumulation order)."""
+    eg = require_gpu()
+    M, N, K = shape
+    A, B = inputs.uniform((M, K), 80 + M), inputs.uniform((K, N), 81 + N)
+    monkeypatch.setenv("EGEMM_FUSED_A", "1")
+    D = _run(eg, A, B, cfg=cfg)
+    _assert_parity(oracle_lib, A, B, D)
+    monkeypatch.setenv("EGEMM_FUSED_A", "0")
+    D0 = _run(eg, A, B, cfg=cfg)
+    assert np.array_equal(D, D0)
+
+
+def test_gemm_fused_a_strided_rows(oracle_lib, monkeypatch):
+    """lda not a multiple of 4 (scalar-load fallback of the converter)."""
+    eg = require_gpu()
+    big = inputs.uniform((400, 515), 90)
+    B = inputs.uniform((513, 256), 91)
+    monkeypatch.setenv("EGEMM_FUSED_A", "1")
+    eg.set_config(2, 256, 0, 128)
+    try:
+        D = to_host(eg.gemm(to_dev(big)[:, 1:514], to_dev(B)))
+    finally:
+        eg.set_config(0, 0, 0, 0)
+    _assert_parity(oracle_lib, big[:, 1:514], B, D)
