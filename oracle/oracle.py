@@ -60,6 +60,10 @@ def lib():
         L.oracle_kmeans_finalize.restype = None
         L.oracle_group_sums.argtypes = [P, I64, I64, P, I64, P, P]
         L.oracle_group_sums.restype = None
+        L.oracle_tc_mma16.argtypes = [P, P, I, ctypes.c_float, I]
+        L.oracle_tc_mma16.restype = ctypes.c_float
+        L.oracle_gemm_alg1_tc.argtypes = [I64, I64, I64, P, P, P, I, I, I, P]
+        L.oracle_gemm_alg1_tc.restype = None
         L.oracle_num_threads.argtypes = []
         L.oracle_num_threads.restype = I
         _lib = L
@@ -227,6 +231,25 @@ def kmeans_finalize(sums, counts, C):
     out = _f32(C).copy()
     lib().oracle_kmeans_finalize(_p(sums), _p(counts), out.shape[0], out.shape[1], _p(out))
     return out
+
+
+def tc_mma16(a, b, c: float = 0.0, use_c: bool = True) -> float:
+    """The profiled tcgen05 kind::f16 MMA step (C implementation) on <= 16 products."""
+    a, b = _f32(a), _f32(b)
+    return float(np.float32(lib().oracle_tc_mma16(_p(a), _p(b), int(a.size), float(c), int(use_c))))
+
+
+def gemm_alg1_tc(A, B, C=None, terms: int = 3, sep: int = 0, kc: int = 64):
+    """Alg. 1 step by step on the profiled tensor-core primitive with promotion every kc
+    (reading R21): the bitwise model of what the kernel computes for (terms, sep, kc)."""
+    A, B = _f32(A), _f32(B)
+    M, K = A.shape
+    N = B.shape[1]
+    D = np.empty((M, N), np.float32)
+    Cp = _f32(C) if C is not None else None
+    lib().oracle_gemm_alg1_tc(M, N, K, _p(A), _p(B), _p(Cp) if Cp is not None else None,
+                              int(terms), int(sep), int(kc), _p(D))
+    return D
 
 
 def group_sums(X, assign, kc: int):

@@ -1,0 +1,51 @@
+"""Bit-exact GEMM parity: the tcgen05 kernel == Alg. 1 executed on the profiled tensor-core
+primitive (oracle.gemm_alg1_tc, reading R21) for every tile configuration / promotion
+interval / term count / accumulator mode, fused and pre-split A, ragged shapes and C.
+The per-element arithmetic of the kernel does not depend on the tile shape, only on
+(terms, sep, Kc), so every configuration must match the model bitwise."""
+import numpy as np
+import pytest
+
+from paper_conf_ppopp_fengwcz0d21_b200 import inputs
+from tests.gpu_util import require_gpu, to_dev, to_host
+
+pytestmark = pytest.mark.gpu
+
+CFGS = [(2, 256, 0, 64), (2, 256, 0, 128), (1, 128, 0, 64), (1, 128, 1, 128), (1, 128, 1, 256),
+        (2, 128, 1, 256)]
+
+
+def _gpu(eg, A, B, C, cfg, terms, fused):
+    eg.set_config(*cfg)
+    import os
+    os.environ["EGEMM_FUSED_A"] = "1" if fused else "0"
+    try:
+        return to_host(eg.gemm(to_dev(A), to_dev(B), to_dev(C) if C is not None else None,
+                               terms=terms))
+    finally:
+        eg.set_config(0, 0, 0, 0)
+        os.environ.pop("EGEMM_FUSED_A", None)
+
+
+@pytest.mark.parametrize("cfg", CFGS)
+@pytest.mark.parametrize("shape", [(256, 256, 256), (300, 200, 1000), (129, 257, 65)])
+def test_bitexact_vs_alg1_model(oracle_lib, cfg, shape):
+    eg = require_gpu()
+    M, N, K = shape
+    A, B = inputs.uniform((M, K), 20 + K), inputs.uniform((K, N), 21 + N)
+    D = _gpu(eg, A, B, None, cfg, 3, False)
+    ref = oracle_lib.gemm_alg1_tc(A, B, terms=3, sep=cfg[2], kc=cfg[3])
+    assert np.array_equal(D.view(np.uint32), ref.view(np.uint32)), \
+        "mismatches: %d" % int((D != ref).sum())
+
+
+@pytest.mark.parametrize("cfg", [(2, 256, 0, 128), (1, 128, 1, 256)])
+@pytest.mark.parametrize("gen", [inputs.stress, inputs.in_zone])
+def test_bitexact_terms4_with_c_and_fused(oracle_lib, cfg, gen):
+    eg = require_gpu()
+    A, B, C = gen((200, 700), 30), gen((700, 300), 31), inputs.uniform((200, 300), 32)
+    for terms in (3, 4):
+        for fused in (False, True):
+            D = _gpu(eg, A, B, C, cfg, terms, fused)
+            ref = oracle_lib.gemm_alg1_tc(A, B, C, terms=terms, sep=cfg[2], kc=cfg[3])
+            assert np.array_equal(D.view(np.uint32), ref.view(np.uint32)), (terms, fused)

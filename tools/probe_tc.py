@@ -56,6 +56,18 @@ def main(out="gpurun_out/probe.npz"):
     A[:, 16] = f16(g.uniform(1, 2, M) * np.exp2(-g.integers(10, 30, M)) * np.where(g.random(M) < .5, -1, 1))
     B[16, :] = f16(g.uniform(1, 2, N))
     sets["s7"] = (A, B)
+    # S8: subnormal fp16 operands (what the lo parts of |x| < 2^-3 become) mixed with normals
+    sub = lambda shape: (g.integers(1, 1024, shape) * 2.0 ** -24 * np.where(g.random(shape) < .5, -1, 1))
+    A = f16(g.uniform(-1, 1, (M, 32)))
+    A[:, :8] = f16(sub((M, 8)))
+    A[:, 16:28] = f16(sub((M, 12)))
+    B = f16(g.uniform(-1, 1, (32, N)))
+    B[4:12, :] = f16(sub((8, N)) * 2.0 ** 10)
+    sets["s8"] = (A, B)
+    # S9: all-subnormal A against normal B, with C from a first MMA of normals
+    A = f16(sub((M, 32)))
+    A[:, :16] = f16(g.uniform(-2.0 ** -10, 2.0 ** -10, (M, 16)))
+    sets["s9"] = (A, f16(g.uniform(-1, 1, (32, N))))
     res = {}
     egemm.set_config(1, 128, 1, 1024)
     for name, (A, B) in sets.items():
