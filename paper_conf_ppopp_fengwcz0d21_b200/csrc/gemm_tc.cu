@@ -71,6 +71,7 @@ struct KParams {
   int64_t lda_f32;
   int vec_a;
   int K;
+  int debug_no_tma;  // EGEMM_DEBUG_NO_TMA=1: skip operand loads (timing diagnostics only)
 };
 
 template <int CG, int BN>
@@ -318,6 +319,11 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
           for (int kb = 0; kb < p.num_kb; kb++) {
             ptx::mbar_wait(&empty[stage], phase ^ 1u);
             uint8_t* sb = stage_base + stage * G::STAGE_BYTES;
+            if (p.debug_no_tma) {  // diagnostics only: MMA-issue ceiling without operand traffic
+              if (leader && !FA) ptx::mbar_arrive(&full[stage]);
+              if (++stage == STAGES) { stage = 0; phase ^= 1u; }
+              continue;
+            }
             if (leader) ptx::mbar_arrive_expect_tx(&full[stage], TX * CG);
             const int k0 = kb * kBK;
             if constexpr (CG == 1) {
@@ -781,6 +787,10 @@ int launch_tc(int64_t M, int64_t N, int64_t K, const TcOperands& ops, const TcCo
   }
   KParams kp = {};
   kp.K = (int)K;
+  {
+    const char* dbg = getenv("EGEMM_DEBUG_NO_TMA");
+    kp.debug_no_tma = (dbg && dbg[0] == '1') ? 1 : 0;
+  }
   if (fa) {
     kp.a_f32 = ops.a_f32;
     kp.lda_f32 = ops.lda_f32;
