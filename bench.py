@@ -119,8 +119,11 @@ def _dist_setup():
     rank = int(os.environ.get("RANK", "0"))
     local = int(os.environ.get("LOCAL_RANK", "0"))
     if world > 1:
-        torch.cuda.set_device(local)
-        dist.init_process_group("nccl")
+        # EGEMM_BENCH_SHARE_GPU=1 (tests only): all ranks on cuda:0 over gloo, to exercise the
+        # multi-rank code path on a single-GPU box; the real runs use NCCL, one GPU per rank
+        shared = os.environ.get("EGEMM_BENCH_SHARE_GPU") == "1"
+        torch.cuda.set_device(0 if shared else local)
+        dist.init_process_group("gloo" if shared else "nccl")
     else:
         torch.cuda.set_device(0)
     return world, rank, local
