@@ -76,6 +76,14 @@ typedef struct {
 int egemm_split(const float* x, int64_t rows, int64_t cols, int64_t ldx, uint16_t* hi,
                 uint16_t* lo, int64_t ldo, int transpose, uint32_t* range_flags, void* stream);
 
+/* Truncate-split, the Markidis variant the paper compares against (Fig. 4a, P:812-824;
+ * Table 1 "Markidis 1-5-20"): hi = fp16_RZ(x), lo = fp16_RZ(x - (float)hi).  Same
+ * arguments and behaviour as egemm_split.  Feed the result to egemm_gemm as pre-split
+ * operands to reproduce the paper's precision comparison (Fig. 7). */
+int egemm_split_trunc(const float* x, int64_t rows, int64_t cols, int64_t ldx, uint16_t* hi,
+                      uint16_t* lo, int64_t ldo, int transpose, uint32_t* range_flags,
+                      void* stream);
+
 /*
  * Extended-precision GEMM (Alg. 1 "Emulation(D, A, B, C)"):
  *   D[M x N] = A[M x K] * B[K x N] (+ C[M x N] if C != NULL)

@@ -227,8 +227,24 @@ int egemm_set_config(int cg, int bn, int sep, int kc) {
   return EGEMM_OK;
 }
 
+static int split_entry(const float* x, int64_t rows, int64_t cols, int64_t ldx, uint16_t* hi,
+                       uint16_t* lo, int64_t ldo, int transpose, uint32_t* range_flags,
+                       void* stream, int mode);
+
 int egemm_split(const float* x, int64_t rows, int64_t cols, int64_t ldx, uint16_t* hi,
                 uint16_t* lo, int64_t ldo, int transpose, uint32_t* range_flags, void* stream) {
+  return split_entry(x, rows, cols, ldx, hi, lo, ldo, transpose, range_flags, stream, 0);
+}
+
+int egemm_split_trunc(const float* x, int64_t rows, int64_t cols, int64_t ldx, uint16_t* hi,
+                      uint16_t* lo, int64_t ldo, int transpose, uint32_t* range_flags,
+                      void* stream) {
+  return split_entry(x, rows, cols, ldx, hi, lo, ldo, transpose, range_flags, stream, 1);
+}
+
+static int split_entry(const float* x, int64_t rows, int64_t cols, int64_t ldx, uint16_t* hi,
+                       uint16_t* lo, int64_t ldo, int transpose, uint32_t* range_flags,
+                       void* stream, int mode) {
   if (rows < 0 || cols < 0) {
     set_last_error("negative size");
     return EGEMM_ERR_INVALID_ARG;
@@ -246,7 +262,8 @@ int egemm_split(const float* x, int64_t rows, int64_t cols, int64_t ldx, uint16_
     set_last_error("no sm_100 device");
     return EGEMM_ERR_CUDA;
   }
-  if (launch_split(x, rows, cols, ldx, hi, lo, ldo, transpose, range_flags, (cudaStream_t)stream)) {
+  if (launch_split(x, rows, cols, ldx, hi, lo, ldo, transpose, range_flags, (cudaStream_t)stream,
+                   mode)) {
     set_last_error("split launch: %s", cudaGetErrorString(cudaGetLastError()));
     return EGEMM_ERR_CUDA;
   }

@@ -7,9 +7,10 @@ namespace egemm {
 
 int num_sms();
 
+// mode 0: round-split (Alg. 1), mode 1: truncate-split (Markidis, NEXT-1 variant)
 int launch_split(const float* x, int64_t rows, int64_t cols, int64_t ldx, uint16_t* hi,
                  uint16_t* lo, int64_t ldo, int transpose, uint32_t* range_flags,
-                 cudaStream_t stream);
+                 cudaStream_t stream, int mode = 0);
 
 // Epilogue policies of the tensor-core kernel.
 enum EpiKind : int { EPI_STORE = 0, EPI_KNN = 1, EPI_KMEANS = 2 };

@@ -33,7 +33,8 @@ class Operand(ctypes.Structure):
                 ("ld", ctypes.c_int64), ("trans", ctypes.c_int), ("ld_split", ctypes.c_int64)]
 
 
-EXPORTS = ["egemm_status_string", "egemm_last_error", "egemm_version", "egemm_split", "egemm_gemm",
+EXPORTS = ["egemm_status_string", "egemm_last_error", "egemm_version", "egemm_split",
+           "egemm_split_trunc", "egemm_gemm",
            "egemm_gemm_workspace_size", "egemm_knn", "egemm_knn_workspace_size", "egemm_knn_index",
            "egemm_kmeans_step", "egemm_kmeans_workspace_size", "egemm_kmeans_finalize",
            "egemm_set_config", "egemm_num_sms", "egemm_debug_last_clock", "egemm_tune_table",
@@ -58,6 +59,8 @@ def load(path: str = LIB_PATH):
     L.egemm_version.restype = I
     L.egemm_split.argtypes = [P, I64, I64, I64, P, P, I64, I, P, P]
     L.egemm_split.restype = I
+    L.egemm_split_trunc.argtypes = [P, I64, I64, I64, P, P, I64, I, P, P]
+    L.egemm_split_trunc.restype = I
     L.egemm_gemm.argtypes = [I64, I64, I64, Operand, Operand, P, I64, P, I64, I, P, SZ, P]
     L.egemm_gemm.restype = I
     L.egemm_gemm_workspace_size.argtypes = [I64, I64, I64, I, I]
@@ -146,9 +149,10 @@ def _workspace(nbytes: int, device, ws=None):
 
 # ---------------------------------------------------------------------------- split
 def split(x: torch.Tensor, transpose: bool = False, range_flags: torch.Tensor | None = None,
-          out: tuple | None = None, stream=None):
+          out: tuple | None = None, stream=None, mode: str = "round"):
     """Round-split fp32 x [rows, cols] -> (hi, lo) fp16 bit patterns as int16 tensors
-    (viewable as torch.float16).  transpose=True returns the [cols, rows] transpose."""
+    (viewable as torch.float16).  transpose=True returns the [cols, rows] transpose.
+    mode="trunc": the Markidis truncate-split (egemm_split_trunc)."""
     L = load()
     _need_cuda(x)
     assert x.dtype == torch.float32 and x.dim() == 2 and x.stride(1) == 1
@@ -159,8 +163,9 @@ def split(x: torch.Tensor, transpose: bool = False, range_flags: torch.Tensor | 
         lo = torch.empty(oshape, dtype=torch.int16, device=x.device)
     else:
         hi, lo = out
-    _check(L.egemm_split(_ptr(x), rows, cols, x.stride(0), _ptr(hi), _ptr(lo), hi.stride(0),
-                         1 if transpose else 0, _ptr(range_flags), _stream(stream)), "egemm_split")
+    fn = {"round": L.egemm_split, "trunc": L.egemm_split_trunc}[mode]
+    _check(fn(_ptr(x), rows, cols, x.stride(0), _ptr(hi), _ptr(lo), hi.stride(0),
+              1 if transpose else 0, _ptr(range_flags), _stream(stream)), "egemm_split")
     return hi, lo
 
 

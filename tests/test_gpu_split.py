@@ -73,3 +73,38 @@ def test_split_empty():
     eg = require_gpu()
     hi, lo = eg.split(torch.empty((0, 5), dtype=torch.float32, device="cuda"))
     assert hi.shape == (0, 5)
+
+
+def test_truncate_split_matches_oracle(oracle_lib):
+    """NEXT-1 variant: egemm_split_trunc == oracle split 'trunc' (RZ hi, RZ lo), bitwise, on a
+    strided sweep of all fp32 patterns plus dense normal-range values."""
+    eg = require_gpu()
+    x = np.concatenate([inputs.all_f32_patterns(0, 1 << 32)[:: 4099].copy(),
+                        inputs.stress(1 << 20, 17), inputs.uniform(1 << 20, 18)])
+    x = x[: (x.size // 64) * 64]
+    ohi, olo = oracle_lib.split(x, "trunc")
+    hi, lo = eg.split(to_dev(x).view(-1, 64), mode="trunc")
+    ok = _cmp(x, u16(hi).ravel(), u16(lo).ravel(), ohi, olo)
+    assert ok.all(), "mismatch at 0x%08x" % int(x.view(np.uint32)[np.argmin(ok)])
+
+
+def test_fig7_direction(oracle_lib):
+    """Fig. 7 on B200 at N = 256 and 1024: round-split EGEMM error sits below
+    the paper's EGEMM-TC series and below truncate-split (Markidis), which sits below
+    the tensor-core-half GEMM (tests/golden/fig7_max_error.txt)."""
+    eg = require_gpu()
+    paper = {256: 1.9e-5, 1024: 8.9e-5}
+    for n in (256, 1024):
+        A, B = inputs.uniform((n, n), 900 + n), inputs.uniform((n, n), 901 + n)
+        rows = np.arange(0, n, max(1, n // 128))
+        V32 = oracle_lib.gemm32_naive(A[rows], B)
+        Ad, Bd = to_dev(A), to_dev(B)
+        err = {}
+        for mode in ("round", "trunc"):
+            D = to_host(eg.gemm(None, None, a_split=eg.split(Ad, mode=mode),
+                                b_split=eg.split(Bd, transpose=True, mode=mode)))
+            err[mode] = oracle_lib.eq10_max_error(D[rows], V32)
+        Dh = to_host(torch.matmul(Ad.half(), Bd.half()).float())
+        err["half"] = oracle_lib.eq10_max_error(Dh[rows], V32)
+        assert err["round"] < paper[n], err
+        assert err["round"] < err["trunc"] < err["half"], err
