@@ -7,10 +7,11 @@
 // P:812-824; NEXT-1):  hi = fp16_RZ(x);  lo = fp16_RZ(x - (float)hi).
 // No -ftz / fast-math: fp32 subnormals and fp16 subnormal lo parts are kept.
 //
-// HBM-bound: 4 B read + 4 B written per element.  The contiguous kernel moves 16 elements
-// per thread and iteration (4 x 16-B loads, 2 x 16-B stores per output) on a grid of
+// HBM-bound: 4 B read + 4 B written per element.  The contiguous kernel moves 8 elements
+// per thread and iteration (2 x 16-B loads, one 16-B store per output) on a grid of
 // 148 x 8 CTAs; the transposing kernel (B stored K x N -> K-major N x K hi / lo) stages
-// 128 x 64 tiles through shared memory and writes 16-B rows.
+// 64 x 64 tiles through shared memory.  (Measured: wider 16-element iterations and
+// 128 x 64 tiles with 16-B stores were slower on B200.)
 #include <cuda_fp16.h>
 #include <cstdint>
 #include "egemm_internal.h"
@@ -44,36 +45,25 @@ __device__ __forceinline__ void flush_flags(uint32_t flags, uint32_t* range_flag
   if (any && (threadIdx.x & 31) == 0) atomicOr(range_flags, any);
 }
 
-// Contiguous x, hi, lo: 16 elements per thread-iteration, scalar tail.
+// Contiguous x, hi, lo: 8 elements per thread-iteration, scalar tail.
 template <int MODE>
 __global__ void __launch_bounds__(256) split_flat_kernel(const float* __restrict__ x, int64_t n,
                                                           uint16_t* __restrict__ hi,
                                                           uint16_t* __restrict__ lo,
                                                           uint32_t* range_flags) {
   uint32_t flags = 0;
-  const int64_t nv = n >> 4;
+  const int64_t nv = n >> 3;  // groups of 8: 2 x 16 B in, 16 B + 16 B out
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
   for (int64_t g = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; g < nv; g += stride) {
-    const float4* src = reinterpret_cast<const float4*>(x) + 4 * g;
-    float4 v[4];
-#pragma unroll
-    for (int i = 0; i < 4; i++) v[i] = __ldcs(src + i);
-    uint32_t h[8], l[8];
-#pragma unroll
-    for (int i = 0; i < 4; i++) {
-      SplitPair p0 = split2<MODE>(v[i].x, v[i].y, flags), p1 = split2<MODE>(v[i].z, v[i].w, flags);
-      h[2 * i] = p0.hi; h[2 * i + 1] = p1.hi;
-      l[2 * i] = p0.lo; l[2 * i + 1] = p1.lo;
-    }
-    uint4* dh = reinterpret_cast<uint4*>(hi) + 2 * g;
-    uint4* dl = reinterpret_cast<uint4*>(lo) + 2 * g;
-    __stcs(dh, make_uint4(h[0], h[1], h[2], h[3]));
-    __stcs(dh + 1, make_uint4(h[4], h[5], h[6], h[7]));
-    __stcs(dl, make_uint4(l[0], l[1], l[2], l[3]));
-    __stcs(dl + 1, make_uint4(l[4], l[5], l[6], l[7]));
+    const float4* src = reinterpret_cast<const float4*>(x) + 2 * g;
+    const float4 a = __ldcs(src), b = __ldcs(src + 1);
+    const SplitPair p0 = split2<MODE>(a.x, a.y, flags), p1 = split2<MODE>(a.z, a.w, flags);
+    const SplitPair p2 = split2<MODE>(b.x, b.y, flags), p3 = split2<MODE>(b.z, b.w, flags);
+    __stcs(reinterpret_cast<uint4*>(hi) + g, make_uint4(p0.hi, p1.hi, p2.hi, p3.hi));
+    __stcs(reinterpret_cast<uint4*>(lo) + g, make_uint4(p0.lo, p1.lo, p2.lo, p3.lo));
   }
-  if (blockIdx.x == 0) {  // scalar tail (n % 16 elements)
-    const int64_t t = (nv << 4) + threadIdx.x;
+  if (blockIdx.x == 0) {  // scalar tail (n % 8 elements)
+    const int64_t t = (nv << 3) + threadIdx.x;
     if (t < n) {
       SplitPair p = split2<MODE>(x[t], 0.f, flags);
       hi[t] = (uint16_t)(p.hi & 0xffffu);
@@ -102,10 +92,10 @@ __global__ void __launch_bounds__(256) split_strided_kernel(const float* __restr
   flush_flags(flags, range_flags);
 }
 
-// Transposing: x is rows x cols (ldx); hi/lo are cols x rows (ldo).  Tiles of 128 x-rows
-// x 64 x-cols: coalesced 8-B loads along x's rows, split, transposed into shared memory,
-// then each output row segment (128 fp16 = 256 B) written as 16-B vectors.
-constexpr int kTR = 128, kTC = 64, kTP = kTR + 8;  // pitch keeps 16-B row alignment
+// Transposing: x is rows x cols (ldx); hi/lo are cols x rows (ldo).  64 x 64 tiles:
+// coalesced loads along x's rows, split, transposed through shared memory (33-word pitch:
+// conflict-light column writes), 4-B stores along the output rows.
+constexpr int kTR = 64, kTC = 64;
 
 template <int MODE>
 __global__ void __launch_bounds__(256) split_transpose_kernel(const float* __restrict__ x,
@@ -114,52 +104,42 @@ __global__ void __launch_bounds__(256) split_transpose_kernel(const float* __res
                                                                uint16_t* __restrict__ hi,
                                                                uint16_t* __restrict__ lo,
                                                                int64_t ldo, uint32_t* range_flags) {
-  __shared__ __align__(16) uint16_t th[kTC][kTP];
-  __shared__ __align__(16) uint16_t tl[kTC][kTP];
+  __shared__ uint32_t th[64][33];  // packed fp16 pairs of tile element [c][r]
+  __shared__ uint32_t tl[64][33];
   uint32_t flags = 0;
   const int64_t r0 = (int64_t)blockIdx.y * kTR, c0 = (int64_t)blockIdx.x * kTC;
   const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;  // 32 x 8
-  const bool vec_in = ((ldx & 1) == 0) && ((reinterpret_cast<uintptr_t>(x) & 7) == 0);
-  const int64_t gc = c0 + 2 * tx;
-#pragma unroll 4
-  for (int i = 0; i < kTR / 8; i++) {
+  for (int i = 0; i < 8; i++) {
     const int r = ty + 8 * i;
-    const int64_t gr = r0 + r;
+    const int64_t gr = r0 + r, gc = c0 + 2 * tx;
     float a = 0.f, b = 0.f;
     if (gr < rows) {
-      const float* src = x + gr * ldx + gc;
-      if (vec_in && gc + 1 < cols) {
-        const float2 t = __ldcs(reinterpret_cast<const float2*>(src));
-        a = t.x;
-        b = t.y;
-      } else {
-        if (gc < cols) a = src[0];
-        if (gc + 1 < cols) b = src[1];
-      }
+      if (gc < cols) a = x[gr * ldx + gc];
+      if (gc + 1 < cols) b = x[gr * ldx + gc + 1];
     }
-    SplitPair p = split2<MODE>(a, b, flags);
-    th[2 * tx][r] = (uint16_t)(p.hi & 0xffffu);
-    th[2 * tx + 1][r] = (uint16_t)(p.hi >> 16);
-    tl[2 * tx][r] = (uint16_t)(p.lo & 0xffffu);
-    tl[2 * tx + 1][r] = (uint16_t)(p.lo >> 16);
+    const SplitPair p = split2<MODE>(a, b, flags);
+    reinterpret_cast<uint16_t*>(&th[2 * tx][0])[r] = (uint16_t)(p.hi & 0xffffu);
+    reinterpret_cast<uint16_t*>(&th[2 * tx + 1][0])[r] = (uint16_t)(p.hi >> 16);
+    reinterpret_cast<uint16_t*>(&tl[2 * tx][0])[r] = (uint16_t)(p.lo & 0xffffu);
+    reinterpret_cast<uint16_t*>(&tl[2 * tx + 1][0])[r] = (uint16_t)(p.lo >> 16);
   }
   __syncthreads();
-  // output rows oc = c0 + c (64 of them), 128 fp16 each = 16 chunks of 8: 4 per thread
-  const bool vec_out = ((ldo & 7) == 0) && ((reinterpret_cast<uintptr_t>(hi) & 15) == 0) &&
-                       ((reinterpret_cast<uintptr_t>(lo) & 15) == 0);
-#pragma unroll
-  for (int i = 0; i < 4; i++) {
-    const int idx = threadIdx.x + 256 * i;  // 0 .. 1023
-    const int c = idx >> 4, ch = idx & 15;
-    const int64_t oc = c0 + c, orow = r0 + ch * 8;
-    if (oc >= cols || orow >= rows) continue;
-    if (vec_out && orow + 8 <= rows) {
-      *reinterpret_cast<uint4*>(hi + oc * ldo + orow) = *reinterpret_cast<const uint4*>(&th[c][ch * 8]);
-      *reinterpret_cast<uint4*>(lo + oc * ldo + orow) = *reinterpret_cast<const uint4*>(&tl[c][ch * 8]);
+  for (int i = 0; i < 8; i++) {  // output row = column c of x; 2 fp16 per thread
+    const int c = ty + 8 * i;
+    const int64_t oc = c0 + c, orow = r0 + 2 * tx;
+    if (oc >= cols) continue;
+    const uint32_t vh = th[c][tx], vl = tl[c][tx];
+    if (orow + 1 < rows && ((ldo & 1) == 0)) {
+      *reinterpret_cast<uint32_t*>(hi + oc * ldo + orow) = vh;
+      *reinterpret_cast<uint32_t*>(lo + oc * ldo + orow) = vl;
     } else {
-      for (int e = 0; e < 8 && orow + e < rows; e++) {
-        hi[oc * ldo + orow + e] = th[c][ch * 8 + e];
-        lo[oc * ldo + orow + e] = tl[c][ch * 8 + e];
+      if (orow < rows) {
+        hi[oc * ldo + orow] = (uint16_t)(vh & 0xffffu);
+        lo[oc * ldo + orow] = (uint16_t)(vl & 0xffffu);
+      }
+      if (orow + 1 < rows) {
+        hi[oc * ldo + orow + 1] = (uint16_t)(vh >> 16);
+        lo[oc * ldo + orow + 1] = (uint16_t)(vl >> 16);
       }
     }
   }
@@ -176,7 +156,7 @@ static void launch_mode(const float* x, int64_t rows, int64_t cols, int64_t ldx,
                        ((uintptr_t)hi % 16 == 0) && ((uintptr_t)lo % 16 == 0));
     const int64_t n = rows * cols;
     if (flat) {
-      int64_t blocks = ((n >> 4) + 255) / 256;
+      int64_t blocks = ((n >> 3) + 255) / 256;
       const int64_t cap = (int64_t)nsm * 8;  // 8 x 256 threads resident per SM
       if (blocks > cap) blocks = cap;
       if (blocks < 1) blocks = 1;
