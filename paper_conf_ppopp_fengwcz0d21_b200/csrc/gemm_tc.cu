@@ -173,7 +173,7 @@ __device__ __forceinline__ void named_bar_sync(int id, int nthreads) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }
 
-template <int CG, int BN, bool SEP, int EPI, int STAGES, int NEPI, bool FA>
+template <int CG, int BN, bool SEP, int EPI, int STAGES, int NEPI, bool FA, bool AR>
 __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
     egemm_tc_kernel(const __grid_constant__ CUtensorMap tm_ahi,
                     const __grid_constant__ CUtensorMap tm_alo,
@@ -192,13 +192,21 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
                                              ~uintptr_t(1023));
+  // AR (A resident, kNN / kMeans with K <= 128): the A tile of a unit is loaded once into
+  // its own buffer and the ring carries only B; otherwise each stage holds A and B.
+  constexpr int SB = AR ? 2 * G::B_BYTES : G::STAGE_BYTES;  // bytes per ring stage
+  constexpr int B_OFF = AR ? 0 : 2 * G::A_BYTES;            // B_hi offset inside a stage
+  constexpr int AR_BYTES = AR ? 2 * 2 * G::A_BYTES : 0;     // 2 k-blocks of A_hi + A_lo
   uint8_t* stage_base = smem;
-  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + STAGES * G::STAGE_BYTES);
+  uint8_t* a_res = smem + STAGES * SB;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + STAGES * SB + AR_BYTES);
   uint64_t* full = bars;
   uint64_t* empty = bars + STAGES;
   uint64_t* acc_full = bars + 2 * STAGES;
   uint64_t* acc_empty = bars + 2 * STAGES + 2;
-  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * STAGES + 4);
+  uint64_t* a_full = bars + 2 * STAGES + 4;
+  uint64_t* a_empty = bars + 2 * STAGES + 5;
+  uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * STAGES + 6);
   uint8_t* scratch = reinterpret_cast<uint8_t*>(bars + 2 * STAGES + 8);  // epilogue merges
 
   const int warp = threadIdx.x >> 5;
@@ -226,6 +234,8 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
       ptx::mbar_init(&acc_full[b], 1);
       ptx::mbar_init(&acc_empty[b], NEPI * CG);  // one arrive per epilogue warp of the pair
     }
+    ptx::mbar_init(a_full, 1);
+    ptx::mbar_init(a_empty, 1);
     ptx::fence_mbar_init();
   }
   if (warp == EG::W_ALLOC) ptx::tmem_alloc<CG>(tmem_slot, TMEM_COLS);
@@ -309,16 +319,32 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
     if (lane == 0) {
       int stage = 0;
       uint32_t phase = 0;
-      // FA: only B comes through TMA (A is written by the converter warps)
-      constexpr uint32_t TX = FA ? 2 * G::B_BYTES : G::STAGE_BYTES;
-      for (int u = cluster; u < p.num_units; u += nclusters) {
+      // FA: only B comes through TMA (A is written by the converter warps); AR: the ring
+      // carries only B, A is loaded once per unit into a_res
+      constexpr uint32_t TX = (FA || AR) ? 2 * G::B_BYTES : G::STAGE_BYTES;
+      uint32_t uctr = 0;
+      for (int u = cluster; u < p.num_units; u += nclusters, uctr++) {
         UnitInfo ui = decode_unit<EPI>(p, u);
         const int arow = ui.m_tile * (kBM * CG) + (int)rank * kBM;
+        if constexpr (AR) {
+          ptx::mbar_wait(a_empty, (uctr & 1u) ^ 1u);  // the previous unit's MMAs are done
+          if (leader) ptx::mbar_arrive_expect_tx(a_full, 2 * G::A_BYTES * p.num_kb * CG);
+          for (int kb = 0; kb < p.num_kb; kb++) {
+            uint8_t* ab = a_res + kb * 2 * G::A_BYTES;
+            if constexpr (CG == 1) {
+              ptx::tma_load_2d(&tm_ahi, a_full, ab, kb * kBK, arow);
+              ptx::tma_load_2d(&tm_alo, a_full, ab + G::A_BYTES, kb * kBK, arow);
+            } else {
+              ptx::tma_load_2d_pair(&tm_ahi, a_full, ab, kb * kBK, arow);
+              ptx::tma_load_2d_pair(&tm_alo, a_full, ab + G::A_BYTES, kb * kBK, arow);
+            }
+          }
+        }
         for (int ns = 0; ns < ui.n_count; ns++) {
           const int brow = (ui.n_begin + ns) * BN + (int)rank * G::BNC;
           for (int kb = 0; kb < p.num_kb; kb++) {
             ptx::mbar_wait(&empty[stage], phase ^ 1u);
-            uint8_t* sb = stage_base + stage * G::STAGE_BYTES;
+            uint8_t* sb = stage_base + stage * SB;
             if (p.debug_no_tma) {  // diagnostics only: MMA-issue ceiling without operand traffic
               if (leader && !FA) ptx::mbar_arrive(&full[stage]);
               if (++stage == STAGES) { stage = 0; phase ^= 1u; }
@@ -327,20 +353,19 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
             if (leader) ptx::mbar_arrive_expect_tx(&full[stage], TX * CG);
             const int k0 = kb * kBK;
             if constexpr (CG == 1) {
-              if (!FA) {
+              if (!FA && !AR) {
                 ptx::tma_load_2d(&tm_ahi, &full[stage], sb, k0, arow);
                 ptx::tma_load_2d(&tm_alo, &full[stage], sb + G::A_BYTES, k0, arow);
               }
-              ptx::tma_load_2d(&tm_bhi, &full[stage], sb + 2 * G::A_BYTES, k0, brow);
-              ptx::tma_load_2d(&tm_blo, &full[stage], sb + 2 * G::A_BYTES + G::B_BYTES, k0, brow);
+              ptx::tma_load_2d(&tm_bhi, &full[stage], sb + B_OFF, k0, brow);
+              ptx::tma_load_2d(&tm_blo, &full[stage], sb + B_OFF + G::B_BYTES, k0, brow);
             } else {
-              if (!FA) {
+              if (!FA && !AR) {
                 ptx::tma_load_2d_pair(&tm_ahi, &full[stage], sb, k0, arow);
                 ptx::tma_load_2d_pair(&tm_alo, &full[stage], sb + G::A_BYTES, k0, arow);
               }
-              ptx::tma_load_2d_pair(&tm_bhi, &full[stage], sb + 2 * G::A_BYTES, k0, brow);
-              ptx::tma_load_2d_pair(&tm_blo, &full[stage], sb + 2 * G::A_BYTES + G::B_BYTES, k0,
-                                    brow);
+              ptx::tma_load_2d_pair(&tm_bhi, &full[stage], sb + B_OFF, k0, brow);
+              ptx::tma_load_2d_pair(&tm_blo, &full[stage], sb + B_OFF + G::B_BYTES, k0, brow);
             }
             if (++stage == STAGES) { stage = 0; phase ^= 1u; }
           }
@@ -357,8 +382,14 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
       int stage = 0;
       uint32_t phase = 0;
       uint32_t chunk_ctr = 0;
-      for (int u = cluster; u < p.num_units; u += nclusters) {
+      uint32_t uctr = 0;
+      const uint32_t abase = ptx::smem_u32(a_res);
+      for (int u = cluster; u < p.num_units; u += nclusters, uctr++) {
         UnitInfo ui = decode_unit<EPI>(p, u);
+        if constexpr (AR) {
+          ptx::mbar_wait(a_full, uctr & 1u);  // this unit's A tile is resident
+          ptx::tc_fence_after();
+        }
         for (int ns = 0; ns < ui.n_count; ns++) {
           for (int ch = 0; ch < nch; ch++) {
             const uint32_t buf = chunk_ctr & 1u;
@@ -372,11 +403,12 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
             for (int kb = kb0; kb < kb1; kb++) {
               ptx::mbar_wait(&full[stage], phase);
               ptx::tc_fence_after();
-              const uint32_t sa = sbase + stage * G::STAGE_BYTES;
-              const uint64_t d_ahi = ptx::sdesc_kmajor_sw128(sa);
-              const uint64_t d_alo = ptx::sdesc_kmajor_sw128(sa + G::A_BYTES);
-              const uint64_t d_bhi = ptx::sdesc_kmajor_sw128(sa + 2 * G::A_BYTES);
-              const uint64_t d_blo = ptx::sdesc_kmajor_sw128(sa + 2 * G::A_BYTES + G::B_BYTES);
+              const uint32_t sa = sbase + stage * SB;
+              const uint32_t aa = AR ? abase + kb * 2 * G::A_BYTES : sa;
+              const uint64_t d_ahi = ptx::sdesc_kmajor_sw128(aa);
+              const uint64_t d_alo = ptx::sdesc_kmajor_sw128(aa + G::A_BYTES);
+              const uint64_t d_bhi = ptx::sdesc_kmajor_sw128(sa + B_OFF);
+              const uint64_t d_blo = ptx::sdesc_kmajor_sw128(sa + B_OFF + G::B_BYTES);
               // Alg. 1 order: the products involving lo first, hi*hi last --
               // here per 64-wide k-block: all cross MMAs, then all hi*hi MMAs.  With one
               // accumulator this keeps |acc| ~2^-11 smaller while the cross terms are
@@ -407,6 +439,10 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
             __syncwarp();
             chunk_ctr++;
           }
+        }
+        if constexpr (AR) {  // the resident A tile is free once this unit's MMAs complete
+          if (ptx::elect_one()) ptx::mma_commit<CG>(a_empty);
+          __syncwarp();
         }
       }
     }
@@ -693,15 +729,17 @@ static bool make_tmap_f16(CUtensorMap* m, const void* base, int64_t rows, int64_
   return r == CUDA_SUCCESS;
 }
 
-template <int CG, int BN, bool SEP, int EPI, int STAGES, bool FA = false>
+template <int CG, int BN, bool SEP, int EPI, int STAGES, bool FA = false, bool AR = false>
 static int launch_variant(const CUtensorMap* maps, const KParams& kp, int max_clusters,
                           cudaStream_t stream) {
   using G = Geo<CG, BN>;
   // kMeans' argmin epilogue is issue-bound next to a 64-deep k-loop: 16 epilogue warps
   constexpr int NEPI = (EPI == EPI_KMEANS) ? 16 : 8;
-  auto kern = egemm_tc_kernel<CG, BN, SEP, EPI, STAGES, NEPI, FA>;
+  auto kern = egemm_tc_kernel<CG, BN, SEP, EPI, STAGES, NEPI, FA, AR>;
   const int scratch = EPI == EPI_KNN ? kBM * kKnnMax * 8 : EPI == EPI_KMEANS ? 2 * 4 * kBM * 4 : 0;
-  const size_t smem = 1024 + (size_t)STAGES * G::STAGE_BYTES + 8 * (2 * STAGES + 8) + scratch;
+  const size_t sb = AR ? 2 * G::B_BYTES : G::STAGE_BYTES;
+  const size_t smem = 1024 + (size_t)STAGES * sb + (AR ? 4 * G::A_BYTES : 0) +
+                      8 * (2 * STAGES + 8) + scratch;
   static bool attr_done = false;  // per instantiation
   if (!attr_done) {
     if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
@@ -736,6 +774,11 @@ static int launch_variant(const CUtensorMap* maps, const KParams& kp, int max_cl
   return 0;
 }
 
+static bool getenv_flag(const char* name) {
+  const char* v = getenv(name);
+  return v && v[0] == '1';
+}
+
 template <int EPI>
 static int dispatch(const CUtensorMap* maps, const KParams& kp, const TcConfig& cfg,
                     cudaStream_t s) {
@@ -751,6 +794,11 @@ static int dispatch(const CUtensorMap* maps, const KParams& kp, const TcConfig& 
                      cfg.sep);
       return 2;
     }
+  } else {
+    // kNN / kMeans with K <= 128: the unit's A tile stays resident (halves L2->smem traffic)
+    if (kp.num_kb <= 2 && cfg.cg == 2 && cfg.bn == 256 && !cfg.sep && !kp.debug_no_tma &&
+        !getenv_flag("EGEMM_NO_ARES"))
+      return launch_variant<2, 256, false, EPI, 4, false, true>(maps, kp, cfg.max_clusters, s);
   }
   if (cfg.cg == 2 && cfg.bn == 256 && !cfg.sep)
     return launch_variant<2, 256, false, EPI, 3>(maps, kp, cfg.max_clusters, s);
