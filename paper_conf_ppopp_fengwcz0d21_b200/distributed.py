@@ -87,6 +87,41 @@ def merge_topk(keys: torch.Tensor, idx: torch.Tensor, k: int):
     return torch.gather(kcat, 1, o2)[:, :k], torch.gather(icat, 1, o2)[:, :k]
 
 
+def knn_references_sharded(X_local: torch.Tensor, x_offset: int, Q: torch.Tensor, k: int,
+                           world: int | None = None, knn_fn=None, **kw):
+    """NEXT-4: kNN with the REFERENCES sharded over ranks (X too big for one GPU); every
+    rank holds all queries Q.  Local top-k of this rank's rows X_local (global row ids
+    x_offset + j) -> all_gather of the [nq, k] (dist, id) lists -> merge by (dist, id).
+    Exchange: 8 * nq * k bytes per rank (tiny next to the GEMM).  ``knn_fn(X, Q, k)`` ->
+    (idx, dist) defaults to egemm.knn; shards with fewer than k rows pad with (+inf, -1).
+    Returns (idx int64 [nq, k], dist fp32 [nq, k]), identical on every rank."""
+    world = world if world is not None else world_size()
+    nq = Q.shape[0]
+    if knn_fn is None:
+        from . import egemm
+        knn_fn = lambda X_, Q_, k_: egemm.knn(X_, Q_, k_, **kw)  # noqa: E731
+    kl = min(k, X_local.shape[0])
+    idx, dst = knn_fn(X_local, Q, kl) if kl > 0 else (None, None)
+    keys = torch.full((nq, k), float("inf"), dtype=dst.dtype if kl > 0 else torch.float32,
+                      device=Q.device)
+    ids = torch.full((nq, k), -1, dtype=torch.int64, device=Q.device)
+    if kl > 0:
+        keys[:, :kl] = dst
+        ids[:, :kl] = idx.long() + x_offset
+    if world > 1:
+        kp = [torch.empty_like(keys) for _ in range(world)]
+        ip = [torch.empty_like(ids) for _ in range(world)]
+        dist.all_gather(kp, keys)
+        dist.all_gather(ip, ids)
+        keys, ids = torch.stack(kp), torch.stack(ip)
+    else:
+        keys, ids = keys[None], ids[None]
+    # padding (+inf, -1) must sort after every real candidate: map -1 to the largest id
+    ids = torch.where(ids < 0, torch.iinfo(torch.int64).max, ids)
+    mk, mi = merge_topk(keys, ids, k)
+    return torch.where(mi == torch.iinfo(torch.int64).max, -1, mi), mk
+
+
 def kmeans_fit(X: torch.Tensor, C: torch.Tensor, iters: int, x_split=None, workspace=None,
                bufs=None, world: int | None = None, step=None, finalize=None):
     """Lloyd iterations on this rank's points X with replicated centroids C (updated in

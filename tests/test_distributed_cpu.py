@@ -121,3 +121,46 @@ def test_kmeans_fit_allreduce_equals_single_process(oracle_lib):
         C = oracle_lib.kmeans_finalize(s, c, C)
     # sums were reduced across ranks in another fp64 order: <= 1 ulp of fp32 (R20 note)
     assert np.allclose(out[0], C, rtol=2.0 ** -23, atol=2.0 ** -30)
+
+
+def _knn_sharded_ranks(rank, world):
+    import oracle
+    X, _, _ = inputs.mixture(3001, 16, 12, 21, sigma=0.2)
+    Q = torch.from_numpy(inputs.uniform((40, 16), 22))
+    lo, hi = edist.shard_bounds(3001, world, rank)
+
+    def knn_fn(X_, Q_, k_):
+        i, d = oracle.knn(X_.numpy(), Q_.numpy(), k_)
+        return torch.from_numpy(i), torch.from_numpy(d)
+
+    i, d = edist.knn_references_sharded(torch.from_numpy(X[lo:hi].copy()), lo, Q, 16,
+                                        world=world, knn_fn=knn_fn)
+    return i.numpy(), d.numpy()
+
+
+def test_knn_references_sharded_equals_single_process(oracle_lib):
+    """NEXT-4: references sharded over 2 ranks + all_gather merge == unsharded exact kNN
+    (fp64 keys: (dist, id) is a total order, so the result is unique)."""
+    out = _run(_knn_sharded_ranks)
+    assert np.array_equal(out[0][0], out[1][0]) and np.array_equal(out[0][1], out[1][1])
+    X, _, _ = inputs.mixture(3001, 16, 12, 21, sigma=0.2)
+    ri, rd = oracle_lib.knn(X, inputs.uniform((40, 16), 22), 16)
+    assert np.array_equal(out[0][0], ri) and np.array_equal(out[0][1], rd)
+
+
+def test_knn_references_sharded_small_shards():
+    """Shards with fewer than k rows pad with (+inf, -1) and never displace real rows."""
+    X = torch.tensor([[0.0], [1.0], [2.0]])
+    Q = torch.tensor([[0.9]])
+
+    def knn_fn(X_, Q_, k_):
+        d = ((X_[None, :, 0] - Q_[:, None, 0]) ** 2).double()
+        dd, ii = torch.sort(d, dim=1, stable=True)
+        return ii[:, :k_], dd[:, :k_]
+
+    parts = [edist.knn_references_sharded(X[a:b], a, Q, 2, world=1, knn_fn=knn_fn)
+             for a, b in ((0, 1), (1, 3))]
+    i0, d0 = parts[0]
+    assert i0.tolist() == [[0, -1]] and d0[0, 1].item() == float("inf")
+    i1, _ = parts[1]
+    assert i1.tolist() == [[1, 2]]

@@ -58,6 +58,25 @@ def test_knn_clustered_and_presplit(oracle_lib):
     assert torch.equal(idx, idx3) and torch.equal(dist, dist3)
 
 
+def test_knn_references_sharded(oracle_lib):
+    """NEXT-4: references split into 3 shards (egemm_knn per shard, ids offset) merged by
+    (dist, id) == the kNN rule against the fp64 oracle over all of X."""
+    from paper_conf_ppopp_fengwcz0d21_b200 import distributed as edist
+    eg = require_gpu()
+    X, Q = inputs.uniform((4100, 96), 60), inputs.uniform((300, 96), 61)
+    Xd, Qd = to_dev(X), to_dev(Q)
+    cuts = [0, 1000, 1010, 4100]  # a shard with fewer than k rows included
+    keys, ids = [], []
+    for a, b in zip(cuts[:-1], cuts[1:]):
+        i, d = edist.knn_references_sharded(Xd[a:b], a, Qd, 16, world=1)
+        ids.append(i)
+        keys.append(d)
+    mk, mi = edist.merge_topk(torch.stack(keys), torch.where(torch.stack(ids) < 0, 1 << 62,
+                                                            torch.stack(ids)), 16)
+    ex = _knn_check(oracle_lib, X, Q, 16, to_host(mi), to_host(mk))
+    assert ex <= 300 // 50
+
+
 def test_knn_self_match_and_duplicates():
     eg = require_gpu()
     X = inputs.uniform((1000, 32), 42)

@@ -53,6 +53,14 @@ def test_16384_cube_sampled(oracle_lib):
     _gemm_sampled(oracle_lib, 16384, 16384, 16384, 115, 215, 16)
 
 
+@pytest.mark.parametrize("shape", [(4096, 4096, 8192), (16384, 4096, 4096), (2048, 2048, 4096),
+                                   (8192, 2048, 2048)])
+def test_skewed_fig9_sampled(oracle_lib, shape):
+    """NEXT-2: Fig. 9's skewed shapes (N, N, 2N) and (4N, N, N), public call."""
+    M, N, K = shape
+    _gemm_sampled(oracle_lib, M, N, K, 300 + M.bit_length(), 400 + K.bit_length(), 32)
+
+
 def test_tall_skinny_full(oracle_lib):
     """configs[2]: M=65536 N=256 K=1024, all rows against the fp64 oracle."""
     _gemm_sampled(oracle_lib, 65536, 256, 1024, 200, 201, 65536)
