@@ -72,6 +72,7 @@ struct KParams {
   int vec_a;
   int K;
   int debug_no_tma;  // EGEMM_DEBUG_NO_TMA=1: skip operand loads (timing diagnostics only)
+  int debug_no_epi;  // EGEMM_DEBUG_NO_EPI=1: skip the promotion's TMEM reads (diagnostics)
 };
 
 template <int CG, int BN>
@@ -488,6 +489,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
             ptx::mbar_wait(&acc_full[buf], use & 1u);
             ptx::tc_fence_after();
             const uint32_t acc_hh = tmem_base + lane_off + (SEP ? 2 * buf : buf) * BN + cgp * COLS;
+            if (!p.debug_no_epi)
 #pragma unroll
             for (int c = 0; c < COLS / 32; c++) {
               float v[32];
@@ -841,6 +843,7 @@ int launch_tc(int64_t M, int64_t N, int64_t K, const TcOperands& ops, const TcCo
   {
     const char* dbg = getenv("EGEMM_DEBUG_NO_TMA");
     kp.debug_no_tma = (dbg && dbg[0] == '1') ? 1 : 0;
+    kp.debug_no_epi = getenv_flag("EGEMM_DEBUG_NO_EPI") ? 1 : 0;
   }
   if (fa) {
     kp.a_f32 = ops.a_f32;

@@ -1,0 +1,119 @@
+"""Where does the GEMM kernel lose MMA-pipe time?  Runs the 8192^3 pre-split GEMM under
+diagnostic switches (EGEMM_DEBUG_NO_TMA: no operand loads; EGEMM_DEBUG_NO_EPI: no promotion
+TMEM reads) and chunk sizes, each with the in-kernel SM-clock probe, and cuBLAS fp16 at the
+same size with nvidia-smi clocks sampled during a long loop.  Tool code (diagnostics only).
+
+usage: python tools/diag_gemm.py [n]
+"""
+import os
+import subprocess
+import sys
+import threading
+
+import torch
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+from paper_conf_ppopp_fengwcz0d21_b200 import egemm  # noqa: E402
+
+
+def timeit(fn, iters=20, warm=5):
+    for _ in range(warm):
+        fn()
+    torch.cuda.synchronize()
+    s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    s.record()
+    for _ in range(iters):
+        fn()
+    e.record()
+    e.synchronize()
+    return s.elapsed_time(e) / iters
+
+
+def smi_clock_during(fn, seconds=2.0):
+    samples, stop = [], threading.Event()
+
+    def poll():
+        while not stop.is_set():
+            try:
+                o = subprocess.run(["nvidia-smi", "--query-gpu=clocks.sm,power.draw",
+                                    "--format=csv,noheader,nounits", "-i", "0"],
+                                   capture_output=True, text=True, timeout=5).stdout
+                a, b = o.strip().split(",")
+                samples.append((float(a), float(b)))
+            except Exception:
+                pass
+            stop.wait(0.05)
+
+    t = threading.Thread(target=poll)
+    t.start()
+    import time
+    t0 = time.time()
+    n = 0
+    while time.time() - t0 < seconds:
+        fn()
+        n += 1
+        if n % 10 == 0:
+            torch.cuda.synchronize()
+    torch.cuda.synchronize()
+    stop.set()
+    t.join()
+    samples = samples[len(samples) // 4:]
+    if not samples:
+        return None, None
+    mh = sorted(s[0] for s in samples)[len(samples) // 2]
+    pw = sorted(s[1] for s in samples)[len(samples) // 2]
+    return mh, pw
+
+
+def main():
+    n = int(sys.argv[1]) if len(sys.argv) > 1 else 8192
+    A = torch.rand(n, n, device="cuda") * 2 - 1
+    B = torch.rand(n, n, device="cuda") * 2 - 1
+    a_s, b_s = egemm.split(A), egemm.split(B, transpose=True)
+    D = torch.empty(n, n, device="cuda")
+    fl3 = 3 * 2.0 * n ** 3
+
+    def run(tag, cfg, env):
+        for k in ("EGEMM_DEBUG_NO_TMA", "EGEMM_DEBUG_NO_EPI"):
+            os.environ.pop(k, None)
+        os.environ.update(env)
+        egemm.set_config(*cfg)
+        f = lambda: egemm.gemm(None, None, a_split=a_s, b_split=b_s, out=D)  # noqa: E731
+        ms = timeit(f)
+        mhz = egemm.debug_last_clock()
+        smi, pw = smi_clock_during(f, 1.5)
+        tf = fl3 / ms / 1e9
+        peak = 148 * 8192 * mhz * 1e6 / 1e12
+        print("%-28s cfg %-18s %.3f ms  %.0f TF(fp16)  kernel %.0f MHz -> %.3f of clock peak | "
+              "smi %s MHz %s W" % (tag, cfg, ms, tf, mhz, tf / peak, smi, pw), flush=True)
+
+    for cfg in ((2, 256, 0, 128), (2, 256, 0, 64), (2, 256, 0, 256), (2, 256, 0, n)):
+        run("normal", cfg, {})
+    cfg = (2, 256, 0, 128)
+    run("no_tma", cfg, {"EGEMM_DEBUG_NO_TMA": "1"})
+    run("no_epi", cfg, {"EGEMM_DEBUG_NO_EPI": "1"})
+    run("no_tma+no_epi", cfg, {"EGEMM_DEBUG_NO_TMA": "1", "EGEMM_DEBUG_NO_EPI": "1"})
+    run("no_tma+no_epi kc=n", (2, 256, 0, n), {"EGEMM_DEBUG_NO_TMA": "1", "EGEMM_DEBUG_NO_EPI": "1"})
+    for k in ("EGEMM_DEBUG_NO_TMA", "EGEMM_DEBUG_NO_EPI"):
+        os.environ.pop(k, None)
+    egemm.set_config(0, 0, 0, 0)
+    Ah, Bh = A.half(), B.half()
+    f = lambda: torch.matmul(Ah, Bh)  # noqa: E731
+    ms = timeit(f)
+    smi, pw = smi_clock_during(f, 1.5)
+    tf = 2.0 * n ** 3 / ms / 1e9
+    print("cublas fp16 %d^3: %.3f ms  %.0f TF | smi %s MHz %s W -> %.3f of smi-clock peak"
+          % (n, ms, tf, smi, pw, tf / (148 * 8192 * smi * 1e6 / 1e12) if smi else 0), flush=True)
+    Ahh = torch.cat([Ah, Ah, Ah], 1)  # K = 3n: the same MMA count as one EGEMM launch
+    Bhh = torch.cat([Bh, Bh, Bh], 0)
+    f = lambda: torch.matmul(Ahh, Bhh)  # noqa: E731
+    ms = timeit(f, 10, 3)
+    smi, pw = smi_clock_during(f, 1.5)
+    tf = 2.0 * n * n * 3 * n / ms / 1e9
+    print("cublas fp16 %dx%dx%d: %.3f ms  %.0f TF | smi %s MHz %s W -> %.3f of smi-clock peak"
+          % (n, n, 3 * n, ms, tf, smi, pw, tf / (148 * 8192 * smi * 1e6 / 1e12) if smi else 0),
+          flush=True)
+
+
+if __name__ == "__main__":
+    main()

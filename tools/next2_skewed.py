@@ -21,8 +21,14 @@ import json
 import os
 import sys
 
-import numpy as np
-import torch
+# cuBLAS 12.9 (system) has the BF16x9 compute type; torch bundles 12.8.  Load the system
+# libraries first (same sonames) so torch and this tool share one cuBLAS 12.9.
+_CUDA_LIB = "/usr/local/cuda/lib64"
+for _so in ("libcublasLt.so.12", "libcublas.so.12"):
+    ctypes.CDLL(os.path.join(_CUDA_LIB, _so), mode=ctypes.RTLD_GLOBAL)
+
+import numpy as np  # noqa: E402
+import torch  # noqa: E402
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
@@ -39,7 +45,7 @@ class Cublas:
     column-major D^T = B^T A^T)."""
 
     def __init__(self):
-        self.L = ctypes.CDLL("/usr/local/cuda/lib64/libcublas.so.12")
+        self.L = ctypes.CDLL(os.path.join(_CUDA_LIB, "libcublas.so.12"))
         self.h = ctypes.c_void_p()
         assert self.L.cublasCreate_v2(ctypes.byref(self.h)) == 0
         self.L.cublasGemmEx.argtypes = [ctypes.c_void_p, ctypes.c_int, ctypes.c_int,
@@ -49,6 +55,9 @@ class Cublas:
                                         ctypes.c_int, ctypes.c_void_p, ctypes.c_void_p,
                                         ctypes.c_int, ctypes.c_int, ctypes.c_int, ctypes.c_int]
         self.L.cublasSetStream_v2(self.h, ctypes.c_void_p(torch.cuda.current_stream().cuda_stream))
+        v = ctypes.c_int()
+        self.L.cublasGetVersion_v2(self.h, ctypes.byref(v))
+        self.version = v.value
 
     def gemm(self, A, B, D, beta=0.0, compute=COMPUTE_32F):
         M, K = A.shape
@@ -128,7 +137,7 @@ def run_shape(cb, M, N, K, sample=64):
 def main():
     ns = [int(a) for a in sys.argv[1:]] or [1024, 2048, 4096, 8192]
     cb = Cublas()
-    out = {"what": "Fig. 9 skewed shapes (P:2002-2081) + Table 5 vendor baselines on one B200; "
+    out = {"cublas_version": cb.version, "what": "Fig. 9 skewed shapes (P:2002-2081) + Table 5 vendor baselines on one B200; "
                    "TFLOP/s = 2MNK / time, splits included; normwise error vs fp64 on 64 rows",
            "shapes": []}
     for n in ns:
