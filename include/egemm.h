@@ -183,6 +183,11 @@ int egemm_num_sms(void);
  * from clock64 / %globaltimer.  Synchronous (copies a device symbol). */
 int egemm_debug_last_clock(double* mhz);
 
+/* Debug: running sums of the same probe over every tensor-core launch since the last
+ * reset: mean SM clock (MHz), CTA-0 SM cycles per launch (clock-independent kernel cost),
+ * number of launches.  reset != 0 zeroes the sums after reading.  Synchronous. */
+int egemm_debug_clock_stats(double* mhz, double* cycles_per_launch, double* launches, int reset);
+
 #ifdef __cplusplus
 }
 #endif

@@ -211,6 +211,11 @@ int egemm_debug_last_clock(double* mhz) {
   return read_clock_probe(mhz) ? EGEMM_ERR_CUDA : EGEMM_OK;
 }
 
+int egemm_debug_clock_stats(double* mhz, double* cycles_per_launch, double* launches, int reset) {
+  if (!mhz || !cycles_per_launch || !launches) return EGEMM_ERR_INVALID_ARG;
+  return read_clock_stats(mhz, cycles_per_launch, launches, reset) ? EGEMM_ERR_CUDA : EGEMM_OK;
+}
+
 int egemm_set_config(int cg, int bn, int sep, int kc) {
   if (cg == 0 && bn == 0 && sep == 0 && kc == 0) {
     g_override = Override();

@@ -78,6 +78,7 @@ int launch_fill_c(int64_t M, int64_t N, const float* C, int64_t ldc, float* D, i
 
 void set_last_error(const char* fmt, ...);
 int read_clock_probe(double* mhz);
+int read_clock_stats(double* mhz, double* cycles_per_launch, double* launches, int reset);
 
 // tune.cu: the measured configuration table
 bool tune_lookup(int op, long long M, long long N, long long K, int* cg, int* bn, int* sep,

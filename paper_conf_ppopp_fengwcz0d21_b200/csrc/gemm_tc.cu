@@ -34,7 +34,7 @@
 
 namespace egemm {
 
-__device__ unsigned long long g_clock_probe[4];
+__device__ unsigned long long g_clock_probe[8];  // [0..3] last launch, [4..6] running sums
 
 __device__ __forceinline__ unsigned long long globaltimer_ns() {
   unsigned long long t;
@@ -688,16 +688,36 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
     ptx::tmem_dealloc<CG>(tmem_base, TMEM_COLS);
   }
   if (blockIdx.x == 0 && threadIdx.x == 0) {
-    g_clock_probe[2] = clock64();
-    g_clock_probe[3] = globaltimer_ns();
+    const unsigned long long c1 = clock64(), t1 = globaltimer_ns();
+    g_clock_probe[2] = c1;
+    g_clock_probe[3] = t1;
+    g_clock_probe[4] += c1 - g_clock_probe[0];
+    g_clock_probe[5] += t1 - g_clock_probe[1];
+    g_clock_probe[6] += 1;
   }
 }
 
 // SM cycles / wall ns of CTA 0 over the last launch (debug: effective SM clock).
 int read_clock_probe(double* mhz) {
-  unsigned long long h[4];
+  unsigned long long h[8];
   if (cudaMemcpyFromSymbol(h, g_clock_probe, sizeof(h)) != cudaSuccess) return 3;
   *mhz = (h[3] > h[1]) ? (double)(h[2] - h[0]) * 1e3 / (double)(h[3] - h[1]) : 0.0;
+  return 0;
+}
+
+// Running sums since the last reset: mean SM clock and CTA-0 cycles per launch.
+int read_clock_stats(double* mhz, double* cycles_per_launch, double* launches, int reset) {
+  unsigned long long h[8];
+  if (cudaMemcpyFromSymbol(h, g_clock_probe, sizeof(h)) != cudaSuccess) return 3;
+  *mhz = h[5] ? (double)h[4] * 1e3 / (double)h[5] : 0.0;
+  *cycles_per_launch = h[6] ? (double)h[4] / (double)h[6] : 0.0;
+  *launches = (double)h[6];
+  if (reset) {
+    unsigned long long z[3] = {0, 0, 0};
+    if (cudaMemcpyToSymbol(g_clock_probe, z, sizeof(z), 4 * sizeof(unsigned long long)) !=
+        cudaSuccess)
+      return 3;
+  }
   return 0;
 }
 

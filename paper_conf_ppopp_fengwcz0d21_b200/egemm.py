@@ -38,6 +38,7 @@ EXPORTS = ["egemm_status_string", "egemm_last_error", "egemm_version", "egemm_sp
            "egemm_gemm_workspace_size", "egemm_knn", "egemm_knn_workspace_size", "egemm_knn_index",
            "egemm_kmeans_step", "egemm_kmeans_workspace_size", "egemm_kmeans_finalize",
            "egemm_set_config", "egemm_num_sms", "egemm_debug_last_clock", "egemm_tune_table",
+           "egemm_debug_clock_stats",
            "egemm_query_config", "egemm_gemm_host", "egemm_gemm_host_workspace_size"]
 
 _lib = None
@@ -82,6 +83,9 @@ def load(path: str = LIB_PATH):
     L.egemm_num_sms.restype = I
     L.egemm_debug_last_clock.argtypes = [ctypes.POINTER(ctypes.c_double)]
     L.egemm_debug_last_clock.restype = I
+    DP = ctypes.POINTER(ctypes.c_double)
+    L.egemm_debug_clock_stats.argtypes = [DP, DP, DP, I]
+    L.egemm_debug_clock_stats.restype = I
     L.egemm_gemm_host.argtypes = [I64, I64, I64, P, I64, P, I64, P, I64, I, P, SZ, P]
     L.egemm_gemm_host.restype = I
     L.egemm_gemm_host_workspace_size.argtypes = [I64, I64, I64]
@@ -110,6 +114,15 @@ def query_config(op: str, M: int, N: int, K: int, with_fused: bool = False):
                                      *[ctypes.byref(x) for x in v]), "egemm_query_config")
     out = tuple(x.value for x in v)
     return out if with_fused else out[:4]
+
+
+def debug_clock_stats(reset: bool = True):
+    """(mean SM MHz, CTA-0 cycles per launch, launches) over the tensor-core launches since
+    the last reset (synchronous; debug)."""
+    v = [ctypes.c_double(0.0) for _ in range(3)]
+    _check(load().egemm_debug_clock_stats(*[ctypes.byref(x) for x in v], int(reset)),
+           "egemm_debug_clock_stats")
+    return tuple(x.value for x in v)
 
 
 def debug_last_clock() -> float:

@@ -73,27 +73,43 @@ def main():
     D = torch.empty(n, n, device="cuda")
     fl3 = 3 * 2.0 * n ** 3
 
-    def run(tag, cfg, env):
+    need = fl3 / (148 * 8192.0)  # SM cycles of pure MMA issue per launch at the dense peak
+
+    def run(tag, cfg, env, seconds=1.5):
         for k in ("EGEMM_DEBUG_NO_TMA", "EGEMM_DEBUG_NO_EPI"):
             os.environ.pop(k, None)
         os.environ.update(env)
         egemm.set_config(*cfg)
         f = lambda: egemm.gemm(None, None, a_split=a_s, b_split=b_s, out=D)  # noqa: E731
-        ms = timeit(f)
-        mhz = egemm.debug_last_clock()
-        smi, pw = smi_clock_during(f, 1.5)
+        timeit(f, 5, 5)
+        egemm.debug_clock_stats(reset=True)
+        import time
+        s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        torch.cuda.synchronize()
+        s.record()
+        t0, it = time.time(), 0
+        while time.time() - t0 < seconds:
+            for _ in range(10):
+                f()
+            it += 10
+            torch.cuda.synchronize()
+        e.record()
+        e.synchronize()
+        ms = s.elapsed_time(e) / it
+        mhz, cyc, nl = egemm.debug_clock_stats(reset=True)
         tf = fl3 / ms / 1e9
-        peak = 148 * 8192 * mhz * 1e6 / 1e12
-        print("%-28s cfg %-18s %.3f ms  %.0f TF(fp16)  kernel %.0f MHz -> %.3f of clock peak | "
-              "smi %s MHz %s W" % (tag, cfg, ms, tf, mhz, tf / peak, smi, pw), flush=True)
+        print("%-22s cfg %-18s %.3f ms  %.0f TF(fp16)  mean %.0f MHz  %.0f kcyc/launch -> "
+              "cycle efficiency %.3f" % (tag, cfg, ms, tf, mhz, cyc / 1e3, need / cyc), flush=True)
 
-    for cfg in ((2, 256, 0, 128), (2, 256, 0, 64), (2, 256, 0, 256), (2, 256, 0, n)):
-        run("normal", cfg, {})
-    cfg = (2, 256, 0, 128)
-    run("no_tma", cfg, {"EGEMM_DEBUG_NO_TMA": "1"})
-    run("no_epi", cfg, {"EGEMM_DEBUG_NO_EPI": "1"})
-    run("no_tma+no_epi", cfg, {"EGEMM_DEBUG_NO_TMA": "1", "EGEMM_DEBUG_NO_EPI": "1"})
-    run("no_tma+no_epi kc=n", (2, 256, 0, n), {"EGEMM_DEBUG_NO_TMA": "1", "EGEMM_DEBUG_NO_EPI": "1"})
+    for rep in range(2):
+        for cfg in ((2, 256, 0, 128), (2, 256, 0, 64), (2, 256, 0, 256), (2, 256, 0, n)):
+            run("normal", cfg, {})
+        cfg = (2, 256, 0, 128)
+        run("no_tma", cfg, {"EGEMM_DEBUG_NO_TMA": "1"})
+        run("no_epi", cfg, {"EGEMM_DEBUG_NO_EPI": "1"})
+        run("no_tma+no_epi", cfg, {"EGEMM_DEBUG_NO_TMA": "1", "EGEMM_DEBUG_NO_EPI": "1"})
+        run("no_tma+no_epi kc=n", (2, 256, 0, n), {"EGEMM_DEBUG_NO_TMA": "1",
+                                                   "EGEMM_DEBUG_NO_EPI": "1"})
     for k in ("EGEMM_DEBUG_NO_TMA", "EGEMM_DEBUG_NO_EPI"):
         os.environ.pop(k, None)
     egemm.set_config(0, 0, 0, 0)
