@@ -65,6 +65,43 @@ def smi_clock_during(fn, seconds=2.0):
     return mh, pw
 
 
+_spin = None
+
+
+def spin_mhz(fn, ms=1500.0):
+    """SM clock (MHz) seen by a 1-warp spin kernel co-resident with fn() looping for ms."""
+    global _spin
+    import ctypes
+    import time
+    if _spin is None:
+        so = os.path.join("gpurun_out", "clockspin.so")
+        src = os.path.join(os.path.dirname(os.path.abspath(__file__)), "csrc", "clockspin.cu")
+        subprocess.run(["nvcc", "-gencode", "arch=compute_100a,code=sm_100a", "-O2", "-shared",
+                        "-Xcompiler", "-fPIC", "-o", so, src], check=True)
+        _spin = ctypes.CDLL(os.path.abspath(so))
+        _spin.clockspin_launch.argtypes = [ctypes.c_double, ctypes.c_void_p]
+        _spin.clockspin_read.argtypes = [ctypes.POINTER(ctypes.c_double)]
+    for _ in range(3):
+        fn()
+    side = torch.cuda.Stream()
+    torch.cuda.synchronize()
+    _spin.clockspin_launch(ms, ctypes.c_void_p(side.cuda_stream))
+    t0, it = time.time(), 0
+    s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    s.record()
+    while time.time() - t0 < ms / 1e3 + 0.2:
+        for _ in range(5):
+            fn()
+        it += 5
+        torch.cuda.synchronize()
+    e.record()
+    e.synchronize()
+    torch.cuda.synchronize()
+    v = ctypes.c_double(0.0)
+    _spin.clockspin_read(ctypes.byref(v))
+    return v.value, s.elapsed_time(e) / it
+
+
 def main():
     n = int(sys.argv[1]) if len(sys.argv) > 1 else 8192
     A = torch.rand(n, n, device="cuda") * 2 - 1
@@ -114,21 +151,18 @@ def main():
         os.environ.pop(k, None)
     egemm.set_config(0, 0, 0, 0)
     Ah, Bh = A.half(), B.half()
-    f = lambda: torch.matmul(Ah, Bh)  # noqa: E731
-    ms = timeit(f)
-    smi, pw = smi_clock_during(f, 1.5)
-    tf = 2.0 * n ** 3 / ms / 1e9
-    print("cublas fp16 %d^3: %.3f ms  %.0f TF | smi %s MHz %s W -> %.3f of smi-clock peak"
-          % (n, ms, tf, smi, pw, tf / (148 * 8192 * smi * 1e6 / 1e12) if smi else 0), flush=True)
     Ahh = torch.cat([Ah, Ah, Ah], 1)  # K = 3n: the same MMA count as one EGEMM launch
     Bhh = torch.cat([Bh, Bh, Bh], 0)
-    f = lambda: torch.matmul(Ahh, Bhh)  # noqa: E731
-    ms = timeit(f, 10, 3)
-    smi, pw = smi_clock_during(f, 1.5)
-    tf = 2.0 * n * n * 3 * n / ms / 1e9
-    print("cublas fp16 %dx%dx%d: %.3f ms  %.0f TF | smi %s MHz %s W -> %.3f of smi-clock peak"
-          % (n, n, 3 * n, ms, tf, smi, pw, tf / (148 * 8192 * smi * 1e6 / 1e12) if smi else 0),
-          flush=True)
+    for tag, f, fl in (("cublas fp16 n^3", lambda: torch.matmul(Ah, Bh), 2.0 * n ** 3),
+                       ("cublas fp16 n x n x 3n", lambda: torch.matmul(Ahh, Bhh), fl3),
+                       ("egemm (2,256,0,128)", None, fl3)):
+        if f is None:
+            egemm.set_config(2, 256, 0, 128)
+            f = lambda: egemm.gemm(None, None, a_split=a_s, b_split=b_s, out=D)  # noqa: E731
+        mhz, ms = spin_mhz(f)
+        tf = fl / ms / 1e9
+        print("%-24s %.3f ms  %.0f TF | spin-probe SM clock %.0f MHz -> cycle efficiency %.3f"
+              % (tag, ms, tf, mhz, tf / (148 * 8192 * mhz * 1e6 / 1e12)), flush=True)
 
 
 if __name__ == "__main__":
