@@ -81,21 +81,23 @@ def spin_mhz(fn, ms=1500.0):
         _spin = ctypes.CDLL(os.path.abspath(so))
         _spin.clockspin_launch.argtypes = [ctypes.c_double, ctypes.c_void_p]
         _spin.clockspin_read.argtypes = [ctypes.POINTER(ctypes.c_double)]
-    for _ in range(3):
-        fn()
-    side = torch.cuda.Stream()
-    torch.cuda.synchronize()
-    _spin.clockspin_launch(ms, ctypes.c_void_p(side.cuda_stream))
-    t0, it = time.time(), 0
-    s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
-    s.record()
-    while time.time() - t0 < ms / 1e3 + 0.2:
-        for _ in range(5):
+    # both on non-default streams: the legacy default stream would serialise them
+    side, work = torch.cuda.Stream(), torch.cuda.Stream()
+    with torch.cuda.stream(work):
+        for _ in range(3):
             fn()
-        it += 5
         torch.cuda.synchronize()
-    e.record()
-    e.synchronize()
+        _spin.clockspin_launch(ms, ctypes.c_void_p(side.cuda_stream))
+        t0, it = time.time(), 0
+        s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        s.record()
+        while time.time() - t0 < ms / 1e3 - 0.2:
+            for _ in range(5):
+                fn()
+            it += 5
+            work.synchronize()
+        e.record()
+        e.synchronize()
     torch.cuda.synchronize()
     v = ctypes.c_double(0.0)
     _spin.clockspin_read(ctypes.byref(v))
