@@ -273,6 +273,10 @@ def main():
         for _ in range(args.warmup):
             step()
         _barrier(world)
+        try:  # zero the kernel's clock-probe sums (synchronous, outside the timed region)
+            egemm.debug_clock_stats(reset=True)
+        except Exception:  # pragma: no cover
+            pass
         clk.mark()
         start.record(stream)
         for i in range(args.steps):
@@ -291,10 +295,10 @@ def main():
     gemm_ms = float(np.mean([e[1].elapsed_time(e[2]) for e in ev]))
     split_ms = float(np.mean([e[0].elapsed_time(e[1]) for e in ev]))
     clocks = clk.summary()
-    try:  # effective SM clock inside the last timed GEMM launch (clock64 / globaltimer)
-        kernel_mhz = egemm.debug_last_clock()
+    try:  # SM clock inside the timed GEMM launches (clock64 / globaltimer of CTA 0, summed)
+        kernel_mhz, kernel_cycles, _ = egemm.debug_clock_stats(reset=True)
     except Exception:  # pragma: no cover
-        kernel_mhz = None
+        kernel_mhz, kernel_cycles = None, None
 
     peaks = _peaks()
     prof = _profile_summary()
@@ -319,6 +323,10 @@ def main():
         "kernel_sm_mhz": round(kernel_mhz, 1) if kernel_mhz else None,
         "frac_of_clock_adjusted_peak": round(achieved / (148 * 8192 * kernel_mhz * 1e-6), 4)
         if kernel_mhz else None,
+        # clock-independent: MMA-issue cycles the launch needs at 8192 fp16 flop/clk/SM over
+        # the SM cycles CTA 0 lived (the power cap sets the clock, the kernel sets this)
+        "cycle_efficiency": round(tensor_flop / (148 * 8192.0) / kernel_cycles, 4)
+        if kernel_cycles else None,
     }
     split_bytes = 8.0 * ((0 if fused_a else m_loc * K) + K * N)
     split_rl = {"kernel": "split (B^T)" if fused_a else "split (A rows + B^T)", "bound": "hbm",
