@@ -69,12 +69,14 @@ def summarize(rep):
     return out
 
 
-def launch_list(path):
+def launch_list(path, first=None):
+    """Per-kernel totals of an ncu launch list; `first` = only the first N launches (the
+    bench's headline warm-up + timed steps come first)."""
     rows = [r for r in csv.reader(open(path)) if len(r) > 10]
     hdr = rows[0]
     ik, iv, iu = hdr.index("Kernel Name"), hdr.index("Metric Value"), hdr.index("Metric Unit")
     agg = {}
-    for r in rows[1:]:
+    for r in rows[1:1 + first if first else None]:
         k = r[ik].split("(")[0][:80]
         ns = float(r[iv].replace(",", "")) * (1e3 if r[iu] == "usecond" else 1e6 if r[iu] == "msecond" else 1)
         a = agg.setdefault(k, [0, 0.0])
@@ -88,16 +90,22 @@ def launch_list(path):
 def main():
     args = sys.argv[1:]
     prefix = args.pop(0)
-    launch = None
+    launch, head = None, None
     if "--launch" in args:
         i = args.index("--launch")
         launch = args[i + 1]
+        del args[i:i + 2]
+    if "--headline" in args:
+        i = args.index("--headline")
+        head = int(args[i + 1])
         del args[i:i + 2]
     res = {"kernels": []}
     for rep in args:
         res["kernels"] += summarize(rep)
     if launch:
         res["launch_list"] = launch_list(launch)
+        if head:
+            res["headline_launches"] = launch_list(launch, head)
     json.dump(res, open(prefix + ".json", "w"), indent=1)
     with open(prefix + ".md", "w") as f:
         for s in res["kernels"]:
@@ -111,6 +119,12 @@ def main():
             f.write("| kernel | launches | total ms | share |\n|---|---|---|---|\n")
             for r in res["launch_list"]:
                 f.write("| %s | %d | %.3f | %.3f |\n" % (r["kernel"], r["launches"], r["total_ms"], r["share"]))
+            if head:
+                f.write("\n### headline step only (first %d launches: warm-up + timed steps)\n\n" % head)
+                f.write("| kernel | launches | total ms | share |\n|---|---|---|---|\n")
+                for r in res["headline_launches"]:
+                    f.write("| %s | %d | %.3f | %.3f |\n" % (r["kernel"], r["launches"], r["total_ms"],
+                                                          r["share"]))
     print("wrote", prefix + ".json", prefix + ".md")
 
 

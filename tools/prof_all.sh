@@ -13,5 +13,5 @@ timeout 600 $NCU -k regex:"egemm_tc_kernel|km_" -c 10 -f -o $O/${R}_kmeans pytho
 timeout 600 ncu --metrics gpu__time_duration.sum --clock-control none -c 400 --csv \
   --log-file $O/${R}_bench_launches.csv python bench.py --steps 2 --warmup 3 > $O/ncu_bench.log 2>&1
 python tools/ncu_summarize.py $O/${R}_ncu $O/${R}_gemm8192.ncu-rep $O/${R}_split.ncu-rep \
-  $O/${R}_knn.ncu-rep $O/${R}_kmeans.ncu-rep --launch $O/${R}_bench_launches.csv
+  $O/${R}_knn.ncu-rep $O/${R}_kmeans.ncu-rep --launch $O/${R}_bench_launches.csv --headline 15
 ls -la $O
