@@ -333,7 +333,7 @@ def main():
                 "achieved": round(split_bytes / (split_ms * 1e-3) / 1e9, 1),
                 "peak": peaks.get("hbm_gbs", 6454.0), "unit": "GB/s",
                 "frac": round(split_bytes / (split_ms * 1e-3) / 1e9 / peaks.get("hbm_gbs", 6454.0), 4),
-                "traffic": prof.get("split_dram_bytes_per_launch")}
+                "traffic": prof.get("split_dram_bytes_per_step")}
 
     # ---- e2e through the public API with host buffers: H2D A shard + B, D2H D shard
     e2e = None
