@@ -140,6 +140,13 @@ def main():
         print("%-22s cfg %-18s %.3f ms  %.0f TF(fp16)  mean %.0f MHz  %.0f kcyc/launch -> "
               "cycle efficiency %.3f" % (tag, cfg, ms, tf, mhz, cyc / 1e3, need / cyc), flush=True)
 
+    # data-dependent MMA power: fp16-exact inputs (every lo = 0) vs U[-1,1] fp32 inputs
+    a_full, b_full = a_s, b_s
+    a_s = egemm.split(A.half().float())
+    b_s = egemm.split(B.half().float(), transpose=True)
+    run("lo=0 (fp16-exact in)", (2, 256, 0, 256), {})
+    a_s, b_s = a_full, b_full
+    run("normal", (2, 256, 0, 256), {})
     for rep in range(2):
         for cfg in ((2, 256, 0, 128), (2, 256, 0, 64), (2, 256, 0, 256), (2, 256, 0, n)):
             run("normal", cfg, {})
@@ -153,6 +160,13 @@ def main():
         os.environ.pop(k, None)
     egemm.set_config(0, 0, 0, 0)
     Ah, Bh = A.half(), B.half()
+    lo_a = (A - Ah.float()).half()
+    lo_b = (B - Bh.float()).half()
+    for tag, f in (("cublas fp16 hi*hi", lambda: torch.matmul(Ah, Bh)),
+                   ("cublas fp16 lo*hi", lambda: torch.matmul(lo_a, Bh)),
+                   ("cublas fp16 hi*hi", lambda: torch.matmul(Ah, Bh))):
+        ms = timeit(f, 200, 50)
+        print("%-24s %.3f ms (steady, 200 calls)" % (tag, ms), flush=True)
     Ahh = torch.cat([Ah, Ah, Ah], 1)  # K = 3n: the same MMA count as one EGEMM launch
     Bhh = torch.cat([Bh, Bh, Bh], 0)
     for tag, f, fl in (("cublas fp16 n^3", lambda: torch.matmul(Ah, Bh), 2.0 * n ** 3),
