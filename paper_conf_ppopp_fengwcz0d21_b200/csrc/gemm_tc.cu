@@ -28,6 +28,7 @@
 #include <cuda_runtime.h>
 #include <cstdint>
 #include <cstdio>
+#include <cstdlib>
 #include <mutex>
 #include "egemm_internal.h"
 #include "ptx.cuh"
@@ -73,6 +74,9 @@ struct KParams {
   int K;
   int debug_no_tma;  // EGEMM_DEBUG_NO_TMA=1: skip operand loads (timing diagnostics only)
   int debug_no_epi;  // EGEMM_DEBUG_NO_EPI=1: skip the promotion's TMEM reads (diagnostics)
+  int debug_mode;    // EGEMM_DEBUG_MODE bits (diagnostics): 1 extra commit per k-block;
+                     // with NO_TMA: 2 MMA warp ignores the full barriers (producer idle),
+                     // 4 no per-k-block commits
 };
 
 template <int CG, int BN>
@@ -324,7 +328,8 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
       // carries only B, A is loaded once per unit into a_res
       constexpr uint32_t TX = (FA || AR) ? 2 * G::B_BYTES : G::STAGE_BYTES;
       uint32_t uctr = 0;
-      for (int u = cluster; u < p.num_units; u += nclusters, uctr++) {
+      const bool idle = p.debug_no_tma && (p.debug_mode & 2);  // diagnostics only
+      for (int u = idle ? p.num_units : cluster; u < p.num_units; u += nclusters, uctr++) {
         UnitInfo ui = decode_unit<EPI>(p, u);
         const int arow = ui.m_tile * (kBM * CG) + (int)rank * kBM;
         if constexpr (AR) {
@@ -402,7 +407,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
             const int kb0 = ch * p.kb_per_chunk;
             const int kb1 = min(p.num_kb, kb0 + p.kb_per_chunk);
             for (int kb = kb0; kb < kb1; kb++) {
-              ptx::mbar_wait(&full[stage], phase);
+              if (!(p.debug_no_tma && (p.debug_mode & 2))) ptx::mbar_wait(&full[stage], phase);
               ptx::tc_fence_after();
               const uint32_t sa = sbase + stage * SB;
               const uint32_t aa = AR ? abase + kb * 2 * G::A_BYTES : sa;
@@ -431,7 +436,8 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
                   const uint32_t first = k > 0 ? 1u : acc0;
                   ptx::mma_f16<CG>(acc_hh, d_ahi + ko, d_bhi + ko, idesc, SEP ? first : 1u);
                 }
-                ptx::mma_commit<CG>(&empty[stage]);
+                if (!(p.debug_no_tma && (p.debug_mode & 4))) ptx::mma_commit<CG>(&empty[stage]);
+                if (p.debug_mode & 1) ptx::mma_commit<CG>(a_empty);  // diagnostics only
               }
               __syncwarp();
               if (++stage == STAGES) { stage = 0; phase ^= 1u; }
@@ -864,6 +870,8 @@ int launch_tc(int64_t M, int64_t N, int64_t K, const TcOperands& ops, const TcCo
     const char* dbg = getenv("EGEMM_DEBUG_NO_TMA");
     kp.debug_no_tma = (dbg && dbg[0] == '1') ? 1 : 0;
     kp.debug_no_epi = getenv_flag("EGEMM_DEBUG_NO_EPI") ? 1 : 0;
+    const char* dm = getenv("EGEMM_DEBUG_MODE");
+    kp.debug_mode = dm ? atoi(dm) : 0;
   }
   if (fa) {
     kp.a_f32 = ops.a_f32;

@@ -115,7 +115,7 @@ def main():
     need = fl3 / (148 * 8192.0)  # SM cycles of pure MMA issue per launch at the dense peak
 
     def run(tag, cfg, env, seconds=1.5):
-        for k in ("EGEMM_DEBUG_NO_TMA", "EGEMM_DEBUG_NO_EPI"):
+        for k in ("EGEMM_DEBUG_NO_TMA", "EGEMM_DEBUG_NO_EPI", "EGEMM_DEBUG_MODE"):
             os.environ.pop(k, None)
         os.environ.update(env)
         egemm.set_config(*cfg)
@@ -140,25 +140,42 @@ def main():
         print("%-22s cfg %-18s %.3f ms  %.0f TF(fp16)  mean %.0f MHz  %.0f kcyc/launch -> "
               "cycle efficiency %.3f" % (tag, cfg, ms, tf, mhz, cyc / 1e3, need / cyc), flush=True)
 
-    # data-dependent MMA power: fp16-exact inputs (every lo = 0) vs U[-1,1] fp32 inputs
-    a_full, b_full = a_s, b_s
-    a_s = egemm.split(A.half().float())
-    b_s = egemm.split(B.half().float(), transpose=True)
-    run("lo=0 (fp16-exact in)", (2, 256, 0, 256), {})
-    a_s, b_s = a_full, b_full
-    run("normal", (2, 256, 0, 256), {})
-    for rep in range(2):
-        for cfg in ((2, 256, 0, 128), (2, 256, 0, 64), (2, 256, 0, 256), (2, 256, 0, n)):
-            run("normal", cfg, {})
-        cfg = (2, 256, 0, 128)
-        run("no_tma", cfg, {"EGEMM_DEBUG_NO_TMA": "1"})
-        run("no_epi", cfg, {"EGEMM_DEBUG_NO_EPI": "1"})
-        run("no_tma+no_epi", cfg, {"EGEMM_DEBUG_NO_TMA": "1", "EGEMM_DEBUG_NO_EPI": "1"})
-        run("no_tma+no_epi kc=n", (2, 256, 0, n), {"EGEMM_DEBUG_NO_TMA": "1",
-                                                   "EGEMM_DEBUG_NO_EPI": "1"})
+    which = os.environ.get("DIAG", "issue")
+    if which == "issue":  # MMA-issue mechanics: barrier handshakes and commits
+        nt = {"EGEMM_DEBUG_NO_TMA": "1", "EGEMM_DEBUG_NO_EPI": "1"}
+        kn = (2, 256, 0, n)
+        run("normal kc=256", (2, 256, 0, 256), {})
+        run("normal kc=n", kn, {})
+        run("mma-only", kn, nt)
+        run("mma-only +extra commit", kn, dict(nt, EGEMM_DEBUG_MODE="1"))
+        run("mma-only no full-wait", kn, dict(nt, EGEMM_DEBUG_MODE="2"))
+        run("mma-only no wait, no commit", kn, dict(nt, EGEMM_DEBUG_MODE="6"))
+        run("mma-only no wait +extra", kn, dict(nt, EGEMM_DEBUG_MODE="3"))
+        run("mma-only kc=256", (2, 256, 0, 256), nt)
+        run("mma-only kc=256 no wait", (2, 256, 0, 256), dict(nt, EGEMM_DEBUG_MODE="2"))
+        os.environ.pop("EGEMM_DEBUG_MODE", None)
+    else:
+        # data-dependent MMA power: fp16-exact inputs (every lo = 0) vs U[-1,1] fp32 inputs
+        a_full, b_full = a_s, b_s
+        a_s = egemm.split(A.half().float())
+        b_s = egemm.split(B.half().float(), transpose=True)
+        run("lo=0 (fp16-exact in)", (2, 256, 0, 256), {})
+        a_s, b_s = a_full, b_full
+        run("normal", (2, 256, 0, 256), {})
+        for rep in range(2):
+            for cfg in ((2, 256, 0, 128), (2, 256, 0, 64), (2, 256, 0, 256), (2, 256, 0, n)):
+                run("normal", cfg, {})
+            cfg = (2, 256, 0, 128)
+            run("no_tma", cfg, {"EGEMM_DEBUG_NO_TMA": "1"})
+            run("no_epi", cfg, {"EGEMM_DEBUG_NO_EPI": "1"})
+            run("no_tma+no_epi", cfg, {"EGEMM_DEBUG_NO_TMA": "1", "EGEMM_DEBUG_NO_EPI": "1"})
+            run("no_tma+no_epi kc=n", (2, 256, 0, n), {"EGEMM_DEBUG_NO_TMA": "1",
+                                                       "EGEMM_DEBUG_NO_EPI": "1"})
     for k in ("EGEMM_DEBUG_NO_TMA", "EGEMM_DEBUG_NO_EPI"):
         os.environ.pop(k, None)
     egemm.set_config(0, 0, 0, 0)
+    if which == "issue":
+        return
     Ah, Bh = A.half(), B.half()
     lo_a = (A - Ah.float()).half()
     lo_b = (B - Bh.float()).half()
