@@ -421,7 +421,29 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
               // added, so the tensor core's truncating alignment (probe model)
               // loses almost nothing on them; only the 4 hi*hi MMAs see the full |acc|.
               const uint32_t acc0 = (kb > kb0) ? 1u : 0u;
-              if (ptx::elect_one()) {
+              if (p.debug_mode & 24) {  // diagnostics only: MMA-order timing variants
+                if (ptx::elect_one()) {
+                  if (p.debug_mode & 8) {  // grouped: all hi*lo, all lo*hi, all hi*hi
+#pragma unroll
+                    for (int k = 0; k < kBK / 16; k++)
+                      ptx::mma_f16<CG>(acc_x, d_ahi + 2 * k, d_blo + 2 * k, idesc, k > 0 ? 1u : acc0);
+#pragma unroll
+                    for (int k = 0; k < kBK / 16; k++)
+                      ptx::mma_f16<CG>(acc_x, d_alo + 2 * k, d_bhi + 2 * k, idesc, 1u);
+#pragma unroll
+                    for (int k = 0; k < kBK / 16; k++)
+                      ptx::mma_f16<CG>(acc_hh, d_ahi + 2 * k, d_bhi + 2 * k, idesc, 1u);
+                  } else {  // per k step: hi*lo, lo*hi, hi*hi
+#pragma unroll
+                    for (int k = 0; k < kBK / 16; k++) {
+                      ptx::mma_f16<CG>(acc_x, d_ahi + 2 * k, d_blo + 2 * k, idesc, k > 0 ? 1u : acc0);
+                      ptx::mma_f16<CG>(acc_x, d_alo + 2 * k, d_bhi + 2 * k, idesc, 1u);
+                      ptx::mma_f16<CG>(acc_hh, d_ahi + 2 * k, d_bhi + 2 * k, idesc, 1u);
+                    }
+                  }
+                  if (!(p.debug_no_tma && (p.debug_mode & 4))) ptx::mma_commit<CG>(&empty[stage]);
+                }
+              } else if (ptx::elect_one()) {
 #pragma unroll
                 for (int k = 0; k < kBK / 16; k++) {
                   const uint64_t ko = (uint64_t)(k * 2);  // +32 B per 16-wide k step (>>4)

@@ -153,6 +153,11 @@ def main():
         run("mma-only no wait +extra", kn, dict(nt, EGEMM_DEBUG_MODE="3"))
         run("mma-only kc=256", (2, 256, 0, 256), nt)
         run("mma-only kc=256 no wait", (2, 256, 0, 256), dict(nt, EGEMM_DEBUG_MODE="2"))
+        for tag, m in (("grouped", 8), ("per-k", 16)):
+            run("mma-only %s" % tag, kn, dict(nt, EGEMM_DEBUG_MODE=str(m)))
+            run("mma-only %s no wait" % tag, kn, dict(nt, EGEMM_DEBUG_MODE=str(m | 2)))
+            run("normal %s kc=n" % tag, kn, {"EGEMM_DEBUG_MODE": str(m)})
+            run("normal %s kc=256" % tag, (2, 256, 0, 256), {"EGEMM_DEBUG_MODE": str(m)})
         os.environ.pop("EGEMM_DEBUG_MODE", None)
     else:
         # data-dependent MMA power: fp16-exact inputs (every lo = 0) vs U[-1,1] fp32 inputs
