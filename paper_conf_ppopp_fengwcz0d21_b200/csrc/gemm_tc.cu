@@ -444,13 +444,26 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
                   if (!(p.debug_no_tma && (p.debug_mode & 4))) ptx::mma_commit<CG>(&empty[stage]);
                 }
               } else if (ptx::elect_one()) {
+                // The lo*lo term is a separate branch, not a predicate: a predicated-off
+                // UTCHMMA still costs tensor-pipe time (measured: 0.88 -> 0.98 of the issue
+                // peak when the @!P UTCHMMAs are gone, tools/diag_gemm.py).
+                if (p.terms == 4) {
 #pragma unroll
-                for (int k = 0; k < kBK / 16; k++) {
-                  const uint64_t ko = (uint64_t)(k * 2);  // +32 B per 16-wide k step (>>4)
-                  const uint32_t first = k > 0 ? 1u : acc0;
-                  ptx::mma_f16<CG>(acc_x, d_ahi + ko, d_blo + ko, idesc, first);
-                  ptx::mma_f16<CG>(acc_x, d_alo + ko, d_bhi + ko, idesc, 1u);
-                  if (p.terms == 4) ptx::mma_f16<CG>(acc_x, d_alo + ko, d_blo + ko, idesc, 1u);
+                  for (int k = 0; k < kBK / 16; k++) {
+                    const uint64_t ko = (uint64_t)(k * 2);
+                    const uint32_t first = k > 0 ? 1u : acc0;
+                    ptx::mma_f16<CG>(acc_x, d_ahi + ko, d_blo + ko, idesc, first);
+                    ptx::mma_f16<CG>(acc_x, d_alo + ko, d_bhi + ko, idesc, 1u);
+                    ptx::mma_f16<CG>(acc_x, d_alo + ko, d_blo + ko, idesc, 1u);
+                  }
+                } else {
+#pragma unroll
+                  for (int k = 0; k < kBK / 16; k++) {
+                    const uint64_t ko = (uint64_t)(k * 2);  // +32 B per 16-wide k step (>>4)
+                    const uint32_t first = k > 0 ? 1u : acc0;
+                    ptx::mma_f16<CG>(acc_x, d_ahi + ko, d_blo + ko, idesc, first);
+                    ptx::mma_f16<CG>(acc_x, d_alo + ko, d_bhi + ko, idesc, 1u);
+                  }
                 }
 #pragma unroll
                 for (int k = 0; k < kBK / 16; k++) {

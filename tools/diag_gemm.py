@@ -144,20 +144,12 @@ def main():
     if which == "issue":  # MMA-issue mechanics: barrier handshakes and commits
         nt = {"EGEMM_DEBUG_NO_TMA": "1", "EGEMM_DEBUG_NO_EPI": "1"}
         kn = (2, 256, 0, n)
-        run("normal kc=256", (2, 256, 0, 256), {})
-        run("normal kc=n", kn, {})
-        run("mma-only", kn, nt)
-        run("mma-only +extra commit", kn, dict(nt, EGEMM_DEBUG_MODE="1"))
-        run("mma-only no full-wait", kn, dict(nt, EGEMM_DEBUG_MODE="2"))
-        run("mma-only no wait, no commit", kn, dict(nt, EGEMM_DEBUG_MODE="6"))
-        run("mma-only no wait +extra", kn, dict(nt, EGEMM_DEBUG_MODE="3"))
+        for kc in (64, 128, 256, n):
+            run("normal kc=%d" % kc, (2, 256, 0, kc), {})
+        run("mma-only kc=n", kn, nt)
         run("mma-only kc=256", (2, 256, 0, 256), nt)
-        run("mma-only kc=256 no wait", (2, 256, 0, 256), dict(nt, EGEMM_DEBUG_MODE="2"))
-        for tag, m in (("grouped", 8), ("per-k", 16)):
-            run("mma-only %s" % tag, kn, dict(nt, EGEMM_DEBUG_MODE=str(m)))
-            run("mma-only %s no wait" % tag, kn, dict(nt, EGEMM_DEBUG_MODE=str(m | 2)))
-            run("normal %s kc=n" % tag, kn, {"EGEMM_DEBUG_MODE": str(m)})
-            run("normal %s kc=256" % tag, (2, 256, 0, 256), {"EGEMM_DEBUG_MODE": str(m)})
+        run("normal grouped kc=256", (2, 256, 0, 256), {"EGEMM_DEBUG_MODE": "8"})
+        run("normal sep (2,128,1,256)", (2, 128, 1, 256), {})
         os.environ.pop("EGEMM_DEBUG_MODE", None)
     else:
         # data-dependent MMA power: fp16-exact inputs (every lo = 0) vs U[-1,1] fp32 inputs
