@@ -30,23 +30,27 @@ def deps():
         glob.glob(os.path.join(CSRC, "*.h"))) + [os.path.join(ROOT, "include", "egemm.h")]
 
 
-def up_to_date() -> bool:
-    if not os.path.exists(LIB):
+def up_to_date(lib: str = LIB) -> bool:
+    if not os.path.exists(lib):
         return False
-    t = os.path.getmtime(LIB)
+    t = os.path.getmtime(lib)
     return all(os.path.getmtime(f) <= t for f in deps())
 
 
-def build(force: bool = False, verbose: bool = False) -> str:
-    if not force and up_to_date():
-        return LIB
+def build(force: bool = False, verbose: bool = False, lib: str = LIB, defines=()) -> str:
+    """Compile every csrc/*.cu and link `lib`.  `defines` (e.g. ["EGEMM_NO_WAIT_HINT"]) build
+    an experiment variant next to the product library (tools/ A/B runs only)."""
+    if not force and up_to_date(lib):
+        return lib
     objs = []
-    tmpdir = os.path.join(PKG, "build")
+    tag = "_".join(defines)
+    tmpdir = os.path.join(PKG, "build", tag) if tag else os.path.join(PKG, "build")
     os.makedirs(tmpdir, exist_ok=True)
     procs = []
     for src in sources():
         obj = os.path.join(tmpdir, os.path.basename(src) + ".o")
-        cmd = [NVCC] + [f for f in FLAGS if f not in ("-shared",)] + ["-c", src, "-o", obj]
+        cmd = [NVCC] + [f for f in FLAGS if f not in ("-shared",)] + ["-D" + d for d in defines] + \
+            ["-c", src, "-o", obj]
         if verbose:
             cmd += ["-Xptxas", "-v"]
         procs.append((src, subprocess.Popen(cmd, stdout=subprocess.PIPE, stderr=subprocess.STDOUT)))
@@ -61,11 +65,11 @@ def build(force: bool = False, verbose: bool = False) -> str:
             sys.stderr.write(out)
     if failed:
         raise RuntimeError("nvcc build failed")
-    tmp = LIB + ".tmp%d" % os.getpid()
+    tmp = lib + ".tmp%d" % os.getpid()
     subprocess.check_call([NVCC, "-shared", "-cudart", "static", "-gencode",
                            "arch=compute_100a,code=sm_100a", "-o", tmp] + objs)
-    os.replace(tmp, LIB)
-    return LIB
+    os.replace(tmp, lib)
+    return lib
 
 
 if __name__ == "__main__":

@@ -52,12 +52,20 @@ __device__ __forceinline__ void mbar_arrive_cluster(uint64_t* bar, uint32_t cta)
       "r"(cta)
       : "memory");
 }
+// The suspend-time hint lets a waiting warp sleep until the phase completes (SASS
+// NANOSLEEP.SYNCS) instead of re-issuing try_wait: idle epilogue / producer warps then stop
+// burning issue slots and power, which the power-capped GEMM turns into clock.
+#ifndef EGEMM_NO_WAIT_HINT
+#define EGEMM_WAIT_HINT ", 0x989680"
+#else
+#define EGEMM_WAIT_HINT ""
+#endif
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   uint32_t addr = smem_u32(bar);
   asm volatile(
       "{\n\t.reg .pred P;\n\t"
       "WAIT_%=:\n\t"
-      "mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1;\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 P, [%0], %1" EGEMM_WAIT_HINT ";\n\t"
       "@!P bra WAIT_%=;\n\t}" ::"r"(addr),
       "r"(parity)
       : "memory");

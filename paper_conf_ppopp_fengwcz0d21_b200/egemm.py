@@ -12,7 +12,8 @@ import os
 import torch
 
 _PKG = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_PKG, "libegemm.so")
+# EGEMM_LIB_PATH: load another build of the same library (A/B experiments in tools/)
+LIB_PATH = os.environ.get("EGEMM_LIB_PATH") or os.path.join(_PKG, "libegemm.so")
 
 OK, ERR_INVALID_ARG, ERR_UNSUPPORTED, ERR_CUDA, ERR_WORKSPACE = 0, 1, 2, 3, 4
 

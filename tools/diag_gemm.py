@@ -144,13 +144,11 @@ def main():
     if which == "issue":  # MMA-issue mechanics: barrier handshakes and commits
         nt = {"EGEMM_DEBUG_NO_TMA": "1", "EGEMM_DEBUG_NO_EPI": "1"}
         kn = (2, 256, 0, n)
-        for kc in (64, 128, 256, n):
-            run("normal kc=%d" % kc, (2, 256, 0, kc), {})
-        run("mma-only kc=n", kn, nt)
-        run("mma-only kc=256", (2, 256, 0, 256), nt)
-        run("normal grouped kc=256", (2, 256, 0, 256), {"EGEMM_DEBUG_MODE": "8"})
-        run("normal sep (2,128,1,256)", (2, 128, 1, 256), {})
-        os.environ.pop("EGEMM_DEBUG_MODE", None)
+        tag = os.path.basename(egemm.LIB_PATH)
+        for rep in range(2):
+            for kc in (128, 256):
+                run("%s kc=%d" % (tag, kc), (2, 256, 0, kc), {})
+        run("%s mma-only kc=256" % tag, (2, 256, 0, 256), nt)
     else:
         # data-dependent MMA power: fp16-exact inputs (every lo = 0) vs U[-1,1] fp32 inputs
         a_full, b_full = a_s, b_s
