@@ -116,7 +116,12 @@ def build_table(log, Ms, Ns, Ks, extra=None):
                             "err_ratio": round(best["err"] / best["err_naive"], 3)})
     # the largest measured bucket in each dimension is open-ended, then bucket order:
     # smallest first so the library's first-match lookup picks the tightest bucket
+    # M > 8192 is only swept for skinny N (<= 1024): the M = 8192 rows of wider N also
+    # cover every larger M
+    wide_top = max([M for M in Ms if M <= 8192], default=None)
     for e in entries:
+        if e["m_max"] == wide_top and e["n_max"] > 1024:
+            e["m_max"] = max(Ms)
         for key, top in (("m_max", max(Ms)), ("n_max", max(Ns)), ("k_max", max(Ks))):
             if e[key] == top:
                 e[key] = 1 << 40
