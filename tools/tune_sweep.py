@@ -6,7 +6,7 @@ of repeats, pre-split operands) and its normwise error vs the fp64 oracle is mea
 row sample; the fastest configuration that meets the accuracy bar (<= 1e-6 and <= 2x the
 naive-fp32 error, BJ north_star) is recorded.  Tool code (calls oracle/ for the error check).
 
-usage: python tools/tune_sweep.py [--quick]
+usage: python tools/tune_sweep.py [--quick] [--prior T]
 """
 import json
 import os
@@ -18,6 +18,7 @@ import torch
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
+sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
 import oracle  # noqa: E402
 from paper_conf_ppopp_fengwcz0d21_b200 import egemm, inputs  # noqa: E402
 
@@ -56,7 +57,7 @@ def timeit(fn, reps=3, batch_ms=60.0):
     return float(np.median(ts))
 
 
-def gemm_bucket(M, N, K, rows=64):
+def gemm_bucket(M, N, K, rows=64, configs=None):
     A, B = inputs.uniform((M, K), 11 + M), inputs.uniform((K, N), 13 + N)
     Ad, Bd = torch.from_numpy(A).cuda(), torch.from_numpy(B).cuda()
     b_split = egemm.split(Bd, transpose=True)
@@ -66,7 +67,7 @@ def gemm_bucket(M, N, K, rows=64):
     en = oracle.normwise_error(oracle.gemm32_naive(A[rs], B), A[rs], B, C64)
     ws = torch.empty(egemm.gemm_workspace_size(M, N, K, False, True), dtype=torch.uint8, device="cuda")
     res = []
-    for cfg in CONFIGS:
+    for cfg in configs or CONFIGS:
         egemm.set_config(*cfg[:4])
         os.environ["EGEMM_FUSED_A"] = str(cfg[4])
         # the user call with an fp32 A (split separately, or fused into the GEMM) and a
@@ -147,12 +148,29 @@ def main():
     Ks = [256, 1024, 2048, 4096, 8192] if not quick else [1024, 8192]
     log = []
     t0 = time.time()
+    # --prior T: measure every config only on the 8192^3 calibration bucket, then only the
+    # analytic model's top T per bucket (NEXT-4; tools/analytic_model.py), widening to all
+    # configs when none of those meets the accuracy bar
+    prior = int(sys.argv[sys.argv.index("--prior") + 1]) if "--prior" in sys.argv else 0
+    model = None
+    if prior:
+        import analytic_model as am
+        cal = {"M": 8192, "N": 8192, "K": 8192, "results": gemm_bucket(8192, 8192, 8192)}
+        model = am.calibrate([cal])
     for M in Ms:
         for N in Ns:
             for K in Ks:
                 if M > 8192 and N > 1024:  # the tall bucket is for skinny N (configs[2])
                     continue
-                res = gemm_bucket(M, N, K)
+                if model and (M, N, K) == (8192, 8192, 8192):
+                    res = cal["results"]
+                elif model:
+                    ranked = sorted(CONFIGS, key=lambda c: am.predict(c, M, N, K, *model))
+                    res = gemm_bucket(M, N, K, configs=ranked[:prior])
+                    if not any(r["ok"] for r in res):
+                        res += gemm_bucket(M, N, K, configs=ranked[prior:])
+                else:
+                    res = gemm_bucket(M, N, K)
                 best = select(res, k_scale(K, Ks))
                 log.append({"M": M, "N": N, "K": K, "results": res})
                 print("M=%5d N=%5d K=%5d best=%s %s" % (M, N, K, best and best["cfg"],
