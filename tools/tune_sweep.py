@@ -6,7 +6,7 @@ of repeats, pre-split operands) and its normwise error vs the fp64 oracle is mea
 row sample; the fastest configuration that meets the accuracy bar (<= 1e-6 and <= 2x the
 naive-fp32 error, BJ north_star) is recorded.  Tool code (calls oracle/ for the error check).
 
-usage: python tools/tune_sweep.py [--quick] [--prior T]
+usage: python tools/tune_sweep.py [--quick] [--prior T] [--out table.json]
 """
 import json
 import os
@@ -180,10 +180,12 @@ def main():
         "device": torch.cuda.get_device_name(),
         "when": time.strftime("%Y-%m-%dT%H:%M:%SZ", time.gmtime()),
         "sweep_seconds": round(time.time() - t0, 1)})
-    json.dump(doc, open(OUT, "w"), indent=1)
+    out = sys.argv[sys.argv.index("--out") + 1] if "--out" in sys.argv else OUT
+    json.dump(doc, open(out, "w"), indent=1)
     os.makedirs(os.path.join(ROOT, "gpurun_out"), exist_ok=True)
-    json.dump(log, open(os.path.join(ROOT, "gpurun_out", "tune_sweep_log.json"), "w"), indent=1)
-    print("wrote", OUT, len(doc["entries"]), "entries")
+    logname = "tune_sweep_prior%d_log.json" % prior if prior else "tune_sweep_log.json"
+    json.dump(log, open(os.path.join(ROOT, "gpurun_out", logname), "w"), indent=1)
+    print("wrote", out, len(doc["entries"]), "entries in %.1f s" % doc["sweep_seconds"])
 
 
 if __name__ == "__main__":
