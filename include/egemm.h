@@ -183,6 +183,24 @@ int egemm_num_sms(void);
  * from clock64 / %globaltimer.  Synchronous (copies a device symbol). */
 int egemm_debug_last_clock(double* mhz);
 
+/*
+ * Tensor-core precision probe (the profiling workflow of Sec. 3.1, generalised to
+ * the floating tcgen05 kinds).  Runs ONE chain of tcgen05.mma (cta_group::1,
+ * M = 128) on a single CTA:  D = C + sum over k of A[:, k] * B[:, k]  in the MMA's own
+ * arithmetic (fp32 D in TMEM), so D can be compared bitwise with CPU models of the MMA.
+ *  kind : 0 = kind::f16 with fp16 operands, 1 = kind::f16 with bf16 operands,
+ *         2 = kind::tf32 (fp32 containers; the hardware reads them as tf32).
+ *  A    : 128 x K row-major (K contiguous), element = 2 B (kinds 0, 1) or 4 B (kind 2).
+ *  B    : N x K row-major (each row one column of the math B), same element type.
+ *  C    : nullable 128 x N fp32 addend (NULL = 0, the first MMA overwrites).
+ *  D    : 128 x N fp32 output.
+ *  N    : multiple of 16 in [16, 256];  K : 1 .. 256 (kinds 0, 1) or 1 .. 128 (kind 2); the
+ *         last MMA's missing k are zero.  One MMA consumes 16 (f16/bf16) or 8 (tf32) k.
+ * Profiling only (slow, one CTA); the GEMM never calls it.
+ */
+int egemm_tc_probe(int kind, int N, int K, const void* A, const void* B, const float* C,
+                   float* D, void* stream);
+
 /* Debug: running sums of the same probe over every tensor-core launch since the last
  * reset: mean SM clock (MHz), CTA-0 SM cycles per launch (clock-independent kernel cost),
  * number of launches.  reset != 0 zeroes the sums after reading.  Synchronous. */

@@ -211,6 +211,28 @@ int egemm_debug_last_clock(double* mhz) {
   return read_clock_probe(mhz) ? EGEMM_ERR_CUDA : EGEMM_OK;
 }
 
+int egemm_tc_probe(int kind, int N, int K, const void* A, const void* B, const float* C,
+                   float* D, void* stream) {
+  if (kind < 0 || kind > 2 || N < 16 || N > 256 || (N % 16) != 0 || K < 1 ||
+      K > (kind == 2 ? 128 : 256)) {
+    set_last_error("egemm_tc_probe: kind %d, N %d, K %d out of range", kind, N, K);
+    return EGEMM_ERR_INVALID_ARG;
+  }
+  if (!A || !B || !D) {
+    set_last_error("egemm_tc_probe: NULL data");
+    return EGEMM_ERR_INVALID_ARG;
+  }
+  if (!device_ok()) {
+    set_last_error("no sm_100 device");
+    return EGEMM_ERR_CUDA;
+  }
+  if (launch_tc_probe(kind, N, K, A, B, C, D, (cudaStream_t)stream)) {
+    set_last_error("egemm_tc_probe: launch failed");
+    return EGEMM_ERR_CUDA;
+  }
+  return EGEMM_OK;
+}
+
 int egemm_debug_clock_stats(double* mhz, double* cycles_per_launch, double* launches, int reset) {
   if (!mhz || !cycles_per_launch || !launches) return EGEMM_ERR_INVALID_ARG;
   return read_clock_stats(mhz, cycles_per_launch, launches, reset) ? EGEMM_ERR_CUDA : EGEMM_OK;

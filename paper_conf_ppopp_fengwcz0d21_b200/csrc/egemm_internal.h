@@ -78,6 +78,8 @@ int launch_fill_c(int64_t M, int64_t N, const float* C, int64_t ldc, float* D, i
 
 void set_last_error(const char* fmt, ...);
 int read_clock_probe(double* mhz);
+int launch_tc_probe(int kind, int N, int K, const void* A, const void* B, const float* C,
+                    float* D, cudaStream_t stream);
 int read_clock_stats(double* mhz, double* cycles_per_launch, double* launches, int reset);
 
 // tune.cu: the measured configuration table

@@ -39,7 +39,7 @@ EXPORTS = ["egemm_status_string", "egemm_last_error", "egemm_version", "egemm_sp
            "egemm_gemm_workspace_size", "egemm_knn", "egemm_knn_workspace_size", "egemm_knn_index",
            "egemm_kmeans_step", "egemm_kmeans_workspace_size", "egemm_kmeans_finalize",
            "egemm_set_config", "egemm_num_sms", "egemm_debug_last_clock", "egemm_tune_table",
-           "egemm_debug_clock_stats",
+           "egemm_debug_clock_stats", "egemm_tc_probe",
            "egemm_query_config", "egemm_gemm_host", "egemm_gemm_host_workspace_size"]
 
 _lib = None
@@ -84,6 +84,8 @@ def load(path: str = LIB_PATH):
     L.egemm_num_sms.restype = I
     L.egemm_debug_last_clock.argtypes = [ctypes.POINTER(ctypes.c_double)]
     L.egemm_debug_last_clock.restype = I
+    L.egemm_tc_probe.argtypes = [I, I, I, P, P, P, P, P]
+    L.egemm_tc_probe.restype = I
     DP = ctypes.POINTER(ctypes.c_double)
     L.egemm_debug_clock_stats.argtypes = [DP, DP, DP, I]
     L.egemm_debug_clock_stats.restype = I
@@ -115,6 +117,29 @@ def query_config(op: str, M: int, N: int, K: int, with_fused: bool = False):
                                      *[ctypes.byref(x) for x in v]), "egemm_query_config")
     out = tuple(x.value for x in v)
     return out if with_fused else out[:4]
+
+
+PROBE_KINDS = {"f16": 0, "bf16": 1, "tf32": 2}
+
+
+def tc_probe(kind: str, A: torch.Tensor, B: torch.Tensor, C: torch.Tensor | None = None,
+             stream=None) -> torch.Tensor:
+    """One tcgen05.mma chain D = C + A @ B^T on a single CTA (M = 128) in the MMA's own
+    arithmetic -- the precision-profiling probe of Sec. 3.1 (egemm_tc_probe).  A [128, K] and
+    B [N, K] are fp16 / bf16 (kinds "f16" / "bf16") or fp32 holding tf32 values ("tf32")."""
+    L = load()
+    _need_cuda(A, B)
+    k = PROBE_KINDS[kind]
+    dt = {0: torch.float16, 1: torch.bfloat16, 2: torch.float32}[k]
+    assert A.dtype == dt and B.dtype == dt and A.shape[0] == 128 and A.shape[1] == B.shape[1]
+    A, B = A.contiguous(), B.contiguous()
+    if C is not None:
+        C = C.contiguous().float()
+    N, K = B.shape
+    D = torch.empty((128, N), dtype=torch.float32, device=A.device)
+    _check(L.egemm_tc_probe(k, N, K, _ptr(A), _ptr(B), _ptr(C), _ptr(D), _stream(stream)),
+           "egemm_tc_probe")
+    return D
 
 
 def debug_clock_stats(reset: bool = True):

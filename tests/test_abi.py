@@ -59,6 +59,9 @@ def test_status_strings_and_host_validation(lib):
     assert lib.egemm_gemm(4, 4, 4, op, op, None, 0, None, 4, 7, None, 0, None) == egemm.ERR_INVALID_ARG
     # empty problems are a no-op
     assert lib.egemm_gemm(0, 4, 4, op, op, None, 0, None, 4, 0, None, 0, None) == egemm.OK
+    assert lib.egemm_tc_probe(3, 64, 16, None, None, None, None, None) == egemm.ERR_INVALID_ARG
+    assert lib.egemm_tc_probe(0, 17, 16, None, None, None, None, None) == egemm.ERR_INVALID_ARG
+    assert lib.egemm_tc_probe(2, 64, 129, None, None, None, None, None) == egemm.ERR_INVALID_ARG
     assert lib.egemm_set_config(3, 256, 0, 0) == egemm.ERR_UNSUPPORTED
     assert lib.egemm_set_config(0, 0, 0, 0) == egemm.OK
 
