@@ -243,6 +243,24 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
     ptx::mbar_init(a_empty, 1);
     ptx::fence_mbar_init();
   }
+  if (!FA && !AR && p.debug_no_tma && (p.debug_mode & 32)) {
+    // diagnostics only: fill the ring with random fp16 operands (hi ~[0.5, 1), lo ~2^-9) so a
+    // NO_TMA run multiplies realistic data -- isolates the power of the operand traffic
+    for (int i = threadIdx.x; i < STAGES * SB / 16; i += blockDim.x) {
+      const int off = (i * 16) % SB;
+      const bool lo_part = (off >= G::A_BYTES && off < 2 * G::A_BYTES) || off >= 2 * G::A_BYTES + G::B_BYTES;
+      uint32_t w[4];
+#pragma unroll
+      for (int j = 0; j < 4; j++) {
+        uint32_t h = (uint32_t)(i * 4 + j + 1) * 2654435761u + blockIdx.x * 40503u;
+        h ^= h >> 15; h *= 2246822519u; h ^= h >> 13;
+        const uint32_t e = lo_part ? 0x1800u : 0x3800u;
+        w[j] = ((h & 0x83FFu) | e) | ((((h >> 16) & 0x83FFu) | e) << 16);
+      }
+      ptx::sts128(ptx::smem_u32(stage_base) + i * 16, w[0], w[1], w[2], w[3]);
+    }
+    ptx::fence_proxy_async_smem();
+  }
   if (warp == EG::W_ALLOC) ptx::tmem_alloc<CG>(tmem_slot, TMEM_COLS);
   ptx::tc_fence_before();
   if constexpr (CG == 2) ptx::cluster_sync(); else __syncthreads();

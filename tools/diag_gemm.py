@@ -141,6 +141,13 @@ def main():
               "cycle efficiency %.3f" % (tag, cfg, ms, tf, mhz, cyc / 1e3, need / cyc), flush=True)
 
     which = os.environ.get("DIAG", "issue")
+    if which == "power":  # operand-traffic power: NO_TMA on realistic (random) smem data
+        for rep in range(2):
+            run("normal kc=256", (2, 256, 0, 256), {})
+            run("no_tma, random smem", (2, 256, 0, 256),
+                {"EGEMM_DEBUG_NO_TMA": "1", "EGEMM_DEBUG_MODE": "32"})
+            run("no_tma, stale smem", (2, 256, 0, 256), {"EGEMM_DEBUG_NO_TMA": "1"})
+        return
     if which == "issue":  # MMA-issue mechanics: barrier handshakes and commits
         nt = {"EGEMM_DEBUG_NO_TMA": "1", "EGEMM_DEBUG_NO_EPI": "1"}
         kn = (2, 256, 0, n)
