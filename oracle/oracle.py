@@ -252,6 +252,58 @@ def gemm_alg1_tc(A, B, C=None, terms: int = 3, sep: int = 0, kc: int = 64):
     return D
 
 
+def rownorm_tree(X):
+    """Squared row norms in the order reading R22 fixes (the paper is silent): in fp64,
+    lane l of 32 sums x_t^2 for t = l, l+32, l+64, ... in order; the 32 lane sums are then
+    combined by the butterfly s_l <- s_l + s_(l xor o) for o = 16, 8, 4, 2, 1; the result
+    is rounded to fp32.  Every x^2 is exact in fp64."""
+    X = np.asarray(X, np.float32).astype(np.float64)
+    n, d = X.shape
+    lanes = np.zeros((n, 32), np.float64)
+    for t0 in range(0, d, 32):
+        blk = X[:, t0:t0 + 32]
+        lanes[:, :blk.shape[1]] += blk * blk  # one exact square added per lane and round
+    idx = np.arange(32)
+    for o in (16, 8, 4, 2, 1):
+        lanes = lanes + lanes[:, idx ^ o]
+    return lanes[:, 0].astype(np.float32)
+
+
+def _kc_single(d: int) -> int:
+    return ((d + 63) // 64) * 64  # one promotion chunk over the whole feature dimension
+
+
+def knn_alg1_tc(X, Q, k: int):
+    """kNN with the distance GEMM done by Alg. 1 on the profiled tensor core (R21, R22):
+    key_ij = RN32(||x_j||^2 - 2 (q_i . x_j)), q_i . x_j = gemm_alg1_tc(Q, X^T, kc = whole d);
+    the k smallest (key, j) ascending; dist = max(0, RN32(||q_i||^2 + key)).  The bitwise
+    model of egemm_knn; the plain definition stays `knn` (exact distances, gap rule R18)."""
+    X, Q = _f32(X), _f32(Q)
+    nx, d = X.shape
+    xn = rownorm_tree(X).astype(np.float64)
+    qn = rownorm_tree(Q).astype(np.float64)
+    dot = gemm_alg1_tc(Q, X.T, terms=3, sep=0, kc=_kc_single(d)).astype(np.float64)
+    # fp64 holds -2 dot + xn exactly whenever it matters for the fp32 rounding: this is fma
+    key = (xn[None, :] - 2.0 * dot).astype(np.float32)
+    order = np.lexsort((np.broadcast_to(np.arange(nx), key.shape), key), axis=1)[:, :k]
+    kk = np.take_along_axis(key, order, 1)
+    dist = (qn[:, None] + kk.astype(np.float64)).astype(np.float32)
+    return order.astype(np.int32), np.maximum(dist, np.float32(0.0))
+
+
+def kmeans_assign_alg1_tc(X, C):
+    """kMeans assignment with Alg. 1 on the profiled tensor core (R21, R22): key_ij =
+    RN32(||c_j||^2 - 2 (x_i . c_j)), assign_i = the lowest j of minimal key.  Returns
+    (assign int32, best key fp32)."""
+    X, C = _f32(X), _f32(C)
+    d = X.shape[1]
+    cn = rownorm_tree(C).astype(np.float64)
+    dot = gemm_alg1_tc(X, C.T, terms=3, sep=0, kc=_kc_single(d)).astype(np.float64)
+    key = (cn[None, :] - 2.0 * dot).astype(np.float32)
+    a = np.argmin(key, axis=1)  # first occurrence: ties -> lowest j
+    return a.astype(np.int32), key[np.arange(len(a)), a]
+
+
 def group_sums(X, assign, kc: int):
     """R20-ordered fp64 sums and int64 counts of X's rows grouped by a given assignment."""
     X = _f32(X)

@@ -136,3 +136,40 @@ def test_kmeans_finalize_and_empty_cluster(oracle_lib):
     ref = oracle_lib.kmeans_finalize(to_host(sums), to_host(counts), C)
     assert np.array_equal(newc, ref)
     assert np.array_equal(newc[31], C[31])
+
+
+# ------------------------------------------------------------------ bitwise (R21 + R22)
+@pytest.mark.parametrize("nx,nq,d,k,path", [(5000, 64, 128, 16, "index"), (777, 50, 100, 5, "f32"),
+                                            (40, 33, 16, 16, "split"), (32768, 24, 128, 16, "index"),
+                                            (3000, 300, 64, 8, "f32")])
+def test_knn_bitexact_vs_alg1_model(oracle_lib, nx, nq, d, k, path):
+    """egemm_knn equals the kNN-on-the-profiled-tensor-core model bitwise: indices AND
+    distances (oracle.knn_alg1_tc: Alg. 1 dot products, R22 norms / key / ordering) -- no
+    gap exemptions."""
+    eg = require_gpu()
+    X, Q = inputs.uniform((nx, d), 70 + d), inputs.uniform((nq, d), 71 + d)
+    Xd, Qd = to_dev(X), to_dev(Q)
+    if path == "index":
+        idx, dist = eg.knn(None, Qd, k, index=eg.knn_index(Xd))
+    elif path == "split":
+        idx, dist = eg.knn(Xd, Qd, k, x_split=eg.split(Xd))
+    else:
+        idx, dist = eg.knn(Xd, Qd, k)
+    ri, rd = oracle_lib.knn_alg1_tc(X, Q, k)
+    assert np.array_equal(to_host(idx), ri)
+    assert np.array_equal(to_host(dist).view(np.uint32), rd.view(np.uint32))
+
+
+@pytest.mark.parametrize("n,d,kc", [(20000, 64, 1024), (3001, 64, 100), (5000, 32, 7), (999, 130, 300)])
+def test_kmeans_assign_bitexact_vs_alg1_model(oracle_lib, n, d, kc):
+    """egemm_kmeans_step's assignment equals the profiled-tensor-core model bitwise, so its
+    fp64 sums equal the oracle's R20 sums of that assignment bitwise: the whole step is
+    exact against the oracle (no gap exemptions)."""
+    eg = require_gpu()
+    X, _, _ = inputs.mixture(n, d, min(kc, 1024), 50 + d, sigma=0.2)
+    C = X[:kc].copy()
+    a, sums, counts, _ = eg.kmeans_step(to_dev(X), to_dev(C))
+    ra, _ = oracle_lib.kmeans_assign_alg1_tc(X, C)
+    assert np.array_equal(to_host(a), ra)
+    rs, rc = oracle_lib.group_sums(X, ra, kc)
+    assert np.array_equal(to_host(sums), rs) and np.array_equal(to_host(counts), rc)

@@ -154,3 +154,56 @@ def test_tc_models_reduce_to_textbook_cases(oracle_lib):
     a3 = [2.0 ** -14] + [0.0] * 15
     b3 = [2.0 ** -14] + [0.0] * 15
     assert m(a3, b3, 1.0, "align", 3) == 1.0 and m(a3, b3, 1.0, "rn") == 1.0
+
+
+# ------------------------------------------------------------------ R22 bitwise app models
+def test_rownorm_tree_vs_exact(oracle_lib):
+    """rownorm_tree (R22) is within 1 fp32 ulp of the correctly rounded exact sum of squares
+    and equal to it for nearly all rows; integer rows are exact."""
+    from fractions import Fraction
+    g = inputs.rng(2201)
+    for d in (1, 33, 100, 128, 257):
+        X = g.uniform(-2, 2, (300, d)).astype(np.float32)
+        tree = oracle_lib.rownorm_tree(X)
+        exact = np.array([float(sum(Fraction(float(v)) ** 2 for v in row)) for row in X],
+                         np.float64).astype(np.float32)
+        ulp = np.spacing(exact)
+        assert np.all(np.abs(tree.astype(np.float64) - exact) <= ulp)
+        assert np.mean(tree == exact) >= 0.97
+    Xi = g.integers(-40, 41, (50, 300)).astype(np.float32)
+    assert np.array_equal(oracle_lib.rownorm_tree(Xi), (Xi.astype(np.int64) ** 2).sum(1).astype(np.float32))
+
+
+def test_knn_alg1_tc_integer_data_is_exact(oracle_lib):
+    """On small integers every step is exact, so the TC model kNN equals the exact kNN."""
+    g = inputs.rng(2202)
+    X = g.integers(-4, 5, (400, 20)).astype(np.float32)
+    Q = g.integers(-4, 5, (37, 20)).astype(np.float32)
+    i1, d1 = oracle_lib.knn_alg1_tc(X, Q, 9)
+    i0, d0 = oracle_lib.knn(X, Q, 9)
+    assert np.array_equal(i1, i0) and np.array_equal(d1.astype(np.float64), d0)
+
+
+def test_knn_alg1_tc_agrees_with_exact_where_gap(oracle_lib):
+    g = inputs.rng(2203)
+    X, Q = g.uniform(-1, 1, (600, 48)), g.uniform(-1, 1, (40, 48))
+    i1, _ = oracle_lib.knn_alg1_tc(X, Q, 8)
+    D = oracle_lib.sqdist(X, Q)
+    for r in range(Q.shape[0]):
+        o = np.argsort(D[r], kind="stable")
+        if D[r, o[8]] - D[r, o[7]] > 1e-5:  # far above the method's error bound here
+            assert set(i1[r]) == set(o[:8])
+
+
+def test_kmeans_assign_alg1_tc_integer_and_ties(oracle_lib):
+    g = inputs.rng(2204)
+    X = g.integers(-3, 4, (500, 12)).astype(np.float32)
+    C = g.integers(-3, 4, (17, 12)).astype(np.float32)
+    C[9] = C[4]  # duplicate centroid: ties must go to the lower index
+    a, best = oracle_lib.kmeans_assign_alg1_tc(X, C)
+    D = ((X[:, None, :].astype(np.int64) - C[None].astype(np.int64)) ** 2).sum(2)
+    assert np.array_equal(a, np.argmin(D, 1))
+    assert not np.any(a == 9)
+    cn = (C.astype(np.int64) ** 2).sum(1)
+    assert np.array_equal(best.astype(np.int64), (D - (X.astype(np.int64) ** 2).sum(1)[:, None])[np.arange(500), a])
+    assert np.all(cn[a] - 2 * (X.astype(np.int64) * C[a].astype(np.int64)).sum(1) == best)
