@@ -1,8 +1,10 @@
-"""GPU parity of egemm_knn / egemm_kmeans_step against the fp64 oracles.
+"""GPU parity of egemm_knn / egemm_kmeans_step against the oracles.
 
-Rule (BASELINE north_star; reading R18): neighbour sets / assignments must be identical
-wherever the oracle's distance gap exceeds the method's error bound tau; rows whose gap
-is within tau are exempt (several answers are then correct) and only checked for validity.
+Two bars.  (1) Against the exact fp64 definitions (BASELINE north_star; reading R18):
+neighbour sets / assignments identical wherever the oracle's distance gap exceeds the
+method's error bound tau; rows within tau are exempt and only checked for validity.
+(2) Against the bitwise models of the method on the profiled tensor core (R21, R22):
+indices, distances and assignments identical bit for bit, no exemptions.
 """
 import numpy as np
 import pytest
