@@ -90,6 +90,10 @@ def test_knn_full_size_sampled_queries(oracle_lib):
         dd = oracle_lib.sqdist(X[idx[i]], Q[i:i + 1])[0]
         assert np.all(np.abs(dist[i] - dd) <= np.array([tau_of[int(j)] for j in idx[i]]) + 1e-6)
     assert exempt <= 2
+    # and bitwise against the profiled-tensor-core model (R22) on 2 of the sampled queries
+    bi, bd = oracle_lib.knn_alg1_tc(X, Q[qs[:2]], k)
+    assert np.array_equal(idx[qs[:2]], bi)
+    assert np.array_equal(dist[qs[:2]].view(np.uint32), bd.view(np.uint32))
 
 
 def test_kmeans_full_size_step_sampled(oracle_lib):
@@ -113,3 +117,6 @@ def test_kmeans_full_size_step_sampled(oracle_lib):
     assert (~strict).sum() <= 0.01 * len(ps)
     ref, rcnt = oracle_lib.group_sums(X, a, kc)
     assert np.array_equal(counts, rcnt) and np.array_equal(sums, ref)
+    # bitwise against the profiled-tensor-core model (R22) on 4096 of the sampled points
+    ba, _ = oracle_lib.kmeans_assign_alg1_tc(X[ps[:4096]], C)
+    assert np.array_equal(a[ps[:4096]], ba)
