@@ -473,11 +473,43 @@ def _apps(world, rank, dev, args):
         del A2, B2, ws2, D2
     except Exception as ex:  # pragma: no cover
         out["tall_skinny"] = {"error": str(ex)[:300]}
+    try:  # configs[1]'s other square sizes (the headline is 8192^3): one public call each,
+        # fp32 in -> fp32 out (splits included), rows sharded, steady-state windows
+        sweep = {}
+        for n2 in (1024, 2048, 4096, 16384):
+            r0, r1 = edist.shard_bounds(n2, world, rank, align=256)
+            A2 = (torch.rand(r1 - r0, n2, device=dev, generator=torch.Generator(dev).manual_seed(n2))
+                  * 2 - 1)
+            B2 = torch.rand(n2, n2, device=dev, generator=torch.Generator(dev).manual_seed(n2 + 1)) * 2 - 1
+            ws2 = torch.empty(egemm.gemm_workspace_size(r1 - r0, n2, n2), dtype=torch.uint8, device=dev)
+            D2 = torch.empty((r1 - r0, n2), device=dev)
+            one = 2.0 * n2 ** 3 / 400e12 * 1e3  # ms, rough
+            reps = max(5, int(150.0 / max(one, 1e-3)))
+            for _ in range(max(3, reps // 5)):
+                egemm.gemm(A2, B2, out=D2, workspace=ws2)
+            _barrier(world)
+            s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            s.record()
+            for _ in range(reps):
+                egemm.gemm(A2, B2, out=D2, workspace=ws2)
+            e.record()
+            _barrier(world)
+            ms = _allmax(s.elapsed_time(e), world) / reps
+            sweep[str(n2)] = {"tflops": round(2.0 * n2 ** 3 / (ms * 1e-3) / 1e12, 1), "ms": round(ms, 4),
+                              "config": list(egemm.query_config("gemm", r1 - r0, n2, n2, with_fused=True))}
+            del A2, B2, ws2, D2
+        out["square_sweep"] = {"metric": "EGEMM FP32-equiv TFLOP/s, N^3 (configs[1] sweep; split included)",
+                               "unit": "TFLOP/s", "by_n": sweep}
+    except Exception as ex:  # pragma: no cover
+        out["square_sweep"] = {"error": str(ex)[:300]}
+    cpu_ok = rank == 0 and world == 1 and not args.no_cpu
     try:
         nx, nq, d, k = 1 << 20, 1 << 16, 128, 16
         q0, q1 = edist.shard_bounds(nq, world, rank)
-        X = torch.from_numpy(inputs.uniform((nx, d), 300)).to(dev)
-        Q = torch.from_numpy(inputs.uniform((nq, d), 301)[q0:q1]).to(dev)
+        Xh = inputs.uniform((nx, d), 300)
+        Qh = inputs.uniform((nq, d), 301)
+        X = torch.from_numpy(Xh).to(dev)
+        Q = torch.from_numpy(Qh[q0:q1]).to(dev)
         t_ib = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
         t_ib[0].record()
         index = egemm.knn_index(X)  # the index build (once): split + norms of X
@@ -502,7 +534,21 @@ def _apps(world, rank, dev, args):
                       "fp32eq_tflops": round(2.0 * nx * nq * d / (ms * 1e-3) / 1e12, 1),
                       "kernel_sm_mhz": round(egemm.debug_last_clock(), 1),
                       "sharding": "queries over %d ranks, X replicated" % world}
-        del X, Q, index, ws
+        if cpu_ok:  # the plain fp64 kNN oracle on a bounded query sample (host cores)
+            import oracle
+            t0 = time.perf_counter()
+            oracle.knn(Xh, Qh[:16], k)
+            per_q = (time.perf_counter() - t0) / 16
+            nqs = int(max(16, min(1024, args.cpu_seconds / 2 / per_q)))
+            t0 = time.perf_counter()
+            oracle.knn(Xh, Qh[:nqs], k)
+            dt = time.perf_counter() - t0
+            out["knn"]["cpu_baseline"] = {"value": round(nqs / dt, 2), "unit": "queries/s",
+                                          "cores": oracle.num_threads(), "kind": "oracle",
+                                          "sample": "oracle.knn (direct fp64 distances) on %d of the "
+                                                    "64K queries against all 1M references, %.1f s"
+                                                    % (nqs, dt)}
+        del X, Q, index, ws, Xh, Qh
     except Exception as ex:  # pragma: no cover
         out["knn"] = {"error": str(ex)[:300]}
     try:
@@ -511,6 +557,20 @@ def _apps(world, rank, dev, args):
         Xh, lab, _ = inputs.mixture(n, d, kc, 400)
         X = torch.from_numpy(Xh[p0:p1]).to(dev)
         C0 = torch.from_numpy(Xh[:kc].copy()).to(dev)
+        if cpu_ok:  # one oracle Lloyd step (fp64 direct distances + R20 sums) on a point sample
+            import oracle
+            ps = 1 << 14
+            t0 = time.perf_counter()
+            oracle.kmeans_step(Xh[:ps], Xh[:kc])
+            per_pt = (time.perf_counter() - t0) / ps
+            ps = int(max(ps, min(n, args.cpu_seconds / 2 / per_pt)))
+            t0 = time.perf_counter()
+            oracle.kmeans_step(Xh[:ps], Xh[:kc])
+            dt = time.perf_counter() - t0
+            kmeans_cpu = {"value": round(dt * n / ps * 1e3, 1), "unit": "ms/iter",
+                          "cores": oracle.num_threads(), "kind": "oracle",
+                          "sample": "oracle.kmeans_step on %d of the 4M points (x %.0f to a full "
+                                    "iteration), %.1f s" % (ps, n / ps, dt)}
         del Xh
         x_split = egemm.split(X)
         C = C0.clone()
@@ -532,6 +592,8 @@ def _apps(world, rank, dev, args):
                          "fp32eq_tflops": round(2.0 * n * kc * d / (ms * 1e-3) / 1e12, 1),
                          "kernel_sm_mhz": round(egemm.debug_last_clock(), 1),
                          "sharding": "points over %d ranks, NCCL all_reduce of sums/counts" % world}
+        if cpu_ok:
+            out["kmeans"]["cpu_baseline"] = kmeans_cpu
     except Exception as ex:  # pragma: no cover
         out["kmeans"] = {"error": str(ex)[:300]}
     return out
