@@ -250,6 +250,8 @@ def main():
     launches_per_step = 2 if fused_a else 3
     ws_a = torch.empty(egemm.gemm_workspace_size(m_loc, N, K, False, True), dtype=torch.uint8,
                        device=dev)
+    ws_p = torch.empty(egemm.gemm_workspace_size(m_loc, N, K, True, True), dtype=torch.uint8,
+                       device=dev)  # the k-pacing counters only (256 B)
 
     def pre():  # the splits outside the GEMM kernel
         if not fused_a:
@@ -260,7 +262,7 @@ def main():
         if fused_a:
             egemm.gemm(A, None, b_split=b_split, out=D, workspace=ws_a)
         else:
-            egemm.gemm(None, None, a_split=a_split, b_split=b_split, out=D)
+            egemm.gemm(None, None, a_split=a_split, b_split=b_split, out=D, workspace=ws_p)
 
     def step():
         pre()

@@ -95,8 +95,11 @@ int egemm_split_trunc(const float* x, int64_t rows, int64_t cols, int64_t ldx, u
  *      alias A or B; D may equal C only if ldd == ldc.
  *  terms : 0 (tuning-table default, 3), 3, or 4.
  *  workspace : device scratch of >= egemm_gemm_workspace_size(...) bytes (256-B aligned),
- *      used for the on-the-fly split of operands given only in fp32.  May be NULL when
- *      that size is 0.
+ *      used for the on-the-fly split of operands given only in fp32 and, in its last
+ *      256 B, for the k-pacing counters that keep the persistent clusters within a few
+ *      k-blocks of each other (L2 reuse of shared tiles).  The pacing is
+ *      optional: a workspace that only covers the splits (NULL when both operands are
+ *      pre-split) is accepted and the kernel runs unpaced; results are identical.
  * M == 0 or N == 0: no-op.  K == 0: D = C (or 0).
  */
 int egemm_gemm(int64_t M, int64_t N, int64_t K, egemm_operand_t A, egemm_operand_t B,

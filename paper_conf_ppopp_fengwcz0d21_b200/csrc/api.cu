@@ -297,14 +297,22 @@ static int split_entry(const float* x, int64_t rows, int64_t cols, int64_t ldx, 
   return EGEMM_OK;
 }
 
-size_t egemm_gemm_workspace_size(int64_t M, int64_t N, int64_t K, int a_presplit,
-                                 int b_presplit) {
+// Bytes the operand splits need; the full workspace size adds kPaceBytes for the k-pacing
+// counters (optional: egemm_gemm runs unpaced when the workspace has no room for them).
+static constexpr size_t kPaceBytes = 256;
+static size_t gemm_operand_ws(int64_t M, int64_t N, int64_t K, int a_presplit, int b_presplit) {
   if (M <= 0 || N <= 0 || K <= 0) return 0;
   Carver cv{nullptr};
   const int64_t ldk = ldk_of(K);
   if (!a_presplit) { cv.take<uint16_t>((size_t)(M * ldk)); cv.take<uint16_t>((size_t)(M * ldk)); }
   if (!b_presplit) { cv.take<uint16_t>((size_t)(N * ldk)); cv.take<uint16_t>((size_t)(N * ldk)); }
   return cv.off;
+}
+
+size_t egemm_gemm_workspace_size(int64_t M, int64_t N, int64_t K, int a_presplit,
+                                 int b_presplit) {
+  if (M <= 0 || N <= 0 || K <= 0) return 0;
+  return gemm_operand_ws(M, N, K, a_presplit, b_presplit) + kPaceBytes;
 }
 
 int egemm_gemm(int64_t M, int64_t N, int64_t K, egemm_operand_t A, egemm_operand_t B,
@@ -333,7 +341,7 @@ int egemm_gemm(int64_t M, int64_t N, int64_t K, egemm_operand_t A, egemm_operand
   int r;
   if ((r = check_operand(A, M, K, false, "A"))) return r;
   if ((r = check_operand(B, N, K, true, "B"))) return r;
-  size_t need = egemm_gemm_workspace_size(M, N, K, A.hi != nullptr, B.hi != nullptr);
+  size_t need = gemm_operand_ws(M, N, K, A.hi != nullptr, B.hi != nullptr);
   if (need > 0 && (!workspace || workspace_bytes < need)) {
     set_last_error("workspace %zu < %zu", workspace_bytes, need);
     return EGEMM_ERR_WORKSPACE;
@@ -361,6 +369,7 @@ int egemm_gemm(int64_t M, int64_t N, int64_t K, egemm_operand_t A, egemm_operand
   epi.ldd = ldd;
   epi.C = C;
   epi.ldc = ldc;
+  if (workspace && workspace_bytes >= cv.off + kPaceBytes) epi.sync = cv.take<uint32_t>(64);
   r = launch_tc(M, N, K, ops, cfg, epi, s);
   return r == 0 ? EGEMM_OK : (r == 2 ? EGEMM_ERR_UNSUPPORTED : EGEMM_ERR_CUDA);
 }

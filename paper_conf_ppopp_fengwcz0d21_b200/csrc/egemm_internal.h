@@ -46,6 +46,7 @@ struct TcEpilogue {
   int64_t ldd;
   const float* C;
   int64_t ldc;
+  uint32_t* sync;      // nullable: 256 B of workspace for the k-pacing counters
   // EPI_KNN / EPI_KMEANS: per-B-row squared norms (||x_j||^2 or ||c_j||^2)
   const float* bnorm;
   // EPI_KNN

@@ -74,10 +74,38 @@ struct KParams {
   int K;
   int debug_no_tma;  // EGEMM_DEBUG_NO_TMA=1: skip operand loads (timing diagnostics only)
   int debug_no_epi;  // EGEMM_DEBUG_NO_EPI=1: skip the promotion's TMEM reads (diagnostics)
+  uint32_t* sync;    // nullable: kSyncR epoch counters (zeroed per launch) for the k-pacing
   int debug_mode;    // EGEMM_DEBUG_MODE bits (diagnostics): 1 extra commit per k-block;
                      // with NO_TMA: 2 MMA warp ignores the full barriers (producer idle),
                      // 4 no per-k-block commits
 };
+
+// ---------------------------------------------------------------- k-pacing (STORE GEMMs)
+// Clusters that share A or B tiles (the 8-m-tile band order) only share them through L2 if
+// they read the same k-slabs at about the same time.  Left free, persistent clusters drift
+// apart over long K and the L2 working set outgrows 126 MB (measured: 57 GB of DRAM reads
+// per 16384^3 launch vs ~2.6 GB at 8192^3), which costs power and hence clock.  Each CTA's
+// producer therefore arrives at a global epoch counter every kSyncE k-blocks and, before
+// loading epoch e, waits until every CTA has started epoch e - kSyncS: the grid stays within
+// ~kSyncS epochs of k.  Counters live in the caller's workspace (kSyncR monotone slots,
+// zeroed per launch); it is a throttle only -- results do not depend on it.
+constexpr int kSyncE = 8;   // k-blocks (of 64) per epoch
+constexpr int kSyncS = 3;   // slack in epochs
+constexpr int kSyncR = 8;   // counter ring (> kSyncS)
+
+__device__ __forceinline__ void sync_arrive(uint32_t* sync, uint32_t e) {
+  atomicAdd(sync + (e % kSyncR), 1u);
+}
+__device__ __forceinline__ void sync_wait(const uint32_t* sync, uint32_t e, uint32_t nctas) {
+  const uint32_t need = nctas * (e / kSyncR + 1);
+  const uint32_t* c = sync + (e % kSyncR);
+  uint32_t v;
+  while (true) {
+    asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(c) : "memory");
+    if ((int32_t)(v - need) >= 0) break;
+    __nanosleep(64);
+  }
+}
 
 template <int CG, int BN>
 struct Geo {
@@ -346,6 +374,8 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
       // carries only B, A is loaded once per unit into a_res
       constexpr uint32_t TX = (FA || AR) ? 2 * G::B_BYTES : G::STAGE_BYTES;
       uint32_t uctr = 0;
+      const bool pace = (EPI == EPI_STORE) && p.sync != nullptr && !p.debug_no_tma;
+      uint32_t gkb = 0;  // k-blocks this CTA has started loading, over all its units
       const bool idle = p.debug_no_tma && (p.debug_mode & 2);  // diagnostics only
       for (int u = idle ? p.num_units : cluster; u < p.num_units; u += nclusters, uctr++) {
         UnitInfo ui = decode_unit<EPI>(p, u);
@@ -367,6 +397,12 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
         for (int ns = 0; ns < ui.n_count; ns++) {
           const int brow = (ui.n_begin + ns) * BN + (int)rank * G::BNC;
           for (int kb = 0; kb < p.num_kb; kb++) {
+            if (pace && (gkb % kSyncE) == 0) {
+              const uint32_t e = gkb / kSyncE;
+              sync_arrive(p.sync, e);
+              if (e >= (uint32_t)kSyncS) sync_wait(p.sync, e - kSyncS, gridDim.x);
+            }
+            gkb++;
             ptx::mbar_wait(&empty[stage], phase ^ 1u);
             uint8_t* sb = stage_base + stage * SB;
             if (p.debug_no_tma) {  // diagnostics only: MMA-issue ceiling without operand traffic
@@ -394,6 +430,11 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
             if (++stage == STAGES) { stage = 0; phase ^= 1u; }
           }
         }
+      }
+      if (pace) {  // out of units: arrive at every remaining epoch so nobody waits on us
+        const uint32_t per_cta = (uint32_t)((p.num_units + nclusters - 1) / nclusters) * p.num_kb;
+        const uint32_t total = (per_cta + kSyncE - 1) / kSyncE;
+        for (uint32_t e = (gkb + kSyncE - 1) / kSyncE; e < total; e++) sync_arrive(p.sync, e);
       }
     }
   } else if (warp == EG::W_MMA) {
@@ -941,6 +982,11 @@ int launch_tc(int64_t M, int64_t N, int64_t K, const TcOperands& ops, const TcCo
   kp.n_tiles = (int)((N + cfg.bn - 1) / cfg.bn);
   kp.D = epi.D;
   kp.ldd = epi.ldd;
+  kp.sync = (epi.kind == EPI_STORE && !getenv_flag("EGEMM_NO_PACE")) ? epi.sync : nullptr;
+  if (kp.sync && cudaMemsetAsync(kp.sync, 0, kSyncR * sizeof(uint32_t), stream) != cudaSuccess) {
+    set_last_error("memset of the pacing counters failed");
+    return 3;
+  }
   kp.C = epi.C;
   kp.ldc = epi.ldc;
   kp.vec_ok = (epi.D && (epi.ldd % 4 == 0) && ((uintptr_t)epi.D % 16 == 0) &&

@@ -68,8 +68,9 @@ def test_status_strings_and_host_validation(lib):
 
 def test_workspace_queries(lib):
     from paper_conf_ppopp_fengwcz0d21_b200 import egemm
-    assert egemm.gemm_workspace_size(256, 256, 256) == 4 * 256 * 256 * 2
-    assert egemm.gemm_workspace_size(256, 256, 256, True, True) == 0
+    # hi + lo of A and B, plus 256 B of k-pacing counters (optional for egemm_gemm)
+    assert egemm.gemm_workspace_size(256, 256, 256) == 4 * 256 * 256 * 2 + 256
+    assert egemm.gemm_workspace_size(256, 256, 256, True, True) == 256
     assert egemm.gemm_workspace_size(0, 5, 5) == 0
     assert egemm.knn_workspace_size(1000, 10, 128, 16) > 0
     assert egemm.kmeans_workspace_size(1000, 64, 10) > 0

@@ -196,3 +196,26 @@ def test_gemm_fused_a_strided_rows(oracle_lib, monkeypatch):
     finally:
         eg.set_config(0, 0, 0, 0)
     _assert_parity(oracle_lib, big[:, 1:514], B, D)
+
+
+@pytest.mark.parametrize("shape", [(2048, 2048, 4096), (1000, 3000, 2500), (300, 256, 64)])
+def test_gemm_k_pacing_does_not_change_results(monkeypatch, shape):
+    """The k-pacing counters (workspace tail) only throttle the producers: paced, unpaced
+    (EGEMM_NO_PACE) and ops-only-workspace runs are bitwise identical, fused or pre-split."""
+    eg = require_gpu()
+    M, N, K = shape
+    A, B = inputs.uniform((M, K), 510), inputs.uniform((K, N), 511)
+    Ad, Bd = to_dev(A), to_dev(B)
+    full = torch.empty(eg.gemm_workspace_size(M, N, K), dtype=torch.uint8, device="cuda")
+    D1 = eg.gemm(Ad, Bd, workspace=full)
+    monkeypatch.setenv("EGEMM_NO_PACE", "1")
+    D2 = eg.gemm(Ad, Bd, workspace=full)
+    monkeypatch.delenv("EGEMM_NO_PACE")
+    ops_only = torch.empty(eg.gemm_workspace_size(M, N, K) - 256, dtype=torch.uint8, device="cuda")
+    D3 = torch.empty((M, N), device="cuda")
+    eg.load().egemm_gemm(M, N, K, eg.operand(Ad), eg.operand(Bd), None, 0,
+                         eg._ptr(D3), N, 0, eg._ptr(ops_only), ops_only.numel(), eg._stream())
+    a_s, b_s = eg.split(Ad), eg.split(Bd, transpose=True)
+    D4 = eg.gemm(None, None, a_split=a_s, b_split=b_s)  # 256-B pacing workspace only
+    for D in (D2, D3, D4):
+        assert torch.equal(D1.view(torch.int32), D.view(torch.int32))

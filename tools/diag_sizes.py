@@ -7,9 +7,14 @@ for n in (8192, 16384, 12288):
     a_s, b_s = egemm.split(A), egemm.split(B, transpose=True)
     D = torch.empty(n, n, device="cuda")
     need = 6.0 * n ** 3 / (148 * 8192.0)
-    for cfg in ((2, 256, 0, 256), (2, 256, 0, 128)):
+    ws = torch.empty(egemm.gemm_workspace_size(n, n, n, True, True), dtype=torch.uint8, device="cuda")
+    for cfg, pace in (((2, 256, 0, 256), 1), ((2, 256, 0, 256), 0), ((2, 256, 0, 256), 1)):
+        if pace:
+            os.environ.pop("EGEMM_NO_PACE", None)
+        else:
+            os.environ["EGEMM_NO_PACE"] = "1"
         egemm.set_config(*cfg)
-        f = lambda: egemm.gemm(None, None, a_split=a_s, b_split=b_s, out=D)
+        f = lambda: egemm.gemm(None, None, a_split=a_s, b_split=b_s, out=D, workspace=ws)
         for _ in range(3): f()
         torch.cuda.synchronize()
         egemm.debug_clock_stats(reset=True)
@@ -20,6 +25,6 @@ for n in (8192, 16384, 12288):
         e.record(); e.synchronize()
         ms = s.elapsed_time(e) / it
         mhz, cyc, nl = egemm.debug_clock_stats(reset=True)
-        print(n, cfg, "%.3f ms %.0f TF-fp16 %.0f MHz cycle-eff %.3f" % (ms, 6.0 * n ** 3 / ms / 1e9, mhz, need / cyc), flush=True)
+        print(n, cfg, "paced" if pace else "free ", "%.3f ms %.0f TF-fp16 %.0f MHz cycle-eff %.3f" % (ms, 6.0 * n ** 3 / ms / 1e9, mhz, need / cyc), flush=True)
     del A, B, a_s, b_s, D
     torch.cuda.empty_cache()
