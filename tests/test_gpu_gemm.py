@@ -198,7 +198,7 @@ def test_gemm_fused_a_strided_rows(oracle_lib, monkeypatch):
     _assert_parity(oracle_lib, big[:, 1:514], B, D)
 
 
-@pytest.mark.parametrize("shape", [(2048, 2048, 4096), (1000, 3000, 2500), (300, 256, 64)])
+@pytest.mark.parametrize("shape", [(2048, 2048, 4096), (1000, 3000, 2504), (300, 256, 64)])
 def test_gemm_k_pacing_does_not_change_results(monkeypatch, shape):
     """The k-pacing counters (workspace tail) only throttle the producers: paced, unpaced
     (EGEMM_NO_PACE) and ops-only-workspace runs are bitwise identical, fused or pre-split."""
