@@ -75,6 +75,7 @@ struct KParams {
   int debug_no_tma;  // EGEMM_DEBUG_NO_TMA=1: skip operand loads (timing diagnostics only)
   int debug_no_epi;  // EGEMM_DEBUG_NO_EPI=1: skip the promotion's TMEM reads (diagnostics)
   uint32_t* sync;    // nullable: kSyncR epoch counters (zeroed per launch) for the k-pacing
+  int pace_e, pace_s;  // k-blocks per epoch, slack in epochs
   int debug_mode;    // EGEMM_DEBUG_MODE bits (diagnostics): 1 extra commit per k-block;
                      // with NO_TMA: 2 MMA warp ignores the full barriers (producer idle),
                      // 4 no per-k-block commits
@@ -89,9 +90,9 @@ struct KParams {
 // loading epoch e, waits until every CTA has started epoch e - kSyncS: the grid stays within
 // ~kSyncS epochs of k.  Counters live in the caller's workspace (kSyncR monotone slots,
 // zeroed per launch); it is a throttle only -- results do not depend on it.
-constexpr int kSyncE = 8;   // k-blocks (of 64) per epoch
-constexpr int kSyncS = 3;   // slack in epochs
-constexpr int kSyncR = 8;   // counter ring (> kSyncS)
+constexpr int kSyncE = 8;   // default k-blocks (of 64) per epoch
+constexpr int kSyncS = 3;   // default slack in epochs
+constexpr int kSyncR = 8;   // counter ring (> slack)
 
 __device__ __forceinline__ void sync_arrive(uint32_t* sync, uint32_t e) {
   atomicAdd(sync + (e % kSyncR), 1u);
@@ -397,10 +398,10 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
         for (int ns = 0; ns < ui.n_count; ns++) {
           const int brow = (ui.n_begin + ns) * BN + (int)rank * G::BNC;
           for (int kb = 0; kb < p.num_kb; kb++) {
-            if (pace && (gkb % kSyncE) == 0) {
-              const uint32_t e = gkb / kSyncE;
+            if (pace && (gkb % (uint32_t)p.pace_e) == 0) {
+              const uint32_t e = gkb / (uint32_t)p.pace_e;
               sync_arrive(p.sync, e);
-              if (e >= (uint32_t)kSyncS) sync_wait(p.sync, e - kSyncS, gridDim.x);
+              if (e >= (uint32_t)p.pace_s) sync_wait(p.sync, e - p.pace_s, gridDim.x);
             }
             gkb++;
             ptx::mbar_wait(&empty[stage], phase ^ 1u);
@@ -433,8 +434,9 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
       }
       if (pace) {  // out of units: arrive at every remaining epoch so nobody waits on us
         const uint32_t per_cta = (uint32_t)((p.num_units + nclusters - 1) / nclusters) * p.num_kb;
-        const uint32_t total = (per_cta + kSyncE - 1) / kSyncE;
-        for (uint32_t e = (gkb + kSyncE - 1) / kSyncE; e < total; e++) sync_arrive(p.sync, e);
+        const uint32_t pe = (uint32_t)p.pace_e;
+        const uint32_t total = (per_cta + pe - 1) / pe;
+        for (uint32_t e = (gkb + pe - 1) / pe; e < total; e++) sync_arrive(p.sync, e);
       }
     }
   } else if (warp == EG::W_MMA) {
@@ -983,6 +985,14 @@ int launch_tc(int64_t M, int64_t N, int64_t K, const TcOperands& ops, const TcCo
   kp.D = epi.D;
   kp.ldd = epi.ldd;
   kp.sync = (epi.kind == EPI_STORE && !getenv_flag("EGEMM_NO_PACE")) ? epi.sync : nullptr;
+  {
+    const char* pe = getenv("EGEMM_PACE_E");
+    const char* ps = getenv("EGEMM_PACE_S");
+    kp.pace_e = pe ? atoi(pe) : kSyncE;
+    kp.pace_s = ps ? atoi(ps) : kSyncS;
+    if (kp.pace_e < 4) kp.pace_e = 4;  // a pair partner runs <= STAGES k-blocks ahead
+    if (kp.pace_s < 2 || kp.pace_s >= kSyncR) kp.pace_s = kSyncS;  // >= 2: no pair deadlock
+  }
   if (kp.sync && cudaMemsetAsync(kp.sync, 0, kSyncR * sizeof(uint32_t), stream) != cudaSuccess) {
     set_last_error("memset of the pacing counters failed");
     return 3;
