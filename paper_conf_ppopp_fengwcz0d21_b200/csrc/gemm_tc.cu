@@ -91,7 +91,7 @@ struct KParams {
 // ~kSyncS epochs of k.  Counters live in the caller's workspace (kSyncR monotone slots,
 // zeroed per launch); it is a throttle only -- results do not depend on it.
 constexpr int kSyncE = 8;   // default k-blocks (of 64) per epoch
-constexpr int kSyncS = 3;   // default slack in epochs
+constexpr int kSyncS = 2;   // default slack in epochs (tools/pace_sweep.py)
 constexpr int kSyncR = 8;   // counter ring (> slack)
 
 __device__ __forceinline__ void sync_arrive(uint32_t* sync, uint32_t e) {
