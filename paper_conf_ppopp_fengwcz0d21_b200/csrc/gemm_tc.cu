@@ -76,6 +76,7 @@ struct KParams {
   int debug_no_epi;  // EGEMM_DEBUG_NO_EPI=1: skip the promotion's TMEM reads (diagnostics)
   uint32_t* sync;    // nullable: kSyncR epoch counters (zeroed per launch) for the k-pacing
   int pace_e, pace_s;  // k-blocks per epoch, slack in epochs
+  int band_m;          // STORE tile order: m-tiles per band
   int debug_mode;    // EGEMM_DEBUG_MODE bits (diagnostics): 1 extra commit per k-block;
                      // with NO_TMA: 2 MMA warp ignores the full barriers (producer idle),
                      // 4 no per-k-block commits
@@ -137,9 +138,9 @@ template <int EPI>
 __device__ __forceinline__ UnitInfo decode_unit(const KParams& p, int u) {
   UnitInfo r;
   if constexpr (EPI == EPI_STORE) {
-    // bands of up to 8 m-tiles, m fastest inside a band: concurrent clusters share A and B
-    // k-slabs in L2.
-    const int GM = 8;
+    // bands of up to band_m (8) m-tiles, m fastest inside a band: concurrent clusters share
+    // A and B k-slabs in L2.
+    const int GM = p.band_m;
     int band = u / (GM * p.n_tiles);
     int m0 = band * GM;
     int gm = min(GM, p.m_tiles - m0);
@@ -992,6 +993,9 @@ int launch_tc(int64_t M, int64_t N, int64_t K, const TcOperands& ops, const TcCo
     kp.pace_s = ps ? atoi(ps) : kSyncS;
     if (kp.pace_e < 4) kp.pace_e = 4;  // a pair partner runs <= STAGES k-blocks ahead
     if (kp.pace_s < 2 || kp.pace_s >= kSyncR) kp.pace_s = kSyncS;  // >= 2: no pair deadlock
+    const char* bm = getenv("EGEMM_BAND");
+    kp.band_m = bm ? atoi(bm) : 8;
+    if (kp.band_m < 1) kp.band_m = 8;
   }
   if (kp.sync && cudaMemsetAsync(kp.sync, 0, kSyncR * sizeof(uint32_t), stream) != cudaSuccess) {
     set_last_error("memset of the pacing counters failed");

@@ -29,6 +29,8 @@ def run(f, n, seconds=1.0):
 def main():
     sizes = [int(a) for a in sys.argv[1:]] or [8192, 16384]
     combos = [(None, None), (4, 2), (4, 3), (8, 2), (8, 3), (8, 4), (16, 2), (16, 3), (32, 2)]
+    if os.environ.get("BANDS"):  # sweep the band height at the default pacing instead
+        combos = [("band", int(b)) for b in os.environ["BANDS"].split(",")]
     for n in sizes:
         A = torch.rand(n, n, device="cuda") * 2 - 1
         B = torch.rand(n, n, device="cuda") * 2 - 1
@@ -38,9 +40,11 @@ def main():
         f = lambda: egemm.gemm(None, None, a_split=a_s, b_split=b_s, out=D, workspace=ws)  # noqa: E731
         for rep in range(2):
             for E, S in combos:
-                for k in ("EGEMM_NO_PACE", "EGEMM_PACE_E", "EGEMM_PACE_S"):
+                for k in ("EGEMM_NO_PACE", "EGEMM_PACE_E", "EGEMM_PACE_S", "EGEMM_BAND"):
                     os.environ.pop(k, None)
-                if E is None:
+                if E == "band":
+                    os.environ["EGEMM_BAND"] = str(S)
+                elif E is None:
                     os.environ["EGEMM_NO_PACE"] = "1"
                 else:
                     os.environ["EGEMM_PACE_E"], os.environ["EGEMM_PACE_S"] = str(E), str(S)
