@@ -380,6 +380,8 @@ int egemm_gemm(int64_t M, int64_t N, int64_t K, egemm_operand_t A, egemm_operand
 // tcgen05 GEMM (caller stream) -> D2H (second copy stream), double-buffered, so the two
 // PCIe directions and the GPU work overlap.  Streams/events are created once per device.
 static int64_t host_chunk_rows(int64_t M) {
+  const int forced = env_int("EGEMM_HOST_CHUNK", 0);  // experiments
+  if (forced > 0) return forced > M ? M : forced;
   int64_t c = ((M / 8 + 255) / 256) * 256;
   if (c < 256) c = 256;
   if (c > 4096) c = 4096;
