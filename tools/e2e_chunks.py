@@ -26,8 +26,24 @@ def main():
         e.record()
         e.synchronize()
         print("%s %.1f GB/s" % (name, 5 * n * n * 4 / (s.elapsed_time(e) * 1e-3) / 1e9), flush=True)
-    del dev
-    for chunk in (0, 256, 512, 1024, 2048):
+    # both directions at once (the e2e pipeline overlaps them)
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    dev2 = torch.empty(n, n, device="cuda")
+    torch.cuda.synchronize()
+    s.record()
+    with torch.cuda.stream(s1):
+        for _ in range(5):
+            dev.copy_(A, non_blocking=True)
+    with torch.cuda.stream(s2):
+        for _ in range(5):
+            D.copy_(dev2, non_blocking=True)
+    torch.cuda.synchronize()
+    e.record()
+    e.synchronize()
+    print("h2d+d2h concurrent: %.1f GB/s per direction"
+          % (5 * n * n * 4 / (s.elapsed_time(e) * 1e-3) / 1e9), flush=True)
+    del dev, dev2
+    for chunk in (0, 512):
         if chunk:
             os.environ["EGEMM_HOST_CHUNK"] = str(chunk)
         else:
