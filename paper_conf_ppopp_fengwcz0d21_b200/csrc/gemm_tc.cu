@@ -98,13 +98,19 @@ constexpr int kSyncR = 8;   // counter ring (> slack)
 __device__ __forceinline__ void sync_arrive(uint32_t* sync, uint32_t e) {
   atomicAdd(sync + (e % kSyncR), 1u);
 }
-__device__ __forceinline__ void sync_wait(const uint32_t* sync, uint32_t e, uint32_t nctas) {
+// Returns false if the wait gave up: pacing assumes every CTA of the grid is resident (one
+// persistent CTA per SM); if another kernel holds SMs and some CTAs have not started, the
+// waiters stop pacing after kSyncTimeoutNs instead of deadlocking, and the kernel runs unpaced.
+constexpr unsigned long long kSyncTimeoutNs = 200000ull;
+__device__ __forceinline__ bool sync_wait(const uint32_t* sync, uint32_t e, uint32_t nctas) {
   const uint32_t need = nctas * (e / kSyncR + 1);
   const uint32_t* c = sync + (e % kSyncR);
   uint32_t v;
+  const unsigned long long t0 = globaltimer_ns();
   while (true) {
     asm volatile("ld.relaxed.gpu.global.u32 %0, [%1];" : "=r"(v) : "l"(c) : "memory");
-    if ((int32_t)(v - need) >= 0) break;
+    if ((int32_t)(v - need) >= 0) return true;
+    if (globaltimer_ns() - t0 > kSyncTimeoutNs) return false;
     __nanosleep(64);
   }
 }
@@ -376,7 +382,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
       // carries only B, A is loaded once per unit into a_res
       constexpr uint32_t TX = (FA || AR) ? 2 * G::B_BYTES : G::STAGE_BYTES;
       uint32_t uctr = 0;
-      const bool pace = (EPI == EPI_STORE) && p.sync != nullptr && !p.debug_no_tma;
+      bool pace = (EPI == EPI_STORE) && p.sync != nullptr && !p.debug_no_tma;
       uint32_t gkb = 0;  // k-blocks this CTA has started loading, over all its units
       const bool idle = p.debug_no_tma && (p.debug_mode & 2);  // diagnostics only
       for (int u = idle ? p.num_units : cluster; u < p.num_units; u += nclusters, uctr++) {
@@ -402,7 +408,8 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
             if (pace && (gkb % (uint32_t)p.pace_e) == 0) {
               const uint32_t e = gkb / (uint32_t)p.pace_e;
               sync_arrive(p.sync, e);
-              if (e >= (uint32_t)p.pace_s) sync_wait(p.sync, e - p.pace_s, gridDim.x);
+              if (e >= (uint32_t)p.pace_s && !sync_wait(p.sync, e - p.pace_s, gridDim.x))
+                pace = false;  // not all CTAs resident: run unpaced (others time out too)
             }
             gkb++;
             ptx::mbar_wait(&empty[stage], phase ^ 1u);

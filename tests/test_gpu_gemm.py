@@ -219,3 +219,28 @@ def test_gemm_k_pacing_does_not_change_results(monkeypatch, shape):
     D4 = eg.gemm(None, None, a_split=a_s, b_split=b_s)  # 256-B pacing workspace only
     for D in (D2, D3, D4):
         assert torch.equal(D1.view(torch.int32), D.view(torch.int32))
+
+
+def test_gemm_concurrent_streams_paced():
+    """Two paced persistent GEMMs on two streams at once cannot all be resident: the pacing
+    waits time out instead of deadlocking, and both results are bitwise the serial ones."""
+    eg = require_gpu()
+    n = 4096
+    A1, B1 = to_dev(inputs.uniform((n, n), 520)), to_dev(inputs.uniform((n, n), 521))
+    A2, B2 = to_dev(inputs.uniform((n, n), 522)), to_dev(inputs.uniform((n, n), 523))
+    ref1, ref2 = eg.gemm(A1, B1), eg.gemm(A2, B2)
+    s1, s2 = torch.cuda.Stream(), torch.cuda.Stream()
+    w1 = torch.empty(eg.gemm_workspace_size(n, n, n), dtype=torch.uint8, device="cuda")
+    w2 = torch.empty(eg.gemm_workspace_size(n, n, n), dtype=torch.uint8, device="cuda")
+    torch.cuda.synchronize()
+    outs = []
+    for _ in range(3):
+        with torch.cuda.stream(s1):
+            D1 = eg.gemm(A1, B1, workspace=w1)
+        with torch.cuda.stream(s2):
+            D2 = eg.gemm(A2, B2, workspace=w2)
+        outs.append((D1, D2))
+    torch.cuda.synchronize()
+    for D1, D2 in outs:
+        assert torch.equal(D1.view(torch.int32), ref1.view(torch.int32))
+        assert torch.equal(D2.view(torch.int32), ref2.view(torch.int32))
