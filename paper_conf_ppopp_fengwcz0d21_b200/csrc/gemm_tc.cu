@@ -654,6 +654,16 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
           const uint32_t use = chunk_ctr >> 1;
           ptx::mbar_wait(&acc_full[buf], use & 1u);
           ptx::tc_fence_after();
+          if (p.debug_no_epi) {  // diagnostics only: release the accumulator untouched
+            ptx::tc_fence_before();
+            __syncwarp();
+            if (lane == 0) {
+              if constexpr (CG == 1) ptx::mbar_arrive(&acc_empty[buf]);
+              else ptx::mbar_arrive_cluster(&acc_empty[buf], 0);
+            }
+            chunk_ctr++;
+            continue;
+          }
           const uint32_t acc_hh = tmem_base + lane_off + (SEP ? 2 * buf : buf) * BN + cgp * COLS;
           // TMEM -> registers software-pipelined: the load of group c+1 is in flight while
           // group c is processed; the accumulator buffer is handed back to the MMA warp as
