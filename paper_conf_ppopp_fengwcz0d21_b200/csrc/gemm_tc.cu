@@ -792,6 +792,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
             const int oi = si[(g - 1) * kBM + r];
             if (ob < best || (ob == best && oi < besti)) { best = ob; besti = oi; }
           }
+          if (p.debug_no_epi) besti = 0;  // diagnostics: keep the downstream kernels in bounds
           if (row < p.M) { p.assign[row] = besti; p.best_key[row] = best; }
         }
         named_bar_sync(1 + q, 32 * GPQ);
