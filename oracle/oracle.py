@@ -64,6 +64,10 @@ def lib():
         L.oracle_tc_mma16.restype = ctypes.c_float
         L.oracle_gemm_alg1_tc.argtypes = [I64, I64, I64, P, P, P, I, I, I, P]
         L.oracle_gemm_alg1_tc.restype = None
+        L.oracle_tf32_parts.argtypes = [ctypes.c_float, P, P, P]
+        L.oracle_tf32_parts.restype = None
+        L.oracle_norm_step.argtypes = [I64, I64, P, P, P]
+        L.oracle_norm_step.restype = None
         L.oracle_num_threads.argtypes = []
         L.oracle_num_threads.restype = I
         _lib = L
@@ -273,18 +277,35 @@ def _kc_single(d: int) -> int:
     return ((d + 63) // 64) * 64  # one promotion chunk over the whole feature dimension
 
 
+def tf32_parts(y: float):
+    """(h, m, l) with y = h + m + l exactly, each part an exact tf32 value (reading R22)."""
+    h, m, l = ctypes.c_float(), ctypes.c_float(), ctypes.c_float()
+    lib().oracle_tf32_parts(float(np.float32(y)), ctypes.byref(h), ctypes.byref(m), ctypes.byref(l))
+    return h.value, m.value, l.value
+
+
+def norm_step(dot, nrm):
+    """acc_ij = TC(dot_ij; 1*h_j + 1*m_j + 1*l_j), (h, m, l) = tf32_parts(-nrm_j / 2): the
+    tensor-core step that adds -||x_j||^2 / 2 after the products (reading R22)."""
+    dot, nrm = _f32(dot), _f32(nrm)
+    M, N = dot.shape
+    out = np.empty((M, N), np.float32)
+    lib().oracle_norm_step(M, N, _p(dot), _p(nrm), _p(out))
+    return out
+
+
 def knn_alg1_tc(X, Q, k: int):
     """kNN with the distance GEMM done by Alg. 1 on the profiled tensor core (R21, R22):
-    key_ij = RN32(||x_j||^2 - 2 (q_i . x_j)), q_i . x_j = gemm_alg1_tc(Q, X^T, kc = whole d);
-    the k smallest (key, j) ascending; dist = max(0, RN32(||q_i||^2 + key)).  The bitwise
-    model of egemm_knn; the plain definition stays `knn` (exact distances, gap rule R18)."""
+    dot = gemm_alg1_tc(Q, X^T, kc = whole d); acc = norm_step(dot, ||x||^2) (one more
+    tensor-core step adding -||x_j||^2 / 2); key_ij = -2 acc_ij (exact); the k smallest
+    (key, j) ascending; dist = max(0, RN32(||q_i||^2 + key)).  The bitwise model of
+    egemm_knn; the plain definition stays `knn` (exact distances, gap rule R18)."""
     X, Q = _f32(X), _f32(Q)
     nx, d = X.shape
-    xn = rownorm_tree(X).astype(np.float64)
+    xn = rownorm_tree(X)
     qn = rownorm_tree(Q).astype(np.float64)
-    dot = gemm_alg1_tc(Q, X.T, terms=3, sep=0, kc=_kc_single(d)).astype(np.float64)
-    # fp64 holds -2 dot + xn exactly whenever it matters for the fp32 rounding: this is fma
-    key = (xn[None, :] - 2.0 * dot).astype(np.float32)
+    dot = gemm_alg1_tc(Q, X.T, terms=3, sep=0, kc=_kc_single(d))
+    key = np.float32(-2.0) * norm_step(dot, xn)
     order = np.lexsort((np.broadcast_to(np.arange(nx), key.shape), key), axis=1)[:, :k]
     kk = np.take_along_axis(key, order, 1)
     dist = (qn[:, None] + kk.astype(np.float64)).astype(np.float32)
@@ -293,13 +314,13 @@ def knn_alg1_tc(X, Q, k: int):
 
 def kmeans_assign_alg1_tc(X, C):
     """kMeans assignment with Alg. 1 on the profiled tensor core (R21, R22): key_ij =
-    RN32(||c_j||^2 - 2 (x_i . c_j)), assign_i = the lowest j of minimal key.  Returns
+    -2 norm_step(x_i . c_j, ||c_j||^2), assign_i = the lowest j of minimal key.  Returns
     (assign int32, best key fp32)."""
     X, C = _f32(X), _f32(C)
     d = X.shape[1]
-    cn = rownorm_tree(C).astype(np.float64)
-    dot = gemm_alg1_tc(X, C.T, terms=3, sep=0, kc=_kc_single(d)).astype(np.float64)
-    key = (cn[None, :] - 2.0 * dot).astype(np.float32)
+    cn = rownorm_tree(C)
+    dot = gemm_alg1_tc(X, C.T, terms=3, sep=0, kc=_kc_single(d))
+    key = np.float32(-2.0) * norm_step(dot, cn)
     a = np.argmin(key, axis=1)  # first occurrence: ties -> lowest j
     return a.astype(np.int32), key[np.arange(len(a)), a]
 
@@ -317,13 +338,16 @@ def group_sums(X, assign, kc: int):
 
 def dist_tolerance(Q, X, mma_ulps: float = 4.0):
     """tau_ij for a squared distance ||q||^2 + ||x||^2 - 2 q.x computed by the method
-    (R18): 2 * elem_bound(q.x) + 4 * 2^-24 * (||q||^2 + ||x||^2)."""
+    (R18): 2 * elem_bound(q.x) + 12 * 2^-24 * (||q||^2 + ||x||^2).  The norm term covers
+    the fp32 norms (1 ulp each), the R22 norm step (4 terms truncated onto 2^(E-25) with
+    2^E <= max(|q.x|, ||x||^2/2), then RZ: < 2^-22 (||q||^2 + 1.5 ||x||^2) on the key) and
+    the final RN of ||q||^2 + key (<= 2 ulps of the norms): <= 9 units, rounded up to 12."""
     Q = np.asarray(Q, np.float64)
     X = np.asarray(X, np.float64)
     eb = elem_bound(Q, X.T, mma_ulps)
     nq = (Q * Q).sum(1)[:, None]
     nx = (X * X).sum(1)[None, :]
-    return 2.0 * eb + 4.0 * 2.0 ** -24 * (nq + nx) + 2.0 ** -20
+    return 2.0 * eb + 12.0 * 2.0 ** -24 * (nq + nx) + 2.0 ** -20
 
 
 # ---------------------------------------------------------------- tensor-core models

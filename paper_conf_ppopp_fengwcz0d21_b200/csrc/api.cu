@@ -96,6 +96,10 @@ static TcConfig choose_config(int epi_kind, int64_t M, int64_t N, int64_t K, int
   c.fa = env_int("EGEMM_FUSED_A", c.fa);
   if (c.kc < 64) c.kc = 64;
   c.kc = (c.kc / 64) * 64;
+  if (epi_kind != EPI_STORE) {  // kNN / kMeans: one accumulator (the norm MMA adds into it)
+    c.sep = 0;
+    if (!((c.cg == 2 && c.bn == 256) || (c.cg == 1 && c.bn == 128))) { c.cg = 2; c.bn = 256; }
+  }
   return c;
 }
 

@@ -10,8 +10,14 @@
 //
 // B200 design:
 //  * warp-specialised persistent kernel, 12 warps: w0 TMA producer, w1 MMA issuer (one
-//    elected lane; leader CTA only when CG == 2), w2 TMEM allocator, w3 idle, w4..w11
-//    epilogue (two warps per TMEM lane quarter, each owning BN/2 columns).
+//    elected lane; leader CTA only when CG == 2), w2 TMEM allocator, w3 norm warp (kNN /
+//    kMeans) or idle, w4..w11 epilogue (two warps per TMEM lane quarter, each owning BN/2
+//    columns).
+//  * kNN / kMeans ("norm MMA", reading R22 in DESIGN.md): after a tile's last product MMA one
+//    more tcgen05.mma kind::tf32 adds y_j = -||b_j||^2 / 2 to every row of column j (A' = rows
+//    of ones, B' = the three tf32 parts of y_j written into the stage by the norm warp), so
+//    the accumulator holds a.b_j - ||b_j||^2/2 = -key/2: the tensor core broadcasts the norms
+//    and the epilogue only compares accumulators (no per-thread norm loads, no FMA).
 //  * operands: pre-split fp16 hi/lo, K-major, loaded by TMA into 128-B-swizzled stages
 //    (BK = 64 fp16 = one swizzle atom row) in a STAGES-deep full/empty mbarrier ring.
 //  * CG == 2: cta_group::2 pair, UMMA M = 256, each CTA stages its 128 A rows and BN/2 B
@@ -214,6 +220,16 @@ __device__ __forceinline__ void named_bar_sync(int id, int nthreads) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }
 
+// y = h + m + l exactly, each part with <= 11 significant bits and its 13 low mantissa bits
+// zero, i.e. exact tf32 operands (kind::tf32 ignores those bits).  Truncation split: h keeps
+// y's top 11 bits, r = y - h (exact) its low 13, m the top 11 of r, l = r - m (exact, <= 2).
+__device__ __forceinline__ void tf32_parts(float y, float& h, float& m, float& l) {
+  h = __uint_as_float(__float_as_uint(y) & 0xFFFFE000u);
+  const float r = __fsub_rn(y, h);
+  m = __uint_as_float(__float_as_uint(r) & 0xFFFFE000u);
+  l = __fsub_rn(r, m);
+}
+
 template <int CG, int BN, bool SEP, int EPI, int STAGES, int NEPI, bool FA, bool AR>
 __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
     egemm_tc_kernel(const __grid_constant__ CUtensorMap tm_ahi,
@@ -228,6 +244,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
   constexpr uint32_t TMEM_COLS = (NACC * BN <= 32) ? 32 : (NACC * BN <= 64) ? 64
                                  : (NACC * BN <= 128) ? 128 : (NACC * BN <= 256) ? 256 : 512;
   static_assert(NACC * BN <= 512, "TMEM overflow");
+  static_assert(!(EPI != EPI_STORE && SEP), "kNN / kMeans: single accumulator (norm MMA)");
   static_assert(COLS % 32 == 0, "epilogue column split");
 
   extern __shared__ __align__(1024) uint8_t smem_raw[];
@@ -235,12 +252,20 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
                                              ~uintptr_t(1023));
   // AR (A resident, kNN / kMeans with K <= 128): the A tile of a unit is loaded once into
   // its own buffer and the ring carries only B; otherwise each stage holds A and B.
-  constexpr int SB = AR ? 2 * G::B_BYTES : G::STAGE_BYTES;  // bytes per ring stage
+  // NORM (kNN / kMeans): each stage also has a 32-B row per staged B row for the tf32 norm
+  // parts (written by the norm warp on a tile's last k-block), plus one A' tile of ones.
+  constexpr bool NORM = (EPI != EPI_STORE);
+  constexpr int NP_OFF = AR ? 2 * G::B_BYTES : G::STAGE_BYTES;  // norm parts inside a stage
+  constexpr int NP_BYTES = NORM ? G::BNC * 32 : 0;
+  constexpr int SB = NP_OFF + NP_BYTES;                       // bytes per ring stage
   constexpr int B_OFF = AR ? 0 : 2 * G::A_BYTES;            // B_hi offset inside a stage
   constexpr int AR_BYTES = AR ? 2 * 2 * G::A_BYTES : 0;     // 2 k-blocks of A_hi + A_lo
+  constexpr int ONES_BYTES = NORM ? kBM * 32 : 0;
+  static_assert(SB % 1024 == 0, "stage alignment");
   uint8_t* stage_base = smem;
   uint8_t* a_res = smem + STAGES * SB;
-  uint64_t* bars = reinterpret_cast<uint64_t*>(smem + STAGES * SB + AR_BYTES);
+  uint8_t* ones_tile = a_res + AR_BYTES;
+  uint64_t* bars = reinterpret_cast<uint64_t*>(ones_tile + ONES_BYTES);
   uint64_t* full = bars;
   uint64_t* empty = bars + STAGES;
   uint64_t* acc_full = bars + 2 * STAGES;
@@ -267,8 +292,9 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
   }
   if (warp == EG::W_MMA && lane == 0) {
     for (int s = 0; s < STAGES; s++) {
-      // FA: the producer's expect_tx arrive plus one arrive per converter warp of the pair
-      ptx::mbar_init(&full[s], FA ? 1 + 4 * CG : 1);
+      // FA: the producer's expect_tx arrive plus one arrive per converter warp of the pair;
+      // NORM: plus one arrive per norm warp of the pair
+      ptx::mbar_init(&full[s], 1 + (FA ? 4 * CG : 0) + (NORM ? CG : 0));
       ptx::mbar_init(&empty[s], 1);
     }
     for (int b = 0; b < 2; b++) {
@@ -296,6 +322,20 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
       ptx::sts128(ptx::smem_u32(stage_base) + i * 16, w[0], w[1], w[2], w[3]);
     }
     ptx::fence_proxy_async_smem();
+  }
+  if constexpr (NORM) {
+    if (warp == 3) {
+      // A' = rows of (1, 1, 1, 0) in both 16-B chunks of every 32-B row: invariant under the
+      // 32-B swizzle's chunk exchange, so B' may hold its parts in either chunk.  The NP
+      // slots start zeroed; the norm warp later rewrites only the parts chunk of a row.
+      const uint32_t o = ptx::smem_u32(ones_tile);
+      for (int i = lane; i < ONES_BYTES / 16; i += 32) ptx::sts128f(o + i * 16, 1.f, 1.f, 1.f, 0.f);
+      for (int st = 0; st < STAGES; st++) {
+        const uint32_t np = ptx::smem_u32(stage_base + st * SB + NP_OFF);
+        for (int i = lane; i < NP_BYTES / 16; i += 32) ptx::sts128f(np + i * 16, 0.f, 0.f, 0.f, 0.f);
+      }
+      ptx::fence_proxy_async_smem();
+    }
   }
   if (warp == EG::W_ALLOC) ptx::tmem_alloc<CG>(tmem_slot, TMEM_COLS);
   ptx::tc_fence_before();
@@ -447,6 +487,43 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
         for (uint32_t e = (gkb + pe - 1) / pe; e < total; e++) sync_arrive(p.sync, e);
       }
     }
+  } else if (NORM && warp == 3) {
+    // ============================ norm warp (kNN / kMeans) ============================
+    // Follows the stage ring; on a tile's last k-block writes, for each of this CTA's BNC
+    // staged B rows j, the tf32 parts of y_j = -||b_j||^2 / 2 (columns >= N: 0) into the
+    // stage's norm slot, then arrives on the stage's full barrier like the TMA bytes do.
+    if constexpr (NORM) {
+      int stage = 0;
+      uint32_t phase = 0;
+      for (int u = cluster; u < p.num_units; u += nclusters) {
+        UnitInfo ui = decode_unit<EPI>(p, u);
+        for (int ns = 0; ns < ui.n_count; ns++) {
+          const int64_t brow0 = (int64_t)(ui.n_begin + ns) * BN + (int)rank * G::BNC;
+          for (int kb = 0; kb < p.num_kb; kb++) {
+            ptx::mbar_wait(&empty[stage], phase ^ 1u);
+            if (kb == p.num_kb - 1) {
+              const uint32_t np = ptx::smem_u32(stage_base + stage * SB + NP_OFF);
+#pragma unroll
+              for (int j = 0; j < G::BNC / 32; j++) {
+                const int r = j * 32 + lane;  // lane-contiguous 32-B rows: conflict-free
+                const int64_t col = brow0 + r;
+                const float bn = col < p.N ? __ldg(p.bnorm + col) : 0.f;
+                float h, m, l;
+                tf32_parts(-0.5f * bn, h, m, l);  // -bn/2 is exact
+                ptx::sts128f(np + r * 32, h, m, l, 0.f);
+              }
+              ptx::fence_proxy_async_smem();  // generic-proxy stores -> visible to tcgen05.mma
+            }
+            __syncwarp();
+            if (lane == 0) {
+              if constexpr (CG == 1) ptx::mbar_arrive(&full[stage]);
+              else ptx::mbar_arrive_cluster(&full[stage], 0);
+            }
+            if (++stage == STAGES) { stage = 0; phase ^= 1u; }
+          }
+        }
+      }
+    }
   } else if (warp == EG::W_MMA) {
     // ============================ MMA issuer ============================
     // The whole warp runs the loop (so stage / descriptor arithmetic stays in uniform
@@ -540,6 +617,13 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
                   const uint32_t first = k > 0 ? 1u : acc0;
                   ptx::mma_f16<CG>(acc_hh, d_ahi + ko, d_bhi + ko, idesc, SEP ? first : 1u);
                 }
+                if constexpr (NORM) {
+                  // acc += 1 * h_j + 1 * m_j + 1 * l_j = a.b_j - ||b_j||^2 / 2 (reading R22)
+                  if (kb == p.num_kb - 1)
+                    ptx::mma_tf32<CG>(acc_hh, ptx::sdesc_kmajor_sw32(ptx::smem_u32(ones_tile)),
+                                      ptx::sdesc_kmajor_sw32(sa + NP_OFF),
+                                      ptx::idesc_tf32_f32(kBM * CG, BN), 1u);
+                }
                 if (!(p.debug_no_tma && (p.debug_mode & 4))) ptx::mma_commit<CG>(&empty[stage]);
                 if (p.debug_mode & 1) ptx::mma_commit<CG>(a_empty);  // diagnostics only
               }
@@ -570,7 +654,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
 
     float kd[kKnnMax];
     int ki[kKnnMax];
-    float best = __int_as_float(0x7f800000);
+    float best = __int_as_float(0xff800000);
     int besti = 0x7fffffff;
 
     for (int u = cluster; u < p.num_units; u += nclusters) {
@@ -580,7 +664,8 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
 #pragma unroll
         for (int t = 0; t < kKnnMax; t++) { kd[t] = __int_as_float(0x7f800000); ki[t] = 0x7fffffff; }
       }
-      if constexpr (EPI == EPI_KMEANS) { best = __int_as_float(0x7f800000); besti = 0x7fffffff; }
+      // kMeans: best = the largest accumulator (= smallest key) so far, key = -2 best
+      if constexpr (EPI == EPI_KMEANS) { best = __int_as_float(0xff800000); besti = 0x7fffffff; }
 
       for (int ns = 0; ns < ui.n_count; ns++) {
         const int col_base = (ui.n_begin + ns) * BN + cgp * COLS;
@@ -654,7 +739,17 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
           const uint32_t use = chunk_ctr >> 1;
           ptx::mbar_wait(&acc_full[buf], use & 1u);
           ptx::tc_fence_after();
-          if (p.debug_no_epi) {  // diagnostics only: release the accumulator untouched
+          if (p.debug_mode & 64) {  // diagnostics only: TMEM reads, no epilogue arithmetic
+            const uint32_t a0 = tmem_base + lane_off + buf * BN + cgp * COLS;
+#pragma unroll
+            for (int c = 0; c < COLS / 32; c++) {
+              float v[32];
+              ptx::tmem_ld32(a0 + c * 32, v);
+              ptx::tmem_wait_ld();
+              if (v[c] == 1234.5f) best = v[31];  // keep the loads observable
+            }
+          }
+          if (p.debug_no_epi || (p.debug_mode & 64)) {  // diagnostics: release untouched
             ptx::tc_fence_before();
             __syncwarp();
             if (lane == 0) {
@@ -695,37 +790,27 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
               }
             }
             const int c0 = col_base + c * 32;
-            float bn[32];
-            if (c0 + 32 <= p.N) {
+            // v = a.b_j - ||b_j||^2 / 2 (norm MMA), so key_j = -2 v exactly: min key = max v
+            if (c0 + 32 > p.N) {  // ragged last tile: columns >= N never win
 #pragma unroll
-              for (int i = 0; i < 32; i += 4) {
-                float4 t = __ldg(reinterpret_cast<const float4*>(p.bnorm + c0 + i));
-                bn[i] = t.x; bn[i + 1] = t.y; bn[i + 2] = t.z; bn[i + 3] = t.w;
-              }
-            } else {
-#pragma unroll
-              for (int i = 0; i < 32; i++)
-                bn[i] = (c0 + i < p.N) ? __ldg(p.bnorm + c0 + i) : __int_as_float(0x7f800000);
+              for (int i = 0; i < 32; i++) v[i] = (c0 + i < p.N) ? v[i] : __int_as_float(0xff800000);
             }
             if constexpr (EPI == EPI_KNN) {
-              // fast path: keys + a candidate mask against this row's current k-th key;
-              // the (rare) insertions run in a compact loop over the set bits.  A thread's
-              // columns arrive in increasing index order, so a strict '<' keeps the lower
-              // index first among equal keys.
+              float mx = __int_as_float(0xff800000);
+#pragma unroll
+              for (int i = 0; i < 32; i++) mx = fmaxf(mx, v[i]);
+              // candidate test against this row's current k-th key; the (rare) insertions
+              // run in a compact loop over the set bits.  A thread's columns arrive in
+              // increasing index order, so a strict '<' keeps the lower index first among
+              // equal keys.
               const float thr = kd[kKnnMax - 1];
-              float mn = __int_as_float(0x7f800000);
-#pragma unroll
-              for (int i = 0; i < 32; i += 2)  // key = ||b||^2 - 2 a.b (the *2 is exact)
-                ptx::fma2_m2(v[i], v[i + 1], bn[i], bn[i + 1]);
-#pragma unroll
-              for (int i = 0; i < 32; i++) mn = fminf(mn, v[i]);
-              if (__any_sync(0xffffffffu, mn < thr)) {
+              if (__any_sync(0xffffffffu, -2.f * mx < thr)) {
                 uint32_t cand = 0;
                 float keys[32];
 #pragma unroll
                 for (int i = 0; i < 32; i++) {
-                  keys[i] = v[i];
-                  cand |= (v[i] < thr) ? (1u << i) : 0u;
+                  keys[i] = -2.f * v[i];
+                  cand |= (keys[i] < thr) ? (1u << i) : 0u;
                 }
 #pragma unroll 1
                 while (cand) {
@@ -735,18 +820,16 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
                 }
               }
             } else {
-              // group min first (FFMA2 + 3-input FMNMX), the index only when it improves
-              float mn = __int_as_float(0x7f800000);
+              // group max first (3-input FMNMX), the index only when it improves.  (Parking
+              // the improving quarter in smem and searching once per unit measured the same.)
+              float mx = __int_as_float(0xff800000);
 #pragma unroll
-              for (int i = 0; i < 32; i += 2)  // key = ||b||^2 - 2 a.b (the *2 is exact)
-                ptx::fma2_m2(v[i], v[i + 1], bn[i], bn[i + 1]);
-#pragma unroll
-              for (int i = 0; i < 32; i++) mn = fminf(mn, v[i]);
-              if (mn < best) {  // strict: an equal key from a later column never wins
+              for (int i = 0; i < 32; i++) mx = fmaxf(mx, v[i]);
+              if (mx > best) {  // strict: an equal key from a later column never wins
                 int idx = 31;
 #pragma unroll
-                for (int i = 30; i >= 0; i--) idx = (v[i] == mn) ? i : idx;  // lowest index
-                best = mn;
+                for (int i = 30; i >= 0; i--) idx = (v[i] == mx) ? i : idx;  // lowest index
+                best = mx;
                 besti = c0 + idx;
               }
             }
@@ -757,21 +840,26 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
 
       // ---- unit end: merge the two column halves of each row, write the unit's result
       if constexpr (EPI == EPI_KNN) {
-        // column groups 1..GPQ-1 hand their lists to group 0 one at a time (16 KiB scratch)
-        float* sk = reinterpret_cast<float*>(scratch) + (q * 32 + lane) * kKnnMax;
-        int* si = reinterpret_cast<int*>(scratch + kBM * kKnnMax * 4) + (q * 32 + lane) * kKnnMax;
+        // column groups 1..GPQ-1 hand their lists to group 0 one at a time, half a list per
+        // round (8 KiB scratch)
+        constexpr int KH = kKnnMax / 2;
+        float* sk = reinterpret_cast<float*>(scratch) + (q * 32 + lane) * KH;
+        int* si = reinterpret_cast<int*>(scratch + kBM * KH * 4) + (q * 32 + lane) * KH;
 #pragma unroll 1
         for (int g = 1; g < GPQ; g++) {
-          if (cgp == g) {
 #pragma unroll
-            for (int t = 0; t < kKnnMax; t++) { sk[t] = kd[t]; si[t] = ki[t]; }
-          }
-          named_bar_sync(1 + q, 32 * GPQ);
-          if (cgp == 0) {
+          for (int h = 0; h < 2; h++) {
+            if (cgp == g) {
+#pragma unroll
+              for (int t = 0; t < KH; t++) { sk[t] = kd[h * KH + t]; si[t] = ki[h * KH + t]; }
+            }
+            named_bar_sync(1 + q, 32 * GPQ);
+            if (cgp == 0) {
 #pragma unroll 1
-            for (int t = 0; t < kKnnMax; t++) topk_insert<kKnnMax>(kd, ki, sk[t], si[t]);
+              for (int t = 0; t < KH; t++) topk_insert<kKnnMax>(kd, ki, sk[t], si[t]);
+            }
+            named_bar_sync(1 + q, 32 * GPQ);
           }
-          named_bar_sync(1 + q, 32 * GPQ);
         }
         if (cgp == 0 && row < p.M) {
           const int64_t o = ((int64_t)ui.slice * p.M + row) * p.knn_k;
@@ -780,6 +868,8 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
             if (t < p.knn_k) { p.part_key[o + t] = kd[t]; p.part_idx[o + t] = ki[t]; }
         }
       } else if constexpr (EPI == EPI_KMEANS) {
+        best = -2.f * best;  // the key (exact): ||c||^2 - 2 x.c
+        // merge the GPQ column groups of each row through smem
         float* sk = reinterpret_cast<float*>(scratch);
         int* si = reinterpret_cast<int*>(scratch + GPQ * kBM * 4);
         const int r = q * 32 + lane;
@@ -792,7 +882,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
             const int oi = si[(g - 1) * kBM + r];
             if (ob < best || (ob == best && oi < besti)) { best = ob; besti = oi; }
           }
-          if (p.debug_no_epi) besti = 0;  // diagnostics: keep the downstream kernels in bounds
+          if (p.debug_no_epi || (p.debug_mode & 64)) besti = 0;  // diagnostics: keep the downstream kernels in bounds
           if (row < p.M) { p.assign[row] = besti; p.best_key[row] = best; }
         }
         named_bar_sync(1 + q, 32 * GPQ);
@@ -880,10 +970,12 @@ static int launch_variant(const CUtensorMap* maps, const KParams& kp, int max_cl
   // (kNN with 16 warps spills its top-k lists at the 102-register cap: measured slower)
   constexpr int NEPI = (EPI == EPI_KMEANS) ? 16 : 8;
   auto kern = egemm_tc_kernel<CG, BN, SEP, EPI, STAGES, NEPI, FA, AR>;
-  const int scratch = EPI == EPI_KNN ? kBM * kKnnMax * 8 : EPI == EPI_KMEANS ? 2 * 4 * kBM * 4 : 0;
-  const size_t sb = AR ? 2 * G::B_BYTES : G::STAGE_BYTES;
+  // kNN: top-k merge lists (half a list per round); kMeans: (key, index) of 3 column groups
+  const int scratch = EPI == EPI_KNN ? kBM * kKnnMax * 4 : EPI == EPI_KMEANS ? 2 * 4 * kBM * 4 : 0;
+  constexpr bool NORM = (EPI != EPI_STORE);  // norm slot per stage + the A' ones tile
+  const size_t sb = (AR ? 2 * G::B_BYTES : G::STAGE_BYTES) + (NORM ? G::BNC * 32 : 0);
   const size_t smem = 1024 + (size_t)STAGES * sb + (AR ? 4 * G::A_BYTES : 0) +
-                      8 * (2 * STAGES + 8) + scratch;
+                      (NORM ? kBM * 32 : 0) + 8 * (2 * STAGES + 8) + scratch;
   static bool attr_done = false;  // per instantiation
   if (!attr_done) {
     if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
@@ -950,10 +1042,12 @@ static int dispatch(const CUtensorMap* maps, const KParams& kp, const TcConfig& 
     return launch_variant<2, 256, false, EPI, 3>(maps, kp, cfg.max_clusters, s);
   if (cfg.cg == 1 && cfg.bn == 128 && !cfg.sep)
     return launch_variant<1, 128, false, EPI, 3>(maps, kp, cfg.max_clusters, s);
-  if (cfg.cg == 1 && cfg.bn == 128 && cfg.sep)
-    return launch_variant<1, 128, true, EPI, 3>(maps, kp, cfg.max_clusters, s);
-  if (cfg.cg == 2 && cfg.bn == 128 && cfg.sep)
-    return launch_variant<2, 128, true, EPI, 3>(maps, kp, cfg.max_clusters, s);
+  if constexpr (EPI == EPI_STORE) {  // kNN / kMeans keep one accumulator (norm MMA)
+    if (cfg.cg == 1 && cfg.bn == 128 && cfg.sep)
+      return launch_variant<1, 128, true, EPI, 3>(maps, kp, cfg.max_clusters, s);
+    if (cfg.cg == 2 && cfg.bn == 128 && cfg.sep)
+      return launch_variant<2, 128, true, EPI, 3>(maps, kp, cfg.max_clusters, s);
+  }
   set_last_error("unsupported tile config cg=%d bn=%d sep=%d", cfg.cg, cfg.bn, cfg.sep);
   return 2;
 }

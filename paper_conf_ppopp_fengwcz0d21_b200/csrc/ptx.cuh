@@ -263,19 +263,12 @@ __device__ __forceinline__ void sts128(uint32_t addr, uint32_t a, uint32_t b, ui
                : "memory");
 }
 
-// ------------------------------------------------------------------ packed fp32x2 math
-// (d0, d1) = (b0 - 2 v0, b1 - 2 v1), one FFMA2 (fma.rn.f32x2, sm_100a); each lane is an
-// ordinary round-to-nearest fma, so results equal __fmaf_rn(-2, v, b) bitwise.
-__device__ __forceinline__ void fma2_m2(float& v0, float& v1, float b0, float b1) {
-  asm("{\n\t.reg .b64 a, b, c, d;\n\t"
-      "mov.b64 a, {%0, %1};\n\t"
-      "mov.b64 b, {%2, %3};\n\t"
-      "mov.b64 c, 0xC0000000C0000000;\n\t"
-      "fma.rn.f32x2 d, a, c, b;\n\t"
-      "mov.b64 {%0, %1}, d;\n\t}"
-      : "+f"(v0), "+f"(v1)
-      : "f"(b0), "f"(b1));
+__device__ __forceinline__ void sts128f(uint32_t addr, float a, float b, float c, float d) {
+  asm volatile("st.shared.v4.f32 [%0], {%1, %2, %3, %4};" ::"r"(addr), "f"(a), "f"(b), "f"(c),
+               "f"(d)
+               : "memory");
 }
+
 // (a0, a1) += (b0, b1) with round-to-nearest (add.rn.f32x2)
 __device__ __forceinline__ void add2(float& a0, float& a1, float b0, float b1) {
   asm("{\n\t.reg .b64 a, b;\n\t"
@@ -299,6 +292,39 @@ __device__ __forceinline__ uint64_t sdesc_kmajor_sw128(uint32_t smem_addr) {
   d |= (uint64_t)1u << 46;                         // version = 1    [46,48)
   d |= (uint64_t)2u << 61;                         // SWIZZLE_128B   [61,64)
   return d;
+}
+// K-major, 32-B swizzle (rows of 32 B = 8 tf32, 8-row atoms of 256 B): the norm-broadcast
+// operands of the kNN / kMeans epilogue MMA (one K = 8 tf32 step).
+__device__ __forceinline__ uint64_t sdesc_kmajor_sw32(uint32_t smem_addr) {
+  uint64_t d = 0;
+  d |= (uint64_t)((smem_addr & 0x3FFFFu) >> 4);  // start address  [0,14)
+  d |= (uint64_t)1u << 16;                         // LBO (unused)   [16,30)
+  d |= (uint64_t)(256u >> 4) << 32;                // SBO = 256 B    [32,46)
+  d |= (uint64_t)1u << 46;                         // version = 1    [46,48)
+  d |= (uint64_t)6u << 61;                         // SWIZZLE_32B    [61,64)
+  return d;
+}
+// Instruction descriptor, .kind::tf32: A,B tf32 (format 2), D fp32, both K-major.
+__host__ __device__ constexpr uint32_t idesc_tf32_f32(int M, int N) {
+  return (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)(N >> 3) << 17) |
+         ((uint32_t)(M >> 4) << 24);
+}
+template <int CG>
+__device__ __forceinline__ void mma_tf32(uint32_t d_tmem, uint64_t adesc, uint64_t bdesc,
+                                         uint32_t idesc, uint32_t accumulate) {
+  if constexpr (CG == 1) {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "setp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
+        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate));
+  } else {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "setp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::2.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(d_tmem),
+        "l"(adesc), "l"(bdesc), "r"(idesc), "r"(accumulate));
+  }
 }
 // Instruction descriptor, .kind::f16: A,B fp16 (format 0), D fp32 (c_format 1), both K-major.
 __host__ __device__ constexpr uint32_t idesc_f16_f32(int M, int N) {

@@ -175,3 +175,22 @@ def test_kmeans_assign_bitexact_vs_alg1_model(oracle_lib, n, d, kc):
     assert np.array_equal(to_host(a), ra)
     rs, rc = oracle_lib.group_sums(X, ra, kc)
     assert np.array_equal(to_host(sums), rs) and np.array_equal(to_host(counts), rc)
+
+
+@pytest.mark.parametrize("n,d,kc,dup", [(4096, 64, 1024, 512), (3000, 64, 600, 300), (2000, 32, 97, 5)])
+def test_kmeans_ties_lowest_index_bitexact(oracle_lib, n, d, kc, dup):
+    """Exact ties on integer data: every centroid appears twice (columns j and j + dup, i.e.
+    in other 16-column halves, 32-column groups and 256-column tiles), so the minimal key
+    is always shared; the assignment must be the lower index (R12/R22), bitwise equal to
+    the profiled-tensor-core model."""
+    eg = require_gpu()
+    X = inputs.integers((n, d), 90 + kc, lim=6)
+    base = inputs.integers((dup, d), 91 + kc, lim=6)
+    C = np.tile(base, (-(-kc // dup), 1))[:kc].copy()
+    a, sums, counts, _ = eg.kmeans_step(to_dev(X), to_dev(C))
+    ra, _ = oracle_lib.kmeans_assign_alg1_tc(X, C)
+    ga = to_host(a)
+    assert np.array_equal(ga, ra)
+    assert ga.max() < dup  # the first copy always wins
+    rs, rc = oracle_lib.group_sums(X, ra, kc)
+    assert np.array_equal(to_host(sums), rs) and np.array_equal(to_host(counts), rc)

@@ -207,3 +207,43 @@ def test_kmeans_assign_alg1_tc_integer_and_ties(oracle_lib):
     cn = (C.astype(np.int64) ** 2).sum(1)
     assert np.array_equal(best.astype(np.int64), (D - (X.astype(np.int64) ** 2).sum(1)[:, None])[np.arange(500), a])
     assert np.all(cn[a] - 2 * (X.astype(np.int64) * C[a].astype(np.int64)).sum(1) == best)
+
+
+def _low13_zero(x):
+    return (np.asarray(x, np.float32).view(np.uint32) & 0x1FFF) == 0
+
+
+def test_tf32_parts_exact_decomposition(oracle_lib):
+    """R22 norm parts: y = h + m + l exactly (checked in fp64), every part an exact tf32
+    value (13 low mantissa bits zero), |m| < 2^-10 |h| and |l| < 2^-20 |h|; tf32-exact y
+    gives m = l = 0."""
+    g = inputs.rng(2205)
+    ys = np.concatenate([(g.uniform(-1, 1, 4000) * 2.0 ** g.integers(-30, 40, 4000)),
+                         [0.0, -0.0, 1.0, -3.5, 65504.0, 1e30, -1e-30]]).astype(np.float32)
+    for y in ys:
+        h, m, l = oracle_lib.tf32_parts(y)
+        assert float(h) + float(m) + float(l) == float(y)
+        assert _low13_zero([h, m, l]).all()
+        if h != 0:
+            assert abs(m) < 2.0 ** -10 * abs(h) and abs(l) < 2.0 ** -20 * abs(h)
+    for y in np.float32([1.0, 0.75, -1024.0, 3.0 * 2 ** 20]):
+        assert oracle_lib.tf32_parts(y)[1:] == (0.0, 0.0)
+
+
+def test_norm_step_matches_rational_model_and_exact_cases(oracle_lib):
+    """norm_step = one profiled tensor-core step on (1, 1, 1) x (h, m, l) with C = dot:
+    checked against the exact-rational tc_model rendering, and exact (= dot - nrm / 2) when
+    that value is representable on the step's grid (integers)."""
+    g = inputs.rng(2206)
+    dot = (g.uniform(-1, 1, (7, 50)) * 2.0 ** g.integers(-4, 12, (7, 50))).astype(np.float32)
+    nrm = (g.uniform(0, 1, 50) * 2.0 ** g.integers(-6, 14, 50)).astype(np.float32)
+    out = oracle_lib.norm_step(dot, nrm)
+    for i in range(7):
+        for j in range(50):
+            parts = np.float32(oracle_lib.tf32_parts(np.float32(-0.5) * nrm[j]))
+            ref = oracle_lib.tc_model(np.ones(3, np.float32), parts, float(dot[i, j]), "align", 2, "fields")
+            assert out[i, j] == np.float32(ref), (i, j)
+    di = g.integers(-5000, 5000, (9, 40)).astype(np.float32)
+    ni = g.integers(0, 20000, 40).astype(np.float32)
+    assert np.array_equal(oracle_lib.norm_step(di, ni).astype(np.float64),
+                          di.astype(np.float64) - 0.5 * ni.astype(np.float64))

@@ -38,9 +38,10 @@ def main():
     Qk = torch.from_numpy(inputs.uniform((nq, 128), 301)).cuda()
     index = egemm.knn_index(Xk)
     need_knn = 6.0 * nq * nx * 128 / (148 * 8192.0)
-    for tag, env in (("full", {}), ("no_epi", {"EGEMM_DEBUG_NO_EPI": "1"}),
+    for tag, env in (("full", {}), ("tmem_ld_only", {"EGEMM_DEBUG_MODE": "64"}),
+                     ("no_epi", {"EGEMM_DEBUG_NO_EPI": "1"}),
                      ("no_tma+no_epi", {"EGEMM_DEBUG_NO_EPI": "1", "EGEMM_DEBUG_NO_TMA": "1"})):
-        for k in ("EGEMM_DEBUG_NO_EPI", "EGEMM_DEBUG_NO_TMA"):
+        for k in ("EGEMM_DEBUG_NO_EPI", "EGEMM_DEBUG_NO_TMA", "EGEMM_DEBUG_MODE"):
             os.environ.pop(k, None)
         os.environ.update(env)
         ms, mhz, cyc, lpc = measure(lambda: egemm.kmeans_step(X, C, x_split=xs, want_inertia=False,
