@@ -196,24 +196,23 @@ __device__ __forceinline__ void topk_insert(float (&kd)[KN], int (&ki)[KN], floa
   }
 }
 
-// streaming insertion (indices arrive in increasing order): strict '<' is enough
+// streaming insertion (indices arrive in increasing order): strict '<' is enough.  All 16
+// comparisons against the old list are independent (c_t = key < kd[t], monotone in t), and
+// each slot takes its left neighbour (c_{t-1}), the new key (c_t only) or itself: no serial
+// compare-swap chain, so the insertion costs ~5 dependent ALU latencies instead of ~48.
 template <int KN>
 __device__ __forceinline__ void topk_insert_stream(float (&kd)[KN], int (&ki)[KN], float key,
                                                    int idx) {
-  if (key < kd[KN - 1]) {
-    kd[KN - 1] = key;
-    ki[KN - 1] = idx;
+  bool c[KN];
 #pragma unroll
-    for (int t = KN - 1; t > 0; t--) {
-      const bool sw = kd[t] < kd[t - 1];
-      const float a = kd[t], b = kd[t - 1];
-      const int ia = ki[t], ib = ki[t - 1];
-      kd[t] = sw ? b : a;
-      kd[t - 1] = sw ? a : b;
-      ki[t] = sw ? ib : ia;
-      ki[t - 1] = sw ? ia : ib;
-    }
+  for (int t = 0; t < KN; t++) c[t] = key < kd[t];
+#pragma unroll
+  for (int t = KN - 1; t > 0; t--) {
+    kd[t] = c[t - 1] ? kd[t - 1] : (c[t] ? key : kd[t]);
+    ki[t] = c[t - 1] ? ki[t - 1] : (c[t] ? idx : ki[t]);
   }
+  kd[0] = c[0] ? key : kd[0];
+  ki[0] = c[0] ? idx : ki[0];
 }
 
 __device__ __forceinline__ void named_bar_sync(int id, int nthreads) {
@@ -966,8 +965,9 @@ template <int CG, int BN, bool SEP, int EPI, int STAGES, bool FA = false, bool A
 static int launch_variant(const CUtensorMap* maps, const KParams& kp, int max_clusters,
                           cudaStream_t stream) {
   using G = Geo<CG, BN>;
-  // kMeans' argmin epilogue is issue-bound next to a 64-deep k-loop: 16 epilogue warps
-  // (kNN with 16 warps spills its top-k lists at the 102-register cap: measured slower)
+  // kMeans' argmin epilogue is issue-bound next to a 64-deep k-loop: 16 epilogue warps.
+  // kNN keeps 8 (with 16 each thread's list sees half the columns, twice the insertions:
+  // measured 3-15 % slower even without spills after the norm MMA freed 32 registers)
   constexpr int NEPI = (EPI == EPI_KMEANS) ? 16 : 8;
   auto kern = egemm_tc_kernel<CG, BN, SEP, EPI, STAGES, NEPI, FA, AR>;
   // kNN: top-k merge lists (half a list per round); kMeans: (key, index) of 3 column groups
