@@ -13,9 +13,11 @@
 //   A  km_hist       per-block histogram H[j][b] (smem atomics)
 //   B1 km_scan_blk   per-centroid exclusive scan over blocks, cnt[j]
 //   B2 km_scan_c     offsets[j], counts[j], chunk_base[j], chunk -> centroid map
-//   C  km_scatter    stable scatter (warp-serial 32-point chunks, match_any ranks)
-//   D  km_chunk      chunk partial sums (+ per-chunk inertia terms)
-//   E  km_combine    sums[j] = sequential sum of its chunk partials (+ inertia_j)
+//   C  km_scatter    stable scatter: the block's 4096 points in W warp sub-ranges, per-warp
+//                    histograms -> per-warp offsets, then match_any ranks (32 points a step)
+//   D  km_chunk      chunk partial sums (+ per-chunk inertia terms); the CTA that finishes
+//                    the last chunk of centroid j (atomic ticket) adds j's chunk partials in
+//                    chunk order: sums[j] (+ inertia_j) -- the old separate combine pass
 //   F  km_inertia    inertia = fixed-order tree sum of inertia_j
 #include <cuda_runtime.h>
 #include <cstdint>
@@ -78,7 +80,8 @@ __global__ void km_scan_blk_kernel(int32_t* __restrict__ H, int nb, int32_t* __r
 __global__ void km_scan_c_kernel(const int32_t* __restrict__ cnt, int64_t kc,
                                  int64_t* __restrict__ offsets, int64_t* __restrict__ counts,
                                  int32_t* __restrict__ chunk_base, int32_t* __restrict__ chunk_j,
-                                 int32_t* __restrict__ n_chunks) {
+                                 int32_t* __restrict__ n_chunks, int32_t* __restrict__ done,
+                                 double* __restrict__ sums, int64_t d, double* __restrict__ in_j) {
   __shared__ int64_t wt64[32];
   __shared__ int32_t wt32[32];
   int64_t carry = 0;
@@ -95,6 +98,11 @@ __global__ void km_scan_c_kernel(const int32_t* __restrict__ cnt, int64_t kc,
       offsets[j] = carry + ex;
       counts[j] = c;
       chunk_base[j] = ccarry + cex;
+      done[j] = 0;  // km_chunk's per-centroid tickets
+      if (c == 0) {  // no chunk will write an empty cluster's sums
+        for (int64_t t = 0; t < d; t++) sums[j * d + t] = 0.0;
+        in_j[j] = 0.0;
+      }
       for (int32_t q = 0; q < nch; q++) chunk_j[ccarry + cex + q] = (int32_t)j;
     }
     carry += tot;
@@ -103,26 +111,50 @@ __global__ void km_scan_c_kernel(const int32_t* __restrict__ cnt, int64_t kc,
   if (threadIdx.x == 0) *n_chunks = ccarry;
 }
 
-__global__ void km_scatter_kernel(const int32_t* __restrict__ assign, int64_t n, int64_t kc,
-                                  const int32_t* __restrict__ H, int nb,
-                                  const int64_t* __restrict__ offsets, int32_t* __restrict__ order) {
-  extern __shared__ int32_t run[];
-  const int lane = threadIdx.x;
-  for (int64_t j = lane; j < kc; j += 32) run[j] = 0;
-  __syncwarp();
+// Stable scatter of one block of kKmBlockPts points: W warps take consecutive sub-ranges;
+// pass 1 counts each warp's members per centroid (match_any: the leader of each peer group
+// adds its popcount, so no atomics), the counts become per-warp start offsets (block base
+// H[a][b] + earlier warps), pass 2 writes order[] with the in-warp ranks.  Same positions as
+// a sequential walk over the block: the order stays stable (ascending i per centroid).
+template <int W>
+__global__ void __launch_bounds__(32 * W) km_scatter_kernel(
+    const int32_t* __restrict__ assign, int64_t n, int64_t kc, const int32_t* __restrict__ H,
+    int nb, const int64_t* __restrict__ offsets, int32_t* __restrict__ order) {
+  extern __shared__ int32_t hw[];  // [W][kc]
+  const int lane = threadIdx.x & 31, w = threadIdx.x >> 5;
+  for (int64_t j = threadIdx.x; j < (int64_t)W * kc; j += blockDim.x) hw[j] = 0;
+  __syncthreads();
   const int64_t i0 = (int64_t)blockIdx.x * kKmBlockPts;
   const int64_t i1 = min(n, i0 + kKmBlockPts);
-  int a_next = (i0 + lane < i1) ? assign[i0 + lane] : -1 - lane;
-  for (int64_t c = i0; c < i1; c += 32) {
+  constexpr int SUB = kKmBlockPts / W;
+  const int64_t s0 = i0 + (int64_t)w * SUB, s1 = min(i1, s0 + SUB);
+  int32_t* mine = hw + (int64_t)w * kc;
+  for (int64_t c = s0; c < s1; c += 32) {
     const int64_t i = c + lane;
-    const bool valid = i < i1;
-    const int a = a_next;
-    a_next = (c + 32 + lane < i1) ? assign[c + 32 + lane] : -1 - lane;  // prefetch
+    const int a = i < s1 ? assign[i] : -1 - lane;
+    const uint32_t peers = __match_any_sync(0xffffffffu, a);
+    if (i < s1 && lane == __ffs(peers) - 1) mine[a] += __popc(peers);
+  }
+  __syncthreads();
+  for (int64_t j = threadIdx.x; j < kc; j += blockDim.x) {  // exclusive prefix over warps
+    int32_t run = H[j * nb + blockIdx.x];
+#pragma unroll
+    for (int v = 0; v < W; v++) {
+      const int32_t t = hw[(int64_t)v * kc + j];
+      hw[(int64_t)v * kc + j] = run;
+      run += t;
+    }
+  }
+  __syncthreads();
+  for (int64_t c = s0; c < s1; c += 32) {
+    const int64_t i = c + lane;
+    const bool valid = i < s1;
+    const int a = valid ? assign[i] : -1 - lane;
     const uint32_t peers = __match_any_sync(0xffffffffu, a);
     const int rank = __popc(peers & ((1u << lane) - 1u));
-    if (valid) order[offsets[a] + H[(int64_t)a * nb + blockIdx.x] + run[a] + rank] = (int32_t)i;
+    if (valid) order[offsets[a] + mine[a] + rank] = (int32_t)i;
     __syncwarp();
-    if (valid && lane == __ffs(peers) - 1) run[a] += __popc(peers);
+    if (valid && lane == __ffs(peers) - 1) mine[a] += __popc(peers);
     __syncwarp();
   }
 }
@@ -137,9 +169,11 @@ __global__ void km_chunk_kernel(const float* __restrict__ X, int64_t d, int64_t 
                                 const int32_t* __restrict__ chunk_j,
                                 const int32_t* __restrict__ n_chunks,
                                 const float* __restrict__ best_key, double* __restrict__ part,
-                                double* __restrict__ part_in) {
+                                double* __restrict__ part_in, int32_t* __restrict__ done,
+                                double* __restrict__ sums, double* __restrict__ in_j) {
   __shared__ int32_t sidx[kKmChunk];
   __shared__ double red[32];
+  __shared__ int last;
   const int g = blockIdx.x;
   if (g >= *n_chunks) return;
   const int j = chunk_j[g];
@@ -180,24 +214,26 @@ __global__ void km_chunk_kernel(const float* __restrict__ X, int64_t d, int64_t 
       part_in[g] = w;
     }
   }
-}
-
-// one CTA per centroid: sums[j][t] = sequential sum of the chunk partials (R20)
-__global__ void km_combine_kernel(const double* __restrict__ part, const double* __restrict__ part_in,
-                                  int64_t d, const int64_t* __restrict__ counts,
-                                  const int32_t* __restrict__ chunk_base, double* __restrict__ sums,
-                                  double* __restrict__ in_j) {
-  const int64_t j = blockIdx.x;
+  // The CTA that completes centroid j's last chunk adds j's chunk partials in chunk order
+  // (R20's second level): which CTA does it does not change the order or the bits.
   const int nch = (int)((counts[j] + kKmChunk - 1) / kKmChunk);
+  __threadfence();  // this thread's partials before the ticket
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    last = (atomicAdd(done + j, 1) == nch - 1);
+    __threadfence();
+  }
+  __syncthreads();
+  if (!last) return;
   const int64_t g0 = chunk_base[j];
-  for (int64_t t = threadIdx.x; t < d; t += blockDim.x) {
-    double s = 0.0;
-    for (int c = 0; c < nch; c++) s = __dadd_rn(s, part[(g0 + c) * d + t]);
-    sums[j * d + t] = s;
+  if (active) {
+    double acc = 0.0;
+    for (int c = 0; c < nch; c++) acc = __dadd_rn(acc, __ldcg(part + (g0 + c) * d + t));
+    sums[j * d + t] = acc;
   }
   if (part_in && threadIdx.x == 0) {
     double w = 0.0;
-    for (int c = 0; c < nch; c++) w += part_in[g0 + c];
+    for (int c = 0; c < nch; c++) w += __ldcg(part_in + g0 + c);
     in_j[j] = w;
   }
 }
@@ -217,7 +253,7 @@ __global__ void km_inertia_kernel(const double* __restrict__ in_j, int64_t kc,
 }
 
 struct KmWs {
-  int32_t *H, *cnt, *chunk_base, *chunk_j, *n_chunks, *order;
+  int32_t *H, *cnt, *chunk_base, *chunk_j, *n_chunks, *order, *done;
   int64_t* offsets;
   double *part, *part_in, *in_j;
 };
@@ -240,6 +276,7 @@ static KmWs carve(void* base, int64_t n, int64_t d, int64_t kc, size_t* total) {
   w.chunk_base = reinterpret_cast<int32_t*>(take(sizeof(int32_t) * (size_t)kc));
   w.chunk_j = reinterpret_cast<int32_t*>(take(sizeof(int32_t) * (size_t)gmax));
   w.n_chunks = reinterpret_cast<int32_t*>(take(sizeof(int32_t)));
+  w.done = reinterpret_cast<int32_t*>(take(sizeof(int32_t) * (size_t)kc));
   w.order = reinterpret_cast<int32_t*>(take(sizeof(int32_t) * (size_t)(n > 0 ? n : 1)));
   w.offsets = reinterpret_cast<int64_t*>(take(sizeof(int64_t) * (size_t)kc));
   w.part = reinterpret_cast<double*>(take(sizeof(double) * (size_t)(gmax * d)));
@@ -274,13 +311,20 @@ int launch_kmeans_accumulate(const float* X, int64_t n, int64_t d, int64_t ldx,
   km_hist_kernel<<<nb, 256, hs, stream>>>(assign, n, kc, w.H, nb);
   km_scan_blk_kernel<<<(unsigned)kc, 256, 0, stream>>>(w.H, nb, w.cnt);
   km_scan_c_kernel<<<1, 1024, 0, stream>>>(w.cnt, kc, w.offsets, counts, w.chunk_base, w.chunk_j,
-                                           w.n_chunks);
-  km_scatter_kernel<<<nb, 32, hs, stream>>>(assign, n, kc, w.H, nb, w.offsets, w.order);
+                                           w.n_chunks, w.done, sums, d, w.in_j);
+  // W warps per scatter block, W per-warp histograms of kc counters in smem (<= 48 KiB)
+  if (kc <= 1536)
+    km_scatter_kernel<8><<<nb, 256, 8 * hs, stream>>>(assign, n, kc, w.H, nb, w.offsets, w.order);
+  else if (kc <= 3072)
+    km_scatter_kernel<4><<<nb, 128, 4 * hs, stream>>>(assign, n, kc, w.H, nb, w.offsets, w.order);
+  else if (kc <= 6144)
+    km_scatter_kernel<2><<<nb, 64, 2 * hs, stream>>>(assign, n, kc, w.H, nb, w.offsets, w.order);
+  else
+    km_scatter_kernel<1><<<nb, 32, hs, stream>>>(assign, n, kc, w.H, nb, w.offsets, w.order);
   km_chunk_kernel<<<(unsigned)gmax, dt, 0, stream>>>(X, d, ldx, w.order, w.offsets, counts,
                                                      w.chunk_base, w.chunk_j, w.n_chunks, best_key,
-                                                     w.part, inertia ? w.part_in : nullptr);
-  km_combine_kernel<<<(unsigned)kc, dt, 0, stream>>>(w.part, inertia ? w.part_in : nullptr, d,
-                                                     counts, w.chunk_base, sums, w.in_j);
+                                                     w.part, inertia ? w.part_in : nullptr, w.done,
+                                                     sums, w.in_j);
   if (inertia) km_inertia_kernel<<<1, 1024, 0, stream>>>(w.in_j, kc, inertia);
   return cudaGetLastError() == cudaSuccess ? 0 : 3;
 }
