@@ -127,6 +127,10 @@ size_t egemm_gemm_host_workspace_size(int64_t M, int64_t N, int64_t K);
  * the k rows x_j of X[nx x d] with the smallest squared distance
  *   dist_ij = ||q_i||^2 + ||x_j||^2 - 2 q_i . x_j ,
  * ascending by (dist, j), dist clamped to >= 0; self matches are kept (reading R11).
+ * Arithmetic (reading R22): q.x_j by Alg. 1 on the tensor core (one promotion
+ * chunk over d), then one more tensor-core step adds -||x_j||^2/2 (three exact tf32 parts
+ * times ones), key = -2 * that accumulator, dist = max(0, fp32(||q||^2 + key)); the results
+ * are bitwise reproducible and equal to the oracle's model of these steps.
  *  X     : the references, trans 0.  Either fp32 rows (then split and normed on the fly)
  *          or the "index" from egemm_knn_index: pre-split hi/lo + x_norms (f32 may be NULL).
  *  x_norms : nullable nx fp32 ||x_j||^2 (fp64-accumulated, from egemm_knn_index).
@@ -147,7 +151,8 @@ int egemm_knn_index(const float* X, int64_t nx, int64_t d, int64_t ldx, uint16_t
 
 /*
  * One Lloyd step of kMeans on the caller's shard of points (the GEMM-based kMeans of [2],
- * P:142-145): assign_i = argmin_j (||c_j||^2 - 2 x_i . c_j) (ties -> lowest j),
+ * P:142-145): assign_i = argmin_j (||c_j||^2 - 2 x_i . c_j) (ties -> lowest j;
+ * the key is formed on the tensor core as in egemm_knn, reading R22),
  * then fp64 partial sums sums[j][:] = sum_{a_i = j} x_i (from the fp32 x) and int64 counts.
  * sums / counts / inertia are OVERWRITTEN.  inertia (nullable) = sum_i dist(x_i, c_{a_i}).
  *  X : f32 required (n x d, trans 0); hi/lo optional (pre-split points).
