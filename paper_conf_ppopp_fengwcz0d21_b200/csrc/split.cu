@@ -10,8 +10,9 @@
 // HBM-bound: 4 B read + 4 B written per element.  The contiguous kernel moves 8 elements
 // per thread and iteration (2 x 16-B loads, one 16-B store per output) on a grid of
 // 148 x 8 CTAs; the transposing kernel (B stored K x N -> K-major N x K hi / lo) stages
-// 64 x 64 tiles through shared memory.  (Measured: wider 16-element iterations and
-// 128 x 64 tiles with 16-B stores were slower on B200.)
+// 64 x 64 tiles through shared memory, splitting row pairs so the transpose moves packed
+// fp16x2 words and writes 16 B per store.  The range-flag tests are compiled out unless
+// the caller passes range_flags.  (Measured: wider 16-element flat iterations were slower.)
 #include <cuda_fp16.h>
 #include <cstdint>
 #include "egemm_internal.h"
@@ -22,7 +23,7 @@ struct SplitPair {
   uint32_t hi, lo;  // two packed fp16 each (element a in the low half)
 };
 
-template <int MODE>
+template <int MODE, bool FLAGS = true>
 __device__ __forceinline__ SplitPair split2(float a, float b, uint32_t& flags) {
   uint32_t h, l;
   if (MODE == 0) asm("cvt.rn.f16x2.f32 %0, %1, %2;" : "=r"(h) : "f"(b), "f"(a));
@@ -32,10 +33,12 @@ __device__ __forceinline__ SplitPair split2(float a, float b, uint32_t& flags) {
   const float ra = __fsub_rn(a, hf.x), rb = __fsub_rn(b, hf.y);  // exact in fp32
   if (MODE == 0) asm("cvt.rn.f16x2.f32 %0, %1, %2;" : "=r"(l) : "f"(rb), "f"(ra));
   else asm("cvt.rz.f16x2.f32 %0, %1, %2;" : "=r"(l) : "f"(rb), "f"(ra));
-  const float aa = fabsf(a), ab = fabsf(b);
-  // bit0: |x| >= 65520 (rounds to inf) or non-finite; bit1: 0 < |x| < 2^-3 (below 21-bit zone)
-  flags |= (!(aa < 65520.f) || !(ab < 65520.f)) ? 1u : 0u;
-  flags |= ((aa > 0.f && aa < 0.125f) || (ab > 0.f && ab < 0.125f)) ? 2u : 0u;
+  if constexpr (FLAGS) {  // only when the caller asked for range_flags
+    const float aa = fabsf(a), ab = fabsf(b);
+    // bit0: |x| >= 65520 (rounds to inf) or non-finite; bit1: 0 < |x| < 2^-3 (below 21-bit zone)
+    flags |= (!(aa < 65520.f) || !(ab < 65520.f)) ? 1u : 0u;
+    flags |= ((aa > 0.f && aa < 0.125f) || (ab > 0.f && ab < 0.125f)) ? 2u : 0u;
+  }
   return SplitPair{h, l};
 }
 
@@ -46,7 +49,7 @@ __device__ __forceinline__ void flush_flags(uint32_t flags, uint32_t* range_flag
 }
 
 // Contiguous x, hi, lo: 8 elements per thread-iteration, scalar tail.
-template <int MODE>
+template <int MODE, bool FLAGS>
 __global__ void __launch_bounds__(256) split_flat_kernel(const float* __restrict__ x, int64_t n,
                                                           uint16_t* __restrict__ hi,
                                                           uint16_t* __restrict__ lo,
@@ -57,8 +60,8 @@ __global__ void __launch_bounds__(256) split_flat_kernel(const float* __restrict
   for (int64_t g = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; g < nv; g += stride) {
     const float4* src = reinterpret_cast<const float4*>(x) + 2 * g;
     const float4 a = __ldcs(src), b = __ldcs(src + 1);
-    const SplitPair p0 = split2<MODE>(a.x, a.y, flags), p1 = split2<MODE>(a.z, a.w, flags);
-    const SplitPair p2 = split2<MODE>(b.x, b.y, flags), p3 = split2<MODE>(b.z, b.w, flags);
+    const SplitPair p0 = split2<MODE, FLAGS>(a.x, a.y, flags), p1 = split2<MODE, FLAGS>(a.z, a.w, flags);
+    const SplitPair p2 = split2<MODE, FLAGS>(b.x, b.y, flags), p3 = split2<MODE, FLAGS>(b.z, b.w, flags);
     __stcs(reinterpret_cast<uint4*>(hi) + g, make_uint4(p0.hi, p1.hi, p2.hi, p3.hi));
     __stcs(reinterpret_cast<uint4*>(lo) + g, make_uint4(p0.lo, p1.lo, p2.lo, p3.lo));
   }
@@ -103,11 +106,13 @@ __global__ void __launch_bounds__(256) split_transpose_kernel(const float* __res
                                                                int64_t ldx,
                                                                uint16_t* __restrict__ hi,
                                                                uint16_t* __restrict__ lo,
-                                                               int64_t ldo, uint32_t* range_flags) {
+                                                               int64_t ldo, uint32_t* range_flags,
+                                                               int skip_full) {
   __shared__ uint32_t th[64][33];  // packed fp16 pairs of tile element [c][r]
   __shared__ uint32_t tl[64][33];
   uint32_t flags = 0;
   const int64_t r0 = (int64_t)blockIdx.y * kTR, c0 = (int64_t)blockIdx.x * kTC;
+  if (skip_full && r0 + kTR <= rows && c0 + kTC <= cols) return;  // done by the fast kernel
   const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;  // 32 x 8
   for (int i = 0; i < 8; i++) {
     const int r = ty + 8 * i;
@@ -146,11 +151,56 @@ __global__ void __launch_bounds__(256) split_transpose_kernel(const float* __res
   flush_flags(flags, range_flags);  // padding elements are 0: they raise no flag
 }
 
+// Transposing, full 64 x 64 tiles with aligned rows (x: 16-B float4 loads; hi / lo: 16-B
+// stores).  Each thread splits the PAIR (x[r][c], x[r+1][c]) into one packed fp16x2 word
+// per output -- already the output's order along r -- so the smem transpose moves 32-bit
+// words and the write-out is one 16-B store per 8 outputs.  Edge tiles (and unaligned
+// operands) take split_transpose_kernel.
+template <int MODE, bool FLAGS>
+__global__ void __launch_bounds__(256) split_transpose_fast_kernel(
+    const float* __restrict__ x, int64_t rows, int64_t cols, int64_t ldx, uint16_t* __restrict__ hi,
+    uint16_t* __restrict__ lo, int64_t ldo, uint32_t* range_flags) {
+  __shared__ uint32_t th[kTC][kTR / 2 + 1];  // [c][r/2]: packed (r, r+1) pairs, 33-word pitch
+  __shared__ uint32_t tl[kTC][kTR / 2 + 1];
+  uint32_t flags = 0;
+  const int64_t r0 = (int64_t)blockIdx.y * kTR, c0 = (int64_t)blockIdx.x * kTC;
+  const int t = threadIdx.x;
+  {
+    const int tx = t & 15, ty = t >> 4;  // 16 column quads x 16 row pairs (two passes)
+#pragma unroll
+    for (int i = 0; i < 2; i++) {
+      const int rp = ty + 16 * i;  // row pair: rows 2 rp, 2 rp + 1
+      const float* src = x + (r0 + 2 * rp) * ldx + c0 + 4 * tx;
+      const float4 u = __ldcs(reinterpret_cast<const float4*>(src));
+      const float4 v = __ldcs(reinterpret_cast<const float4*>(src + ldx));
+      const SplitPair p0 = split2<MODE, FLAGS>(u.x, v.x, flags);
+      const SplitPair p1 = split2<MODE, FLAGS>(u.y, v.y, flags);
+      const SplitPair p2 = split2<MODE, FLAGS>(u.z, v.z, flags);
+      const SplitPair p3 = split2<MODE, FLAGS>(u.w, v.w, flags);
+      th[4 * tx][rp] = p0.hi; th[4 * tx + 1][rp] = p1.hi; th[4 * tx + 2][rp] = p2.hi; th[4 * tx + 3][rp] = p3.hi;
+      tl[4 * tx][rp] = p0.lo; tl[4 * tx + 1][rp] = p1.lo; tl[4 * tx + 2][rp] = p2.lo; tl[4 * tx + 3][rp] = p3.lo;
+    }
+  }
+  __syncthreads();
+#pragma unroll
+  for (int i = 0; i < 2; i++) {  // 64 output rows x 8 chunks of 8 fp16 = 512 chunks
+    const int q = t + 256 * i;
+    const int c = q >> 3, k = q & 7;
+    const uint4 vh = make_uint4(th[c][4 * k], th[c][4 * k + 1], th[c][4 * k + 2], th[c][4 * k + 3]);
+    const uint4 vl = make_uint4(tl[c][4 * k], tl[c][4 * k + 1], tl[c][4 * k + 2], tl[c][4 * k + 3]);
+    const int64_t o = (c0 + c) * ldo + r0 + 8 * k;
+    __stcs(reinterpret_cast<uint4*>(hi + o), vh);
+    __stcs(reinterpret_cast<uint4*>(lo + o), vl);
+  }
+  if constexpr (FLAGS) flush_flags(flags, range_flags);
+}
+
 template <int MODE>
 static void launch_mode(const float* x, int64_t rows, int64_t cols, int64_t ldx, uint16_t* hi,
                         uint16_t* lo, int64_t ldo, int transpose, uint32_t* range_flags,
                         cudaStream_t stream) {
   const int nsm = num_sms();
+  const bool fl = range_flags != nullptr;
   if (!transpose) {
     const bool flat = (ldx == cols && ldo == cols && ((uintptr_t)x % 16 == 0) &&
                        ((uintptr_t)hi % 16 == 0) && ((uintptr_t)lo % 16 == 0));
@@ -160,7 +210,8 @@ static void launch_mode(const float* x, int64_t rows, int64_t cols, int64_t ldx,
       const int64_t cap = (int64_t)nsm * 8;  // 8 x 256 threads resident per SM
       if (blocks > cap) blocks = cap;
       if (blocks < 1) blocks = 1;
-      split_flat_kernel<MODE><<<(unsigned)blocks, 256, 0, stream>>>(x, n, hi, lo, range_flags);
+      if (fl) split_flat_kernel<MODE, true><<<(unsigned)blocks, 256, 0, stream>>>(x, n, hi, lo, range_flags);
+      else split_flat_kernel<MODE, false><<<(unsigned)blocks, 256, 0, stream>>>(x, n, hi, lo, nullptr);
     } else {
       int64_t blocks = (n + 255) / 256;
       const int64_t cap = (int64_t)nsm * 8;
@@ -170,8 +221,21 @@ static void launch_mode(const float* x, int64_t rows, int64_t cols, int64_t ldx,
     }
   } else {
     dim3 grid((unsigned)((cols + kTC - 1) / kTC), (unsigned)((rows + kTR - 1) / kTR));
-    split_transpose_kernel<MODE><<<grid, 256, 0, stream>>>(x, rows, cols, ldx, hi, lo, ldo,
-                                                           range_flags);
+    const bool fast = (ldx % 4 == 0) && ((uintptr_t)x % 16 == 0) && (ldo % 8 == 0) &&
+                      ((uintptr_t)hi % 16 == 0) && ((uintptr_t)lo % 16 == 0);
+    const dim3 full((unsigned)(cols / kTC), (unsigned)(rows / kTR));
+    if (fast && full.x > 0 && full.y > 0) {
+      if (fl)
+        split_transpose_fast_kernel<MODE, true><<<full, 256, 0, stream>>>(x, rows, cols, ldx, hi, lo,
+                                                                          ldo, range_flags);
+      else
+        split_transpose_fast_kernel<MODE, false><<<full, 256, 0, stream>>>(x, rows, cols, ldx, hi, lo,
+                                                                           ldo, nullptr);
+    }
+    const bool edges = !fast || (cols % kTC) != 0 || (rows % kTR) != 0 || full.x == 0 || full.y == 0;
+    if (edges)
+      split_transpose_kernel<MODE><<<grid, 256, 0, stream>>>(x, rows, cols, ldx, hi, lo, ldo,
+                                                             range_flags, fast ? 1 : 0);
   }
 }
 

@@ -46,6 +46,25 @@ def test_split_transpose_and_ragged(oracle_lib, shape):
     assert np.array_equal(u16(hiT), ohi.T) and np.array_equal(u16(loT), olo.T)
 
 
+@pytest.mark.parametrize("shape", [(64, 64), (2048, 4096), (4100, 130)])
+def test_split_transpose_all_patterns_sampled(oracle_lib, shape):
+    """The tiled transposing kernel (full 64 x 64 tiles; edge tiles on the generic kernel)
+    bit-exact on fp32 patterns drawn from all of [0, 2^32) -- NaN / inf / subnormal
+    included -- with and without range_flags."""
+    eg = require_gpu()
+    n = shape[0] * shape[1]
+    bits = inputs.rng(13 + shape[0]).integers(0, 1 << 32, size=n, dtype=np.uint64).astype(np.uint32)
+    x = bits.view(np.float32).reshape(shape)
+    ohi, olo = oracle_lib.split(x.ravel())
+    ohi, olo = ohi.reshape(shape), olo.reshape(shape)
+    for flags in (None, torch.zeros(1, dtype=torch.int32, device="cuda")):
+        hiT, loT = eg.split(to_dev(x), transpose=True, range_flags=flags)
+        ok = _cmp(x.T.ravel(), u16(hiT).ravel(), u16(loT).ravel(), ohi.T.ravel(), olo.T.ravel())
+        assert ok.all()
+        if flags is not None:
+            assert int(to_host(flags)[0]) == 3  # inf/NaN and tiny values are present
+
+
 def test_split_strided_view(oracle_lib):
     eg = require_gpu()
     big = inputs.uniform((300, 512), 12)
