@@ -77,6 +77,7 @@ struct KParams {
   const float* a_f32;
   int64_t lda_f32;
   int vec_a;
+  int a_pf;         // FA: k-blocks of fp32 A prefetched into L2 ahead of the converters (0: off)
   int K;
   int debug_no_tma;  // EGEMM_DEBUG_NO_TMA=1: skip operand loads (timing diagnostics only)
   int debug_no_epi;  // EGEMM_DEBUG_NO_EPI=1: skip the promotion's TMEM reads (diagnostics)
@@ -282,10 +283,8 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
   const bool leader = (rank == 0);
 
   if (warp == EG::W_PROD && lane == 0) {
-    if (!FA) {
-      ptx::prefetch_tmap(&tm_ahi);
-      ptx::prefetch_tmap(&tm_alo);
-    }
+    if (!FA || p.a_pf) ptx::prefetch_tmap(&tm_ahi);  // FA: tm_ahi maps the fp32 A (L2 prefetch)
+    if (!FA) ptx::prefetch_tmap(&tm_alo);
     ptx::prefetch_tmap(&tm_bhi);
     ptx::prefetch_tmap(&tm_blo);
   }
@@ -451,6 +450,14 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
                 pace = false;  // not all CTAs resident: run unpaced (others time out too)
             }
             gkb++;
+            if (FA && p.a_pf) {
+              // the converters' fp32 A tile a_pf k-blocks ahead (and the unit's first ones):
+              // their LDGs then hit L2 instead of waiting for DRAM
+              const int kf = kb + p.a_pf;
+              if (kb == 0)
+                for (int j = 0; j < p.a_pf && j < p.num_kb; j++) ptx::tma_prefetch_2d_l2(&tm_ahi, j * kBK, arow);
+              if (ns == 0 && kf < p.num_kb) ptx::tma_prefetch_2d_l2(&tm_ahi, kf * kBK, arow);
+            }
             ptx::mbar_wait(&empty[stage], phase ^ 1u);
             uint8_t* sb = stage_base + stage * SB;
             if (p.debug_no_tma) {  // diagnostics only: MMA-issue ceiling without operand traffic
@@ -961,6 +968,22 @@ static bool make_tmap_f16(CUtensorMap* m, const void* base, int64_t rows, int64_
   return r == CUDA_SUCCESS;
 }
 
+// fp32 [rows x cols] row-major (row stride ld elements), box {64, box_rows}, no swizzle:
+// only used for L2 prefetches of the fused-split A operand.
+static bool make_tmap_f32(CUtensorMap* m, const void* base, int64_t rows, int64_t cols, int64_t ld,
+                          int box_rows) {
+  auto enc = get_encode();
+  if (!enc) return false;
+  cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {(cuuint64_t)(ld * 4)};
+  cuuint32_t box[2] = {64u, (cuuint32_t)box_rows};
+  cuuint32_t estr[2] = {1u, 1u};
+  CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<void*>(base), dims, strides,
+                   box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                   CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  return r == CUDA_SUCCESS;
+}
+
 template <int CG, int BN, bool SEP, int EPI, int STAGES, bool FA = false, bool AR = false>
 static int launch_variant(const CUtensorMap* maps, const KParams& kp, int max_clusters,
                           cudaStream_t stream) {
@@ -1069,7 +1092,7 @@ int launch_tc(int64_t M, int64_t N, int64_t K, const TcOperands& ops, const TcCo
     set_last_error("cuTensorMapEncodeTiled failed (alignment: base 16 B, ld %% 8 == 0)");
     return 2;
   }
-  if (fa) {  // A is converted in-kernel; its maps are unused (pass B's as placeholders)
+  if (fa) {  // A is converted in-kernel: maps[0] = fp32 A for the L2 prefetch (else a placeholder)
     maps[0] = maps[2];
     maps[1] = maps[3];
   }
@@ -1086,6 +1109,11 @@ int launch_tc(int64_t M, int64_t N, int64_t K, const TcOperands& ops, const TcCo
     kp.a_f32 = ops.a_f32;
     kp.lda_f32 = ops.lda_f32;
     kp.vec_a = ((ops.lda_f32 % 4) == 0 && ((uintptr_t)ops.a_f32 % 16) == 0) ? 1 : 0;
+    const char* pf = getenv("EGEMM_A_PREFETCH");
+    kp.a_pf = pf ? atoi(pf) : 2;  // measured: 2 > 4 > 8 > 0 at 65536 x 256 x 1024
+    if (kp.a_pf < 0) kp.a_pf = 0;
+    if (kp.a_pf && !(kp.vec_a && make_tmap_f32(&maps[0], ops.a_f32, M, K, ops.lda_f32, kBM)))
+      kp.a_pf = 0;
   }
   kp.M = (int)M;
   kp.N = (int)N;

@@ -127,6 +127,13 @@ __device__ __forceinline__ void tma_load_2d_pair(const void* tmap, uint64_t* bar
       "l"(reinterpret_cast<uint64_t>(tmap)), "r"(b), "r"(c0), "r"(c1)
       : "memory");
 }
+// Bulk prefetch of a 2-D tensor tile into L2 (no smem, no barrier).
+__device__ __forceinline__ void tma_prefetch_2d_l2(const void* tmap, int32_t c0, int32_t c1) {
+  asm volatile("cp.async.bulk.prefetch.tensor.2d.L2.global.tile [%0, {%1, %2}];" ::"l"(
+                   reinterpret_cast<uint64_t>(tmap)),
+               "r"(c0), "r"(c1)
+               : "memory");
+}
 __device__ __forceinline__ void tma_store_2d(const void* tmap, const void* src, int32_t c0,
                                              int32_t c1) {
   asm volatile(
