@@ -195,3 +195,20 @@ def test_kmeans_ties_lowest_index_bitexact(oracle_lib, n, d, kc, dup):
     assert ga.max() < dup  # the first copy always wins
     rs, rc = oracle_lib.group_sums(X, ra, kc)
     assert np.array_equal(to_host(sums), rs) and np.array_equal(to_host(counts), rc)
+
+
+@pytest.mark.parametrize("scale", [2.0 ** 12, 2.0 ** -9])
+def test_knn_kmeans_norm_step_extreme_magnitudes(oracle_lib, scale):
+    """The R22 norm step on large (||x||^2 ~ 2^30) and tiny (~2^-12) norms: the tf32 parts
+    keep the full fp32 value at any magnitude, and the GPU still equals the model bitwise."""
+    eg = require_gpu()
+    X = (inputs.uniform((3000, 64), 95) * scale).astype(np.float32)
+    Q = (inputs.uniform((70, 64), 96) * scale).astype(np.float32)
+    idx, dist = eg.knn(to_dev(X), to_dev(Q), 8)
+    ri, rd = oracle_lib.knn_alg1_tc(X, Q, 8)
+    assert np.array_equal(to_host(idx), ri)
+    assert np.array_equal(to_host(dist).view(np.uint32), rd.view(np.uint32))
+    C = X[:100].copy()
+    a, _, _, _ = eg.kmeans_step(to_dev(X), to_dev(C))
+    ra, _ = oracle_lib.kmeans_assign_alg1_tc(X, C)
+    assert np.array_equal(to_host(a), ra)
