@@ -78,6 +78,7 @@ struct KParams {
   int64_t lda_f32;
   int vec_a;
   int a_pf;         // FA: k-blocks of fp32 A prefetched into L2 ahead of the converters (0: off)
+  int a_staged;     // FA: tm_ahi maps fp32 A with 32-column 128-B-swizzled boxes (AS variant)
   int K;
   int debug_no_tma;  // EGEMM_DEBUG_NO_TMA=1: skip operand loads (timing diagnostics only)
   int debug_no_epi;  // EGEMM_DEBUG_NO_EPI=1: skip the promotion's TMEM reads (diagnostics)
@@ -230,7 +231,7 @@ __device__ __forceinline__ void tf32_parts(float y, float& h, float& m, float& l
   l = __fsub_rn(r, m);
 }
 
-template <int CG, int BN, bool SEP, int EPI, int STAGES, int NEPI, bool FA, bool AR>
+template <int CG, int BN, bool SEP, int EPI, int STAGES, int NEPI, bool FA, bool AR, bool AS>
 __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
     egemm_tc_kernel(const __grid_constant__ CUtensorMap tm_ahi,
                     const __grid_constant__ CUtensorMap tm_alo,
@@ -262,9 +263,16 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
   constexpr int AR_BYTES = AR ? 2 * 2 * G::A_BYTES : 0;     // 2 k-blocks of A_hi + A_lo
   constexpr int ONES_BYTES = NORM ? kBM * 32 : 0;
   static_assert(SB % 1024 == 0, "stage alignment");
+  // AS (fused A, TMA-staged): the fp32 A tiles land in their own ring (NSTG x 128 rows x 64
+  // fp32, two 128-B-swizzled boxes of 32 columns), loaded ahead by warp 7; the converters
+  // split from smem instead of waiting on their own global loads.
+  constexpr int NSTG = AS ? 3 : 0;
+  constexpr int STG_BYTES = kBM * kBK * 4;
+  static_assert(!AS || FA, "AS is a fused-A mode");
   uint8_t* stage_base = smem;
   uint8_t* a_res = smem + STAGES * SB;
-  uint8_t* ones_tile = a_res + AR_BYTES;
+  uint8_t* a_stg = a_res + AR_BYTES;
+  uint8_t* ones_tile = a_stg + NSTG * STG_BYTES;
   uint64_t* bars = reinterpret_cast<uint64_t*>(ones_tile + ONES_BYTES);
   uint64_t* full = bars;
   uint64_t* empty = bars + STAGES;
@@ -273,7 +281,9 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
   uint64_t* a_full = bars + 2 * STAGES + 4;
   uint64_t* a_empty = bars + 2 * STAGES + 5;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * STAGES + 6);
-  uint8_t* scratch = reinterpret_cast<uint8_t*>(bars + 2 * STAGES + 8);  // epilogue merges
+  uint64_t* sfull = bars + 2 * STAGES + 8;   // AS: fp32 A tile landed (TMA bytes)
+  uint64_t* sempty = sfull + NSTG;           // AS: consumed by the 4 converter warps
+  uint8_t* scratch = reinterpret_cast<uint8_t*>(bars + 2 * STAGES + 8 + 2 * NSTG);  // merges
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
@@ -301,6 +311,10 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
     }
     ptx::mbar_init(a_full, 1);
     ptx::mbar_init(a_empty, 1);
+    for (int i = 0; i < NSTG; i++) {
+      ptx::mbar_init(&sfull[i], 1);
+      ptx::mbar_init(&sempty[i], 4);
+    }
     ptx::fence_mbar_init();
   }
   if (!FA && !AR && p.debug_no_tma && (p.debug_mode & 32)) {
@@ -360,6 +374,8 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
     if constexpr (FA) {
       int stage = 0;
       uint32_t phase = 0;
+      int si = 0;          // AS: staging ring slot / parity
+      uint32_t sph = 0;
       const int c = lane & 7;         // 16-B chunk (8 fp16) of the 128-B row
       const int rsub = lane >> 3;     // 4 rows per warp instruction
       for (int u = cluster; u < p.num_units; u += nclusters) {
@@ -367,6 +383,40 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
         const int64_t arow0 = (int64_t)ui.m_tile * (kBM * CG) + rank * kBM;
         for (int ns = 0; ns < ui.n_count; ns++) {
           for (int kb = 0; kb < p.num_kb; kb++) {
+            if constexpr (AS) {
+              // fp32 tile from the TMA ring: row r, 8 values k = 8c..8c+7 are fp32 16-B
+              // chunks 2(c%4), 2(c%4)+1 of box c/4, at chunk position j ^ (r & 7) (SW128)
+              ptx::mbar_wait(&sfull[si], sph);
+              ptx::mbar_wait(&empty[stage], phase ^ 1u);
+              const uint32_t sb = ptx::smem_u32(stage_base + stage * G::STAGE_BYTES);
+              const uint32_t xb = ptx::smem_u32(a_stg + si * STG_BYTES) + (c >> 2) * (STG_BYTES / 2);
+              const int j0 = (c & 3) * 2;
+#pragma unroll
+              for (int it = 0; it < 8; it++) {
+                const int r = warp * 32 + it * 4 + rsub;
+                const uint32_t rb = xb + r * 128;
+                const float4 u0 = ptx::lds128f(rb + ((j0 ^ (r & 7)) << 4));
+                const float4 u1 = ptx::lds128f(rb + (((j0 + 1) ^ (r & 7)) << 4));
+                uint32_t hi[4], lo[4];
+                ptx::split2(u0.x, u0.y, hi[0], lo[0]);
+                ptx::split2(u0.z, u0.w, hi[1], lo[1]);
+                ptx::split2(u1.x, u1.y, hi[2], lo[2]);
+                ptx::split2(u1.z, u1.w, hi[3], lo[3]);
+                const uint32_t off = (uint32_t)(r * 128 + ((c ^ (r & 7)) << 4));
+                ptx::sts128(sb + off, hi[0], hi[1], hi[2], hi[3]);
+                ptx::sts128(sb + G::A_BYTES + off, lo[0], lo[1], lo[2], lo[3]);
+              }
+              ptx::fence_proxy_async_smem();  // generic-proxy stores -> visible to tcgen05.mma
+              __syncwarp();
+              if (lane == 0) {
+                if constexpr (CG == 1) ptx::mbar_arrive(&full[stage]);
+                else ptx::mbar_arrive_cluster(&full[stage], 0);
+                ptx::mbar_arrive(&sempty[si]);
+              }
+              if (++stage == STAGES) { stage = 0; phase ^= 1u; }
+              if (++si == NSTG) { si = 0; sph ^= 1u; }
+              continue;
+            }
             ptx::mbar_wait(&empty[stage], phase ^ 1u);
             const uint32_t sb = ptx::smem_u32(stage_base + stage * G::STAGE_BYTES);
             const int k = kb * kBK + c * 8;
@@ -450,7 +500,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
                 pace = false;  // not all CTAs resident: run unpaced (others time out too)
             }
             gkb++;
-            if (FA && p.a_pf) {
+            if (FA && !AS && p.a_pf) {
               // the converters' fp32 A tile a_pf k-blocks ahead (and the unit's first ones):
               // their LDGs then hit L2 instead of waiting for DRAM
               const int kf = kb + p.a_pf;
@@ -491,6 +541,28 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
         const uint32_t pe = (uint32_t)p.pace_e;
         const uint32_t total = (per_cta + pe - 1) / pe;
         for (uint32_t e = (gkb + pe - 1) / pe; e < total; e++) sync_arrive(p.sync, e);
+      }
+    }
+  } else if (AS && warp == 7) {
+    // ==================== fp32 A staging producer (fused A, AS) ====================
+    if constexpr (AS) {
+      if (lane == 0) {
+        int si = 0;
+        uint32_t sph = 0;
+        for (int u = cluster; u < p.num_units; u += nclusters) {
+          UnitInfo ui = decode_unit<EPI>(p, u);
+          const int arow = ui.m_tile * (kBM * CG) + (int)rank * kBM;
+          for (int ns = 0; ns < ui.n_count; ns++) {
+            for (int kb = 0; kb < p.num_kb; kb++) {
+              ptx::mbar_wait(&sempty[si], sph ^ 1u);
+              ptx::mbar_arrive_expect_tx(&sfull[si], STG_BYTES);
+              uint8_t* dst = a_stg + si * STG_BYTES;
+              ptx::tma_load_2d(&tm_ahi, &sfull[si], dst, kb * kBK, arow);
+              ptx::tma_load_2d(&tm_ahi, &sfull[si], dst + STG_BYTES / 2, kb * kBK + 32, arow);
+              if (++si == NSTG) { si = 0; sph ^= 1u; }
+            }
+          }
+        }
       }
     }
   } else if (NORM && warp == 3) {
@@ -971,20 +1043,22 @@ static bool make_tmap_f16(CUtensorMap* m, const void* base, int64_t rows, int64_
 // fp32 [rows x cols] row-major (row stride ld elements), box {64, box_rows}, no swizzle:
 // only used for L2 prefetches of the fused-split A operand.
 static bool make_tmap_f32(CUtensorMap* m, const void* base, int64_t rows, int64_t cols, int64_t ld,
-                          int box_rows) {
+                          int box_rows, int box_cols = 64, bool sw128 = false) {
   auto enc = get_encode();
   if (!enc) return false;
   cuuint64_t dims[2] = {(cuuint64_t)cols, (cuuint64_t)rows};
   cuuint64_t strides[1] = {(cuuint64_t)(ld * 4)};
-  cuuint32_t box[2] = {64u, (cuuint32_t)box_rows};
+  cuuint32_t box[2] = {(cuuint32_t)box_cols, (cuuint32_t)box_rows};
   cuuint32_t estr[2] = {1u, 1u};
   CUresult r = enc(m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, const_cast<void*>(base), dims, strides,
-                   box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_NONE,
+                   box, estr, CU_TENSOR_MAP_INTERLEAVE_NONE,
+                   sw128 ? CU_TENSOR_MAP_SWIZZLE_128B : CU_TENSOR_MAP_SWIZZLE_NONE,
                    CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
   return r == CUDA_SUCCESS;
 }
 
-template <int CG, int BN, bool SEP, int EPI, int STAGES, bool FA = false, bool AR = false>
+template <int CG, int BN, bool SEP, int EPI, int STAGES, bool FA = false, bool AR = false,
+          bool AS = false>
 static int launch_variant(const CUtensorMap* maps, const KParams& kp, int max_clusters,
                           cudaStream_t stream) {
   using G = Geo<CG, BN>;
@@ -992,13 +1066,14 @@ static int launch_variant(const CUtensorMap* maps, const KParams& kp, int max_cl
   // kNN keeps 8 (with 16 each thread's list sees half the columns, twice the insertions:
   // measured 3-15 % slower even without spills after the norm MMA freed 32 registers)
   constexpr int NEPI = (EPI == EPI_KMEANS) ? 16 : 8;
-  auto kern = egemm_tc_kernel<CG, BN, SEP, EPI, STAGES, NEPI, FA, AR>;
+  auto kern = egemm_tc_kernel<CG, BN, SEP, EPI, STAGES, NEPI, FA, AR, AS>;
   // kNN: top-k merge lists (half a list per round); kMeans: (key, index) of 3 column groups
   const int scratch = EPI == EPI_KNN ? kBM * kKnnMax * 4 : EPI == EPI_KMEANS ? 2 * 4 * kBM * 4 : 0;
   constexpr bool NORM = (EPI != EPI_STORE);  // norm slot per stage + the A' ones tile
   const size_t sb = (AR ? 2 * G::B_BYTES : G::STAGE_BYTES) + (NORM ? G::BNC * 32 : 0);
   const size_t smem = 1024 + (size_t)STAGES * sb + (AR ? 4 * G::A_BYTES : 0) +
-                      (NORM ? kBM * 32 : 0) + 8 * (2 * STAGES + 8) + scratch;
+                      (NORM ? kBM * 32 : 0) + (AS ? 3 * kBM * kBK * 4 + 8 * 6 : 0) +
+                      8 * (2 * STAGES + 8) + scratch;
   static bool attr_done = false;  // per instantiation
   if (!attr_done) {
     if (cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)smem) !=
@@ -1043,6 +1118,9 @@ static int dispatch(const CUtensorMap* maps, const KParams& kp, const TcConfig& 
                     cudaStream_t s) {
   if constexpr (EPI == EPI_STORE) {
     if (kp.a_f32) {  // fused A split (converter warpgroup)
+      // aligned fp32 A: TMA-staged (2 MMA stages + 3 fp32 staging slots); else LDG converters
+      if (cfg.cg == 2 && cfg.bn == 256 && !cfg.sep && kp.a_staged)
+        return launch_variant<2, 256, false, EPI, 2, true, false, true>(maps, kp, cfg.max_clusters, s);
       if (cfg.cg == 2 && cfg.bn == 256 && !cfg.sep)
         return launch_variant<2, 256, false, EPI, 3, true>(maps, kp, cfg.max_clusters, s);
       if (cfg.cg == 2 && cfg.bn == 128 && cfg.sep)
@@ -1112,6 +1190,10 @@ int launch_tc(int64_t M, int64_t N, int64_t K, const TcOperands& ops, const TcCo
     const char* pf = getenv("EGEMM_A_PREFETCH");
     kp.a_pf = pf ? atoi(pf) : 2;  // measured: 2 > 4 > 8 > 0 at 65536 x 256 x 1024
     if (kp.a_pf < 0) kp.a_pf = 0;
+    const char* st = getenv("EGEMM_A_STAGED");
+    kp.a_staged = (st ? atoi(st) : 1) && kp.vec_a && cfg.cg == 2 && cfg.bn == 256 && !cfg.sep &&
+                  make_tmap_f32(&maps[0], ops.a_f32, M, K, ops.lda_f32, kBM, 32, true);
+    if (kp.a_staged) kp.a_pf = 0;
     if (kp.a_pf && !(kp.vec_a && make_tmap_f32(&maps[0], ops.a_f32, M, K, ops.lda_f32, kBM)))
       kp.a_pf = 0;
   }
