@@ -489,16 +489,39 @@ def _apps(world, rank, dev, args):
             reps = max(5, int(150.0 / max(one, 1e-3)))
             for _ in range(max(3, reps // 5)):
                 egemm.gemm(A2, B2, out=D2, workspace=ws2)
+            # small sizes: the public call is captured once into a CUDA graph (its 2-3 launches)
+            # and replayed, so the host-side Python/ctypes cost of a call does not set the rate
+            graph = None
+            if n2 <= 4096:
+                try:
+                    cs = torch.cuda.Stream()
+                    cs.wait_stream(torch.cuda.current_stream())
+                    with torch.cuda.stream(cs):
+                        egemm.gemm(A2, B2, out=D2, workspace=ws2, stream=cs)
+                    torch.cuda.current_stream().wait_stream(cs)
+                    graph = torch.cuda.CUDAGraph()
+                    with torch.cuda.graph(graph):
+                        egemm.gemm(A2, B2, out=D2, workspace=ws2,
+                                   stream=torch.cuda.current_stream())
+                    for _ in range(3):
+                        graph.replay()
+                except Exception:  # pragma: no cover -- fall back to direct calls
+                    graph = None
+            run = graph.replay if graph is not None else (
+                lambda: egemm.gemm(A2, B2, out=D2, workspace=ws2))
             _barrier(world)
             s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
             s.record()
             for _ in range(reps):
-                egemm.gemm(A2, B2, out=D2, workspace=ws2)
+                run()
             e.record()
             _barrier(world)
             ms = _allmax(s.elapsed_time(e), world) / reps
             sweep[str(n2)] = {"tflops": round(2.0 * n2 ** 3 / (ms * 1e-3) / 1e12, 1), "ms": round(ms, 4),
-                              "config": list(egemm.query_config("gemm", r1 - r0, n2, n2, with_fused=True))}
+                              "config": list(egemm.query_config("gemm", r1 - r0, n2, n2, with_fused=True)),
+                              "timing": "CUDA-graph replay of egemm_gemm" if graph is not None
+                              else "direct egemm_gemm calls"}
+            del graph
             del A2, B2, ws2, D2
         out["square_sweep"] = {"metric": "EGEMM FP32-equiv TFLOP/s, N^3 (configs[1] sweep; split included)",
                                "unit": "TFLOP/s", "by_n": sweep}
