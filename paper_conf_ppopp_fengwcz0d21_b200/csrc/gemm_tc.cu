@@ -221,6 +221,7 @@ __device__ __forceinline__ void named_bar_sync(int id, int nthreads) {
   asm volatile("bar.sync %0, %1;" ::"r"(id), "r"(nthreads) : "memory");
 }
 
+
 // y = h + m + l exactly, each part with <= 11 significant bits and its 13 low mantissa bits
 // zero, i.e. exact tf32 operands (kind::tf32 ignores those bits).  Truncation split: h keeps
 // y's top 11 bits, r = y - h (exact) its low 13, m the top 11 of r, l = r - m (exact, <= 2).
@@ -256,6 +257,11 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
   // NORM (kNN / kMeans): each stage also has a 32-B row per staged B row for the tf32 norm
   // parts (written by the norm warp on a tile's last k-block), plus one A' tile of ones.
   constexpr bool NORM = (EPI != EPI_STORE);
+  // KREG (kNN, 8 epilogue warps): a thread's whole column share of a tile (COLS fp32) is
+  // loaded from TMEM at once and the accumulator handed back before any of it is ranked, so
+  // the top-k work of tile t overlaps the MMAs of tiles t+1 and t+2; the registers come from
+  // the control warpgroup (setmaxnreg 56 / 216: 4x32x56 + 8x32x216 <= 64K).
+  constexpr bool KREG = (EPI == EPI_KNN) && AR && !FA && NEPI == 8 && COLS == 128;
   constexpr int NP_OFF = AR ? 2 * G::B_BYTES : G::STAGE_BYTES;  // norm parts inside a stage
   constexpr int NP_BYTES = NORM ? G::BNC * 32 : 0;
   constexpr int SB = NP_OFF + NP_BYTES;                       // bytes per ring stage
@@ -460,7 +466,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
       }
     }
   } else if (warp < EG::EPI0) {
-   if constexpr (FA) asm volatile("setmaxnreg.dec.sync.aligned.u32 56;");
+   if constexpr (FA || KREG) asm volatile("setmaxnreg.dec.sync.aligned.u32 56;");
    if (warp == EG::W_PROD) {
     // ============================ TMA producer ============================
     if (lane == 0) {
@@ -722,6 +728,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
    }
   } else {
     if constexpr (FA) asm volatile("setmaxnreg.inc.sync.aligned.u32 176;");
+    if constexpr (KREG) asm volatile("setmaxnreg.inc.sync.aligned.u32 216;");
     // ============================ epilogue ============================
     const int ew = warp - EG::EPI0;
     const int q = warp & 3;         // TMEM lane quarter this warp may access
@@ -732,6 +739,10 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
 
     float kd[kKnnMax];
     int ki[kKnnMax];
+    // KREG: the two column groups of a row exchange their sorted key lists once per tile
+    // (double-buffered smem slots after the merge scratch, named barrier 5 + q)
+    uint32_t xgen = 0;
+    float* const xch = reinterpret_cast<float*>(scratch + kBM * kKnnMax * 4);
     float best = __int_as_float(0xff800000);
     int besti = 0x7fffffff;
 
@@ -838,6 +849,93 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
             continue;
           }
           const uint32_t acc_hh = tmem_base + lane_off + (SEP ? 2 * buf : buf) * BN + cgp * COLS;
+          if constexpr (KREG) {
+            float v[COLS];
+#pragma unroll
+            for (int c = 0; c < COLS / 32; c++) ptx::tmem_ld32(acc_hh + c * 32, v + c * 32);
+            ptx::tmem_wait_ld();
+            ptx::tc_fence_before();
+            __syncwarp();
+            if (lane == 0) {
+              if constexpr (CG == 1) ptx::mbar_arrive(&acc_empty[buf]);
+              else ptx::mbar_arrive_cluster(&acc_empty[buf], 0);
+            }
+            // Filter bound u = the 16th smallest key of (own list) U (the partner group's list
+            // as published after the previous tile of this unit).  Both lists hold distinct
+            // real columns of this row, so at least 16 keys <= u exist and a key > u can never
+            // reach the row's final top 16 (a key == u still may, by index: kept).  The union
+            // bound cuts the insertions to about those of one list over both column halves.
+            float u = kd[kKnnMax - 1];
+            {
+              if (ns > 0) {  // (ns == 0: the last publication belongs to the previous unit's rows)
+                const uint32_t pb = ptx::smem_u32(
+                    xch + ((((xgen - 1) & 1u) * GPQ + (cgp ^ 1)) * kBM + q * 32 + lane) * kKnnMax);
+                float b[kKnnMax];
+#pragma unroll
+                for (int t = 0; t < kKnnMax / 4; t++) {
+                  const float4 w = ptx::lds128f(pb + 16 * t);
+                  b[4 * t] = w.x; b[4 * t + 1] = w.y; b[4 * t + 2] = w.z; b[4 * t + 3] = w.w;
+                }
+                // 16th smallest of two sorted 16-lists: min over splits i of max(A[i-1], B[15-i])
+                float m = fminf(b[kKnnMax - 1], kd[kKnnMax - 1]);
+#pragma unroll
+                for (int i = 1; i < kKnnMax; i++) m = fminf(m, fmaxf(kd[i - 1], b[kKnnMax - 1 - i]));
+                u = m;
+              }
+            }
+            // key < own 16th (strict: stream order) and key <= u, in accumulator space
+            // (key = -2 v): v > -kd15/2 and v >= -u/2
+            const float vt = fmaxf(-0.5f * kd[kKnnMax - 1], nextafterf(-0.5f * u, __int_as_float(0xff800000)));
+#pragma unroll
+            for (int c = 0; c < COLS / 32; c++) {
+              float* g = v + c * 32;
+              const int c0 = col_base + c * 32;
+              if (c0 + 32 > p.N) {  // ragged last tile: columns >= N never win
+#pragma unroll
+                for (int i = 0; i < 32; i++) g[i] = (c0 + i < p.N) ? g[i] : __int_as_float(0xff800000);
+              }
+              // v = a.b_j - ||b_j||^2/2, key_j = -2 v (exact).  key < thr <=> v > -thr/2 (the
+              // threshold is itself -2 v_k: halving it is exact), so the filter compares the
+              // accumulators directly; the group maximum by a tree (depth 5, not a chain of 16).
+              float t16[16];
+#pragma unroll
+              for (int i = 0; i < 16; i++) t16[i] = fmaxf(g[2 * i], g[2 * i + 1]);
+#pragma unroll
+              for (int w = 8; w >= 1; w >>= 1)
+#pragma unroll
+                for (int i = 0; i < w; i++) t16[i] = fmaxf(t16[i], t16[i + w]);
+              if (__any_sync(0xffffffffu, t16[0] > vt) && !(p.debug_mode & 128)) {
+                uint32_t cand = 0;
+                float vv[32];
+#pragma unroll
+                for (int i = 0; i < 32; i++) {
+                  vv[i] = g[i];
+                  cand |= (g[i] > vt) ? (1u << i) : 0u;
+                }
+                // a thread's columns arrive in increasing index order: strict '<' inside the
+                // insertion keeps the lower index first among equal keys
+#pragma unroll 1
+                while (cand) {
+                  const int i = __ffs(cand) - 1;
+                  cand &= cand - 1u;
+                  topk_insert_stream<kKnnMax>(kd, ki, -2.f * vv[i], c0 + i);
+                }
+              }
+            }
+            {  // publish this tile's list for the partner group
+              const uint32_t ob = ptx::smem_u32(
+                  xch + (((xgen & 1u) * GPQ + cgp) * kBM + q * 32 + lane) * kKnnMax);
+#pragma unroll
+              for (int t = 0; t < kKnnMax / 4; t++)
+                ptx::sts128f(ob + 16 * t, kd[4 * t], kd[4 * t + 1], kd[4 * t + 2], kd[4 * t + 3]);
+              // lockstep per tile (a bar.arrive / bar.sync pair could let one warp arrive
+              // twice before the other syncs, merging two barrier generations)
+              named_bar_sync(5 + q, 64);
+              xgen++;
+            }
+            chunk_ctr++;
+            continue;
+          }
           // TMEM -> registers software-pipelined: the load of group c+1 is in flight while
           // group c is processed; the accumulator buffer is handed back to the MMA warp as
           // soon as the last group has landed in registers.
@@ -882,7 +980,8 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
               // increasing index order, so a strict '<' keeps the lower index first among
               // equal keys.
               const float thr = kd[kKnnMax - 1];
-              if (__any_sync(0xffffffffu, -2.f * mx < thr)) {
+              // (debug bit 128, diagnostics only: never take the candidate path)
+              if (__any_sync(0xffffffffu, -2.f * mx < thr) && !(p.debug_mode & 128)) {
                 uint32_t cand = 0;
                 float keys[32];
 #pragma unroll
@@ -1068,7 +1167,10 @@ static int launch_variant(const CUtensorMap* maps, const KParams& kp, int max_cl
   constexpr int NEPI = (EPI == EPI_KMEANS) ? 16 : 8;
   auto kern = egemm_tc_kernel<CG, BN, SEP, EPI, STAGES, NEPI, FA, AR, AS>;
   // kNN: top-k merge lists (half a list per round); kMeans: (key, index) of 3 column groups
-  const int scratch = EPI == EPI_KNN ? kBM * kKnnMax * 4 : EPI == EPI_KMEANS ? 2 * 4 * kBM * 4 : 0;
+  // (+ kNN KREG: two generations x two column groups x 128 rows of 16-key lists)
+  constexpr bool KREG = (EPI == EPI_KNN) && AR && !FA && NEPI == 8 && BN / (NEPI / 4) == 128;
+  const int scratch = EPI == EPI_KNN ? kBM * kKnnMax * 4 + (KREG ? 2 * 2 * kBM * kKnnMax * 4 : 0)
+                      : EPI == EPI_KMEANS ? 2 * 4 * kBM * 4 : 0;
   constexpr bool NORM = (EPI != EPI_STORE);  // norm slot per stage + the A' ones tile
   const size_t sb = (AR ? 2 * G::B_BYTES : G::STAGE_BYTES) + (NORM ? G::BNC * 32 : 0);
   const size_t smem = 1024 + (size_t)STAGES * sb + (AR ? 4 * G::A_BYTES : 0) +
@@ -1137,7 +1239,7 @@ static int dispatch(const CUtensorMap* maps, const KParams& kp, const TcConfig& 
     // reloads are cheap and the variant measured slightly slower)
     if (EPI == EPI_KNN && kp.num_kb <= 2 && cfg.cg == 2 && cfg.bn == 256 && !cfg.sep &&
         !kp.debug_no_tma && !getenv_flag("EGEMM_NO_ARES"))
-      return launch_variant<2, 256, false, EPI, 4, false, true>(maps, kp, cfg.max_clusters, s);
+      return launch_variant<2, 256, false, EPI, 3, false, true>(maps, kp, cfg.max_clusters, s);
   }
   if (cfg.cg == 2 && cfg.bn == 256 && !cfg.sep)
     return launch_variant<2, 256, false, EPI, 3>(maps, kp, cfg.max_clusters, s);
