@@ -999,6 +999,8 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
             } else {
               // group max first (3-input FMNMX), the index only when it improves.  (Parking
               // the improving quarter in smem and searching once per unit measured the same.)
+              // (a depth-5 tree here, or loading both groups and releasing the accumulator
+              // before the search, measured slower than this chain with 16 warps)
               float mx = __int_as_float(0xff800000);
 #pragma unroll
               for (int i = 0; i < 32; i++) mx = fmaxf(mx, v[i]);

@@ -162,6 +162,23 @@ def test_knn_bitexact_vs_alg1_model(oracle_lib, nx, nq, d, k, path):
     assert np.array_equal(to_host(dist).view(np.uint32), rd.view(np.uint32))
 
 
+@pytest.mark.parametrize("nx,d,dup,nq", [(6000, 64, 700, 300), (9000, 128, 37, 200), (4096, 32, 256, 64)])
+def test_knn_ties_lowest_index_bitexact(oracle_lib, nx, d, dup, nq):
+    """Exact key ties on integer data: the references are `dup` distinct rows repeated down
+    the index (copies in other 32-column groups, column halves and 256-column tiles), so the
+    16 nearest keys are shared by several columns and the lower indices must win.  This is
+    where the filter bound of the kNN epilogue (the 16th key of the union of a row's two
+    column-group lists, kept inclusive) could drop a tied column; bitwise vs the model."""
+    eg = require_gpu()
+    base = inputs.integers((dup, d), 95 + d, lim=4)
+    X = np.tile(base, (-(-nx // dup), 1))[:nx].copy()
+    Q = inputs.integers((nq, d), 96 + d, lim=4)
+    idx, dist = eg.knn(None, to_dev(Q), 16, index=eg.knn_index(to_dev(X)))
+    ri, rd = oracle_lib.knn_alg1_tc(X, Q, 16)
+    assert np.array_equal(to_host(idx), ri)
+    assert np.array_equal(to_host(dist).view(np.uint32), rd.view(np.uint32))
+
+
 @pytest.mark.parametrize("n,d,kc", [(20000, 64, 1024), (3001, 64, 100), (5000, 32, 7), (999, 130, 300),
                                     (9000, 16, 2000), (7000, 8, 7000)])
 def test_kmeans_assign_bitexact_vs_alg1_model(oracle_lib, n, d, kc):
