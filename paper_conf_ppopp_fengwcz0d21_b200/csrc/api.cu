@@ -54,7 +54,7 @@ static bool fused_a_supported(const TcConfig& c) {
 
 static bool valid_config(int cg, int bn, int sep) {
   return (cg == 2 && bn == 256 && sep == 0) || (cg == 1 && bn == 128) ||
-         (cg == 2 && bn == 128 && sep == 1);
+         (cg == 2 && bn == 128 && sep == 1) || (cg == 2 && bn == 224 && sep == 0);
 }
 
 static TcConfig choose_config(int epi_kind, int64_t M, int64_t N, int64_t K, int terms) {

@@ -247,7 +247,9 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
                                  : (NACC * BN <= 128) ? 128 : (NACC * BN <= 256) ? 256 : 512;
   static_assert(NACC * BN <= 512, "TMEM overflow");
   static_assert(!(EPI != EPI_STORE && SEP), "kNN / kMeans: single accumulator (norm MMA)");
-  static_assert(COLS % 32 == 0, "epilogue column split");
+  static_assert(COLS % 32 == 0 || (EPI == EPI_STORE && COLS % 16 == 0), "epilogue column split");
+  // TMEM -> register load width of the STORE epilogue (BN = 224: 112 columns per warp)
+  constexpr int LDW = (COLS % 32 == 0) ? 32 : 16;
 
   extern __shared__ __align__(1024) uint8_t smem_raw[];
   uint8_t* smem = reinterpret_cast<uint8_t*>((reinterpret_cast<uintptr_t>(smem_raw) + 1023) &
@@ -775,17 +777,19 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
             const uint32_t acc_hh = tmem_base + lane_off + (SEP ? 2 * buf : buf) * BN + cgp * COLS;
             if (!p.debug_no_epi)
 #pragma unroll
-            for (int c = 0; c < COLS / 32; c++) {
-              float v[32];
-              ptx::tmem_ld32(acc_hh + c * 32, v);
+            for (int c = 0; c < COLS / LDW; c++) {
+              float v[LDW];
+              if constexpr (LDW == 32) ptx::tmem_ld32(acc_hh + c * LDW, v);
+              else ptx::tmem_ld16(acc_hh + c * LDW, v);
               ptx::tmem_wait_ld();
 #pragma unroll
-              for (int i = 0; i < 32; i++) tot[c * 32 + i] = __fadd_rn(tot[c * 32 + i], v[i]);
+              for (int i = 0; i < LDW; i++) tot[c * LDW + i] = __fadd_rn(tot[c * LDW + i], v[i]);
               if constexpr (SEP) {
-                ptx::tmem_ld32(acc_hh + BN + c * 32, v);
+                if constexpr (LDW == 32) ptx::tmem_ld32(acc_hh + BN + c * LDW, v);
+                else ptx::tmem_ld16(acc_hh + BN + c * LDW, v);
                 ptx::tmem_wait_ld();
 #pragma unroll
-                for (int i = 0; i < 32; i++) totx[c * 32 + i] = __fadd_rn(totx[c * 32 + i], v[i]);
+                for (int i = 0; i < LDW; i++) totx[c * LDW + i] = __fadd_rn(totx[c * LDW + i], v[i]);
               }
             }
             ptx::tc_fence_before();
@@ -1245,6 +1249,12 @@ static int dispatch(const CUtensorMap* maps, const KParams& kp, const TcConfig& 
   }
   if (cfg.cg == 2 && cfg.bn == 256 && !cfg.sep)
     return launch_variant<2, 256, false, EPI, 3>(maps, kp, cfg.max_clusters, s);
+  if constexpr (EPI == EPI_STORE) {
+    // 256 x 224 pair tiles: ceil(N / 224) n-tiles make whole waves of 74 clusters where
+    // 256-wide tiles leave a partial one (e.g. M = 1024 or 2048 rows of N = 8192 per rank)
+    if (cfg.cg == 2 && cfg.bn == 224 && !cfg.sep)
+      return launch_variant<2, 224, false, EPI, 3>(maps, kp, cfg.max_clusters, s);
+  }
   if (cfg.cg == 1 && cfg.bn == 128 && !cfg.sep)
     return launch_variant<1, 128, false, EPI, 3>(maps, kp, cfg.max_clusters, s);
   if constexpr (EPI == EPI_STORE) {  // kNN / kMeans keep one accumulator (norm MMA)

@@ -12,7 +12,7 @@ from tests.gpu_util import require_gpu, to_dev, to_host
 pytestmark = pytest.mark.gpu
 
 CFGS = [(2, 256, 0, 64), (2, 256, 0, 128), (1, 128, 0, 64), (1, 128, 1, 128), (1, 128, 1, 256),
-        (2, 128, 1, 256)]
+        (2, 128, 1, 256), (2, 224, 0, 128), (2, 224, 0, 256)]
 
 
 def _gpu(eg, A, B, C, cfg, terms, fused):

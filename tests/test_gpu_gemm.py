@@ -17,7 +17,7 @@ pytestmark = pytest.mark.gpu
 # tile configs the tuning table can select (cg, bn, sep, Kc); longer Kc without SEP is an
 # error-sweep experiment only (tools/error_sweep.py): it exceeds the 2x naive-fp32 bar.
 CONFIGS = [(2, 256, 0, 64), (1, 128, 0, 64), (1, 128, 1, 256), (2, 128, 1, 256), (2, 256, 0, 128),
-           (1, 128, 1, 128)]
+           (1, 128, 1, 128), (2, 224, 0, 128)]
 
 
 def _run(eg, A, B, C=None, terms=0, cfg=None):

@@ -31,7 +31,7 @@ OUT = os.path.join(ROOT, "paper_conf_ppopp_fengwcz0d21_b200", "tune_table.json")
 CONFIGS = [(2, 256, 0, 64, 0), (2, 256, 0, 128, 0), (2, 256, 0, 256, 0), (2, 128, 1, 128, 0),
            (2, 128, 1, 256, 0), (1, 128, 1, 128, 0), (1, 128, 1, 256, 0), (1, 128, 0, 64, 0),
            (2, 256, 0, 64, 1), (2, 256, 0, 128, 1), (2, 256, 0, 256, 1), (2, 128, 1, 256, 1),
-           (1, 128, 1, 256, 1)]
+           (1, 128, 1, 256, 1), (2, 224, 0, 64, 0), (2, 224, 0, 128, 0), (2, 224, 0, 256, 0)]
 
 
 def timeit(fn, reps=3, batch_ms=60.0):
@@ -168,7 +168,8 @@ def main():
         print("rebuilt", OUT, len(doc["entries"]), "entries")
         return
     quick = "--quick" in sys.argv
-    Ms = [128, 256, 1024, 4096, 8192, 65536] if not quick else [128, 1024, 8192]
+    # 2048: the per-rank rows of the 4-GPU row-sharded 8192^3 bench (1024: 8 GPUs)
+    Ms = [128, 256, 1024, 2048, 4096, 8192, 65536] if not quick else [128, 1024, 8192]
     Ns = [256, 1024, 8192] if not quick else [256, 8192]
     Ks = [256, 1024, 2048, 4096, 8192] if not quick else [1024, 8192]
     log = []
