@@ -209,6 +209,9 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--n", type=int, default=8192)
+    ap.add_argument("--as-rank-of", type=int, default=1,
+                    help="diagnostics: on one GPU, time rank 0's share of a world of this size "
+                         "(M / W rows); value and n_gpus then describe that one rank")
     ap.add_argument("--no-apps", action="store_true", help="skip the kNN / kMeans objects")
     ap.add_argument("--no-cpu", action="store_true", help="skip the cpu_baseline oracle timing")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
@@ -229,7 +232,11 @@ def main():
     dev = torch.device("cuda", torch.cuda.current_device())
     n = args.n
     M, N, K = n, n, n
-    r0, r1 = edist.shard_bounds(M, world, rank, align=256)
+    if world == 1 and args.as_rank_of > 1:  # diagnostics only (see --as-rank-of)
+        r0, r1 = edist.shard_bounds(M, args.as_rank_of, 0, align=256)
+        M = r1 - r0
+    else:
+        r0, r1 = edist.shard_bounds(M, world, rank, align=256)
     m_loc = r1 - r0
     # ---- inputs: A rows of this rank, B broadcast once from rank 0 (outside timing)
     A_host = inputs.uniform((M, K), 101)[r0:r1]
@@ -246,21 +253,30 @@ def main():
     # The tuning table decides whether A's round-split runs inside the GEMM (converter
     # warpgroup, a-2 fused mode) or as a separate egemm_split pass; B^T is split by
     # egemm_split either way.
-    fused_a = bool(egemm.query_config("gemm", m_loc, N, K, with_fused=True)[4])
-    launches_per_step = 2 if fused_a else 3
+    # B arrives as fp32 every step: the table's fp32-B rows decide whether B^T is split by a
+    # separate egemm_split pass or inside the GEMM (fused-B converters, e.g. the short per-rank
+    # row blocks of 4 / 8 GPUs); else whether A is split inside the GEMM.
+    fused_b = egemm.query_config("gemm_b32", m_loc, N, K, with_fused=True)[4] == 2
+    fused_a = not fused_b and bool(egemm.query_config("gemm", m_loc, N, K, with_fused=True)[4] & 1)
+    launches_per_step = 2 if (fused_a or fused_b) else 3
     ws_a = torch.empty(egemm.gemm_workspace_size(m_loc, N, K, False, True), dtype=torch.uint8,
                        device=dev)
     ws_p = torch.empty(egemm.gemm_workspace_size(m_loc, N, K, True, True), dtype=torch.uint8,
                        device=dev)  # the k-pacing counters only (256 B)
+    ws_b = torch.empty(egemm.gemm_workspace_size(m_loc, N, K, True, False), dtype=torch.uint8,
+                       device=dev) if fused_b else None
 
     def pre():  # the splits outside the GEMM kernel
         if not fused_a:
             egemm.split(A, out=a_split)
-        egemm.split(B, transpose=True, out=b_split)
+        if not fused_b:
+            egemm.split(B, transpose=True, out=b_split)
 
     def gemm_call():
         if fused_a:
             egemm.gemm(A, None, b_split=b_split, out=D, workspace=ws_a)
+        elif fused_b:
+            egemm.gemm(None, B, a_split=a_split, out=D, workspace=ws_b)
         else:
             egemm.gemm(None, None, a_split=a_split, b_split=b_split, out=D, workspace=ws_p)
 
@@ -310,7 +326,8 @@ def main():
     peak = peaks.get("bf16_tflops_sustained", 1409.0)
     roofline = {
         "kernel": "egemm_tc_kernel cfg=%s%s (tcgen05)" % (
-            egemm.query_config("gemm", m_loc, N, K), " + fused A split" if fused_a else ""),
+            egemm.query_config("gemm_b32" if fused_b else "gemm", m_loc, N, K),
+            " + fused A split" if fused_a else " + fused B split" if fused_b else ""),
         "bound": "tensor", "achieved": round(achieved, 1), "peak": peak, "unit": "TFLOP/s",
         "frac": round(achieved / peak, 4),
         "peak_kind": "measured fp16/bf16 dense, sustained (MEASURED_PEAKS.json bf16_tflops_sustained)",
@@ -330,8 +347,9 @@ def main():
         "cycle_efficiency": round(tensor_flop / (148 * 8192.0) / kernel_cycles, 4)
         if kernel_cycles else None,
     }
-    split_bytes = 8.0 * ((0 if fused_a else m_loc * K) + K * N)
-    split_rl = {"kernel": "split (B^T)" if fused_a else "split (A rows + B^T)", "bound": "hbm",
+    split_bytes = 8.0 * ((0 if fused_a else m_loc * K) + (0 if fused_b else K * N))
+    split_rl = {"kernel": "split (B^T)" if fused_a else "split (A rows)" if fused_b else "split (A rows + B^T)",
+                "bound": "hbm",
                 "achieved": round(split_bytes / (split_ms * 1e-3) / 1e9, 1),
                 "peak": peaks.get("hbm_gbs", 6454.0), "unit": "GB/s",
                 "frac": round(split_bytes / (split_ms * 1e-3) / 1e9 / peaks.get("hbm_gbs", 6454.0), 4),
@@ -426,6 +444,7 @@ def main():
             "data": "synthetic U[-1,1] fp32, seeded PCG64 (inputs > L2, no flush needed)",
             "config": {"workload": "egemm %d^3 (BASELINE configs[1]), row-sharded C" % n,
                        "M": M, "N": N, "K": K, "terms": terms, "rows_per_rank": m_loc,
+                       **({"as_rank_of": args.as_rank_of} if args.as_rank_of > 1 and world == 1 else {}),
                        "l2": "every operand 256 MiB > 126 MB L2",
                        "parallelism": "dp%d rows" % world},
             "gpu_launches": launches_per_step * args.steps,

@@ -178,9 +178,11 @@ int egemm_set_config(int cg, int bn, int sep, int kc);
  * Sec. 6): path of the loaded tune_table.json ("" = built-in defaults) and,
  * through *entries (nullable), its number of entries.  Host-only. */
 const char* egemm_tune_table(int* entries);
-/* The configuration the library would use for op (0 gemm, 1 knn, 2 kmeans) at M, N, K
- * (after table, egemm_set_config and EGEMM_* overrides).  *fused_a (nullable) = 1 when an
- * fp32 row-major A would be round-split inside the GEMM kernel (a-2 fused mode). */
+/* The configuration the library would use for op (0 gemm with a pre-split B, 1 knn,
+ * 2 kmeans, 3 gemm whose B is fp32 K x N row-major, i.e. its round-split is part of the
+ * call) at M, N, K (after table, egemm_set_config and EGEMM_* overrides).  *fused_a
+ * (nullable): 1 when an fp32 row-major A would be round-split inside the GEMM kernel, 2 when
+ * (op 3) the fp32 B would be round-split inside the GEMM kernel (a-2 fused modes), else 0. */
 int egemm_query_config(int op, int64_t M, int64_t N, int64_t K, int* cg, int* bn, int* sep,
                        int* kc, int* fused_a);
 

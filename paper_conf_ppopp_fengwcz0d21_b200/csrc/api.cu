@@ -57,7 +57,12 @@ static bool valid_config(int cg, int bn, int sep) {
          (cg == 2 && bn == 128 && sep == 1) || (cg == 2 && bn == 224 && sep == 0);
 }
 
-static TcConfig choose_config(int epi_kind, int64_t M, int64_t N, int64_t K, int terms) {
+static bool fused_b_supported(const TcConfig& c) { return c.cg == 2 && c.bn == 256 && !c.sep; }
+
+// b_f32: a STORE GEMM whose B is fp32 (split inside the call): the table's "gemm_b32" rows
+// (which may pick the fused-B kernel) first, then the "gemm" rows.
+static TcConfig choose_config(int epi_kind, int64_t M, int64_t N, int64_t K, int terms,
+                              bool b_f32 = false) {
   TcConfig c = {};
   c.terms = terms;
   c.max_clusters = 0;
@@ -71,7 +76,10 @@ static TcConfig choose_config(int epi_kind, int64_t M, int64_t N, int64_t K, int
   if (epi_kind == EPI_STORE && M <= 128) { c.cg = 1; c.bn = 128; c.sep = 1; }
   {  // the measured table (tools/tune_sweep.py -> tune_table.json) overrides the defaults
     int cg, bn, sep, kc, fa;
-    if (tune_lookup(epi_kind, M, N, K, &cg, &bn, &sep, &kc, &fa) && valid_config(cg, bn, sep)) {
+    bool hit = epi_kind == EPI_STORE && b_f32 &&
+               tune_lookup(kOpGemmB32, M, N, K, &cg, &bn, &sep, &kc, &fa) && valid_config(cg, bn, sep);
+    if (!hit) hit = tune_lookup(epi_kind, M, N, K, &cg, &bn, &sep, &kc, &fa) && valid_config(cg, bn, sep);
+    if (hit) {
       c.cg = cg;
       c.bn = bn;
       c.sep = sep;
@@ -200,13 +208,18 @@ const char* egemm_tune_table(int* entries) {
 
 int egemm_query_config(int op, int64_t M, int64_t N, int64_t K, int* cg, int* bn, int* sep,
                        int* kc, int* fused_a) {
-  if (op < 0 || op > 2 || !cg || !bn || !sep || !kc) return EGEMM_ERR_INVALID_ARG;
-  TcConfig c = choose_config(op, M, N, K, 3);
+  if (op < 0 || op > 3 || !cg || !bn || !sep || !kc) return EGEMM_ERR_INVALID_ARG;
+  const bool b32 = op == kOpGemmB32;
+  TcConfig c = choose_config(b32 ? EPI_STORE : op, M, N, K, 3, b32);
   *cg = c.cg;
   *bn = c.bn;
   *sep = c.sep;
   *kc = c.kc;
-  if (fused_a) *fused_a = (op == EPI_STORE && c.fa && fused_a_supported(c)) ? 1 : 0;
+  if (fused_a) {
+    const bool store = op == EPI_STORE || b32;
+    const int a = (store && (c.fa & 1) && fused_a_supported(c)) ? 1 : 0;
+    *fused_a = a ? 1 : (b32 && (c.fa & 2) && fused_b_supported(c)) ? 2 : 0;
+  }
   return EGEMM_OK;
 }
 
@@ -352,9 +365,13 @@ int egemm_gemm(int64_t M, int64_t N, int64_t K, egemm_operand_t A, egemm_operand
   }
   Carver cv{reinterpret_cast<char*>(workspace)};
   TcOperands ops = {};
-  TcConfig cfg = choose_config(EPI_STORE, M, N, K, terms);
-  // fp32 row-major A can be round-split inside the GEMM (converter warps, a-2 fused mode)
-  const bool fuse_a = cfg.fa && !A.hi && !A.trans && fused_a_supported(cfg);
+  TcConfig cfg = choose_config(EPI_STORE, M, N, K, terms, B.f32 && !B.hi && !B.trans);
+  // fp32 row-major A (fa bit 0) or fp32 K x N row-major B (fa bit 1) can be round-split
+  // inside the GEMM (converter warps, a-2 fused mode); B needs 16-B aligned rows (TMA)
+  const bool fuse_a = (cfg.fa & 1) && !A.hi && !A.trans && fused_a_supported(cfg);
+  const bool fuse_b = !fuse_a && (cfg.fa & 2) && !B.hi && B.f32 && !B.trans &&
+                      fused_b_supported(cfg) && (B.ld % 4) == 0 &&
+                      (reinterpret_cast<uintptr_t>(B.f32) % 16) == 0;
   if (fuse_a) {
     ops.a_f32 = A.f32;
     ops.lda_f32 = A.ld;
@@ -366,7 +383,14 @@ int egemm_gemm(int64_t M, int64_t N, int64_t K, egemm_operand_t A, egemm_operand
   // B logical K x N: as an operand it is N rows x K; f32 trans==0 means stored K x N.
   egemm_operand_t Bt = B;
   Bt.trans = !B.trans;
-  if ((r = stage_operand(Bt, N, K, cv, &ops.b_hi, &ops.b_lo, &ops.ldb, s))) return r;
+  if (fuse_b) {
+    ops.b_f32 = B.f32;
+    ops.ldb_f32 = B.ld;
+    cv.take<uint16_t>((size_t)(N * ldk_of(K)));  // keep the workspace layout unchanged
+    cv.take<uint16_t>((size_t)(N * ldk_of(K)));
+  } else if ((r = stage_operand(Bt, N, K, cv, &ops.b_hi, &ops.b_lo, &ops.ldb, s))) {
+    return r;
+  }
   TcEpilogue epi = {};
   epi.kind = EPI_STORE;
   epi.D = D;

@@ -14,6 +14,9 @@ int launch_split(const float* x, int64_t rows, int64_t cols, int64_t ldx, uint16
 
 // Epilogue policies of the tensor-core kernel.
 enum EpiKind : int { EPI_STORE = 0, EPI_KNN = 1, EPI_KMEANS = 2 };
+// tuning-table op of a GEMM whose B arrives as fp32 (its round-split is part of the call,
+// so the table may pick the fused-B kernel); a STORE launch
+constexpr int kOpGemmB32 = 3;
 
 // Operands of one launch of the tcgen05 kernel.  hi/lo are fp16 bit patterns, K-major:
 // A is rows_a x K (row stride lda elements), B is rows_b x K (row stride ldb).
@@ -27,6 +30,9 @@ struct TcOperands {
   // fused A split: fp32 A (rows_a x K, row stride lda_f32); a_hi / a_lo then unused
   const float* a_f32;
   int64_t lda_f32;
+  // fused B split: fp32 B stored K x N row-major (row stride ldb_f32); b_hi / b_lo unused
+  const float* b_f32;
+  int64_t ldb_f32;
 };
 
 struct TcConfig {
@@ -36,7 +42,7 @@ struct TcConfig {
   int kc;        // promotion interval in k elements (multiple of 64)
   int terms;     // 3 or 4
   int max_clusters;  // 0 = all SMs
-  int fa;        // fused A split allowed (fp32 A converted by in-kernel converter warps)
+  int fa;        // fused splits allowed, bit mask: 1 = A, 2 = B (in-kernel converter warps)
 };
 
 struct TcEpilogue {

@@ -85,6 +85,7 @@ struct KParams {
   uint32_t* sync;    // nullable: kSyncR epoch counters (zeroed per launch) for the k-pacing
   int pace_e, pace_s;  // k-blocks per epoch, slack in epochs
   int band_m;          // STORE tile order: m-tiles per band
+  int fb;            // fused B split (host-side dispatch flag; tm_bhi maps the fp32 B)
   int debug_mode;    // EGEMM_DEBUG_MODE bits (diagnostics): 1 extra commit per k-block;
                      // with NO_TMA: 2 MMA warp ignores the full barriers (producer idle),
                      // 4 no per-k-block commits
@@ -232,14 +233,17 @@ __device__ __forceinline__ void tf32_parts(float y, float& h, float& m, float& l
   l = __fsub_rn(r, m);
 }
 
-template <int CG, int BN, bool SEP, int EPI, int STAGES, int NEPI, bool FA, bool AR, bool AS>
-__global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
+template <int CG, int BN, bool SEP, int EPI, int STAGES, int NEPI, bool FA, bool AR, bool AS, bool FB>
+__global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
     egemm_tc_kernel(const __grid_constant__ CUtensorMap tm_ahi,
                     const __grid_constant__ CUtensorMap tm_alo,
                     const __grid_constant__ CUtensorMap tm_bhi,
                     const __grid_constant__ CUtensorMap tm_blo, const KParams p) {
   using G = Geo<CG, BN>;
-  using EG = EpiGeo<NEPI, FA>;
+  // FB (fused B split): the converter warpgroup builds B_hi / B_lo from TMA-staged fp32 B
+  // tiles (row-major K x N, transposed to K-major on the way) while A comes pre-split by TMA
+  constexpr bool CONV = FA || FB;
+  using EG = EpiGeo<NEPI, CONV>;
   constexpr int GPQ = EG::GPQ;
   constexpr int COLS = BN / GPQ;  // columns per epilogue warp
   constexpr int NACC = SEP ? 4 : 2;
@@ -274,9 +278,11 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
   // AS (fused A, TMA-staged): the fp32 A tiles land in their own ring (NSTG x 128 rows x 64
   // fp32, two 128-B-swizzled boxes of 32 columns), loaded ahead by warp 7; the converters
   // split from smem instead of waiting on their own global loads.
-  constexpr int NSTG = AS ? 3 : 0;
+  constexpr int NSTG = (AS || FB) ? 3 : 0;
   constexpr int STG_BYTES = kBM * kBK * 4;
   static_assert(!AS || FA, "AS is a fused-A mode");
+  static_assert(!(FA && FB), "one fused operand at a time");
+  static_assert(!FB || (CG == 2 && BN == 256 && EPI == EPI_STORE && !SEP), "FB: 256 x 256 pair tiles");
   uint8_t* stage_base = smem;
   uint8_t* a_res = smem + STAGES * SB;
   uint8_t* a_stg = a_res + AR_BYTES;
@@ -302,7 +308,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
 
   if (warp == EG::W_PROD && lane == 0) {
     if (!FA || p.a_pf) ptx::prefetch_tmap(&tm_ahi);  // FA: tm_ahi maps the fp32 A (L2 prefetch)
-    if (!FA) ptx::prefetch_tmap(&tm_alo);
+    if (!FA) ptx::prefetch_tmap(&tm_alo);  // (FB: tm_bhi maps the fp32 B, tm_blo a copy)
     ptx::prefetch_tmap(&tm_bhi);
     ptx::prefetch_tmap(&tm_blo);
   }
@@ -310,7 +316,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
     for (int s = 0; s < STAGES; s++) {
       // FA: the producer's expect_tx arrive plus one arrive per converter warp of the pair;
       // NORM: plus one arrive per norm warp of the pair
-      ptx::mbar_init(&full[s], 1 + (FA ? 4 * CG : 0) + (NORM ? CG : 0));
+      ptx::mbar_init(&full[s], 1 + (CONV ? 4 * CG : 0) + (NORM ? CG : 0));
       ptx::mbar_init(&empty[s], 1);
     }
     for (int b = 0; b < 2; b++) {
@@ -372,8 +378,55 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
   // FA register budget per warpgroup (512 threads share 64K registers): converters 96,
   // producer / MMA / allocator 56, the two epilogue warpgroups 176 (running totals).  Each
   // setmaxnreg sits at the top of its warpgroup's branch so it dominates that role's code.
-  if (FA && warp < 4) {
-    if constexpr (FA) asm volatile("setmaxnreg.dec.sync.aligned.u32 96;");
+  if (CONV && warp < 4) {
+    if constexpr (CONV) asm volatile("setmaxnreg.dec.sync.aligned.u32 96;");
+    if constexpr (FB) {
+      // ================= fused round-split of B (converter warpgroup) =================
+      // Alg. 1 l.3 for B inside the GEMM.  The fp32 tile of this CTA's 128
+      // B columns x 64 k (4 TMA boxes of 32 columns, 128-B swizzled rows of k) sits in the
+      // staging ring; thread t takes column n = t, reads its 8 k-chunks down the rows
+      // (a warp reads one 128-B row per instruction: conflict-free), splits them and stores
+      // 16-B hi / lo chunks into row n of the K-major 128-B-swizzled B stage.
+      int stage = 0;
+      uint32_t phase = 0;
+      int si = 0;
+      uint32_t sph = 0;
+      const int n = threadIdx.x;  // 0 .. 127
+      const int cn = (n & 31) >> 2;
+      const uint32_t colx = (uint32_t)((n >> 5) * (STG_BYTES / 4) + (n & 3) * 4);
+      for (int u = cluster; u < p.num_units; u += nclusters) {
+        UnitInfo ui = decode_unit<EPI>(p, u);
+        for (int ns = 0; ns < ui.n_count; ns++) {
+          for (int kb = 0; kb < p.num_kb; kb++) {
+            ptx::mbar_wait(&sfull[si], sph);
+            ptx::mbar_wait(&empty[stage], phase ^ 1u);
+            const uint32_t sb = ptx::smem_u32(stage_base + stage * G::STAGE_BYTES) + 2 * G::A_BYTES;
+            const uint32_t xb = ptx::smem_u32(a_stg + si * STG_BYTES) + colx;
+#pragma unroll
+            for (int c = 0; c < kBK / 8; c++) {
+              float x[8];
+#pragma unroll
+              for (int i = 0; i < 8; i++)  // k = 8c + i: row k, chunk cn at position cn ^ i
+                x[i] = ptx::lds32f(xb + (c * 8 + i) * 128 + ((cn ^ i) << 4));
+              uint32_t hi[4], lo[4];
+#pragma unroll
+              for (int e = 0; e < 4; e++) ptx::split2(x[2 * e], x[2 * e + 1], hi[e], lo[e]);
+              const uint32_t off = (uint32_t)(n * 128 + ((c ^ (n & 7)) << 4));
+              ptx::sts128(sb + off, hi[0], hi[1], hi[2], hi[3]);
+              ptx::sts128(sb + G::B_BYTES + off, lo[0], lo[1], lo[2], lo[3]);
+            }
+            ptx::fence_proxy_async_smem();  // generic-proxy stores -> visible to tcgen05.mma
+            __syncwarp();
+            if (lane == 0) {
+              ptx::mbar_arrive_cluster(&full[stage], 0);
+              ptx::mbar_arrive(&sempty[si]);
+            }
+            if (++stage == STAGES) { stage = 0; phase ^= 1u; }
+            if (++si == NSTG) { si = 0; sph ^= 1u; }
+          }
+        }
+      }
+    }
     // ================= fused round-split of A (converter warpgroup) =================
     // Alg. 1 l.2 inside the GEMM: each thread loads 8 consecutive fp32 of one
     // A row (2 x 16 B), splits them (cvt.rn) and stores the 16 B hi / lo chunks straight
@@ -468,7 +521,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
       }
     }
   } else if (warp < EG::EPI0) {
-   if constexpr (FA || KREG) asm volatile("setmaxnreg.dec.sync.aligned.u32 56;");
+   if constexpr (CONV || KREG) asm volatile("setmaxnreg.dec.sync.aligned.u32 56;");
    if (warp == EG::W_PROD) {
     // ============================ TMA producer ============================
     if (lane == 0) {
@@ -476,7 +529,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
       uint32_t phase = 0;
       // FA: only B comes through TMA (A is written by the converter warps); AR: the ring
       // carries only B, A is loaded once per unit into a_res
-      constexpr uint32_t TX = (FA || AR) ? 2 * G::B_BYTES : G::STAGE_BYTES;
+      constexpr uint32_t TX = (FA || AR) ? 2 * G::B_BYTES : FB ? 2 * G::A_BYTES : G::STAGE_BYTES;
       uint32_t uctr = 0;
       bool pace = (EPI == EPI_STORE) && p.sync != nullptr && !p.debug_no_tma;
       uint32_t gkb = 0;  // k-blocks this CTA has started loading, over all its units
@@ -519,7 +572,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
             ptx::mbar_wait(&empty[stage], phase ^ 1u);
             uint8_t* sb = stage_base + stage * SB;
             if (p.debug_no_tma) {  // diagnostics only: MMA-issue ceiling without operand traffic
-              if (leader && !FA) ptx::mbar_arrive(&full[stage]);
+              if (leader && !CONV) ptx::mbar_arrive(&full[stage]);
               if (++stage == STAGES) { stage = 0; phase ^= 1u; }
               continue;
             }
@@ -530,15 +583,19 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
                 ptx::tma_load_2d(&tm_ahi, &full[stage], sb, k0, arow);
                 ptx::tma_load_2d(&tm_alo, &full[stage], sb + G::A_BYTES, k0, arow);
               }
-              ptx::tma_load_2d(&tm_bhi, &full[stage], sb + B_OFF, k0, brow);
-              ptx::tma_load_2d(&tm_blo, &full[stage], sb + B_OFF + G::B_BYTES, k0, brow);
+              if (!FB) {
+                ptx::tma_load_2d(&tm_bhi, &full[stage], sb + B_OFF, k0, brow);
+                ptx::tma_load_2d(&tm_blo, &full[stage], sb + B_OFF + G::B_BYTES, k0, brow);
+              }
             } else {
               if (!FA && !AR) {
                 ptx::tma_load_2d_pair(&tm_ahi, &full[stage], sb, k0, arow);
                 ptx::tma_load_2d_pair(&tm_alo, &full[stage], sb + G::A_BYTES, k0, arow);
               }
-              ptx::tma_load_2d_pair(&tm_bhi, &full[stage], sb + B_OFF, k0, brow);
-              ptx::tma_load_2d_pair(&tm_blo, &full[stage], sb + B_OFF + G::B_BYTES, k0, brow);
+              if (!FB) {
+                ptx::tma_load_2d_pair(&tm_bhi, &full[stage], sb + B_OFF, k0, brow);
+                ptx::tma_load_2d_pair(&tm_blo, &full[stage], sb + B_OFF + G::B_BYTES, k0, brow);
+              }
             }
             if (++stage == STAGES) { stage = 0; phase ^= 1u; }
           }
@@ -549,6 +606,29 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
         const uint32_t pe = (uint32_t)p.pace_e;
         const uint32_t total = (per_cta + pe - 1) / pe;
         for (uint32_t e = (gkb + pe - 1) / pe; e < total; e++) sync_arrive(p.sync, e);
+      }
+    }
+  } else if (FB && warp == 7) {
+    // ==================== fp32 B staging producer (fused B) ====================
+    if constexpr (FB) {
+      if (lane == 0) {
+        int si = 0;
+        uint32_t sph = 0;
+        for (int u = cluster; u < p.num_units; u += nclusters) {
+          UnitInfo ui = decode_unit<EPI>(p, u);
+          for (int ns = 0; ns < ui.n_count; ns++) {
+            const int n0 = (ui.n_begin + ns) * BN + (int)rank * G::BNC;
+            for (int kb = 0; kb < p.num_kb; kb++) {
+              ptx::mbar_wait(&sempty[si], sph ^ 1u);
+              ptx::mbar_arrive_expect_tx(&sfull[si], STG_BYTES);
+              uint8_t* dst = a_stg + si * STG_BYTES;
+#pragma unroll
+              for (int j = 0; j < G::BNC / 32; j++)
+                ptx::tma_load_2d(&tm_bhi, &sfull[si], dst + j * (STG_BYTES / 4), n0 + 32 * j, kb * kBK);
+              if (++si == NSTG) { si = 0; sph ^= 1u; }
+            }
+          }
+        }
       }
     }
   } else if (AS && warp == 7) {
@@ -729,7 +809,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA>::THREADS, 1)
     }
    }
   } else {
-    if constexpr (FA) asm volatile("setmaxnreg.inc.sync.aligned.u32 176;");
+    if constexpr (CONV) asm volatile("setmaxnreg.inc.sync.aligned.u32 176;");
     if constexpr (KREG) asm volatile("setmaxnreg.inc.sync.aligned.u32 216;");
     // ============================ epilogue ============================
     const int ew = warp - EG::EPI0;
@@ -1163,7 +1243,7 @@ static bool make_tmap_f32(CUtensorMap* m, const void* base, int64_t rows, int64_
 }
 
 template <int CG, int BN, bool SEP, int EPI, int STAGES, bool FA = false, bool AR = false,
-          bool AS = false>
+          bool AS = false, bool FB = false>
 static int launch_variant(const CUtensorMap* maps, const KParams& kp, int max_clusters,
                           cudaStream_t stream) {
   using G = Geo<CG, BN>;
@@ -1171,7 +1251,7 @@ static int launch_variant(const CUtensorMap* maps, const KParams& kp, int max_cl
   // kNN keeps 8 (with 16 each thread's list sees half the columns, twice the insertions:
   // measured 3-15 % slower even without spills after the norm MMA freed 32 registers)
   constexpr int NEPI = (EPI == EPI_KMEANS) ? 16 : 8;
-  auto kern = egemm_tc_kernel<CG, BN, SEP, EPI, STAGES, NEPI, FA, AR, AS>;
+  auto kern = egemm_tc_kernel<CG, BN, SEP, EPI, STAGES, NEPI, FA, AR, AS, FB>;
   // kNN: top-k merge lists (half a list per round); kMeans: (key, index) of 3 column groups
   // (+ kNN KREG: two generations x two column groups x 128 rows of 16-key lists)
   constexpr bool KREG = (EPI == EPI_KNN) && AR && !FA && NEPI == 8 && BN / (NEPI / 4) == 128;
@@ -1180,7 +1260,7 @@ static int launch_variant(const CUtensorMap* maps, const KParams& kp, int max_cl
   constexpr bool NORM = (EPI != EPI_STORE);  // norm slot per stage + the A' ones tile
   const size_t sb = (AR ? 2 * G::B_BYTES : G::STAGE_BYTES) + (NORM ? G::BNC * 32 : 0);
   const size_t smem = 1024 + (size_t)STAGES * sb + (AR ? 4 * G::A_BYTES : 0) +
-                      (NORM ? kBM * 32 : 0) + (AS ? 3 * kBM * kBK * 4 + 8 * 6 : 0) +
+                      (NORM ? kBM * 32 : 0) + ((AS || FB) ? 3 * kBM * kBK * 4 + 8 * 6 : 0) +
                       8 * (2 * STAGES + 8) + scratch;
   static bool attr_done = false;  // per instantiation
   if (!attr_done) {
@@ -1198,7 +1278,7 @@ static int launch_variant(const CUtensorMap* maps, const KParams& kp, int max_cl
   if (clusters < 1) clusters = 1;
   cudaLaunchConfig_t cfg = {};
   cfg.gridDim = dim3((unsigned)(clusters * CG), 1, 1);
-  cfg.blockDim = dim3(EpiGeo<NEPI, FA>::THREADS, 1, 1);
+  cfg.blockDim = dim3(EpiGeo<NEPI, FA || FB>::THREADS, 1, 1);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = stream;
   cudaLaunchAttribute attr[1];
@@ -1225,6 +1305,12 @@ template <int EPI>
 static int dispatch(const CUtensorMap* maps, const KParams& kp, const TcConfig& cfg,
                     cudaStream_t s) {
   if constexpr (EPI == EPI_STORE) {
+    if (kp.fb) {  // fused B split: TMA-staged fp32 B (2 MMA stages + 3 fp32 staging slots)
+      if (cfg.cg == 2 && cfg.bn == 256 && !cfg.sep)
+        return launch_variant<2, 256, false, EPI, 2, false, false, false, true>(maps, kp, cfg.max_clusters, s);
+      set_last_error("fused B split: unsupported tile config cg=%d bn=%d sep=%d", cfg.cg, cfg.bn, cfg.sep);
+      return 2;
+    }
     if (kp.a_f32) {  // fused A split (converter warpgroup)
       // aligned fp32 A: TMA-staged (2 MMA stages + 3 fp32 staging slots); else LDG converters
       if (cfg.cg == 2 && cfg.bn == 256 && !cfg.sep && kp.a_staged)
@@ -1277,10 +1363,12 @@ int launch_tc(int64_t M, int64_t N, int64_t K, const TcOperands& ops, const TcCo
   CUtensorMap maps[4];
   const int bnc = cfg.bn / cfg.cg;
   const bool fa = ops.a_f32 != nullptr && epi.kind == EPI_STORE;
+  const bool fb = ops.b_f32 != nullptr && epi.kind == EPI_STORE && !fa;
   if ((!fa && (!make_tmap_f16(&maps[0], ops.a_hi, M, K, ops.lda, kBM) ||
                !make_tmap_f16(&maps[1], ops.a_lo, M, K, ops.lda, kBM))) ||
-      !make_tmap_f16(&maps[2], ops.b_hi, N, K, ops.ldb, bnc) ||
-      !make_tmap_f16(&maps[3], ops.b_lo, N, K, ops.ldb, bnc)) {
+      (!fb && (!make_tmap_f16(&maps[2], ops.b_hi, N, K, ops.ldb, bnc) ||
+               !make_tmap_f16(&maps[3], ops.b_lo, N, K, ops.ldb, bnc))) ||
+      (fb && !make_tmap_f32(&maps[2], ops.b_f32, K, N, ops.ldb_f32, kBK, 32, true))) {
     set_last_error("cuTensorMapEncodeTiled failed (alignment: base 16 B, ld %% 8 == 0)");
     return 2;
   }
@@ -1288,8 +1376,10 @@ int launch_tc(int64_t M, int64_t N, int64_t K, const TcOperands& ops, const TcCo
     maps[0] = maps[2];
     maps[1] = maps[3];
   }
+  if (fb) maps[3] = maps[2];  // fp32 B (row-major K x N) in 32-column 128-B-swizzled boxes
   KParams kp = {};
   kp.K = (int)K;
+  kp.fb = fb ? 1 : 0;
   {
     const char* dbg = getenv("EGEMM_DEBUG_NO_TMA");
     kp.debug_no_tma = (dbg && dbg[0] == '1') ? 1 : 0;

@@ -99,7 +99,8 @@ static bool parse_entry(const char*& p, TuneEntry* e) {
     if (key == "op") {
       std::string v;
       if (!parse_string(p, &v)) return false;
-      e->op = v == "gemm" ? EPI_STORE : v == "knn" ? EPI_KNN : v == "kmeans" ? EPI_KMEANS : -1;
+      e->op = v == "gemm" ? EPI_STORE : v == "knn" ? EPI_KNN : v == "kmeans" ? EPI_KMEANS
+              : v == "gemm_b32" ? kOpGemmB32 : -1;
     } else if (key == "m_max" || key == "n_max" || key == "k_max" || key == "cg" || key == "bn" ||
                key == "sep" || key == "kc" || key == "fa") {
       char* end = nullptr;

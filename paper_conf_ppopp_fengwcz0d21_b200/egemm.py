@@ -110,10 +110,11 @@ def tune_table():
 
 
 def query_config(op: str, M: int, N: int, K: int, with_fused: bool = False):
-    """The (cg, bn, sep, kc) the library picks for op in {'gemm','knn','kmeans'}
-    (+ fused_a flag when with_fused)."""
+    """The (cg, bn, sep, kc) the library picks for op in {'gemm' (pre-split B), 'knn',
+    'kmeans', 'gemm_b32' (fp32 B split inside the call)} (+ the fused-split flag when
+    with_fused: 1 = A, 2 = B round-split inside the GEMM kernel, 0 = none)."""
     v = [ctypes.c_int(0) for _ in range(5)]
-    _check(load().egemm_query_config({"gemm": 0, "knn": 1, "kmeans": 2}[op], M, N, K,
+    _check(load().egemm_query_config({"gemm": 0, "knn": 1, "kmeans": 2, "gemm_b32": 3}[op], M, N, K,
                                      *[ctypes.byref(x) for x in v]), "egemm_query_config")
     out = tuple(x.value for x in v)
     return out if with_fused else out[:4]

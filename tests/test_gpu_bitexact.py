@@ -16,9 +16,11 @@ CFGS = [(2, 256, 0, 64), (2, 256, 0, 128), (1, 128, 0, 64), (1, 128, 1, 128), (1
 
 
 def _gpu(eg, A, B, C, cfg, terms, fused):
+    """fused: 0 pre-split operands, 1 A split inside the GEMM, 2 B split inside the GEMM
+    (the library falls back to pre-split where the tile config has no such variant)."""
     eg.set_config(*cfg)
     import os
-    os.environ["EGEMM_FUSED_A"] = "1" if fused else "0"
+    os.environ["EGEMM_FUSED_A"] = str(int(fused))
     try:
         return to_host(eg.gemm(to_dev(A), to_dev(B), to_dev(C) if C is not None else None,
                                terms=terms))
@@ -45,7 +47,22 @@ def test_bitexact_terms4_with_c_and_fused(oracle_lib, cfg, gen):
     eg = require_gpu()
     A, B, C = gen((200, 700), 30), gen((700, 300), 31), inputs.uniform((200, 300), 32)
     for terms in (3, 4):
-        for fused in (False, True):
+        for fused in (0, 1, 2):
             D = _gpu(eg, A, B, C, cfg, terms, fused)
             ref = oracle_lib.gemm_alg1_tc(A, B, C, terms=terms, sep=cfg[2], kc=cfg[3])
             assert np.array_equal(D.view(np.uint32), ref.view(np.uint32)), (terms, fused)
+
+
+@pytest.mark.parametrize("shape", [(256, 256, 256), (300, 300, 1000), (129, 260, 65), (512, 1024, 2048),
+                                   (1000, 516, 4100)])
+@pytest.mark.parametrize("kc", [64, 256])
+def test_bitexact_fused_b(oracle_lib, shape, kc):
+    """B round-split inside the GEMM (converter warpgroup transposing TMA-staged fp32 B
+    tiles into the K-major stage) == the model bitwise, ragged N / K included."""
+    eg = require_gpu()
+    M, N, K = shape
+    A, B = inputs.uniform((M, K), 40 + K), inputs.uniform((K, N), 41 + N)
+    D = _gpu(eg, A, B, None, (2, 256, 0, kc), 3, 2)
+    ref = oracle_lib.gemm_alg1_tc(A, B, terms=3, sep=0, kc=kc)
+    assert np.array_equal(D.view(np.uint32), ref.view(np.uint32)), \
+        "mismatches: %d" % int((D != ref).sum())

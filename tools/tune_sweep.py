@@ -142,7 +142,68 @@ def build_table(log, Ms, Ns, Ks, extra=None, keep=None, margin=0.0):
     return doc
 
 
+B32_RULE = ("op gemm_b32 (B arrives as fp32: its round-split is part of the call): the fastest of "
+            "the gemm row's pick (B split by egemm_split) and the fused-B kernels (2, 256, 0, Kc, "
+            "fa=2) under the same accuracy rule")
+
+
+def b32_sweep(Ms, Ns, Ks):
+    """Buckets of the fp32-B user call gemm(A, B): the library's op-0 pick (separate B^T
+    split inside the call) against the fused-B kernel at Kc 64 / 128 / 256."""
+    log = []
+    for M in Ms:
+        for N in Ns:
+            for K in Ks:
+                if M > 8192 and N > 1024:
+                    continue
+                pick = list(egemm.query_config("gemm", M, N, K, with_fused=True))
+                cfgs = [tuple(pick)] + [(2, 256, 0, kc, 2) for kc in (64, 128, 256)]
+                A, B = inputs.uniform((M, K), 11 + M), inputs.uniform((K, N), 13 + N)
+                Ad, Bd = torch.from_numpy(A).cuda(), torch.from_numpy(B).cuda()
+                D = torch.empty((M, N), device="cuda")
+                rs = np.sort(inputs.rng(M + N + K).choice(M, size=min(64, M), replace=False))
+                C64 = oracle.gemm64(A[rs], B)
+                en = oracle.normwise_error(oracle.gemm32_naive(A[rs], B), A[rs], B, C64)
+                ws = torch.empty(egemm.gemm_workspace_size(M, N, K, False, False), dtype=torch.uint8,
+                                 device="cuda")
+                res = []
+                for cfg in cfgs:
+                    egemm.set_config(*cfg[:4])
+                    os.environ["EGEMM_FUSED_A"] = str(cfg[4])
+                    t = timeit(lambda: egemm.gemm(Ad, Bd, out=D, workspace=ws))
+                    e = oracle.normwise_error(D.cpu().numpy()[rs], A[rs], B, C64)
+                    res.append({"cfg": list(cfg), "ms": t, "err": e, "err_naive": en,
+                                "ok": bool(e <= 1e-6 and e <= 2 * en)})
+                egemm.set_config(0, 0, 0, 0)
+                os.environ.pop("EGEMM_FUSED_A", None)
+                best = select(res, k_scale(K, Ks))
+                log.append({"M": M, "N": N, "K": K, "results": res})
+                print("b32 M=%5d N=%5d K=%5d best=%s %s" % (M, N, K, best and best["cfg"],
+                      " ".join("%s:%.3fms%s" % (r["cfg"], r["ms"], "" if r["ok"] else "x") for r in res)),
+                      flush=True)
+                del Ad, Bd, D, ws
+    return log
+
+
 def main():
+    if "--b32" in sys.argv:  # add the fp32-B rows (op gemm_b32) to the current table
+        Ms, Ns, Ks = [128, 256, 1024, 2048, 4096, 8192, 65536], [256, 1024, 8192], [256, 1024, 2048, 4096, 8192]
+        if "--from-log" in sys.argv:
+            log = json.load(open(sys.argv[sys.argv.index("--from-log") + 1]))
+        else:
+            log = b32_sweep(Ms, Ns, Ks)
+            os.makedirs(os.path.join(ROOT, "gpurun_out"), exist_ok=True)
+            json.dump(log, open(os.path.join(ROOT, "gpurun_out", "tune_sweep_b32_log.json"), "w"), indent=1)
+        doc = build_table(log, Ms, Ns, Ks)
+        for e in doc["entries"]:
+            e["op"] = "gemm_b32"
+        table = json.load(open(OUT))
+        table["entries"] = [e for e in table["entries"] if e["op"] != "gemm_b32"] + doc["entries"]
+        table["rule_gemm_b32"] = B32_RULE
+        out = sys.argv[sys.argv.index("--out") + 1] if "--out" in sys.argv else OUT
+        json.dump(table, open(out, "w"), indent=1)
+        print("wrote", out, len(doc["entries"]), "gemm_b32 entries")
+        return
     if "--from-log" in sys.argv:  # re-derive the table from a committed sweep log
         log = json.load(open(sys.argv[sys.argv.index("--from-log") + 1]))
         Ms, Ns, Ks = (sorted({b[k] for b in log}) for k in ("M", "N", "K"))
