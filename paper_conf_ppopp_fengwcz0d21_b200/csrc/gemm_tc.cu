@@ -824,6 +824,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
     // KREG: the two column groups of a row exchange their sorted key lists once per tile
     // (double-buffered smem slots after the merge scratch, named barrier 5 + q)
     uint32_t xgen = 0;
+    uint32_t km_units = 0;  // kMeans: units finished (merge-slot parity)
     float* const xch = reinterpret_cast<float*>(scratch + kBM * kKnnMax * 4);
     float best = __int_as_float(0xff800000);
     int besti = 0x7fffffff;
@@ -1132,9 +1133,14 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
         }
       } else if constexpr (EPI == EPI_KMEANS) {
         best = -2.f * best;  // the key (exact): ||c||^2 - 2 x.c
-        // merge the GPQ column groups of each row through smem
-        float* sk = reinterpret_cast<float*>(scratch);
-        int* si = reinterpret_cast<int*>(scratch + GPQ * kBM * 4);
+        // merge the GPQ column groups of each row through smem.  The slots alternate with the
+        // unit's parity, so only group 0 waits (one barrier per unit): a group writes the
+        // same slots again two units later, after the next unit's barrier, which group 0
+        // reaches only once it has read these.
+        uint8_t* slot = scratch + (km_units & 1u) * (2 * GPQ * kBM * 4);
+        km_units++;
+        float* sk = reinterpret_cast<float*>(slot);
+        int* si = reinterpret_cast<int*>(slot + GPQ * kBM * 4);
         const int r = q * 32 + lane;
         if (cgp > 0) { sk[(cgp - 1) * kBM + r] = best; si[(cgp - 1) * kBM + r] = besti; }
         named_bar_sync(1 + q, 32 * GPQ);
@@ -1148,7 +1154,6 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
           if (p.debug_no_epi || (p.debug_mode & 64)) besti = 0;  // diagnostics: keep the downstream kernels in bounds
           if (row < p.M) { p.assign[row] = besti; p.best_key[row] = best; }
         }
-        named_bar_sync(1 + q, 32 * GPQ);
       }
     }
   }
@@ -1256,7 +1261,7 @@ static int launch_variant(const CUtensorMap* maps, const KParams& kp, int max_cl
   // (+ kNN KREG: two generations x two column groups x 128 rows of 16-key lists)
   constexpr bool KREG = (EPI == EPI_KNN) && AR && !FA && NEPI == 8 && BN / (NEPI / 4) == 128;
   const int scratch = EPI == EPI_KNN ? kBM * kKnnMax * 4 + (KREG ? 2 * 2 * kBM * kKnnMax * 4 : 0)
-                      : EPI == EPI_KMEANS ? 2 * 4 * kBM * 4 : 0;
+                      : EPI == EPI_KMEANS ? 2 * 2 * 4 * kBM * 4 : 0;
   constexpr bool NORM = (EPI != EPI_STORE);  // norm slot per stage + the A' ones tile
   const size_t sb = (AR ? 2 * G::B_BYTES : G::STAGE_BYTES) + (NORM ? G::BNC * 32 : 0);
   const size_t smem = 1024 + (size_t)STAGES * sb + (AR ? 4 * G::A_BYTES : 0) +
