@@ -127,17 +127,29 @@ __global__ void __launch_bounds__(32 * W) km_scatter_kernel(
   const int64_t i0 = (int64_t)blockIdx.x * kKmBlockPts;
   const int64_t i1 = min(n, i0 + kKmBlockPts);
   constexpr int SUB = kKmBlockPts / W;
+  constexpr int B = 16;  // assignments held in registers per lane (the loads of a batch overlap)
   const int64_t s0 = i0 + (int64_t)w * SUB, s1 = min(i1, s0 + SUB);
   int32_t* mine = hw + (int64_t)w * kc;
-  for (int64_t c = s0; c < s1; c += 32) {
-    const int64_t i = c + lane;
-    const int a = i < s1 ? assign[i] : -1 - lane;
-    const uint32_t peers = __match_any_sync(0xffffffffu, a);
-    if (i < s1 && lane == __ffs(peers) - 1) mine[a] += __popc(peers);
+  for (int64_t cb = s0; cb < s1; cb += 32 * B) {
+    int av[B];
+#pragma unroll
+    for (int t = 0; t < B; t++) {
+      const int64_t i = cb + 32 * t + lane;
+      av[t] = i < s1 ? assign[i] : -1 - lane;
+    }
+#pragma unroll
+    for (int t = 0; t < B; t++) {
+      const int64_t i = cb + 32 * t + lane;
+      const uint32_t peers = __match_any_sync(0xffffffffu, av[t]);
+      if (i < s1 && lane == __ffs(peers) - 1) mine[av[t]] += __popc(peers);
+      __syncwarp();  // the next batch's leader of this centroid may be another lane
+    }
   }
   __syncthreads();
-  for (int64_t j = threadIdx.x; j < kc; j += blockDim.x) {  // exclusive prefix over warps
-    int32_t run = H[j * nb + blockIdx.x];
+  // exclusive prefix over warps, starting at the centroid's global offset plus the counts of
+  // the earlier blocks: hw then holds each warp's first output position per centroid
+  for (int64_t j = threadIdx.x; j < kc; j += blockDim.x) {
+    int32_t run = (int32_t)offsets[j] + H[j * nb + blockIdx.x];
 #pragma unroll
     for (int v = 0; v < W; v++) {
       const int32_t t = hw[(int64_t)v * kc + j];
@@ -146,16 +158,25 @@ __global__ void __launch_bounds__(32 * W) km_scatter_kernel(
     }
   }
   __syncthreads();
-  for (int64_t c = s0; c < s1; c += 32) {
-    const int64_t i = c + lane;
-    const bool valid = i < s1;
-    const int a = valid ? assign[i] : -1 - lane;
-    const uint32_t peers = __match_any_sync(0xffffffffu, a);
-    const int rank = __popc(peers & ((1u << lane) - 1u));
-    if (valid) order[offsets[a] + mine[a] + rank] = (int32_t)i;
-    __syncwarp();
-    if (valid && lane == __ffs(peers) - 1) mine[a] += __popc(peers);
-    __syncwarp();
+  for (int64_t cb = s0; cb < s1; cb += 32 * B) {
+    int av[B];
+#pragma unroll
+    for (int t = 0; t < B; t++) {
+      const int64_t i = cb + 32 * t + lane;
+      av[t] = i < s1 ? assign[i] : -1 - lane;
+    }
+#pragma unroll
+    for (int t = 0; t < B; t++) {
+      const int64_t i = cb + 32 * t + lane;
+      const bool valid = i < s1;
+      const int a = av[t];
+      const uint32_t peers = __match_any_sync(0xffffffffu, a);
+      const int rank = __popc(peers & ((1u << lane) - 1u));
+      if (valid) order[mine[a] + rank] = (int32_t)i;
+      __syncwarp();
+      if (valid && lane == __ffs(peers) - 1) mine[a] += __popc(peers);
+      __syncwarp();
+    }
   }
 }
 
@@ -232,6 +253,116 @@ __global__ void km_chunk_kernel(const float* __restrict__ X, int64_t d, int64_t 
     sums[j * d + t] = acc;
   }
   if (part_in && threadIdx.x == 0) {
+    double w = 0.0;
+    for (int c = 0; c < nch; c++) w += __ldcg(part_in + g0 + c);
+    in_j[j] = w;
+  }
+}
+
+// The same chunk sums with float4 rows: a sub-group of TPC = d / 4 lanes (1 .. 32, inside one
+// warp) takes one chunk, each lane 4 dimensions, 8 chunks per CTA.  Per dimension the rows are
+// still added one by one in the chunk's order from 0.0 (R20), so the partials are bitwise those
+// of km_chunk_kernel; a lane now keeps 4 independent fp64 chains and issues one 16-B load per
+// row instead of four 4-B loads (the scalar kernel was issue-bound: ~26 instructions per
+// element, 68 % issue utilisation).
+constexpr int kKmVecChunks = 8;
+template <bool INERTIA>
+__global__ void km_chunk_vec_kernel(const float* __restrict__ X, int64_t d, int64_t ldx,
+                                    const int32_t* __restrict__ order,
+                                    const int64_t* __restrict__ offsets,
+                                    const int64_t* __restrict__ counts,
+                                    const int32_t* __restrict__ chunk_base,
+                                    const int32_t* __restrict__ chunk_j,
+                                    const int32_t* __restrict__ n_chunks,
+                                    const float* __restrict__ best_key, double* __restrict__ part,
+                                    double* __restrict__ part_in, int32_t* __restrict__ done,
+                                    double* __restrict__ sums, double* __restrict__ in_j, int tpc_log2) {
+  __shared__ int32_t sidx[kKmVecChunks][kKmChunk];
+  const int tpc = 1 << tpc_log2;
+  const int sub = (int)threadIdx.x >> tpc_log2;
+  const int lt = (int)threadIdx.x & (tpc - 1);
+  const int g = (int)blockIdx.x * kKmVecChunks + sub;
+  const bool valid = g < *n_chunks;
+  int j = 0, nrow = 0;
+  int64_t c0 = 0;
+  if (valid) {
+    j = chunk_j[g];
+    c0 = (int64_t)(g - chunk_base[j]) * kKmChunk;
+    nrow = (int)min((int64_t)kKmChunk, counts[j] - c0);
+    const int32_t* ord = order + offsets[j] + c0;
+    for (int r = lt; r < nrow; r += tpc) sidx[sub][r] = ord[r];
+  }
+  __syncthreads();
+  const int32_t* si = sidx[sub];
+  const float4* X4 = reinterpret_cast<const float4*>(X) + lt;
+  const int64_t ld4 = ldx >> 2;
+  double s[4] = {0.0, 0.0, 0.0, 0.0}, q[4] = {0.0, 0.0, 0.0, 0.0};
+  int r = 0;
+  for (; r + 8 <= nrow; r += 8) {
+    float4 v[8];
+#pragma unroll
+    for (int i = 0; i < 8; i++) v[i] = __ldg(X4 + (int64_t)si[r + i] * ld4);
+#pragma unroll
+    for (int i = 0; i < 8; i++) {
+      const double a[4] = {(double)v[i].x, (double)v[i].y, (double)v[i].z, (double)v[i].w};
+#pragma unroll
+      for (int k = 0; k < 4; k++) {
+        s[k] = __dadd_rn(s[k], a[k]);
+        if (INERTIA) q[k] = __fma_rn(a[k], a[k], q[k]);
+      }
+    }
+  }
+  for (; r < nrow; r++) {
+    const float4 v = __ldg(X4 + (int64_t)si[r] * ld4);
+    const double a[4] = {(double)v.x, (double)v.y, (double)v.z, (double)v.w};
+#pragma unroll
+    for (int k = 0; k < 4; k++) {
+      s[k] = __dadd_rn(s[k], a[k]);
+      if (INERTIA) q[k] = __fma_rn(a[k], a[k], q[k]);
+    }
+  }
+  double* pg = part + (int64_t)g * d + 4 * lt;
+  if (valid) {
+    reinterpret_cast<double2*>(pg)[0] = make_double2(s[0], s[1]);
+    reinterpret_cast<double2*>(pg)[1] = make_double2(s[2], s[3]);
+  }
+  // sub-group lanes [sub * tpc, sub * tpc + tpc) of this warp
+  const int wl = (int)threadIdx.x & 31;
+  const int lead = wl & ~(tpc - 1);
+  const unsigned wmask = blockDim.x >= 32 ? 0xffffffffu : ((1u << blockDim.x) - 1u);
+  if (INERTIA) {
+    // fixed-order inertia terms: the lane's 4 dims, its strided share of the rows' best keys,
+    // then an xor tree over the sub-group (deterministic; compared to the oracle within 1e-5)
+    double w = (q[0] + q[1]) + (q[2] + q[3]);
+    for (int rr = lt; rr < nrow; rr += tpc) w += (double)best_key[si[rr]];
+    for (int o = tpc >> 1; o > 0; o >>= 1) w += __shfl_xor_sync(wmask, w, o);
+    if (valid && lt == 0) part_in[g] = w;
+  }
+  // the lane that completes centroid j's last chunk adds j's chunk partials in chunk order
+  // (R20's second level) -- as in km_chunk_kernel
+  const int nch = valid ? (int)((counts[j] + kKmChunk - 1) / kKmChunk) : 0;
+  __threadfence();
+  int last = 0;
+  if (valid && lt == 0) {
+    last = (atomicAdd(done + j, 1) == nch - 1);
+    __threadfence();
+  }
+  last = __shfl_sync(wmask, last, lead);
+  if (!valid || !last) return;
+  const int64_t g0 = chunk_base[j];
+  double acc[4] = {0.0, 0.0, 0.0, 0.0};
+  for (int c = 0; c < nch; c++) {
+    const double2* pp = reinterpret_cast<const double2*>(part + (g0 + c) * d + 4 * lt);
+    const double2 a0 = __ldcg(pp), a1 = __ldcg(pp + 1);
+    acc[0] = __dadd_rn(acc[0], a0.x);
+    acc[1] = __dadd_rn(acc[1], a0.y);
+    acc[2] = __dadd_rn(acc[2], a1.x);
+    acc[3] = __dadd_rn(acc[3], a1.y);
+  }
+  double2* sj = reinterpret_cast<double2*>(sums + (int64_t)j * d + 4 * lt);
+  sj[0] = make_double2(acc[0], acc[1]);
+  sj[1] = make_double2(acc[2], acc[3]);
+  if (INERTIA && lt == 0) {
     double w = 0.0;
     for (int c = 0; c < nch; c++) w += __ldcg(part_in + g0 + c);
     in_j[j] = w;
@@ -324,10 +455,28 @@ int launch_kmeans_accumulate(const float* X, int64_t n, int64_t d, int64_t ldx,
     km_scatter_kernel<2><<<nb, 64, 2 * hs, stream>>>(assign, n, kc, w.H, nb, w.offsets, w.order);
   else
     km_scatter_kernel<1><<<nb, 32, hs, stream>>>(assign, n, kc, w.H, nb, w.offsets, w.order);
-  km_chunk_kernel<<<(unsigned)gmax, dt, 0, stream>>>(X, d, ldx, w.order, w.offsets, counts,
-                                                     w.chunk_base, w.chunk_j, w.n_chunks, best_key,
-                                                     w.part, inertia ? w.part_in : nullptr, w.done,
-                                                     sums, w.in_j);
+  int tpc_log2 = -1;  // float4 rows: d / 4 lanes per chunk, a power of two <= 32
+  if (d % 4 == 0 && ldx % 4 == 0 && (reinterpret_cast<uintptr_t>(X) % 16) == 0 &&
+      (reinterpret_cast<uintptr_t>(sums) % 16) == 0)
+    for (int l = 0; l <= 5; l++)
+      if ((int64_t)(4 << l) == d) tpc_log2 = l;
+  if (tpc_log2 >= 0) {
+    const unsigned blocks = (unsigned)((gmax + kKmVecChunks - 1) / kKmVecChunks);
+    const unsigned threads = (unsigned)(kKmVecChunks << tpc_log2);
+    if (inertia)
+      km_chunk_vec_kernel<true><<<blocks, threads, 0, stream>>>(
+          X, d, ldx, w.order, w.offsets, counts, w.chunk_base, w.chunk_j, w.n_chunks, best_key,
+          w.part, w.part_in, w.done, sums, w.in_j, tpc_log2);
+    else
+      km_chunk_vec_kernel<false><<<blocks, threads, 0, stream>>>(
+          X, d, ldx, w.order, w.offsets, counts, w.chunk_base, w.chunk_j, w.n_chunks, best_key,
+          w.part, nullptr, w.done, sums, w.in_j, tpc_log2);
+  } else {
+    km_chunk_kernel<<<(unsigned)gmax, dt, 0, stream>>>(X, d, ldx, w.order, w.offsets, counts,
+                                                       w.chunk_base, w.chunk_j, w.n_chunks, best_key,
+                                                       w.part, inertia ? w.part_in : nullptr, w.done,
+                                                       sums, w.in_j);
+  }
   if (inertia) km_inertia_kernel<<<1, 1024, 0, stream>>>(w.in_j, kc, inertia);
   return cudaGetLastError() == cudaSuccess ? 0 : 3;
 }

@@ -180,7 +180,7 @@ def test_knn_ties_lowest_index_bitexact(oracle_lib, nx, d, dup, nq):
 
 
 @pytest.mark.parametrize("n,d,kc", [(20000, 64, 1024), (3001, 64, 100), (5000, 32, 7), (999, 130, 300),
-                                    (9000, 16, 2000), (7000, 8, 7000)])
+                                    (9000, 16, 2000), (7000, 8, 7000), (3000, 4, 50), (5000, 128, 300)])
 def test_kmeans_assign_bitexact_vs_alg1_model(oracle_lib, n, d, kc):
     """egemm_kmeans_step's assignment equals the profiled-tensor-core model bitwise, so its
     fp64 sums equal the oracle's R20 sums of that assignment bitwise: the whole step is
