@@ -208,7 +208,9 @@ def main():
     ap.add_argument("--steps", type=int, default=200)  # ~0.5 s timed: clocks settle, sampler sees it
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
-    ap.add_argument("--n", type=int, default=8192)
+    # (--size: the same, for torchrun command lines, whose parser takes "--n" as an
+    # abbreviation of its own options)
+    ap.add_argument("--n", "--size", dest="n", type=int, default=8192)
     ap.add_argument("--as-rank-of", type=int, default=1,
                     help="diagnostics: on one GPU, time rank 0's share of a world of this size "
                          "(M / W rows); value and n_gpus then describe that one rank")
