@@ -216,6 +216,11 @@ int egemm_tc_probe(int kind, int N, int K, const void* A, const void* B, const f
  * number of launches.  reset != 0 zeroes the sums after reading.  Synchronous. */
 int egemm_debug_clock_stats(double* mhz, double* cycles_per_launch, double* launches, int reset);
 
+/* Debug: a device event counter bumped by diagnostic kernel modes (EGEMM_DEBUG_MODE bit 256:
+ * kNN candidate-path entries, one per warp and 32-column group).  reset != 0 zeroes it
+ * after reading.  Synchronous. */
+int egemm_debug_counter(unsigned long long* value, int reset);
+
 #ifdef __cplusplus
 }
 #endif

@@ -255,6 +255,11 @@ int egemm_debug_clock_stats(double* mhz, double* cycles_per_launch, double* laun
   return read_clock_stats(mhz, cycles_per_launch, launches, reset) ? EGEMM_ERR_CUDA : EGEMM_OK;
 }
 
+int egemm_debug_counter(unsigned long long* value, int reset) {
+  if (!value) return EGEMM_ERR_INVALID_ARG;
+  return read_debug_counter(value, reset) ? EGEMM_ERR_CUDA : EGEMM_OK;
+}
+
 int egemm_set_config(int cg, int bn, int sep, int kc) {
   if (cg == 0 && bn == 0 && sep == 0 && kc == 0) {
     g_override = Override();
@@ -564,13 +569,16 @@ int egemm_gemm_host(int64_t M, int64_t N, int64_t K, const float* A_host, int64_
   return EGEMM_OK;
 }
 
+// N-slices per query block (wave balance over the persistent clusters); slices of the same
+// rows share their k-th-key bound (row_bound), so later slices skip most of the warm-up.
+constexpr int kKnnMaxSlices = 16;
 static int knn_slices(int64_t nq, int64_t nx, int cg, int bn) {
   const int64_t m_tiles = (nq + 128 * cg - 1) / (128 * cg);
   const int64_t n_tiles = (nx + bn - 1) / bn;
   const int64_t clusters = num_sms() / cg > 0 ? num_sms() / cg : 1;
   int best = 1;
   double best_eff = 0.0;
-  for (int s = 1; s <= 8 && s <= n_tiles; s++) {
+  for (int s = 1; s <= kKnnMaxSlices && s <= n_tiles; s++) {
     int64_t units = m_tiles * s;
     int64_t waves = (units + clusters - 1) / clusters;
     double eff = (double)units / (double)(waves * clusters);
@@ -589,8 +597,9 @@ size_t egemm_knn_workspace_size(int64_t nx, int64_t nq, int64_t d, int k, int x_
   cv.take<uint16_t>((size_t)(nq * ldk));
   cv.take<float>((size_t)nx);
   cv.take<float>((size_t)nq);
-  cv.take<float>((size_t)(8 * nq * k));
-  cv.take<int32_t>((size_t)(8 * nq * k));
+  cv.take<float>((size_t)(kKnnMaxSlices * nq * k));
+  cv.take<int32_t>((size_t)(kKnnMaxSlices * nq * k));
+  cv.take<float>((size_t)nq);
   return cv.off;
 }
 
@@ -658,8 +667,13 @@ int egemm_knn(egemm_operand_t X, const float* x_norms, int64_t nx, egemm_operand
   if ((r = stage_operand(Qs, nq, d, cv, &ops.a_hi, &ops.a_lo, &ops.lda, s))) return r;
   float* xnorm = cv.take<float>((size_t)nx);
   float* qnorm = cv.take<float>((size_t)nq);
-  float* pkey = cv.take<float>((size_t)(8 * nq * k));
-  int32_t* pidx = cv.take<int32_t>((size_t)(8 * nq * k));
+  float* pkey = cv.take<float>((size_t)(kKnnMaxSlices * nq * k));
+  int32_t* pidx = cv.take<int32_t>((size_t)(kKnnMaxSlices * nq * k));
+  float* rbound = cv.take<float>((size_t)nq);
+  if (cudaMemsetAsync(rbound, 0xFF, sizeof(float) * (size_t)nq, s) != cudaSuccess) {
+    set_last_error("memset of the row bounds failed");
+    return EGEMM_ERR_CUDA;
+  }
   if (x_norms) xnorm = const_cast<float*>(x_norms);
   else if (launch_rownorm(X.f32, nx, d, X.ld, xnorm, s)) return EGEMM_ERR_CUDA;
   if (launch_rownorm(Q.f32, nq, d, Q.ld, qnorm, s)) return EGEMM_ERR_CUDA;
@@ -668,6 +682,7 @@ int egemm_knn(egemm_operand_t X, const float* x_norms, int64_t nx, egemm_operand
   epi.bnorm = xnorm;
   epi.knn_k = k;
   epi.n_slices = knn_slices(nq, nx, cfg.cg, cfg.bn);
+  epi.row_bound = rbound;
   epi.part_key = pkey;
   epi.part_idx = pidx;
   r = launch_tc(nq, nx, d, ops, cfg, epi, s);

@@ -58,6 +58,7 @@ struct TcEpilogue {
   // EPI_KNN
   int knn_k;
   int n_slices;
+  float* row_bound;    // [M], bytes 0xFF (NaN = no bound yet) before the launch; nullable
   float* part_key;     // [n_slices][M][knn_k]
   int32_t* part_idx;   // [n_slices][M][knn_k]
   // EPI_KMEANS
@@ -88,6 +89,7 @@ int read_clock_probe(double* mhz);
 int launch_tc_probe(int kind, int N, int K, const void* A, const void* B, const float* C,
                     float* D, cudaStream_t stream);
 int read_clock_stats(double* mhz, double* cycles_per_launch, double* launches, int reset);
+int read_debug_counter(unsigned long long* value, int reset);
 
 // tune.cu: the measured configuration table
 bool tune_lookup(int op, long long M, long long N, long long K, int* cg, int* bn, int* sep,

@@ -69,6 +69,7 @@ struct KParams {
   int vec_ok;
   const float* bnorm;
   int knn_k;
+  float* row_bound;  // kNN (nullable): per query row, a shared upper bound on its k-th key
   float* part_key;
   int32_t* part_idx;
   int32_t* assign;
@@ -825,6 +826,8 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
     // (double-buffered smem slots after the merge scratch, named barrier 5 + q)
     uint32_t xgen = 0;
     uint32_t km_units = 0;  // kMeans: units finished (merge-slot parity)
+    float gpend = __int_as_float(0x7fffffff);  // kNN: the row bound loaded at the last exchange
+    float gcur = __int_as_float(0x7fffffff);   // kNN: the row bound in use (NaN: none)
     float* const xch = reinterpret_cast<float*>(scratch + kBM * kKnnMax * 4);
     float best = __int_as_float(0xff800000);
     int besti = 0x7fffffff;
@@ -968,6 +971,27 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
                 u = m;
               }
             }
+            // Every 8 tiles the bound is also exchanged with the row's other N-slices through
+            // global memory (plain loads / stores: any value ever stored is a valid bound, a
+            // lost update only loosens it; NaN = none yet).  A slice that starts after
+            // another slice of the same rows then skips most of its list warm-up.
+            // The unit's first tile waits for the load; later exchanges use the value loaded
+            // at the previous one (issued 8 tiles earlier, off the critical path).
+            // The bound in use (gcur) applies to every tile; it is refreshed every 8 tiles.
+            if (p.row_bound && !(p.debug_mode & 512) && row < p.M) {
+              if ((ns & 7) == 0) {
+                float* gb = p.row_bound + row;
+                if (ns == 0) {
+                  asm volatile("ld.relaxed.gpu.global.f32 %0, [%1];" : "=f"(gcur) : "l"(gb) : "memory");
+                } else {
+                  if (!(gpend <= u))
+                    asm volatile("st.relaxed.gpu.global.f32 [%0], %1;" ::"l"(gb), "f"(u) : "memory");
+                  gcur = fminf(gcur, gpend);
+                }
+                asm volatile("ld.relaxed.gpu.global.f32 %0, [%1];" : "=f"(gpend) : "l"(gb) : "memory");
+              }
+              u = fminf(u, gcur);
+            }
             // key < own 16th (strict: stream order) and key <= u, in accumulator space
             // (key = -2 v): v > -kd15/2 and v >= -u/2
             const float vt = fmaxf(-0.5f * kd[kKnnMax - 1], nextafterf(-0.5f * u, __int_as_float(0xff800000)));
@@ -990,6 +1014,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
 #pragma unroll
                 for (int i = 0; i < w; i++) t16[i] = fmaxf(t16[i], t16[i + w]);
               if (__any_sync(0xffffffffu, t16[0] > vt) && !(p.debug_mode & 128)) {
+                if ((p.debug_mode & 256) && lane == 0) atomicAdd(&g_clock_probe[7], 1ull);
                 uint32_t cand = 0;
                 float vv[32];
 #pragma unroll
@@ -1174,6 +1199,19 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
     g_clock_probe[5] += t1 - g_clock_probe[1];
     g_clock_probe[6] += 1;
   }
+}
+
+// Debug event counter (g_clock_probe[7]).
+int read_debug_counter(unsigned long long* value, int reset) {
+  if (cudaMemcpyFromSymbol(value, g_clock_probe, sizeof(unsigned long long),
+                           7 * sizeof(unsigned long long)) != cudaSuccess)
+    return 3;
+  if (reset) {
+    const unsigned long long z = 0;
+    if (cudaMemcpyToSymbol(g_clock_probe, &z, sizeof(z), 7 * sizeof(unsigned long long)) != cudaSuccess)
+      return 3;
+  }
+  return 0;
 }
 
 // SM cycles / wall ns of CTA 0 over the last launch (debug: effective SM clock).
@@ -1440,6 +1478,7 @@ int launch_tc(int64_t M, int64_t N, int64_t K, const TcOperands& ops, const TcCo
                   : 0;
   kp.bnorm = epi.bnorm;
   kp.knn_k = epi.knn_k;
+  kp.row_bound = epi.row_bound;
   kp.part_key = epi.part_key;
   kp.part_idx = epi.part_idx;
   kp.assign = epi.assign;

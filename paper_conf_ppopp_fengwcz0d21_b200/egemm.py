@@ -39,7 +39,7 @@ EXPORTS = ["egemm_status_string", "egemm_last_error", "egemm_version", "egemm_sp
            "egemm_gemm_workspace_size", "egemm_knn", "egemm_knn_workspace_size", "egemm_knn_index",
            "egemm_kmeans_step", "egemm_kmeans_workspace_size", "egemm_kmeans_finalize",
            "egemm_set_config", "egemm_num_sms", "egemm_debug_last_clock", "egemm_tune_table",
-           "egemm_debug_clock_stats", "egemm_tc_probe",
+           "egemm_debug_clock_stats", "egemm_debug_counter", "egemm_tc_probe",
            "egemm_query_config", "egemm_gemm_host", "egemm_gemm_host_workspace_size"]
 
 _lib = None
@@ -89,6 +89,8 @@ def load(path: str = LIB_PATH):
     DP = ctypes.POINTER(ctypes.c_double)
     L.egemm_debug_clock_stats.argtypes = [DP, DP, DP, I]
     L.egemm_debug_clock_stats.restype = I
+    L.egemm_debug_counter.argtypes = [ctypes.POINTER(ctypes.c_ulonglong), I]
+    L.egemm_debug_counter.restype = I
     L.egemm_gemm_host.argtypes = [I64, I64, I64, P, I64, P, I64, P, I64, I, P, SZ, P]
     L.egemm_gemm_host.restype = I
     L.egemm_gemm_host_workspace_size.argtypes = [I64, I64, I64]
@@ -150,6 +152,13 @@ def debug_clock_stats(reset: bool = True):
     _check(load().egemm_debug_clock_stats(*[ctypes.byref(x) for x in v], int(reset)),
            "egemm_debug_clock_stats")
     return tuple(x.value for x in v)
+
+
+def debug_counter(reset: bool = True) -> int:
+    """The device debug event counter (EGEMM_DEBUG_MODE bit 256: kNN candidate-path entries)."""
+    v = ctypes.c_ulonglong(0)
+    _check(load().egemm_debug_counter(ctypes.byref(v), int(reset)), "egemm_debug_counter")
+    return int(v.value)
 
 
 def debug_last_clock() -> float:
