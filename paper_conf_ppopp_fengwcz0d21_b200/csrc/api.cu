@@ -48,13 +48,13 @@ static int env_int(const char* name, int dflt) {
 }
 
 static bool fused_a_supported(const TcConfig& c) {
-  return (c.cg == 2 && c.bn == 256 && !c.sep) || (c.cg == 2 && c.bn == 128 && c.sep) ||
+  return (c.cg == 2 && c.bn == 256 && !c.sep) || (c.cg == 2 && c.bn == 128) ||
          (c.cg == 1 && c.bn == 128 && c.sep);
 }
 
 static bool valid_config(int cg, int bn, int sep) {
   return (cg == 2 && bn == 256 && sep == 0) || (cg == 1 && bn == 128) ||
-         (cg == 2 && bn == 128 && sep == 1) || (cg == 2 && bn == 224 && sep == 0);
+         (cg == 2 && bn == 128) || (cg == 2 && bn == 224 && sep == 0);
 }
 
 static bool fused_b_supported(const TcConfig& c) { return c.cg == 2 && c.bn == 256 && !c.sep; }

@@ -1362,6 +1362,8 @@ static int dispatch(const CUtensorMap* maps, const KParams& kp, const TcConfig& 
         return launch_variant<2, 256, false, EPI, 3, true>(maps, kp, cfg.max_clusters, s);
       if (cfg.cg == 2 && cfg.bn == 128 && cfg.sep)
         return launch_variant<2, 128, true, EPI, 3, true>(maps, kp, cfg.max_clusters, s);
+      if (cfg.cg == 2 && cfg.bn == 128 && !cfg.sep)
+        return launch_variant<2, 128, false, EPI, 3, true>(maps, kp, cfg.max_clusters, s);
       if (cfg.cg == 1 && cfg.bn == 128 && cfg.sep)
         return launch_variant<1, 128, true, EPI, 3, true>(maps, kp, cfg.max_clusters, s);
       set_last_error("fused A split: unsupported tile config cg=%d bn=%d sep=%d", cfg.cg, cfg.bn,
@@ -1383,6 +1385,10 @@ static int dispatch(const CUtensorMap* maps, const KParams& kp, const TcConfig& 
     // 256-wide tiles leave a partial one (e.g. M = 1024 or 2048 rows of N = 8192 per rank)
     if (cfg.cg == 2 && cfg.bn == 224 && !cfg.sep)
       return launch_variant<2, 224, false, EPI, 3>(maps, kp, cfg.max_clusters, s);
+    // 256 x 128 pair tiles, one accumulator in ping-pong, 4 stages of 48 KiB: twice the
+    // units of 256-wide tiles for short-N shapes (tall-skinny: 512 units = 6.9 waves)
+    if (cfg.cg == 2 && cfg.bn == 128 && !cfg.sep)
+      return launch_variant<2, 128, false, EPI, 4>(maps, kp, cfg.max_clusters, s);
   }
   if (cfg.cg == 1 && cfg.bn == 128 && !cfg.sep)
     return launch_variant<1, 128, false, EPI, 3>(maps, kp, cfg.max_clusters, s);

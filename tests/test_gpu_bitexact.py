@@ -12,7 +12,7 @@ from tests.gpu_util import require_gpu, to_dev, to_host
 pytestmark = pytest.mark.gpu
 
 CFGS = [(2, 256, 0, 64), (2, 256, 0, 128), (1, 128, 0, 64), (1, 128, 1, 128), (1, 128, 1, 256),
-        (2, 128, 1, 256), (2, 224, 0, 128), (2, 224, 0, 256)]
+        (2, 128, 1, 256), (2, 224, 0, 128), (2, 224, 0, 256), (2, 128, 0, 64)]
 
 
 def _gpu(eg, A, B, C, cfg, terms, fused):
@@ -41,7 +41,7 @@ def test_bitexact_vs_alg1_model(oracle_lib, cfg, shape):
         "mismatches: %d" % int((D != ref).sum())
 
 
-@pytest.mark.parametrize("cfg", [(2, 256, 0, 128), (1, 128, 1, 256)])
+@pytest.mark.parametrize("cfg", [(2, 256, 0, 128), (1, 128, 1, 256), (2, 128, 0, 64)])
 @pytest.mark.parametrize("gen", [inputs.stress, inputs.in_zone])
 def test_bitexact_terms4_with_c_and_fused(oracle_lib, cfg, gen):
     eg = require_gpu()

@@ -33,7 +33,7 @@ def main():
     need = 6.0 * M * N * K / (148 * 8192.0)
     ws = torch.empty(egemm.gemm_workspace_size(M, N, K, False, True), dtype=torch.uint8, device="cuda")
     print("tensor-bound cycles (all 148 SMs busy):", int(need))
-    for cfg in ((2, 256, 0, 64), (2, 256, 0, 128), (2, 128, 1, 128), (1, 128, 0, 64)):
+    for cfg in ((2, 256, 0, 64), (2, 256, 0, 128), (2, 128, 1, 128), (2, 128, 0, 64), (2, 128, 0, 128), (1, 128, 0, 64)):
         egemm.set_config(*cfg)
         ms, mhz, cyc = timed(lambda: egemm.gemm(None, None, a_split=a_s, b_split=b_s, out=D))
         print("presplit GEMM", cfg, "%.4f ms  %.0f MHz  %.0f kcyc  eff %.3f" % (ms, mhz, cyc / 1e3, need / cyc))
