@@ -370,7 +370,8 @@ int egemm_gemm(int64_t M, int64_t N, int64_t K, egemm_operand_t A, egemm_operand
   }
   Carver cv{reinterpret_cast<char*>(workspace)};
   TcOperands ops = {};
-  TcConfig cfg = choose_config(EPI_STORE, M, N, K, terms, B.f32 && !B.hi && !B.trans);
+  // B arriving as fp32 (either orientation): its split is part of this call -> "gemm_b32" rows
+  TcConfig cfg = choose_config(EPI_STORE, M, N, K, terms, B.f32 && !B.hi);
   // fp32 row-major A (fa bit 0) or fp32 K x N row-major B (fa bit 1) can be round-split
   // inside the GEMM (converter warps, a-2 fused mode); B needs 16-B aligned rows (TMA)
   const bool fuse_a = (cfg.fa & 1) && !A.hi && !A.trans && fused_a_supported(cfg);

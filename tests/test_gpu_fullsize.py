@@ -30,7 +30,8 @@ def _gemm_sampled(oracle_lib, M, N, K, seed_a, seed_b, n_rows, presplit=False):
     assert np.all(np.abs(D[rows].astype(np.float64) - C64) <= bound)
     # bitwise: the sampled rows equal Alg. 1 on the profiled tensor core (R21) for the
     # (terms, sep, Kc) the tuning table picked for this launch
-    cg, bn, sep, kc = eg.query_config("gemm", M, N, K)
+    # (an fp32-B call looks up the "gemm_b32" rows, a pre-split call the "gemm" rows)
+    cg, bn, sep, kc = eg.query_config("gemm" if presplit else "gemm_b32", M, N, K)
     br = rows[: min(len(rows), 8)]
     ref = oracle_lib.gemm_alg1_tc(A[br], B, terms=3, sep=sep, kc=kc)
     assert np.array_equal(D[br].view(np.uint32), ref.view(np.uint32))

@@ -91,7 +91,11 @@ def test_gemm_transposed_and_presplit(oracle_lib):
     D2 = to_host(eg.gemm(Ad, to_dev(np.ascontiguousarray(B.T)), b_trans=True))
     a_split = eg.split(Ad)
     b_split = eg.split(Bd, transpose=True)
-    D3 = to_host(eg.gemm(None, None, a_split=a_split, b_split=b_split))
+    eg.set_config(*eg.query_config("gemm_b32", 256, 512, 384))  # same (sep, Kc) as D1
+    try:
+        D3 = to_host(eg.gemm(None, None, a_split=a_split, b_split=b_split))
+    finally:
+        eg.set_config(0, 0, 0, 0)
     assert np.array_equal(D1, D2) and np.array_equal(D1, D3)
     _assert_parity(oracle_lib, A, B, D1)
 
@@ -216,7 +220,13 @@ def test_gemm_k_pacing_does_not_change_results(monkeypatch, shape):
     eg.load().egemm_gemm(M, N, K, eg.operand(Ad), eg.operand(Bd), None, 0,
                          eg._ptr(D3), N, 0, eg._ptr(ops_only), ops_only.numel(), eg._stream())
     a_s, b_s = eg.split(Ad), eg.split(Bd, transpose=True)
-    D4 = eg.gemm(None, None, a_split=a_s, b_split=b_s)  # 256-B pacing workspace only
+    # the pre-split call looks up the "gemm" table rows, the fp32-B calls above the
+    # "gemm_b32" rows: pin the latter's (cg, bn, sep, Kc) -- the bits depend on (sep, Kc)
+    eg.set_config(*eg.query_config("gemm_b32", M, N, K))
+    try:
+        D4 = eg.gemm(None, None, a_split=a_s, b_split=b_s)  # 256-B pacing workspace only
+    finally:
+        eg.set_config(0, 0, 0, 0)
     for D in (D2, D3, D4):
         assert torch.equal(D1.view(torch.int32), D.view(torch.int32))
 
