@@ -14,7 +14,7 @@
 //   B1 km_scan_blk   per-centroid exclusive scan over blocks, cnt[j]
 //   B2 km_scan_c     offsets[j], counts[j], chunk_base[j], chunk -> centroid map
 //   C  km_scatter    stable scatter: the block's 4096 points in W warp sub-ranges, per-warp
-//                    histograms -> per-warp offsets, then match_any ranks (32 points a step)
+//                    histograms -> per-warp offsets, then in-warp ranks from per-bit ballots
 //   D  km_chunk      chunk partial sums (+ per-chunk inertia terms); the CTA that finishes
 //                    the last chunk of centroid j (atomic ticket) adds j's chunk partials in
 //                    chunk order: sums[j] (+ inertia_j) -- the old separate combine pass
@@ -112,10 +112,23 @@ __global__ void km_scan_c_kernel(const int32_t* __restrict__ cnt, int64_t kc,
 }
 
 // Stable scatter of one block of kKmBlockPts points: W warps take consecutive sub-ranges;
-// pass 1 counts each warp's members per centroid (match_any: the leader of each peer group
+// pass 1 counts each warp's members per centroid (peer lanes by ballots: the leader of each group
 // adds its popcount, so no atomics), the counts become per-warp start offsets (block base
 // H[a][b] + earlier warps), pass 2 writes order[] with the in-warp ranks.  Same positions as
 // a sequential walk over the block: the order stays stable (ascending i per centroid).
+// Lanes of the warp holding the same centroid as this lane (valid lanes only): one ballot
+// per bit of the centroid index instead of __match_any_sync, whose result latency bounded the
+// scatter (ncu: the stalls sat on the instructions consuming MATCH).
+__device__ __forceinline__ uint32_t same_key_lanes(int a, bool valid, int nbits) {
+  uint32_t m = __ballot_sync(0xffffffffu, valid);
+  for (int b = 0; b < nbits; b++) {
+    const bool bit = (a >> b) & 1;
+    const uint32_t bb = __ballot_sync(0xffffffffu, bit);
+    m &= bit ? bb : ~bb;
+  }
+  return m;
+}
+
 template <int W>
 __global__ void __launch_bounds__(32 * W) km_scatter_kernel(
     const int32_t* __restrict__ assign, int64_t n, int64_t kc, const int32_t* __restrict__ H,
@@ -130,17 +143,18 @@ __global__ void __launch_bounds__(32 * W) km_scatter_kernel(
   constexpr int B = 16;  // assignments held in registers per lane (the loads of a batch overlap)
   const int64_t s0 = i0 + (int64_t)w * SUB, s1 = min(i1, s0 + SUB);
   int32_t* mine = hw + (int64_t)w * kc;
+  const int nbits = kc > 1 ? 32 - __clz((int)(kc - 1)) : 0;
   for (int64_t cb = s0; cb < s1; cb += 32 * B) {
     int av[B];
 #pragma unroll
     for (int t = 0; t < B; t++) {
       const int64_t i = cb + 32 * t + lane;
-      av[t] = i < s1 ? assign[i] : -1 - lane;
+      av[t] = i < s1 ? assign[i] : 0;
     }
 #pragma unroll
     for (int t = 0; t < B; t++) {
       const int64_t i = cb + 32 * t + lane;
-      const uint32_t peers = __match_any_sync(0xffffffffu, av[t]);
+      const uint32_t peers = same_key_lanes(av[t], i < s1, nbits);
       if (i < s1 && lane == __ffs(peers) - 1) mine[av[t]] += __popc(peers);
       __syncwarp();  // the next batch's leader of this centroid may be another lane
     }
@@ -163,14 +177,14 @@ __global__ void __launch_bounds__(32 * W) km_scatter_kernel(
 #pragma unroll
     for (int t = 0; t < B; t++) {
       const int64_t i = cb + 32 * t + lane;
-      av[t] = i < s1 ? assign[i] : -1 - lane;
+      av[t] = i < s1 ? assign[i] : 0;
     }
 #pragma unroll
     for (int t = 0; t < B; t++) {
       const int64_t i = cb + 32 * t + lane;
       const bool valid = i < s1;
       const int a = av[t];
-      const uint32_t peers = __match_any_sync(0xffffffffu, a);
+      const uint32_t peers = same_key_lanes(a, valid, nbits);
       const int rank = __popc(peers & ((1u << lane) - 1u));
       if (valid) order[mine[a] + rank] = (int32_t)i;
       __syncwarp();
