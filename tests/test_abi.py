@@ -98,6 +98,35 @@ def test_tune_table_lookup(tmp_path):
     assert out == "2 (1, 128, 1, 128) (2, 256, 0, 128) (2, 256, 0, 128)", out
 
 
+def test_tune_table_gemm_b32_rows(tmp_path):
+    """The fp32-B rows ("gemm_b32", the B split is part of the call) are consulted for that op
+    only, fall back to the "gemm" rows where they have no bucket, and report the fused-B
+    flag (2) for the fused-B kernel; the shipped table parses completely."""
+    import json
+    import subprocess
+    import sys
+    t = {"entries": [
+        {"op": "gemm", "m_max": 1 << 40, "n_max": 1 << 40, "k_max": 1 << 40, "cg": 2, "bn": 224,
+         "sep": 0, "kc": 256, "fa": 0},
+        {"op": "gemm_b32", "m_max": 1024, "n_max": 1 << 40, "k_max": 1 << 40, "cg": 2, "bn": 256,
+         "sep": 0, "kc": 256, "fa": 2}]}
+    p = tmp_path / "t.json"
+    p.write_text(json.dumps(t))
+    code = ("import sys; sys.path.insert(0, %r); from paper_conf_ppopp_fengwcz0d21_b200 import egemm;"
+            "print(egemm.query_config('gemm_b32', 1024, 8192, 8192, with_fused=True),"
+            " egemm.query_config('gemm', 1024, 8192, 8192, with_fused=True),"
+            " egemm.query_config('gemm_b32', 4096, 8192, 8192, with_fused=True))" % ROOT)
+    out = subprocess.check_output([sys.executable, "-c", code],
+                                  env=dict(os.environ, EGEMM_TUNE_TABLE=str(p))).decode().strip()
+    assert out == "(2, 256, 0, 256, 2) (2, 224, 0, 256, 0) (2, 224, 0, 256, 0)", out
+    shipped = json.load(open(os.path.join(ROOT, "paper_conf_ppopp_fengwcz0d21_b200", "tune_table.json")))
+    code = ("import sys; sys.path.insert(0, %r); from paper_conf_ppopp_fengwcz0d21_b200 import egemm;"
+            "print(egemm.tune_table()[1])" % ROOT)
+    env = {k: v for k, v in os.environ.items() if k != "EGEMM_TUNE_TABLE"}
+    n = int(subprocess.check_output([sys.executable, "-c", code], env=env).decode().strip())
+    assert n == len(shipped["entries"])
+
+
 def test_no_gpu_means_loud_failure(lib):
     """Without a device the compute entry points fail loudly (no CPU fallback)."""
     import torch
