@@ -143,7 +143,9 @@ def test_kmeans_finalize_and_empty_cluster(oracle_lib):
 # ------------------------------------------------------------------ bitwise (R21 + R22)
 @pytest.mark.parametrize("nx,nq,d,k,path", [(5000, 64, 128, 16, "index"), (777, 50, 100, 5, "f32"),
                                             (40, 33, 16, 16, "split"), (32768, 24, 128, 16, "index"),
-                                            (3000, 300, 64, 8, "f32")])
+                                            (3000, 300, 64, 8, "f32"),
+                                            # d > 128: the streaming-A kernel variant (4+ k-blocks)
+                                            (2000, 100, 200, 16, "index"), (1000, 40, 520, 8, "f32")])
 def test_knn_bitexact_vs_alg1_model(oracle_lib, nx, nq, d, k, path):
     """egemm_knn equals the kNN-on-the-profiled-tensor-core model bitwise: indices AND
     distances (oracle.knn_alg1_tc: Alg. 1 dot products, R22 norms / key / ordering) -- no
