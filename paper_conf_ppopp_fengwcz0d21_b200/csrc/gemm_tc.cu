@@ -279,7 +279,9 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
   // AS (fused A, TMA-staged): the fp32 A tiles land in their own ring (NSTG x 128 rows x 64
   // fp32, two 128-B-swizzled boxes of 32 columns), loaded ahead by warp 7; the converters
   // split from smem instead of waiting on their own global loads.
-  constexpr int NSTG = (AS || FB) ? 3 : 0;
+  // AS: the fp32 A tile (32 KiB = the A_hi + A_lo bytes of a stage) lands in the stage's own A
+  // region and the converters split it in place; FB keeps a 3-slot fp32 staging ring.
+  constexpr int NSTG = FB ? 3 : 0;
   constexpr int STG_BYTES = kBM * kBK * 4;
   static_assert(!AS || FA, "AS is a fused-A mode");
   static_assert(!(FA && FB), "one fused operand at a time");
@@ -298,7 +300,8 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * STAGES + 6);
   uint64_t* sfull = bars + 2 * STAGES + 8;   // AS: fp32 A tile landed (TMA bytes)
   uint64_t* sempty = sfull + NSTG;           // AS: consumed by the 4 converter warps
-  uint8_t* scratch = reinterpret_cast<uint8_t*>(bars + 2 * STAGES + 8 + 2 * NSTG);  // merges
+  uint64_t* afull = sempty + NSTG;           // AS: a stage's fp32 A tile landed (TMA bytes)
+  uint8_t* scratch = reinterpret_cast<uint8_t*>(bars + 2 * STAGES + 8 + 2 * NSTG + (AS ? STAGES : 0));  // merges
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
@@ -326,6 +329,8 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
     }
     ptx::mbar_init(a_full, 1);
     ptx::mbar_init(a_empty, 1);
+    if constexpr (AS)
+      for (int s = 0; s < STAGES; s++) ptx::mbar_init(&afull[s], 1);
     for (int i = 0; i < NSTG; i++) {
       ptx::mbar_init(&sfull[i], 1);
       ptx::mbar_init(&sempty[i], 4);
@@ -446,24 +451,31 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
         for (int ns = 0; ns < ui.n_count; ns++) {
           for (int kb = 0; kb < p.num_kb; kb++) {
             if constexpr (AS) {
-              // fp32 tile from the TMA ring: row r, 8 values k = 8c..8c+7 are fp32 16-B
-              // chunks 2(c%4), 2(c%4)+1 of box c/4, at chunk position j ^ (r & 7) (SW128)
-              ptx::mbar_wait(&sfull[si], sph);
-              ptx::mbar_wait(&empty[stage], phase ^ 1u);
+              // the stage's A region holds the fp32 tile (2 boxes of 32 columns, SW128): row r,
+              // 8 values k = 8c..8c+7 are fp32 16-B chunks 2(c%4), 2(c%4)+1 of box c/4 at chunk
+              // position j ^ (r & 7).  All 4 converter warps read their 64 values first, meet
+              // at a named barrier, then overwrite the region with the hi / lo K-major tiles.
+              ptx::mbar_wait(&afull[stage], phase);  // (the producer waited for the free stage)
               const uint32_t sb = ptx::smem_u32(stage_base + stage * G::STAGE_BYTES);
-              const uint32_t xb = ptx::smem_u32(a_stg + si * STG_BYTES) + (c >> 2) * (STG_BYTES / 2);
+              const uint32_t xb = sb + (c >> 2) * (STG_BYTES / 2);
               const int j0 = (c & 3) * 2;
+              float4 u[16];
 #pragma unroll
               for (int it = 0; it < 8; it++) {
                 const int r = warp * 32 + it * 4 + rsub;
                 const uint32_t rb = xb + r * 128;
-                const float4 u0 = ptx::lds128f(rb + ((j0 ^ (r & 7)) << 4));
-                const float4 u1 = ptx::lds128f(rb + (((j0 + 1) ^ (r & 7)) << 4));
+                u[2 * it] = ptx::lds128f(rb + ((j0 ^ (r & 7)) << 4));
+                u[2 * it + 1] = ptx::lds128f(rb + (((j0 + 1) ^ (r & 7)) << 4));
+              }
+              named_bar_sync(9, 128);  // every fp32 value of the tile is in registers
+#pragma unroll
+              for (int it = 0; it < 8; it++) {
+                const int r = warp * 32 + it * 4 + rsub;
                 uint32_t hi[4], lo[4];
-                ptx::split2(u0.x, u0.y, hi[0], lo[0]);
-                ptx::split2(u0.z, u0.w, hi[1], lo[1]);
-                ptx::split2(u1.x, u1.y, hi[2], lo[2]);
-                ptx::split2(u1.z, u1.w, hi[3], lo[3]);
+                ptx::split2(u[2 * it].x, u[2 * it].y, hi[0], lo[0]);
+                ptx::split2(u[2 * it].z, u[2 * it].w, hi[1], lo[1]);
+                ptx::split2(u[2 * it + 1].x, u[2 * it + 1].y, hi[2], lo[2]);
+                ptx::split2(u[2 * it + 1].z, u[2 * it + 1].w, hi[3], lo[3]);
                 const uint32_t off = (uint32_t)(r * 128 + ((c ^ (r & 7)) << 4));
                 ptx::sts128(sb + off, hi[0], hi[1], hi[2], hi[3]);
                 ptx::sts128(sb + G::A_BYTES + off, lo[0], lo[1], lo[2], lo[3]);
@@ -473,10 +485,8 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
               if (lane == 0) {
                 if constexpr (CG == 1) ptx::mbar_arrive(&full[stage]);
                 else ptx::mbar_arrive_cluster(&full[stage], 0);
-                ptx::mbar_arrive(&sempty[si]);
               }
               if (++stage == STAGES) { stage = 0; phase ^= 1u; }
-              if (++si == NSTG) { si = 0; sph ^= 1u; }
               continue;
             }
             ptx::mbar_wait(&empty[stage], phase ^ 1u);
@@ -579,6 +589,11 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
             }
             if (leader) ptx::mbar_arrive_expect_tx(&full[stage], TX * CG);
             const int k0 = kb * kBK;
+            if constexpr (AS) {  // this CTA's fp32 A tile into the stage's A region
+              ptx::mbar_arrive_expect_tx(&afull[stage], STG_BYTES);
+              ptx::tma_load_2d(&tm_ahi, &afull[stage], sb, k0, arow);
+              ptx::tma_load_2d(&tm_ahi, &afull[stage], sb + STG_BYTES / 2, k0 + 32, arow);
+            }
             if constexpr (CG == 1) {
               if (!FA && !AR) {
                 ptx::tma_load_2d(&tm_ahi, &full[stage], sb, k0, arow);
@@ -626,28 +641,6 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
 #pragma unroll
               for (int j = 0; j < G::BNC / 32; j++)
                 ptx::tma_load_2d(&tm_bhi, &sfull[si], dst + j * (STG_BYTES / 4), n0 + 32 * j, kb * kBK);
-              if (++si == NSTG) { si = 0; sph ^= 1u; }
-            }
-          }
-        }
-      }
-    }
-  } else if (AS && warp == 7) {
-    // ==================== fp32 A staging producer (fused A, AS) ====================
-    if constexpr (AS) {
-      if (lane == 0) {
-        int si = 0;
-        uint32_t sph = 0;
-        for (int u = cluster; u < p.num_units; u += nclusters) {
-          UnitInfo ui = decode_unit<EPI>(p, u);
-          const int arow = ui.m_tile * (kBM * CG) + (int)rank * kBM;
-          for (int ns = 0; ns < ui.n_count; ns++) {
-            for (int kb = 0; kb < p.num_kb; kb++) {
-              ptx::mbar_wait(&sempty[si], sph ^ 1u);
-              ptx::mbar_arrive_expect_tx(&sfull[si], STG_BYTES);
-              uint8_t* dst = a_stg + si * STG_BYTES;
-              ptx::tma_load_2d(&tm_ahi, &sfull[si], dst, kb * kBK, arow);
-              ptx::tma_load_2d(&tm_ahi, &sfull[si], dst + STG_BYTES / 2, kb * kBK + 32, arow);
               if (++si == NSTG) { si = 0; sph ^= 1u; }
             }
           }
@@ -1303,7 +1296,7 @@ static int launch_variant(const CUtensorMap* maps, const KParams& kp, int max_cl
   constexpr bool NORM = (EPI != EPI_STORE);  // norm slot per stage + the A' ones tile
   const size_t sb = (AR ? 2 * G::B_BYTES : G::STAGE_BYTES) + (NORM ? G::BNC * 32 : 0);
   const size_t smem = 1024 + (size_t)STAGES * sb + (AR ? 4 * G::A_BYTES : 0) +
-                      (NORM ? kBM * 32 : 0) + ((AS || FB) ? 3 * kBM * kBK * 4 + 8 * 6 : 0) +
+                      (NORM ? kBM * 32 : 0) + (FB ? 3 * kBM * kBK * 4 + 8 * 6 : 0) + (AS ? 8 * STAGES : 0) +
                       8 * (2 * STAGES + 8) + scratch;
   static bool attr_done = false;  // per instantiation
   if (!attr_done) {
@@ -1357,7 +1350,7 @@ static int dispatch(const CUtensorMap* maps, const KParams& kp, const TcConfig& 
     if (kp.a_f32) {  // fused A split (converter warpgroup)
       // aligned fp32 A: TMA-staged (2 MMA stages + 3 fp32 staging slots); else LDG converters
       if (cfg.cg == 2 && cfg.bn == 256 && !cfg.sep && kp.a_staged)
-        return launch_variant<2, 256, false, EPI, 2, true, false, true>(maps, kp, cfg.max_clusters, s);
+        return launch_variant<2, 256, false, EPI, 3, true, false, true>(maps, kp, cfg.max_clusters, s);
       if (cfg.cg == 2 && cfg.bn == 256 && !cfg.sep)
         return launch_variant<2, 256, false, EPI, 3, true>(maps, kp, cfg.max_clusters, s);
       if (cfg.cg == 2 && cfg.bn == 128 && cfg.sep)
