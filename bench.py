@@ -503,12 +503,14 @@ def main():
 def _apps(world, rank, dev, args):
     """kNN (configs[3]) and kMeans (configs[4]) timings, queries / points sharded."""
     import torch
+    # --as-rank-of W on one GPU: shard as rank 0 of W ranks (per-rank shapes; no collectives)
+    sw = args.as_rank_of if (world == 1 and args.as_rank_of > 1) else world
     from paper_conf_ppopp_fengwcz0d21_b200 import egemm, inputs
     from paper_conf_ppopp_fengwcz0d21_b200 import distributed as edist
     out = {}
     try:  # configs[2]: tall-skinny M=65536 N=256 K=1024 (rows sharded), fp32 in -> fp32 out
         M2, N2, K2 = 65536, 256, 1024
-        r0, r1 = edist.shard_bounds(M2, world, rank, align=256)
+        r0, r1 = edist.shard_bounds(M2, sw, rank, align=256)
         A2 = torch.from_numpy(inputs.uniform((M2, K2), 200)[r0:r1]).to(dev)
         B2 = torch.from_numpy(inputs.uniform((K2, N2), 201)).to(dev)
         ws2 = torch.empty(egemm.gemm_workspace_size(r1 - r0, N2, K2), dtype=torch.uint8, device=dev)
@@ -527,7 +529,7 @@ def _apps(world, rank, dev, args):
         out["tall_skinny"] = {"metric": "EGEMM FP32-equiv TFLOP/s, M=65536 N=256 K=1024 (split included)",
                               "value": round(2.0 * M2 * N2 * K2 / (ms * 1e-3) / 1e12, 1),
                               "unit": "TFLOP/s", "ms": round(ms, 4),
-                              "config": list(egemm.query_config("gemm", r1 - r0, N2, K2))}
+                              "config": list(egemm.query_config("gemm_b32", r1 - r0, N2, K2, with_fused=True))}
         del A2, B2, ws2, D2
     except Exception as ex:  # pragma: no cover
         out["tall_skinny"] = {"error": str(ex)[:300]}
@@ -535,7 +537,7 @@ def _apps(world, rank, dev, args):
         # fp32 in -> fp32 out (splits included), rows sharded, steady-state windows
         sweep = {}
         for n2 in (1024, 2048, 4096, 16384):
-            r0, r1 = edist.shard_bounds(n2, world, rank, align=256)
+            r0, r1 = edist.shard_bounds(n2, sw, rank, align=256)
             A2 = (torch.rand(r1 - r0, n2, device=dev, generator=torch.Generator(dev).manual_seed(n2))
                   * 2 - 1)
             B2 = torch.rand(n2, n2, device=dev, generator=torch.Generator(dev).manual_seed(n2 + 1)) * 2 - 1
@@ -574,7 +576,7 @@ def _apps(world, rank, dev, args):
             _barrier(world)
             ms = _allmax(s.elapsed_time(e), world) / reps
             sweep[str(n2)] = {"tflops": round(2.0 * n2 ** 3 / (ms * 1e-3) / 1e12, 1), "ms": round(ms, 4),
-                              "config": list(egemm.query_config("gemm", r1 - r0, n2, n2, with_fused=True)),
+                              "config": list(egemm.query_config("gemm_b32", r1 - r0, n2, n2, with_fused=True)),
                               "timing": "CUDA-graph replay of egemm_gemm" if graph is not None
                               else "direct egemm_gemm calls"}
             del graph
@@ -586,7 +588,7 @@ def _apps(world, rank, dev, args):
     cpu_ok = rank == 0 and world == 1 and not args.no_cpu
     try:
         nx, nq, d, k = 1 << 20, 1 << 16, 128, 16
-        q0, q1 = edist.shard_bounds(nq, world, rank)
+        q0, q1 = edist.shard_bounds(nq, sw, rank)
         Xh = inputs.uniform((nx, d), 300)
         Qh = inputs.uniform((nq, d), 301)
         X = torch.from_numpy(Xh).to(dev)
@@ -614,7 +616,8 @@ def _apps(world, rank, dev, args):
                       "ms_per_batch": round(ms, 3), "index_build_ms": round(t_ib[0].elapsed_time(t_ib[1]), 3),
                       "fp32eq_tflops": round(2.0 * nx * nq * d / (ms * 1e-3) / 1e12, 1),
                       "kernel_sm_mhz": round(egemm.debug_last_clock(), 1),
-                      "sharding": "queries over %d ranks, X replicated" % world}
+                      "sharding": "queries over %d ranks, X replicated%s" % (
+                          sw, " (rank 0 of them timed alone)" if sw != world else "")}
         if cpu_ok:  # the plain fp64 kNN oracle on a bounded query sample (host cores)
             import oracle
             t0 = time.perf_counter()
@@ -634,7 +637,7 @@ def _apps(world, rank, dev, args):
         out["knn"] = {"error": str(ex)[:300]}
     try:
         n, d, kc, iters = 1 << 22, 64, 1024, 20
-        p0, p1 = edist.shard_bounds(n, world, rank)
+        p0, p1 = edist.shard_bounds(n, sw, rank)
         Xh, lab, _ = inputs.mixture(n, d, kc, 400)
         X = torch.from_numpy(Xh[p0:p1]).to(dev)
         C0 = torch.from_numpy(Xh[:kc].copy()).to(dev)
@@ -672,7 +675,8 @@ def _apps(world, rank, dev, args):
                          "value": round(ms, 4), "unit": "ms/iter", "iterations": iters,
                          "fp32eq_tflops": round(2.0 * n * kc * d / (ms * 1e-3) / 1e12, 1),
                          "kernel_sm_mhz": round(egemm.debug_last_clock(), 1),
-                         "sharding": "points over %d ranks, NCCL all_reduce of sums/counts" % world}
+                         "sharding": "points over %d ranks, NCCL all_reduce of sums/counts%s" % (
+                             sw, " (rank 0 of them timed alone, no all_reduce)" if sw != world else "")}
         if cpu_ok:
             out["kmeans"]["cpu_baseline"] = kmeans_cpu
     except Exception as ex:  # pragma: no cover
