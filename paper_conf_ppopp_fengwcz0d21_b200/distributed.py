@@ -133,9 +133,19 @@ def kmeans_fit(X: torch.Tensor, C: torch.Tensor, iters: int, x_split=None, works
         X_, C_, x_split=x_split, want_inertia=False, workspace=workspace, out=out))
     finalize = finalize or egemm.kmeans_finalize
     assign = None
+    packed = None
     for _ in range(iters):
         assign, sums, counts, _ = step(X, C, bufs)
-        allreduce_sum_(sums, world)
-        allreduce_sum_(counts, world)
+        if world > 1:
+            # one collective per iteration: the fp64 sums and the counts (as fp64: exact below
+            # 2^53) travel in one buffer -- a single NCCL launch / latency instead of two
+            ns, nc = sums.numel(), counts.numel()
+            if packed is None or packed.numel() != ns + nc or packed.device != sums.device:
+                packed = torch.empty(ns + nc, dtype=torch.float64, device=sums.device)
+            packed[:ns].copy_(sums.reshape(-1))
+            packed[ns:].copy_(counts)
+            dist.all_reduce(packed, op=dist.ReduceOp.SUM)
+            sums.copy_(packed[:ns].view_as(sums))
+            counts.copy_(packed[ns:])
         finalize(sums, counts, C)
     return assign
