@@ -29,6 +29,14 @@
 //    matching bits) to Kc-long sums -- the TMEM analogue of the paper's FRAG caching of
 //    C across the k-loop (Table 2).  SEP additionally keeps the
 //    hi*hi and cross products in separate accumulators (needs 4 x BN TMEM columns).
+//  * tiles: BN = 256, 224 (whole waves of 74 clusters for N = 8192 at short M) or 128 per
+//    CTA pair; CG == 1: 128 x 128.
+//  * fused splits (a converter warpgroup in front, setmaxnreg 96 / 56 / 176): FA converts
+//    fp32 A (LDG, or AS: the TMA-staged fp32 tile converted in place in the stage's A
+//    region); FB converts TMA-staged fp32 B (K x N row-major) into the K-major B stage.
+//  * kNN epilogue (KREG): the tile is loaded from TMEM and released before ranking; the two
+//    column groups of a row filter on the union of their lists (smem exchange per tile) and
+//    the row's N-slices share that bound through global memory.
 #include <cuda.h>
 #include <cudaTypedefs.h>
 #include <cuda_runtime.h>
