@@ -57,7 +57,9 @@ static bool valid_config(int cg, int bn, int sep) {
          (cg == 2 && bn == 128) || (cg == 2 && bn == 224 && sep == 0);
 }
 
-static bool fused_b_supported(const TcConfig& c) { return c.cg == 2 && c.bn == 256 && !c.sep; }
+static bool fused_b_supported(const TcConfig& c) {
+  return c.cg == 2 && (c.bn == 256 || c.bn == 224) && !c.sep;
+}
 
 // b_f32: a STORE GEMM whose B is fp32 (split inside the call): the table's "gemm_b32" rows
 // (which may pick the fused-B kernel) first, then the "gemm" rows.

@@ -293,7 +293,8 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
   constexpr int STG_BYTES = kBM * kBK * 4;
   static_assert(!AS || FA, "AS is a fused-A mode");
   static_assert(!(FA && FB), "one fused operand at a time");
-  static_assert(!FB || (CG == 2 && BN == 256 && EPI == EPI_STORE && !SEP), "FB: 256 x 256 pair tiles");
+  static_assert(!FB || (CG == 2 && (BN == 256 || BN == 224) && EPI == EPI_STORE && !SEP),
+                "FB: 256 x 256 or 256 x 224 pair tiles");
   uint8_t* stage_base = smem;
   uint8_t* a_res = smem + STAGES * SB;
   uint8_t* a_stg = a_res + AR_BYTES;
@@ -396,18 +397,18 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
     if constexpr (CONV) asm volatile("setmaxnreg.dec.sync.aligned.u32 96;");
     if constexpr (FB) {
       // ================= fused round-split of B (converter warpgroup) =================
-      // Alg. 1 l.3 for B inside the GEMM.  The fp32 tile of this CTA's 128
-      // B columns x 64 k (4 TMA boxes of 32 columns, 128-B swizzled rows of k) sits in the
-      // staging ring; thread t takes column n = t, reads its 8 k-chunks down the rows
-      // (a warp reads one 128-B row per instruction: conflict-free), splits them and stores
-      // 16-B hi / lo chunks into row n of the K-major 128-B-swizzled B stage.
+      // Alg. 1 l.3 for B inside the GEMM.  The fp32 tile of this CTA's BNC
+      // (128 or 112) B columns x 64 k (one unswizzled TMA box, rows of k contiguous) sits in
+      // the staging ring; thread t takes column n = t, reads its 8 k-chunks down the rows
+      // (a warp reads 32 consecutive words of one row per instruction: conflict-free), splits
+      // them and stores 16-B hi / lo chunks into row n of the K-major 128-B-swizzled B stage.
       int stage = 0;
       uint32_t phase = 0;
       int si = 0;
       uint32_t sph = 0;
-      const int n = threadIdx.x;  // 0 .. 127
-      const int cn = (n & 31) >> 2;
-      const uint32_t colx = (uint32_t)((n >> 5) * (STG_BYTES / 4) + (n & 3) * 4);
+      const int n = threadIdx.x;  // 0 .. 127 (columns >= BNC idle)
+      constexpr int ROWB = G::BNC * 4;  // bytes per staged k-row
+      const bool act = n < G::BNC;
       for (int u = cluster; u < p.num_units; u += nclusters) {
         UnitInfo ui = decode_unit<EPI>(p, u);
         for (int ns = 0; ns < ui.n_count; ns++) {
@@ -415,13 +416,13 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
             ptx::mbar_wait(&sfull[si], sph);
             ptx::mbar_wait(&empty[stage], phase ^ 1u);
             const uint32_t sb = ptx::smem_u32(stage_base + stage * G::STAGE_BYTES) + 2 * G::A_BYTES;
-            const uint32_t xb = ptx::smem_u32(a_stg + si * STG_BYTES) + colx;
+            const uint32_t xb = ptx::smem_u32(a_stg + si * STG_BYTES) + 4 * n;
 #pragma unroll
             for (int c = 0; c < kBK / 8; c++) {
+              if (!act) break;
               float x[8];
 #pragma unroll
-              for (int i = 0; i < 8; i++)  // k = 8c + i: row k, chunk cn at position cn ^ i
-                x[i] = ptx::lds32f(xb + (c * 8 + i) * 128 + ((cn ^ i) << 4));
+              for (int i = 0; i < 8; i++) x[i] = ptx::lds32f(xb + (c * 8 + i) * ROWB);  // k = 8c + i
               uint32_t hi[4], lo[4];
 #pragma unroll
               for (int e = 0; e < 4; e++) ptx::split2(x[2 * e], x[2 * e + 1], hi[e], lo[e]);
@@ -644,11 +645,9 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
             const int n0 = (ui.n_begin + ns) * BN + (int)rank * G::BNC;
             for (int kb = 0; kb < p.num_kb; kb++) {
               ptx::mbar_wait(&sempty[si], sph ^ 1u);
-              ptx::mbar_arrive_expect_tx(&sfull[si], STG_BYTES);
+              ptx::mbar_arrive_expect_tx(&sfull[si], G::BNC * kBK * 4);
               uint8_t* dst = a_stg + si * STG_BYTES;
-#pragma unroll
-              for (int j = 0; j < G::BNC / 32; j++)
-                ptx::tma_load_2d(&tm_bhi, &sfull[si], dst + j * (STG_BYTES / 4), n0 + 32 * j, kb * kBK);
+              ptx::tma_load_2d(&tm_bhi, &sfull[si], dst, n0, kb * kBK);
               if (++si == NSTG) { si = 0; sph ^= 1u; }
             }
           }
@@ -1352,6 +1351,8 @@ static int dispatch(const CUtensorMap* maps, const KParams& kp, const TcConfig& 
     if (kp.fb) {  // fused B split: TMA-staged fp32 B (2 MMA stages + 3 fp32 staging slots)
       if (cfg.cg == 2 && cfg.bn == 256 && !cfg.sep)
         return launch_variant<2, 256, false, EPI, 2, false, false, false, true>(maps, kp, cfg.max_clusters, s);
+      if (cfg.cg == 2 && cfg.bn == 224 && !cfg.sep)
+        return launch_variant<2, 224, false, EPI, 2, false, false, false, true>(maps, kp, cfg.max_clusters, s);
       set_last_error("fused B split: unsupported tile config cg=%d bn=%d sep=%d", cfg.cg, cfg.bn, cfg.sep);
       return 2;
     }
@@ -1418,7 +1419,7 @@ int launch_tc(int64_t M, int64_t N, int64_t K, const TcOperands& ops, const TcCo
                !make_tmap_f16(&maps[1], ops.a_lo, M, K, ops.lda, kBM))) ||
       (!fb && (!make_tmap_f16(&maps[2], ops.b_hi, N, K, ops.ldb, bnc) ||
                !make_tmap_f16(&maps[3], ops.b_lo, N, K, ops.ldb, bnc))) ||
-      (fb && !make_tmap_f32(&maps[2], ops.b_f32, K, N, ops.ldb_f32, kBK, 32, true))) {
+      (fb && !make_tmap_f32(&maps[2], ops.b_f32, K, N, ops.ldb_f32, kBK, bnc, false))) {
     set_last_error("cuTensorMapEncodeTiled failed (alignment: base 16 B, ld %% 8 == 0)");
     return 2;
   }
@@ -1426,7 +1427,7 @@ int launch_tc(int64_t M, int64_t N, int64_t K, const TcOperands& ops, const TcCo
     maps[0] = maps[2];
     maps[1] = maps[3];
   }
-  if (fb) maps[3] = maps[2];  // fp32 B (row-major K x N) in 32-column 128-B-swizzled boxes
+  if (fb) maps[3] = maps[2];  // fp32 B (row-major K x N) in unswizzled 64 x BNC boxes
   KParams kp = {};
   kp.K = (int)K;
   kp.fb = fb ? 1 : 0;

@@ -55,14 +55,14 @@ def test_bitexact_terms4_with_c_and_fused(oracle_lib, cfg, gen):
 
 @pytest.mark.parametrize("shape", [(256, 256, 256), (300, 300, 1000), (129, 260, 65), (512, 1024, 2048),
                                    (1000, 516, 4100)])
-@pytest.mark.parametrize("kc", [64, 256])
-def test_bitexact_fused_b(oracle_lib, shape, kc):
+@pytest.mark.parametrize("kc,bn", [(64, 256), (256, 256), (128, 224)])
+def test_bitexact_fused_b(oracle_lib, shape, kc, bn):
     """B round-split inside the GEMM (converter warpgroup transposing TMA-staged fp32 B
     tiles into the K-major stage) == the model bitwise, ragged N / K included."""
     eg = require_gpu()
     M, N, K = shape
     A, B = inputs.uniform((M, K), 40 + K), inputs.uniform((K, N), 41 + N)
-    D = _gpu(eg, A, B, None, (2, 256, 0, kc), 3, 2)
+    D = _gpu(eg, A, B, None, (2, bn, 0, kc), 3, 2)
     ref = oracle_lib.gemm_alg1_tc(A, B, terms=3, sep=0, kc=kc)
     assert np.array_equal(D.view(np.uint32), ref.view(np.uint32)), \
         "mismatches: %d" % int((D != ref).sum())

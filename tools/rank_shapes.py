@@ -35,7 +35,7 @@ def main():
             print("ranks=%d M=%5d cfg=%-18s gemm %.4f ms  %.1f TF fp32-eq" % (world, m, cfg, t, flop / t / 1e9),
                   flush=True)
         # B round-split inside the GEMM (fa bit 1): no separate B^T split pass per step
-        for cfg in [(2, 256, 0, 256), (2, 256, 0, 128)]:
+        for cfg in [(2, 256, 0, 256), (2, 224, 0, 256)]:
             egemm.set_config(*cfg)
             os.environ["EGEMM_FUSED_A"] = "2"
             t = timeit(lambda: egemm.gemm(None, B, a_split=a_split, out=D, workspace=ws))

@@ -158,7 +158,8 @@ def b32_sweep(Ms, Ns, Ks):
                 if M > 8192 and N > 1024:
                     continue
                 pick = list(egemm.query_config("gemm", M, N, K, with_fused=True))
-                cfgs = [tuple(pick)] + [(2, 256, 0, kc, 2) for kc in (64, 128, 256)]
+                cfgs = [tuple(pick)] + [(2, 256, 0, kc, 2) for kc in (64, 128, 256)] + \
+                    [(2, 224, 0, kc, 2) for kc in (128, 256)]
                 A, B = inputs.uniform((M, K), 11 + M), inputs.uniform((K, N), 13 + N)
                 Ad, Bd = torch.from_numpy(A).cuda(), torch.from_numpy(B).cuda()
                 D = torch.empty((M, N), device="cuda")
