@@ -58,16 +58,16 @@ def lib():
         L.oracle_kmeans_step.restype = None
         L.oracle_kmeans_finalize.argtypes = [P, P, I64, I64, P]
         L.oracle_kmeans_finalize.restype = None
-        L.oracle_group_sums.argtypes = [P, I64, I64, P, I64, P, P]
-        L.oracle_group_sums.restype = None
+        L.oracle_kmeans_sums.argtypes = [P, I64, I64, P, I64, P, P]
+        L.oracle_kmeans_sums.restype = None
+        L.oracle_rownorm.argtypes = [P, I64, I64, P]
+        L.oracle_rownorm.restype = None
         L.oracle_tc_mma16.argtypes = [P, P, I, ctypes.c_float, I]
         L.oracle_tc_mma16.restype = ctypes.c_float
-        L.oracle_gemm_alg1_tc.argtypes = [I64, I64, I64, P, P, P, I, I, I, P]
+        L.oracle_gemm_alg1_tc.argtypes = [I64, I64, I64, P, P, P, I, I, I64, P]
         L.oracle_gemm_alg1_tc.restype = None
-        L.oracle_tf32_parts.argtypes = [ctypes.c_float, P, P, P]
-        L.oracle_tf32_parts.restype = None
-        L.oracle_norm_step.argtypes = [I64, I64, P, P, P]
-        L.oracle_norm_step.restype = None
+        L.oracle_tc_rows.argtypes = [I64, I64, I, P, P, P, P]
+        L.oracle_tc_rows.restype = None
         L.oracle_num_threads.argtypes = []
         L.oracle_num_threads.restype = I
         _lib = L
@@ -180,19 +180,52 @@ def split_abs_bound(x):
     return np.maximum(np.abs(np.asarray(x, np.float64)) * 2.0 ** -22, 2.0 ** -25)
 
 
-def elem_bound(A, B, mma_ulps: float = 4.0, terms: int = 3):
-    """Worst-case |D_gpu - (AB)_ij| (reading R18): split residuals of both operands, the
-    dropped lo*lo term, and `mma_ulps` fp32 ulps of sum_k |a||b| per tensor-core MMA
-    (3 MMAs per 16-wide k-step) plus the promotions and the final combine."""
+MMA_ULPS = 5.25  # per MMA step of the probed primitive: 17 terms truncated (< 17 g) + RZ (< 1 ulp)
+
+
+def elem_bound(A, B, terms: int = 3, kc: int = 0, mma_ulps: float = MMA_ULPS):
+    """Worst-case |D - (AB)_ij| of Alg. 1 on the profiled tensor core (reading R18), derived
+    from the probed primitive: one MMA step truncates each of its <= 17 terms
+    onto the grid g = 2^(E-25) with 2^E <= max |term| <= S (S = sum of |terms|), then rounds
+    toward zero: error < 17 g + ulp(S) <= 5.25 * 2^-23 * S.  Inside a promotion chunk every
+    step's S is at most the chunk's sum of |products| (<= 1.01 sum_k |a_k||b_k| over the
+    chunk), so the chained steps of all chunks add <= 5.25 * 1.01 * terms * ceil(kc/16)
+    * 2^-23 * sum_k |a||b|; each promotion add, the SEP combine and + C add half an ulp.
+    Plus the split residuals of both operands and, for terms = 3, the dropped lo*lo term.
+    kc <= 0 or kc >= K: one chain over all of K (the loosest case)."""
     A = np.abs(np.asarray(A, np.float64))
     B = np.abs(np.asarray(B, np.float64))
     K = A.shape[1]
+    kce = K if (kc <= 0 or kc >= K) else kc
     eA, eB = split_abs_bound(A), split_abs_bound(B)
     absAB = A @ B
     t_split = eA @ B + A @ eB + eA @ eB
     t_lolo = 0.0 if terms == 4 else (A * 2.0 ** -11 + 2.0 ** -24) @ (B * 2.0 ** -11 + 2.0 ** -24)
-    n_round = mma_ulps * (3 * math.ceil(K / 16) + 4)
+    n_round = mma_ulps * 1.01 * terms * math.ceil(max(kce, 1) / 16) + 0.5 * (math.ceil(K / max(kce, 1)) + 2)
     return t_split + t_lolo + n_round * 2.0 ** -23 * absAB
+
+
+NORM_UNITS = 9.0  # units of 2^-24 (||q||^2 + ||x||^2) in dist_tolerance (derivation below)
+
+
+def dist_tolerance(Q, X):
+    """tau_ij for a squared distance ||q||^2 + ||x||^2 - 2 q.x computed by the method
+    (reading R18): 2 * elem_bound(q.x) + 9 * 2^-24 * (||q||^2 + ||x||^2).
+
+    The norm term (derived; pinned against the exact-rational model in
+    tests/test_kernel_model.py): the norm step adds y = -||x||^2/2 to the fp32 dot with one
+    step of the probed primitive (4 terms dot, h, m, l truncated onto g = 2^(E-25), 2^E <=
+    max(|dot|, |y|); result RZ with |result| < 2^(E+2), ulp <= 8 g): error < 12 g, doubled
+    in key = -2 acc: < 24 * 2^-25 max(|dot|, |y|) <= 6 * 2^-24 (||q||^2 + ||x||^2) since
+    |dot| <= ||q|| ||x|| <= (||q||^2 + ||x||^2)/2.  The fp32 norms add 1 unit (RN, 2^-24
+    relative each) and the final RN of ||q||^2 + key (|dist| <= 2 (||q||^2 + ||x||^2))
+    2 units: 9 units."""
+    Q = np.asarray(Q, np.float64)
+    X = np.asarray(X, np.float64)
+    eb = elem_bound(Q, X.T, terms=3, kc=0)
+    nq = (Q * Q).sum(1)[:, None]
+    nx = (X * X).sum(1)[None, :]
+    return 2.0 * eb + NORM_UNITS * 2.0 ** -24 * (nq + nx)
 
 
 # ---------------------------------------------------------------- kNN / kMeans oracles
@@ -229,6 +262,30 @@ def kmeans_step(X, C):
     return assign, sums, counts, float(inertia[0]), best
 
 
+def kmeans_sums(X, assign, kc: int):
+    """(sums fp64 [kc, d], counts int64 [kc]) of a given assignment: the plain definition,
+    sums_j = sum of (double) x_i over a_i == j in ascending i (SURVEY c-6)."""
+    X = _f32(X)
+    a = np.ascontiguousarray(assign, np.int32)
+    n, d = X.shape
+    sums = np.empty((kc, d), np.float64)
+    counts = np.empty(kc, np.int64)
+    lib().oracle_kmeans_sums(_p(X), n, d, _p(a), kc, _p(sums), _p(counts))
+    return sums, counts
+
+
+def kmeans_sums_bound(X, assign, kc: int):
+    """SURVEY c-20: any fp64 summation order of sums_j is within
+    counts_j * 2^-52 * sum_{a_i = j} |x_i| of the plain ascending-i sum (both are within
+    half that of the exact sum)."""
+    X = np.abs(np.asarray(X, np.float64))
+    a = np.asarray(assign, np.int64)
+    absx = np.zeros((kc, X.shape[1]), np.float64)
+    np.add.at(absx, a, X)
+    cnt = np.bincount(a, minlength=kc)
+    return cnt[:, None] * 2.0 ** -52 * absx
+
+
 def kmeans_finalize(sums, counts, C):
     sums = np.ascontiguousarray(sums, np.float64)
     counts = np.ascontiguousarray(counts, np.int64)
@@ -238,14 +295,29 @@ def kmeans_finalize(sums, counts, C):
 
 
 def tc_mma16(a, b, c: float = 0.0, use_c: bool = True) -> float:
-    """The profiled tcgen05 kind::f16 MMA step (C implementation) on <= 16 products."""
+    """The profiled tcgen05 MMA step (C implementation) on <= 16 products."""
     a, b = _f32(a), _f32(b)
     return float(np.float32(lib().oracle_tc_mma16(_p(a), _p(b), int(a.size), float(c), int(use_c))))
 
 
-def gemm_alg1_tc(A, B, C=None, terms: int = 3, sep: int = 0, kc: int = 64):
-    """Alg. 1 step by step on the profiled tensor-core primitive with promotion every kc
-    (reading R21): the bitwise model of what the kernel computes for (terms, sep, kc)."""
+def tc_rows(a, b, c=None):
+    """The profiled MMA step in matrix form: out[i, j] = TC(c[i, j]; sum_t a[i, t] b[j, t])
+    for a [M, n], b [N, n] with n <= 16 (c None: no addend)."""
+    a, b = _f32(a), _f32(b)
+    M, n = a.shape
+    N = b.shape[0]
+    assert b.shape[1] == n and n <= 16
+    cp = _f32(c) if c is not None else None
+    out = np.empty((M, N), np.float32)
+    lib().oracle_tc_rows(M, N, n, _p(a), _p(b), _p(cp) if cp is not None else None, _p(out))
+    return out
+
+
+def gemm_alg1_tc(A, B, C=None, terms: int = 3, sep: int = 0, kc: int = 0):
+    """Alg. 1 step by step on the profiled tensor-core primitive: per 16-wide
+    k-slice in ascending k, [lo*lo,] lo*hi, hi*lo, hi*hi chained through one fp32
+    accumulator; promotion into an fp32 total every kc k-elements (reading R21; kc = 0:
+    the paper's single chain over K); sep = 1: hi*hi in its own chain; + C at the end (R7)."""
     A, B = _f32(A), _f32(B)
     M, K = A.shape
     N = B.shape[1]
@@ -256,98 +328,12 @@ def gemm_alg1_tc(A, B, C=None, terms: int = 3, sep: int = 0, kc: int = 64):
     return D
 
 
-def rownorm_tree(X):
-    """Squared row norms in the order reading R22 fixes (the paper is silent): in fp64,
-    lane l of 32 sums x_t^2 for t = l, l+32, l+64, ... in order; the 32 lane sums are then
-    combined by the butterfly s_l <- s_l + s_(l xor o) for o = 16, 8, 4, 2, 1; the result
-    is rounded to fp32.  Every x^2 is exact in fp64."""
-    X = np.asarray(X, np.float32).astype(np.float64)
-    n, d = X.shape
-    lanes = np.zeros((n, 32), np.float64)
-    for t0 in range(0, d, 32):
-        blk = X[:, t0:t0 + 32]
-        lanes[:, :blk.shape[1]] += blk * blk  # one exact square added per lane and round
-    idx = np.arange(32)
-    for o in (16, 8, 4, 2, 1):
-        lanes = lanes + lanes[:, idx ^ o]
-    return lanes[:, 0].astype(np.float32)
-
-
-def _kc_single(d: int) -> int:
-    return ((d + 63) // 64) * 64  # one promotion chunk over the whole feature dimension
-
-
-def tf32_parts(y: float):
-    """(h, m, l) with y = h + m + l exactly, each part an exact tf32 value (reading R22)."""
-    h, m, l = ctypes.c_float(), ctypes.c_float(), ctypes.c_float()
-    lib().oracle_tf32_parts(float(np.float32(y)), ctypes.byref(h), ctypes.byref(m), ctypes.byref(l))
-    return h.value, m.value, l.value
-
-
-def norm_step(dot, nrm):
-    """acc_ij = TC(dot_ij; 1*h_j + 1*m_j + 1*l_j), (h, m, l) = tf32_parts(-nrm_j / 2): the
-    tensor-core step that adds -||x_j||^2 / 2 after the products (reading R22)."""
-    dot, nrm = _f32(dot), _f32(nrm)
-    M, N = dot.shape
-    out = np.empty((M, N), np.float32)
-    lib().oracle_norm_step(M, N, _p(dot), _p(nrm), _p(out))
-    return out
-
-
-def knn_alg1_tc(X, Q, k: int):
-    """kNN with the distance GEMM done by Alg. 1 on the profiled tensor core (R21, R22):
-    dot = gemm_alg1_tc(Q, X^T, kc = whole d); acc = norm_step(dot, ||x||^2) (one more
-    tensor-core step adding -||x_j||^2 / 2); key_ij = -2 acc_ij (exact); the k smallest
-    (key, j) ascending; dist = max(0, RN32(||q_i||^2 + key)).  The bitwise model of
-    egemm_knn; the plain definition stays `knn` (exact distances, gap rule R18)."""
-    X, Q = _f32(X), _f32(Q)
-    nx, d = X.shape
-    xn = rownorm_tree(X)
-    qn = rownorm_tree(Q).astype(np.float64)
-    dot = gemm_alg1_tc(Q, X.T, terms=3, sep=0, kc=_kc_single(d))
-    key = np.float32(-2.0) * norm_step(dot, xn)
-    order = np.lexsort((np.broadcast_to(np.arange(nx), key.shape), key), axis=1)[:, :k]
-    kk = np.take_along_axis(key, order, 1)
-    dist = (qn[:, None] + kk.astype(np.float64)).astype(np.float32)
-    return order.astype(np.int32), np.maximum(dist, np.float32(0.0))
-
-
-def kmeans_assign_alg1_tc(X, C):
-    """kMeans assignment with Alg. 1 on the profiled tensor core (R21, R22): key_ij =
-    -2 norm_step(x_i . c_j, ||c_j||^2), assign_i = the lowest j of minimal key.  Returns
-    (assign int32, best key fp32)."""
-    X, C = _f32(X), _f32(C)
-    d = X.shape[1]
-    cn = rownorm_tree(C)
-    dot = gemm_alg1_tc(X, C.T, terms=3, sep=0, kc=_kc_single(d))
-    key = np.float32(-2.0) * norm_step(dot, cn)
-    a = np.argmin(key, axis=1)  # first occurrence: ties -> lowest j
-    return a.astype(np.int32), key[np.arange(len(a)), a]
-
-
-def group_sums(X, assign, kc: int):
-    """R20-ordered fp64 sums and int64 counts of X's rows grouped by a given assignment."""
+def rownorm(X):
+    """||x_i||^2: fp64 sum of the (exact) squares in ascending t, rounded once to fp32."""
     X = _f32(X)
-    a = np.ascontiguousarray(assign, np.int32)
-    n, d = X.shape
-    sums = np.empty((kc, d), np.float64)
-    counts = np.empty(kc, np.int64)
-    lib().oracle_group_sums(_p(X), n, d, _p(a), kc, _p(sums), _p(counts))
-    return sums, counts
-
-
-def dist_tolerance(Q, X, mma_ulps: float = 4.0):
-    """tau_ij for a squared distance ||q||^2 + ||x||^2 - 2 q.x computed by the method
-    (R18): 2 * elem_bound(q.x) + 12 * 2^-24 * (||q||^2 + ||x||^2).  The norm term covers
-    the fp32 norms (1 ulp each), the R22 norm step (4 terms truncated onto 2^(E-25) with
-    2^E <= max(|q.x|, ||x||^2/2), then RZ: < 2^-22 (||q||^2 + 1.5 ||x||^2) on the key) and
-    the final RN of ||q||^2 + key (<= 2 ulps of the norms): <= 9 units, rounded up to 12."""
-    Q = np.asarray(Q, np.float64)
-    X = np.asarray(X, np.float64)
-    eb = elem_bound(Q, X.T, mma_ulps)
-    nq = (Q * Q).sum(1)[:, None]
-    nx = (X * X).sum(1)[None, :]
-    return 2.0 * eb + 12.0 * 2.0 ** -24 * (nq + nx) + 2.0 ** -20
+    out = np.empty(X.shape[0], np.float32)
+    lib().oracle_rownorm(_p(X), X.shape[0], X.shape[1], _p(out))
+    return out
 
 
 # ---------------------------------------------------------------- tensor-core models

@@ -1,7 +1,8 @@
-"""Pins for the Alg.-1-on-the-profiled-tensor-core oracle (oracle.gemm_alg1_tc, reading R21):
-the C primitive against the exact-rational Python model of the same definition, closed
-forms (integers, fp16-exact inputs, K <= 16), the element error bound, and the design's
-promotion claim (shorter chunks -> smaller error)."""
+"""Pins for the Alg.-1-on-the-profiled-tensor-core oracle (oracle.gemm_alg1_tc; Alg. 1
+P:749-755 in the paper's step order, promotion reading R21): the C primitive against the
+exact-rational Python model of the same definition, a worked example whose result depends
+on Alg. 1's order (derived by hand below), closed forms (integers, A = signed permutation,
+fp16-exact inputs, K <= 16), the element error bound, and the promotion claim."""
 import numpy as np
 import pytest
 
@@ -38,13 +39,56 @@ def test_tc_mma16_exact_when_representable(oracle_lib):
     assert oracle_lib.tc_mma16(a, b, 7.0, use_c=False) == 2 + 0.5 - 3 + 2
 
 
-@pytest.mark.parametrize("sep,kc", [(0, 64), (0, 128), (1, 256)])
+@pytest.mark.parametrize("sep,kc", [(0, 64), (0, 128), (1, 256), (0, 0), (1, 48)])
 def test_alg1_tc_integers_exact(oracle_lib, sep, kc):
     """Integer inputs |x| <= 32, K = 2048: every partial sum is an exact fp32 integer, so
     truncation never fires and the model equals the integer GEMM bitwise."""
     A, B = inputs.integers((9, 2048), 1), inputs.integers((2048, 11), 2)
     D = oracle_lib.gemm_alg1_tc(A, B, sep=sep, kc=kc)
     assert np.array_equal(D, (A.astype(np.int64) @ B.astype(np.int64)).astype(np.float32))
+
+
+def test_alg1_order_worked_example(oracle_lib):
+    """Alg. 1's order decides the result.  a = b = 1.5 + 2^-22 (fp32-exact) split into
+    hi = 1.5, lo = 2^-22 (an fp16 subnormal).  Products: hi*hi = 2.25, lo*hi = hi*lo =
+    3 * 2^-23.  In the paper's order (l.6 lo*hi, l.7 hi*lo, l.8 hi*hi) the two cross terms
+    meet first: 3*2^-23 + 3*2^-23 = 3*2^-22 exactly; the last step adds 2.25 with
+    E = e(1.5) + e(1.5) = 0, grid 2^-25, on which 3*2^-22 lies, so D = 2.25 + 3*2^-22
+    (representable: the fp32 ulp at 2.25 is 2^-22) = the exact 3-term sum.  hi*hi first
+    would round toward zero after each cross term: 2.25 + 3*2^-23 -> 2.25 + 2^-22, then
+    2.25 + 5*2^-23 -> 2.25 + 2*2^-22 -- one ulp lower.  terms = 4 puts lo*lo = 2^-44 first;
+    it is dropped by the last step's 2^-25 grid: the same D."""
+    x = np.float32(1.5 + 2.0 ** -22)
+    A, B = np.array([[x]], np.float32), np.array([[x]], np.float32)
+    want = np.float32(2.25 + 3 * 2.0 ** -22)
+    assert float(want) == 2.25 + 3 * 2.0 ** -22
+    for terms in (3, 4):
+        assert oracle_lib.gemm_alg1_tc(A, B, terms=terms)[0, 0] == want
+    # the same pair inside a longer K (zeros elsewhere) and with the promotion chunking
+    Ak = np.zeros((1, 48), np.float32)
+    Bk = np.zeros((48, 1), np.float32)
+    Ak[0, 37], Bk[37, 0] = x, x
+    for kc in (0, 16, 32):
+        assert oracle_lib.gemm_alg1_tc(Ak, Bk, kc=kc)[0, 0] == want
+
+
+def test_alg1_signed_permutation_reconstructs_hi_plus_lo(oracle_lib):
+    """A = a signed permutation scaled by powers of two: every output is one product chain
+    2^s * (lo_b ... ) with lo_a = 0, i.e. TC(TC(0; 2^s lo_b); 2^s hi_b) = 2^s (hi_b + lo_b)
+    exactly (hi + lo has <= 22 significant bits), whatever the 16-wide slice it sits in."""
+    g = inputs.rng(11)
+    n = 40
+    perm = g.permutation(n)
+    sgn = g.choice([-1.0, 1.0], n)
+    pw = 2.0 ** g.integers(-3, 4, n)
+    A = np.zeros((n, n), np.float32)
+    A[np.arange(n), perm] = sgn * pw
+    B = inputs.uniform((n, 7), 12)
+    hi, lo = oracle_lib.split(B)
+    hl = (oracle_lib.h2f(hi) + oracle_lib.h2f(lo)).astype(np.float32)
+    want = (sgn * pw)[:, None].astype(np.float32) * hl[perm]
+    for kc in (0, 16):
+        assert np.array_equal(oracle_lib.gemm_alg1_tc(A, B, kc=kc), want)
 
 
 def test_alg1_tc_fp16_inputs_k16_is_one_mma(oracle_lib):
@@ -58,24 +102,25 @@ def test_alg1_tc_fp16_inputs_k16_is_one_mma(oracle_lib):
             assert D[i, j] == np.float32(oracle_lib.tc_model(A[i], B[:, j], 0.0, "align", 2))
 
 
-@pytest.mark.parametrize("terms,sep,kc", [(3, 0, 64), (3, 0, 128), (3, 1, 256), (4, 0, 64)])
+@pytest.mark.parametrize("terms,sep,kc", [(3, 0, 64), (3, 0, 128), (3, 1, 256), (4, 0, 64), (3, 0, 0), (4, 1, 0)])
 def test_alg1_tc_within_bounds(oracle_lib, terms, sep, kc):
     A, B = inputs.uniform((48, 1000), 5), inputs.uniform((1000, 40), 6)
     C = inputs.uniform((48, 40), 7)
     D = oracle_lib.gemm_alg1_tc(A, B, C, terms=terms, sep=sep, kc=kc)
     C64 = oracle_lib.gemm64(A, B, C)
-    assert np.all(np.abs(D - C64) <= oracle_lib.elem_bound(A, B, terms=terms) + 2.0 ** -23 * np.abs(C))
+    assert np.all(np.abs(D - C64) <= oracle_lib.elem_bound(A, B, terms=terms, kc=kc) + 2.0 ** -23 * np.abs(C))
     e = oracle_lib.normwise_error(D, A, B, C64)
     en = oracle_lib.normwise_error(oracle_lib.gemm32_naive(A, B, C), A, B, C64)
-    assert e <= 2 * en
+    if kc:  # the single chain (kc = 0) is the unpromoted paper design: bound only
+        assert e <= 2 * en
 
 
 def test_alg1_tc_promotion_reduces_error(oracle_lib):
-    """with the truncating primitive a single accumulator over all of K is
+    """with the truncating primitive the paper's single chain over all of K is
     several times worse than naive fp32; promotion every 64 k brings it below."""
     A, B = inputs.uniform((24, 4096), 8), inputs.uniform((4096, 24), 9)
     C64 = oracle_lib.gemm64(A, B)
-    e_long = oracle_lib.normwise_error(oracle_lib.gemm_alg1_tc(A, B, kc=4096), A, B, C64)
+    e_long = oracle_lib.normwise_error(oracle_lib.gemm_alg1_tc(A, B, kc=0), A, B, C64)
     e_64 = oracle_lib.normwise_error(oracle_lib.gemm_alg1_tc(A, B, kc=64), A, B, C64)
     en = oracle_lib.normwise_error(oracle_lib.gemm32_naive(A, B), A, B, C64)
     assert e_long > 2 * en and e_64 < en

@@ -66,34 +66,65 @@ def test_kmeans_integer_sums_exact_and_empty_cluster(oracle_lib):
     assert np.array_equal(newc[1], C[1])  # empty cluster keeps its centroid (R12)
 
 
-def test_kmeans_sums_fixed_order_r20(oracle_lib):
-    """Reading R20: group members in ascending i, chunks of 256 summed sequentially, then
-    the chunk sums sequentially -- checked against a pure-Python rendering of that order
-    and against the exact rational sum (fp64 rounding bound)."""
+def test_kmeans_sums_plain_order(oracle_lib):
+    """SURVEY c-6: sums_j = sum of (double) x_i over the members of j in ascending i.
+    Closed form: members 2^53, 1, -2^53 (all fp32) in that order give (2^53 + 1) - 2^53 = 0
+    (2^53 + 1 rounds to the even 2^53), where any order adding the 1 last would give 1.
+    And on mixed data the sums are within n 2^-52 sum |x| of the exact rational sums."""
     from fractions import Fraction
+    X = np.array([[2.0 ** 53], [1.0], [-2.0 ** 53]], np.float32)
+    _, sums, counts, _, _ = oracle_lib.kmeans_step(X, np.zeros((1, 1), np.float32))
+    assert counts[0] == 3 and sums[0, 0] == 0.0
     X, lab, cent = inputs.mixture(3000, 3, 2, 9, sigma=0.5)
     a, sums, counts, _, _ = oracle_lib.kmeans_step(X, cent)
     for j in range(2):
         mem = [i for i in range(3000) if a[i] == j]
         assert counts[j] == len(mem) and len(mem) > 600
         for t in range(3):
-            tot = 0.0
-            for c0 in range(0, len(mem), 256):
-                part = 0.0
-                for i in mem[c0:c0 + 256]:
-                    part = part + float(X[i, t])
-                tot = tot + part
-            assert sums[j, t] == tot
             exact = sum(Fraction(float(X[i, t])) for i in mem)
             mag = sum(abs(float(X[i, t])) for i in mem)
             assert abs(Fraction(sums[j, t]) - exact) <= Fraction(len(mem) * 2.0 ** -52 * mag)
 
 
-def test_group_sums_equals_step_sums(oracle_lib):
-    X, _, cent = inputs.mixture(5000, 6, 3, 10, sigma=0.3)
-    a, sums, counts, _, _ = oracle_lib.kmeans_step(X, cent)
-    s2, c2 = oracle_lib.group_sums(X, a, 3)
-    assert np.array_equal(s2, sums) and np.array_equal(c2, counts)
+def test_rownorm_plain_definition(oracle_lib):
+    """||x||^2 = fp32(fp64 sum of squares in ascending t).  Closed form for the order:
+    (2^12, 1, 2^-15 x 4): in ascending t the fp64 sum is 2^24 + 1 (each 2^-30 falls below
+    half an fp64 ulp of 2^24), an fp32 tie that rounds to the even 2^24; the reverse order
+    keeps 4 * 2^-30 = 2^-28 and would round up to 2^24 + 2.  Integer rows are exact; random
+    rows equal the correctly rounded exact value (the fp64 error, <= d 2^-53 of the sum,
+    cannot move an fp32 rounding except within that distance of a midpoint)."""
+    from fractions import Fraction
+    x = np.array([[2.0 ** 12, 1.0] + [2.0 ** -15] * 4], np.float32)
+    assert oracle_lib.rownorm(x)[0] == np.float32(2.0 ** 24)
+    assert oracle_lib.rownorm(x[:, ::-1])[0] == np.float32(2.0 ** 24 + 2)
+    g = inputs.rng(2201)
+    Xi = g.integers(-40, 41, (50, 300)).astype(np.float32)
+    assert np.array_equal(oracle_lib.rownorm(Xi), (Xi.astype(np.int64) ** 2).sum(1).astype(np.float32))
+    for d in (1, 33, 128, 257):
+        X = g.uniform(-2, 2, (200, d)).astype(np.float32)
+        got = oracle_lib.rownorm(X)
+        for r in range(X.shape[0]):
+            ex = sum(Fraction(float(v)) ** 2 for v in X[r])
+            want = np.float32(oracle_lib.oracle._round_f32(ex, "rn"))  # correctly rounded
+            w = Fraction(float(want))
+            mids = [(w + Fraction(float(np.nextafter(want, np.float32(t))))) / 2 for t in (0, np.inf)]
+            if min(abs(ex - m) for m in mids) > Fraction(d) * Fraction(2.0 ** -52) * ex:
+                assert got[r] == want, (d, r)
+
+
+def test_sqdist_closed_forms(oracle_lib):
+    """Integer rows: exact integer distances; d = 1: (q - x)^2; symmetric in its arguments."""
+    g = inputs.rng(2210)
+    X = g.integers(-50, 51, (30, 17)).astype(np.float32)
+    Q = g.integers(-50, 51, (9, 17)).astype(np.float32)
+    D = oracle_lib.sqdist(X, Q)
+    ref = ((Q[:, None, :].astype(np.int64) - X[None].astype(np.int64)) ** 2).sum(2)
+    assert np.array_equal(D, ref.astype(np.float64))
+    x1, q1 = np.float32([[0.1], [-3.5]]), np.float32([[2.25]])
+    assert np.array_equal(oracle_lib.sqdist(x1, q1)[0],
+                          [(2.25 - float(np.float32(0.1))) ** 2, (2.25 + 3.5) ** 2])
+    U, V = inputs.uniform((12, 8), 2211), inputs.uniform((7, 8), 2212)
+    assert np.array_equal(oracle_lib.sqdist(U, V), oracle_lib.sqdist(V, U).T)
 
 
 def test_kmeans_ties_lowest_index(oracle_lib):
@@ -154,96 +185,3 @@ def test_tc_models_reduce_to_textbook_cases(oracle_lib):
     a3 = [2.0 ** -14] + [0.0] * 15
     b3 = [2.0 ** -14] + [0.0] * 15
     assert m(a3, b3, 1.0, "align", 3) == 1.0 and m(a3, b3, 1.0, "rn") == 1.0
-
-
-# ------------------------------------------------------------------ R22 bitwise app models
-def test_rownorm_tree_vs_exact(oracle_lib):
-    """rownorm_tree (R22) is within 1 fp32 ulp of the correctly rounded exact sum of squares
-    and equal to it for nearly all rows; integer rows are exact."""
-    from fractions import Fraction
-    g = inputs.rng(2201)
-    for d in (1, 33, 100, 128, 257):
-        X = g.uniform(-2, 2, (300, d)).astype(np.float32)
-        tree = oracle_lib.rownorm_tree(X)
-        exact = np.array([float(sum(Fraction(float(v)) ** 2 for v in row)) for row in X],
-                         np.float64).astype(np.float32)
-        ulp = np.spacing(exact)
-        assert np.all(np.abs(tree.astype(np.float64) - exact) <= ulp)
-        assert np.mean(tree == exact) >= 0.97
-    Xi = g.integers(-40, 41, (50, 300)).astype(np.float32)
-    assert np.array_equal(oracle_lib.rownorm_tree(Xi), (Xi.astype(np.int64) ** 2).sum(1).astype(np.float32))
-
-
-def test_knn_alg1_tc_integer_data_is_exact(oracle_lib):
-    """On small integers every step is exact, so the TC model kNN equals the exact kNN."""
-    g = inputs.rng(2202)
-    X = g.integers(-4, 5, (400, 20)).astype(np.float32)
-    Q = g.integers(-4, 5, (37, 20)).astype(np.float32)
-    i1, d1 = oracle_lib.knn_alg1_tc(X, Q, 9)
-    i0, d0 = oracle_lib.knn(X, Q, 9)
-    assert np.array_equal(i1, i0) and np.array_equal(d1.astype(np.float64), d0)
-
-
-def test_knn_alg1_tc_agrees_with_exact_where_gap(oracle_lib):
-    g = inputs.rng(2203)
-    X, Q = g.uniform(-1, 1, (600, 48)), g.uniform(-1, 1, (40, 48))
-    i1, _ = oracle_lib.knn_alg1_tc(X, Q, 8)
-    D = oracle_lib.sqdist(X, Q)
-    for r in range(Q.shape[0]):
-        o = np.argsort(D[r], kind="stable")
-        if D[r, o[8]] - D[r, o[7]] > 1e-5:  # far above the method's error bound here
-            assert set(i1[r]) == set(o[:8])
-
-
-def test_kmeans_assign_alg1_tc_integer_and_ties(oracle_lib):
-    g = inputs.rng(2204)
-    X = g.integers(-3, 4, (500, 12)).astype(np.float32)
-    C = g.integers(-3, 4, (17, 12)).astype(np.float32)
-    C[9] = C[4]  # duplicate centroid: ties must go to the lower index
-    a, best = oracle_lib.kmeans_assign_alg1_tc(X, C)
-    D = ((X[:, None, :].astype(np.int64) - C[None].astype(np.int64)) ** 2).sum(2)
-    assert np.array_equal(a, np.argmin(D, 1))
-    assert not np.any(a == 9)
-    cn = (C.astype(np.int64) ** 2).sum(1)
-    assert np.array_equal(best.astype(np.int64), (D - (X.astype(np.int64) ** 2).sum(1)[:, None])[np.arange(500), a])
-    assert np.all(cn[a] - 2 * (X.astype(np.int64) * C[a].astype(np.int64)).sum(1) == best)
-
-
-def _low13_zero(x):
-    return (np.asarray(x, np.float32).view(np.uint32) & 0x1FFF) == 0
-
-
-def test_tf32_parts_exact_decomposition(oracle_lib):
-    """R22 norm parts: y = h + m + l exactly (checked in fp64), every part an exact tf32
-    value (13 low mantissa bits zero), |m| < 2^-10 |h| and |l| < 2^-20 |h|; tf32-exact y
-    gives m = l = 0."""
-    g = inputs.rng(2205)
-    ys = np.concatenate([(g.uniform(-1, 1, 4000) * 2.0 ** g.integers(-30, 40, 4000)),
-                         [0.0, -0.0, 1.0, -3.5, 65504.0, 1e30, -1e-30]]).astype(np.float32)
-    for y in ys:
-        h, m, l = oracle_lib.tf32_parts(y)
-        assert float(h) + float(m) + float(l) == float(y)
-        assert _low13_zero([h, m, l]).all()
-        if h != 0:
-            assert abs(m) < 2.0 ** -10 * abs(h) and abs(l) < 2.0 ** -20 * abs(h)
-    for y in np.float32([1.0, 0.75, -1024.0, 3.0 * 2 ** 20]):
-        assert oracle_lib.tf32_parts(y)[1:] == (0.0, 0.0)
-
-
-def test_norm_step_matches_rational_model_and_exact_cases(oracle_lib):
-    """norm_step = one profiled tensor-core step on (1, 1, 1) x (h, m, l) with C = dot:
-    checked against the exact-rational tc_model rendering, and exact (= dot - nrm / 2) when
-    that value is representable on the step's grid (integers)."""
-    g = inputs.rng(2206)
-    dot = (g.uniform(-1, 1, (7, 50)) * 2.0 ** g.integers(-4, 12, (7, 50))).astype(np.float32)
-    nrm = (g.uniform(0, 1, 50) * 2.0 ** g.integers(-6, 14, 50)).astype(np.float32)
-    out = oracle_lib.norm_step(dot, nrm)
-    for i in range(7):
-        for j in range(50):
-            parts = np.float32(oracle_lib.tf32_parts(np.float32(-0.5) * nrm[j]))
-            ref = oracle_lib.tc_model(np.ones(3, np.float32), parts, float(dot[i, j]), "align", 2, "fields")
-            assert out[i, j] == np.float32(ref), (i, j)
-    di = g.integers(-5000, 5000, (9, 40)).astype(np.float32)
-    ni = g.integers(0, 20000, 40).astype(np.float32)
-    assert np.array_equal(oracle_lib.norm_step(di, ni).astype(np.float64),
-                          di.astype(np.float64) - 0.5 * ni.astype(np.float64))
