@@ -112,9 +112,12 @@ size_t egemm_gemm_workspace_size(int64_t M, int64_t N, int64_t K, int a_presplit
  * (row-major, strides lda / ldb / ldd in elements; host memory should be pinned for the
  * copies to be asynchronous).  B is copied and split once; row chunks of A are then copied
  * in, split, multiplied and copied out double-buffered, so both PCIe directions overlap the
- * tensor-core work.  Uses two internal copy streams created once per device (the only
- * resources the library creates).  Asynchronous w.r.t. the host like the other calls:
- * D_host is complete when `stream` has completed.  K must be > 0.
+ * tensor-core work.  Uses two internal copy streams and events created once per device (the
+ * only resources the library creates); concurrent calls on the same device from several
+ * host threads are serialised by a per-device lock held while a call enqueues its work and
+ * ordered on the device (a call's copies wait for the previous call's last kernel).
+ * Asynchronous w.r.t. the host like the other calls: D_host is complete when `stream` has
+ * completed.  K must be > 0.
  */
 int egemm_gemm_host(int64_t M, int64_t N, int64_t K, const float* A_host, int64_t lda,
                     const float* B_host, int64_t ldb, float* D_host, int64_t ldd, int terms,
@@ -129,19 +132,35 @@ size_t egemm_gemm_host_workspace_size(int64_t M, int64_t N, int64_t K);
  * ascending by (dist, j), dist clamped to >= 0; self matches are kept (reading R11).
  * Arithmetic (reading R22): q.x_j by Alg. 1 on the tensor core (one promotion
  * chunk over d), then one more tensor-core step adds -||x_j||^2/2 (three exact tf32 parts
- * times ones), key = -2 * that accumulator, dist = max(0, fp32(||q||^2 + key)); the results
- * are bitwise reproducible and equal to the oracle's model of these steps.
+ * times ones), key = -2 * that accumulator, dist = max(0, fp32(||q||^2 + key)); the norms
+ * are fp32(fp64 sum of squares in ascending t).  Results are bitwise reproducible (the
+ * regression model is tests/kernel_model.py).
  *  X     : the references, trans 0.  Either fp32 rows (then split and normed on the fly)
  *          or the "index" from egemm_knn_index: pre-split hi/lo + x_norms (f32 may be NULL).
  *  x_norms : nullable nx fp32 ||x_j||^2 (fp64-accumulated, from egemm_knn_index).
  *  Q     : fp32 query rows (trans 0, ld >= d), split and normed on the fly.
- *  k     : 1 <= k <= 16 and k <= nx.
+ *  k     : 1 <= k <= 64 and k <= nx (register lists of 16, 32 or 64 entries per thread).
  *  out_idx  : nq x k int32;  out_dist : nq x k fp32.
  */
 int egemm_knn(egemm_operand_t X, const float* x_norms, int64_t nx, egemm_operand_t Q, int64_t nq,
               int64_t d, int k, int32_t* out_idx, float* out_dist, void* workspace,
               size_t workspace_bytes, void* stream);
 size_t egemm_knn_workspace_size(int64_t nx, int64_t nq, int64_t d, int k, int x_presplit);
+
+/*
+ * Merge of sorted partial kNN lists (the second step of the GEMM-based kNN when the
+ * references are split -- across the N-slices of one egemm_knn call, or across ranks that
+ * each hold a shard of the references): for each query i, the k smallest
+ * (key, idx) pairs, ascending, of the union of n_lists lists
+ *   keys[l][i][0 .. k_in), idx[l][i][0 .. k_in)   (each list ascending by (key, idx)),
+ * with idx < 0 (or INT32_MAX) marking an empty slot.  Indices must be distinct across
+ * lists (disjoint reference sets).  out_key[i][t] = key, or max(0, qnorm[i] + key) when
+ * qnorm != NULL (the kNN distance, reading R11); empty output slots get idx -1, key +inf.
+ *  n_lists in [1, 64], 1 <= k <= k_in * n_lists, k <= 64, k_in <= 1024.  One warp per query;
+ *  exact (each pair's rank is counted, no approximation).
+ */
+int egemm_knn_merge(const float* keys, const int32_t* idx, int n_lists, int64_t nq, int k_in, int k,
+                    const float* qnorm, int32_t* out_idx, float* out_key, void* stream);
 
 /* kNN index build: round-split of the references X[nx x d] (row stride ldx) into K-major
  * hi/lo (row stride ld_split, a multiple of 8) and their squared norms ||x_j||^2
@@ -168,21 +187,46 @@ size_t egemm_kmeans_workspace_size(int64_t n, int64_t d, int64_t kc, int x_presp
 int egemm_kmeans_finalize(const double* sums, const int64_t* counts, int64_t kc, int64_t d,
                           float* centroids, void* stream);
 
-/* Tile configuration used by the next calls of this thread (the tuning-table override).
- * cg in {1,2}, bn in {128,256}, sep in {0,1}, kc a multiple of 64 (0 = default).
- * Pass all zeros to restore the tuning table.  Returns EGEMM_ERR_UNSUPPORTED for a
- * combination the library was not built with. */
+/*
+ * A launch configuration: the value of one tuning-table entry, and the
+ * thread-local override of the table.  0 (or -1 where noted) = "not set / the table's".
+ *  cg, bn, sep : tile = cta_group (1, 2), MMA N per tile (128, 224, 256), separate hi*hi
+ *                accumulator (0, 1).  Valid: (2,256,0) (2,224,0) (2,128,0|1) (1,128,0|1).
+ *  kc          : promotion interval in k (multiple of 64).
+ *  stages      : smem ring depth (2..4, per tile what fits 227 KiB; 0 = default).
+ *  fused       : -1 table; 0 pre-split operands; 1 fp32 A split inside the GEMM kernel;
+ *                2 fp32 B split inside the GEMM kernel (a-2 fused modes).
+ *  terms       : 3 or 4 products (0 = the call's / table's).
+ *  n_slices    : kNN N-slices per query block (1..16; 0 = table / wave-balance formula).
+ *  epi_warps   : kMeans epilogue warps (8 or 16; 0 = table / 16).
+ *  a_resident  : kNN query tile resident in smem (-1 = when d <= 128, 0 = never).
+ *  pace        : k-pacing of STORE GEMMs (-1 = table / on, 0 = off).
+ *  max_clusters: persistent clusters launched (0 = one per SM pair / SM).
+ */
+typedef struct {
+  int cg, bn, sep, kc, stages, fused, terms, n_slices, epi_warps, a_resident, pace, max_clusters;
+} egemm_config_t;
+
+/* Thread-local override of the tuning table for the next calls of this thread: fields set
+ * in *cfg replace the table's (a tile override also selects the pre-split path unless
+ * `fused` is set).  NULL restores the table.  EGEMM_ERR_UNSUPPORTED for a value the library
+ * was not built with. */
+int egemm_set_config_ex(const egemm_config_t* cfg);
+/* Shorthand: tile (cg, bn, sep) and kc only (fused = 0); all zeros restores the table. */
 int egemm_set_config(int cg, int bn, int sep, int kc);
+/* The configuration the library would use for op (0 gemm with a pre-split B, 1 knn,
+ * 2 kmeans, 3 gemm whose B is fp32, split inside the call) at (M, N, K) = (rows of A /
+ * queries / points, columns of B / references / centroids, K / d), after the table and
+ * this thread's override. */
+int egemm_query_config_ex(int op, int64_t M, int64_t N, int64_t K, egemm_config_t* out);
 
 /* The measured configuration table (replaces the paper's analytic model,
  * Sec. 6): path of the loaded tune_table.json ("" = built-in defaults) and,
  * through *entries (nullable), its number of entries.  Host-only. */
 const char* egemm_tune_table(int* entries);
-/* The configuration the library would use for op (0 gemm with a pre-split B, 1 knn,
- * 2 kmeans, 3 gemm whose B is fp32 K x N row-major, i.e. its round-split is part of the
- * call) at M, N, K (after table, egemm_set_config and EGEMM_* overrides).  *fused_a
- * (nullable): 1 when an fp32 row-major A would be round-split inside the GEMM kernel, 2 when
- * (op 3) the fp32 B would be round-split inside the GEMM kernel (a-2 fused modes), else 0. */
+/* The (cg, bn, sep, kc, fused) part of egemm_query_config_ex.  *fused_a (nullable): 1 when
+ * an fp32 row-major A would be round-split inside the GEMM kernel, 2 when (op 3) the fp32 B
+ * would be, else 0. */
 int egemm_query_config(int op, int64_t M, int64_t N, int64_t K, int* cg, int* bn, int* sep,
                        int* kc, int* fused_a);
 
@@ -216,9 +260,9 @@ int egemm_tc_probe(int kind, int N, int K, const void* A, const void* B, const f
  * number of launches.  reset != 0 zeroes the sums after reading.  Synchronous. */
 int egemm_debug_clock_stats(double* mhz, double* cycles_per_launch, double* launches, int reset);
 
-/* Debug: a device event counter bumped by diagnostic kernel modes (EGEMM_DEBUG_MODE bit 256:
- * kNN candidate-path entries, one per warp and 32-column group).  reset != 0 zeroes it
- * after reading.  Synchronous. */
+/* Debug: a device event counter bumped by diagnostic kernel modes (a library built with
+ * EGEMM_DIAG=1, EGEMM_DEBUG_MODE bit 256: kNN candidate-path entries, one per warp and
+ * 32-column group).  reset != 0 zeroes it after reading.  Synchronous. */
 int egemm_debug_counter(unsigned long long* value, int reset);
 
 #ifdef __cplusplus

@@ -7,6 +7,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <mutex>
+#include <thread>
 #include "../../include/egemm.h"
 #include "egemm_internal.h"
 
@@ -35,17 +36,43 @@ static bool device_ok() {
   return major == 10 && minor == 0;
 }
 
-// ------------------------------------------------------------------ tuning table
-// Measured choices (tune/README in DESIGN.md): key = (op, M/N/K buckets).
-struct Override {
-  int cg = 0, bn = 0, sep = 0, kc = 0;
-};
-static thread_local Override g_override;
-
+// ------------------------------------------------------------------ environment knobs
 static int env_int(const char* name, int dflt) {
   const char* v = getenv(name);
   return (v && *v) ? atoi(v) : dflt;
 }
+
+const Knobs& knobs() {
+  static Knobs k;
+  static std::once_flag once;
+  std::call_once(once, [] {
+    k.pace_e = env_int("EGEMM_PACE_E", 0);
+    k.pace_s = env_int("EGEMM_PACE_S", 0);
+    k.no_pace = env_int("EGEMM_NO_PACE", 0) == 1;
+    k.band = env_int("EGEMM_BAND", 0);
+    k.a_pf = env_int("EGEMM_A_PREFETCH", 2);
+    if (k.a_pf < 0) k.a_pf = 0;
+    k.a_staged = env_int("EGEMM_A_STAGED", 1);
+    k.as_pf = env_int("EGEMM_AS_PREFETCH", 0);
+    if (k.as_pf < 0) k.as_pf = 0;
+    k.host_chunk = env_int("EGEMM_HOST_CHUNK", 0);
+#if EGEMM_DIAG
+    k.dbg_no_tma = env_int("EGEMM_DEBUG_NO_TMA", 0) == 1;
+    k.dbg_no_epi = env_int("EGEMM_DEBUG_NO_EPI", 0) == 1;
+    k.dbg_mode = env_int("EGEMM_DEBUG_MODE", 0);
+#else
+    k.dbg_no_tma = k.dbg_no_epi = k.dbg_mode = 0;
+#endif
+  });
+  return k;
+}
+
+// ------------------------------------------------------------------ tuning table
+// Measured choices (tools/tune_sweep.py -> tune_table.json): key = (op,
+// M/N/K buckets), value = the launch configuration.  The thread-local override
+// (egemm_set_config / egemm_set_config_ex) replaces what it sets.
+static thread_local egemm_config_t g_override = {};
+static thread_local bool g_override_on = false;
 
 static bool fused_a_supported(const TcConfig& c) {
   return (c.cg == 2 && c.bn == 256 && !c.sep) || (c.cg == 2 && c.bn == 128) ||
@@ -62,52 +89,64 @@ static bool fused_b_supported(const TcConfig& c) {
 }
 
 // b_f32: a STORE GEMM whose B is fp32 (split inside the call): the table's "gemm_b32" rows
-// (which may pick the fused-B kernel) first, then the "gemm" rows.
+// (which may pick the fused-B kernel) first, then the "gemm" rows.  terms: the call's
+// argument (0 = the table's choice).
 static TcConfig choose_config(int epi_kind, int64_t M, int64_t N, int64_t K, int terms,
                               bool b_f32 = false) {
   TcConfig c = {};
-  c.terms = terms;
+  c.terms = 3;
   c.max_clusters = 0;
-  // default: CTA pair, 256 x 256 tiles, single accumulator in ping-pong
-  c.cg = 2;
+  c.cg = 2;  // default: CTA pair, 256 x 256 tiles, single accumulator in ping-pong
   c.bn = 256;
   c.sep = 0;
-  // promotion every 64 k (one stage): measured fastest after the barrier fix and the most
-  // accurate single-accumulator setting (tools/error_sweep.py)
-  c.kc = 64;
+  c.kc = 64;  // promotion every 64 k: the most accurate single-accumulator setting
+  c.ares = -1;
+  c.pace = 1;
   if (epi_kind == EPI_STORE && M <= 128) { c.cg = 1; c.bn = 128; c.sep = 1; }
-  {  // the measured table (tools/tune_sweep.py -> tune_table.json) overrides the defaults
-    int cg, bn, sep, kc, fa;
-    bool hit = epi_kind == EPI_STORE && b_f32 &&
-               tune_lookup(kOpGemmB32, M, N, K, &cg, &bn, &sep, &kc, &fa) && valid_config(cg, bn, sep);
-    if (!hit) hit = tune_lookup(epi_kind, M, N, K, &cg, &bn, &sep, &kc, &fa) && valid_config(cg, bn, sep);
+  {
+    TuneEntry t;
+    bool hit = epi_kind == EPI_STORE && b_f32 && tune_lookup(kOpGemmB32, M, N, K, &t) &&
+               valid_config(t.cg, t.bn, t.sep);
+    if (!hit) hit = tune_lookup(epi_kind, M, N, K, &t) && valid_config(t.cg, t.bn, t.sep);
     if (hit) {
-      c.cg = cg;
-      c.bn = bn;
-      c.sep = sep;
-      c.fa = fa;
-      if (kc > 0) c.kc = kc;
+      c.cg = t.cg;
+      c.bn = t.bn;
+      c.sep = t.sep;
+      c.fa = t.fa;
+      if (t.kc > 0) c.kc = t.kc;
+      if (t.terms == 3 || t.terms == 4) c.terms = t.terms;
+      c.stages = t.stages;
+      c.nslices = t.nslices;
+      c.nepi = t.nepi;
+      if (t.ares >= 0) c.ares = t.ares;
     }
   }
+  if (terms == 3 || terms == 4) c.terms = terms;  // the call's explicit term count wins
   if (epi_kind != EPI_STORE) c.kc = (int)(((K + 63) / 64) * 64);
-  // thread-local API override, then environment (experiments)
-  if (g_override.cg) {
-    c.cg = g_override.cg;
-    c.bn = g_override.bn;
-    c.sep = g_override.sep;
-    c.fa = 0;  // an explicit tile override measures the pre-split path unless EGEMM_FUSED_A
+  if (g_override_on) {  // thread-local API override
+    const egemm_config_t& o = g_override;
+    if (o.cg) {
+      c.cg = o.cg;
+      c.bn = o.bn;
+      c.sep = o.sep;
+      c.fa = 0;  // an explicit tile override measures the pre-split path unless `fused` says
+      c.stages = 0;
+    }
+    if (o.kc && epi_kind == EPI_STORE) c.kc = o.kc;
+    if (o.fused >= 0) c.fa = o.fused;
+    if (o.stages) c.stages = o.stages;
+    if (o.terms == 3 || o.terms == 4) c.terms = o.terms;
+    if (o.n_slices) c.nslices = o.n_slices;
+    if (o.epi_warps) c.nepi = o.epi_warps;
+    if (o.a_resident >= 0) c.ares = o.a_resident;
+    if (o.pace >= 0) c.pace = o.pace;
+    if (o.max_clusters) c.max_clusters = o.max_clusters;
   }
-  if (g_override.kc && epi_kind == EPI_STORE) c.kc = g_override.kc;
-  c.cg = env_int("EGEMM_CG", c.cg);
-  c.bn = env_int("EGEMM_BN", c.bn);
-  c.sep = env_int("EGEMM_SEP", c.sep);
-  if (epi_kind == EPI_STORE) c.kc = env_int("EGEMM_KC", c.kc);
-  c.max_clusters = env_int("EGEMM_MAX_CLUSTERS", 0);
-  c.fa = env_int("EGEMM_FUSED_A", c.fa);
   if (c.kc < 64) c.kc = 64;
   c.kc = (c.kc / 64) * 64;
   if (epi_kind != EPI_STORE) {  // kNN / kMeans: one accumulator (the norm MMA adds into it)
     c.sep = 0;
+    c.terms = 3;
     if (!((c.cg == 2 && c.bn == 256) || (c.cg == 1 && c.bn == 128))) { c.cg = 2; c.bn = 256; }
   }
   return c;
@@ -208,20 +247,45 @@ const char* egemm_tune_table(int* entries) {
   return tune_table_path();
 }
 
+static int knn_slices(int64_t nq, int64_t nx, int cg, int bn);
+
+static void to_public(const TcConfig& c, int op, egemm_config_t* o) {
+  const bool b32 = op == kOpGemmB32;
+  const bool store = op == EPI_STORE || b32;
+  o->cg = c.cg;
+  o->bn = c.bn;
+  o->sep = c.sep;
+  o->kc = c.kc;
+  o->stages = c.stages;
+  const int a = (store && (c.fa & 1) && fused_a_supported(c)) ? 1 : 0;
+  o->fused = a ? 1 : (b32 && (c.fa & 2) && fused_b_supported(c)) ? 2 : 0;
+  o->terms = c.terms;
+  o->n_slices = c.nslices;
+  o->epi_warps = op == EPI_KMEANS ? (c.nepi == 8 ? 8 : 16) : 0;
+  o->a_resident = c.ares;
+  o->pace = c.pace;
+  o->max_clusters = c.max_clusters;
+}
+
 int egemm_query_config(int op, int64_t M, int64_t N, int64_t K, int* cg, int* bn, int* sep,
                        int* kc, int* fused_a) {
   if (op < 0 || op > 3 || !cg || !bn || !sep || !kc) return EGEMM_ERR_INVALID_ARG;
+  egemm_config_t o;
+  egemm_query_config_ex(op, M, N, K, &o);
+  *cg = o.cg;
+  *bn = o.bn;
+  *sep = o.sep;
+  *kc = o.kc;
+  if (fused_a) *fused_a = o.fused;
+  return EGEMM_OK;
+}
+
+int egemm_query_config_ex(int op, int64_t M, int64_t N, int64_t K, egemm_config_t* out) {
+  if (op < 0 || op > 3 || !out) return EGEMM_ERR_INVALID_ARG;
   const bool b32 = op == kOpGemmB32;
-  TcConfig c = choose_config(b32 ? EPI_STORE : op, M, N, K, 3, b32);
-  *cg = c.cg;
-  *bn = c.bn;
-  *sep = c.sep;
-  *kc = c.kc;
-  if (fused_a) {
-    const bool store = op == EPI_STORE || b32;
-    const int a = (store && (c.fa & 1) && fused_a_supported(c)) ? 1 : 0;
-    *fused_a = a ? 1 : (b32 && (c.fa & 2) && fused_b_supported(c)) ? 2 : 0;
-  }
+  TcConfig c = choose_config(b32 ? EPI_STORE : op, M, N, K, 0, b32);
+  if (op == EPI_KNN && c.nslices <= 0) c.nslices = knn_slices(M, N, c.cg, c.bn);
+  to_public(c, op, out);
   return EGEMM_OK;
 }
 
@@ -263,18 +327,37 @@ int egemm_debug_counter(unsigned long long* value, int reset) {
 }
 
 int egemm_set_config(int cg, int bn, int sep, int kc) {
-  if (cg == 0 && bn == 0 && sep == 0 && kc == 0) {
-    g_override = Override();
+  if (cg == 0 && bn == 0 && sep == 0 && kc == 0) return egemm_set_config_ex(nullptr);
+  egemm_config_t o = {};
+  o.cg = cg;
+  o.bn = bn;
+  o.sep = sep;
+  o.kc = kc;
+  o.fused = -1;
+  o.a_resident = -1;
+  o.pace = -1;
+  return egemm_set_config_ex(&o);
+}
+
+int egemm_set_config_ex(const egemm_config_t* cfg) {
+  if (!cfg) {
+    g_override = egemm_config_t{};
+    g_override_on = false;
     return EGEMM_OK;
   }
-  if (!valid_config(cg, bn, sep) || kc < 0 || (kc % 64) != 0) {
-    set_last_error("unsupported config cg=%d bn=%d sep=%d kc=%d", cg, bn, sep, kc);
+  const egemm_config_t& o = *cfg;
+  if ((o.cg && !valid_config(o.cg, o.bn, o.sep)) || o.kc < 0 || (o.kc % 64) != 0 ||
+      o.fused < -1 || o.fused > 2 || o.stages < 0 || o.stages > 4 ||
+      !(o.terms == 0 || o.terms == 3 || o.terms == 4) || o.n_slices < 0 || o.n_slices > 16 ||
+      !(o.epi_warps == 0 || o.epi_warps == 8 || o.epi_warps == 16) || o.a_resident < -1 ||
+      o.a_resident > 1 || o.pace < -1 || o.pace > 1 || o.max_clusters < 0) {
+    set_last_error("unsupported config cg=%d bn=%d sep=%d kc=%d fused=%d stages=%d terms=%d "
+                   "n_slices=%d epi_warps=%d", o.cg, o.bn, o.sep, o.kc, o.fused, o.stages, o.terms,
+                   o.n_slices, o.epi_warps);
     return EGEMM_ERR_UNSUPPORTED;
   }
-  g_override.cg = cg;
-  g_override.bn = bn;
-  g_override.sep = sep;
-  g_override.kc = kc;
+  g_override = o;
+  g_override_on = true;
   return EGEMM_OK;
 }
 
@@ -416,7 +499,7 @@ int egemm_gemm(int64_t M, int64_t N, int64_t K, egemm_operand_t A, egemm_operand
 // tcgen05 GEMM (caller stream) -> D2H (second copy stream), double-buffered, so the two
 // PCIe directions and the GPU work overlap.  Streams/events are created once per device.
 static int64_t host_chunk_rows(int64_t M) {
-  const int forced = env_int("EGEMM_HOST_CHUNK", 0);  // experiments
+  const int forced = knobs().host_chunk;  // experiments
   if (forced > 0) return forced > M ? M : forced;
   int64_t c = ((M / 8 + 255) / 256) * 256;
   if (c < 256) c = 256;
@@ -426,8 +509,9 @@ static int64_t host_chunk_rows(int64_t M) {
 
 struct HostPipe {
   bool init = false;
+  std::mutex mu;  // held by one call's whole enqueue sequence (the events are shared)
   cudaStream_t s_in = nullptr, s_out = nullptr;
-  cudaEvent_t ev_start, ev_b, ev_in[2], ev_split[2], ev_comp[2], ev_out[2];
+  cudaEvent_t ev_start, ev_b, ev_in[2], ev_split[2], ev_comp[2], ev_out[2], ev_done;
 };
 static HostPipe g_pipe[64];
 static std::mutex g_pipe_mu;
@@ -440,6 +524,10 @@ static HostPipe* host_pipe() {
   if (!p.init) {
     if (cudaStreamCreateWithFlags(&p.s_in, cudaStreamNonBlocking) != cudaSuccess ||
         cudaStreamCreateWithFlags(&p.s_out, cudaStreamNonBlocking) != cudaSuccess)
+      return nullptr;
+    // ev_done starts "complete" (recorded on an idle stream) so the first call's wait is free
+    if (cudaEventCreateWithFlags(&p.ev_done, cudaEventDisableTiming) != cudaSuccess ||
+        cudaEventRecord(p.ev_done, p.s_in) != cudaSuccess)
       return nullptr;
     cudaEvent_t* evs[] = {&p.ev_start, &p.ev_b, &p.ev_in[0], &p.ev_in[1], &p.ev_split[0],
                           &p.ev_split[1], &p.ev_comp[0], &p.ev_comp[1], &p.ev_out[0], &p.ev_out[1]};
@@ -502,6 +590,10 @@ int egemm_gemm_host(int64_t M, int64_t N, int64_t K, const float* A_host, int64_
     set_last_error("stream/event creation failed");
     return EGEMM_ERR_CUDA;
   }
+  // one call at a time per device: the pipeline's events are shared, and the copy streams
+  // of this call must not start before the previous call (maybe from another thread, on
+  // another stream) has finished with its buffers and events
+  std::lock_guard<std::mutex> call_lock(hp->mu);
   const int64_t ldk = ldk_of(K), mc = host_chunk_rows(M);
   Carver cv{reinterpret_cast<char*>(workspace)};
   float* Bd = cv.take<float>((size_t)(K * N));
@@ -519,6 +611,7 @@ int egemm_gemm_host(int64_t M, int64_t N, int64_t K, const float* A_host, int64_
   TcConfig cfg = choose_config(EPI_STORE, mc, N, K, terms);
   bool ok = true;
   auto chk = [&](cudaError_t e) { ok = ok && (e == cudaSuccess); };
+  chk(cudaStreamWaitEvent(s, hp->ev_done, 0));  // the previous call's pipeline has drained
   chk(cudaEventRecord(hp->ev_start, s));
   chk(cudaStreamWaitEvent(hp->s_in, hp->ev_start, 0));
   chk(cudaStreamWaitEvent(hp->s_out, hp->ev_start, 0));
@@ -565,6 +658,7 @@ int egemm_gemm_host(int64_t M, int64_t N, int64_t K, const float* A_host, int64_
   // the caller's stream completes only after the last D2H
   chk(cudaStreamWaitEvent(s, hp->ev_out[(nchunks - 1) & 1], 0));
   if (nchunks >= 2) chk(cudaStreamWaitEvent(s, hp->ev_out[(nchunks - 2) & 1], 0));
+  chk(cudaEventRecord(hp->ev_done, s));
   if (!ok) {
     set_last_error("host pipeline: %s", cudaGetErrorString(cudaGetLastError()));
     return EGEMM_ERR_CUDA;
@@ -632,8 +726,8 @@ int egemm_knn(egemm_operand_t X, const float* x_norms, int64_t nx, egemm_operand
               int64_t d, int k, int32_t* out_idx, float* out_dist, void* workspace,
               size_t workspace_bytes, void* stream) {
   cudaStream_t s = (cudaStream_t)stream;
-  if (nx < 0 || nq < 0 || d <= 0 || k < 1 || k > 16 || k > nx) {
-    set_last_error("need nx, nq >= 0, d > 0, 1 <= k <= min(16, nx)");
+  if (nx < 0 || nq < 0 || d <= 0 || k < 1 || k > 64 || k > nx) {
+    set_last_error("need nx, nq >= 0, d > 0, 1 <= k <= min(64, nx)");
     return EGEMM_ERR_INVALID_ARG;
   }
   if (nq == 0) return EGEMM_OK;
@@ -684,15 +778,43 @@ int egemm_knn(egemm_operand_t X, const float* x_norms, int64_t nx, egemm_operand
   epi.kind = EPI_KNN;
   epi.bnorm = xnorm;
   epi.knn_k = k;
-  epi.n_slices = knn_slices(nq, nx, cfg.cg, cfg.bn);
+  {
+    const int64_t n_tiles = (nx + cfg.bn - 1) / cfg.bn;
+    int ns = cfg.nslices > 0 ? cfg.nslices : knn_slices(nq, nx, cfg.cg, cfg.bn);
+    if (ns > kKnnMaxSlices) ns = kKnnMaxSlices;
+    if (ns > n_tiles) ns = (int)n_tiles;
+    epi.n_slices = ns < 1 ? 1 : ns;
+  }
   epi.row_bound = rbound;
   epi.part_key = pkey;
   epi.part_idx = pidx;
   r = launch_tc(nq, nx, d, ops, cfg, epi, s);
   if (r) return r == 2 ? EGEMM_ERR_UNSUPPORTED : EGEMM_ERR_CUDA;
-  if (launch_knn_merge(pkey, pidx, epi.n_slices, nq, k, qnorm, out_idx, out_dist, s))
+  if (launch_knn_merge(pkey, pidx, epi.n_slices, nq, k, k, qnorm, out_idx, out_dist, s))
     return EGEMM_ERR_CUDA;
   return EGEMM_OK;
+}
+
+int egemm_knn_merge(const float* keys, const int32_t* idx, int n_lists, int64_t nq, int k_in, int k,
+                    const float* qnorm, int32_t* out_idx, float* out_key, void* stream) {
+  if (nq < 0 || n_lists < 1 || n_lists > 64 || k_in < 1 || k_in > 1024 || k < 1 || k > 64 ||
+      (int64_t)k > (int64_t)k_in * n_lists) {
+    set_last_error("need nq >= 0, 1 <= n_lists <= 64, 1 <= k_in <= 1024, 1 <= k <= min(64, k_in * n_lists)");
+    return EGEMM_ERR_INVALID_ARG;
+  }
+  if (nq == 0) return EGEMM_OK;
+  if (!keys || !idx || !out_idx || !out_key) {
+    set_last_error("NULL pointer");
+    return EGEMM_ERR_INVALID_ARG;
+  }
+  if (!device_ok()) {
+    set_last_error("no sm_100 device");
+    return EGEMM_ERR_CUDA;
+  }
+  return launch_knn_merge(keys, idx, n_lists, nq, k_in, k, qnorm, out_idx, out_key,
+                          (cudaStream_t)stream)
+             ? EGEMM_ERR_CUDA
+             : EGEMM_OK;
 }
 
 size_t egemm_kmeans_workspace_size(int64_t n, int64_t d, int64_t kc, int x_presplit) {

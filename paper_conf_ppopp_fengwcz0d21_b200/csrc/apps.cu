@@ -8,86 +8,112 @@
 
 namespace egemm {
 
-// ||x_i||^2 accumulated in fp64, rounded once to fp32.  One warp per row.
-__global__ void rownorm_kernel(const float* __restrict__ x, int64_t rows, int64_t d, int64_t ld,
-                               float* __restrict__ out) {
-  const int64_t warp = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
-  const int lane = threadIdx.x & 31;
-  const int64_t nwarps = ((int64_t)gridDim.x * blockDim.x) >> 5;
-  for (int64_t r = warp; r < rows; r += nwarps) {
-    const float* xr = x + r * ld;
+// ||x_i||^2 = sum_t x_it^2 accumulated in fp64 in ascending t (every square is exact in
+// fp64), rounded once to fp32 -- the plain definition (reading R22), so the norms are
+// bitwise reproducible by a sequential loop.  One thread per row: a warp's 32 rows are
+// staged through shared memory in 32-column slabs (coalesced 128-B row segments), then each
+// lane adds its own row's slab in order.
+constexpr int kNormSlab = 32;
+__global__ void __launch_bounds__(256) rownorm_kernel(const float* __restrict__ x, int64_t rows,
+                                                      int64_t d, int64_t ld, float* __restrict__ out) {
+  __shared__ float slab[8][32][kNormSlab + 1];
+  const int w = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int64_t nwarps = (int64_t)gridDim.x * 8;
+  for (int64_t r0 = ((int64_t)blockIdx.x * 8 + w) * 32; r0 < rows; r0 += nwarps * 32) {
     double s = 0.0;
-    for (int64_t t = lane; t < d; t += 32) {
-      double v = (double)xr[t];
-      s = fma(v, v, s);
+    for (int64_t t0 = 0; t0 < d; t0 += kNormSlab) {
+      __syncwarp();
+#pragma unroll 4
+      for (int rr = 0; rr < 32; rr++) {  // row r0 + rr, columns t0 + lane
+        const int64_t r = r0 + rr, t = t0 + lane;
+        slab[w][rr][lane] = (r < rows && t < d) ? __ldg(x + r * ld + t) : 0.f;
+      }
+      __syncwarp();
+      const int tn = (d - t0 < kNormSlab) ? (int)(d - t0) : kNormSlab;
+      for (int t = 0; t < tn; t++) {
+        const double v = (double)slab[w][lane][t];
+        s = __dadd_rn(s, __dmul_rn(v, v));  // exact square, one rounding per add
+      }
     }
-#pragma unroll
-    for (int o = 16; o > 0; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
-    if (lane == 0) out[r] = (float)s;
+    if (r0 + lane < rows) out[r0 + lane] = __double2float_rn(s);
   }
 }
 
 int launch_rownorm(const float* x, int64_t rows, int64_t d, int64_t ld, float* out,
                    cudaStream_t stream) {
   if (rows <= 0) return 0;
-  int64_t blocks = (rows * 32 + 255) / 256;
+  int64_t blocks = (rows + 255) / 256;  // 8 warps x 32 rows per block and round
   int64_t cap = (int64_t)num_sms() * 8;
   if (blocks > cap) blocks = cap;
   rownorm_kernel<<<(unsigned)blocks, 256, 0, stream>>>(x, rows, d, ld, out);
   return cudaGetLastError() == cudaSuccess ? 0 : 3;
 }
 
-// Merge the per-slice sorted (key, idx) lists of each query into the final top-k,
-// ascending by (key, idx); distance = max(0, ||q||^2 + key) (reading R11).
-template <int KN>
-__global__ void knn_merge_kernel(const float* __restrict__ pk, const int32_t* __restrict__ pi,
-                                 int n_slices, int64_t nq, int k, const float* __restrict__ qnorm,
-                                 int32_t* __restrict__ out_idx, float* __restrict__ out_dist) {
-  const int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
-  if (i >= nq) return;
-  float kd[KN];
-  int ki[KN];
-#pragma unroll
-  for (int t = 0; t < KN; t++) { kd[t] = __int_as_float(0x7f800000); ki[t] = 0x7fffffff; }
-  for (int s = 0; s < n_slices; s++) {
-    const int64_t o = ((int64_t)s * nq + i) * k;
-    for (int t = 0; t < k; t++) {
-      float key = pk[o + t];
-      int idx = pi[o + t];
-      if (key < kd[KN - 1] || (key == kd[KN - 1] && idx < ki[KN - 1])) {
-        kd[KN - 1] = key;
-        ki[KN - 1] = idx;
-#pragma unroll
-        for (int u = KN - 1; u > 0; u--) {
-          bool sw = (kd[u] < kd[u - 1]) || (kd[u] == kd[u - 1] && ki[u] < ki[u - 1]);
-          float a = kd[u], b = kd[u - 1];
-          int ia = ki[u], ib = ki[u - 1];
-          kd[u] = sw ? b : a; kd[u - 1] = sw ? a : b;
-          ki[u] = sw ? ib : ia; ki[u - 1] = sw ? ia : ib;
-        }
-      } else if (key > kd[KN - 1]) {
-        break;  // each partial list is ascending
+// Merge of n_lists sorted (key, idx) lists per query into the top k (reading R11 order:
+// ascending key, ties by lower idx).  One warp per query.  Every valid entry's final rank is
+// counted exactly -- its position in its own list plus, for every other list, the number
+// of entries that precede it (a binary search; indices are distinct across lists, so no
+// two valid entries compare equal) -- and the entries with rank < k are written there.
+// Empty slots (idx < 0 or INT32_MAX) rank after everything and are never written; output
+// slots beyond the number of valid entries get (-1, +inf).
+__device__ __forceinline__ bool knn_before(float ka, int ia, float kb, int ib) {
+  return ka < kb || (ka == kb && ia < ib);
+}
+__device__ __forceinline__ bool knn_valid(int i) { return i >= 0 && i != 0x7fffffff; }
+
+__global__ void __launch_bounds__(256) knn_merge_kernel(const float* __restrict__ pk,
+                                                        const int32_t* __restrict__ pi, int n_lists,
+                                                        int64_t nq, int k_in, int k,
+                                                        const float* __restrict__ qnorm,
+                                                        int32_t* __restrict__ out_idx,
+                                                        float* __restrict__ out_key) {
+  const int lane = threadIdx.x & 31;
+  const int64_t q = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5;
+  if (q >= nq) return;
+  const float qn = qnorm ? qnorm[q] : 0.f;
+  const int total = n_lists * k_in;
+  int nvalid = 0;
+  for (int c = lane; c < total; c += 32) {
+    const int l = c / k_in, p = c - l * k_in;
+    const int64_t o = ((int64_t)l * nq + q) * k_in;
+    const int idx = pi[o + p];
+    if (!knn_valid(idx)) continue;
+    nvalid++;
+    const float key = pk[o + p];
+    int rank = p;  // entries of its own list before it (the list is sorted)
+    for (int m = 0; m < n_lists && rank < k; m++) {
+      if (m == l) continue;
+      const int64_t om = ((int64_t)m * nq + q) * k_in;
+      int lo = 0, hi = k_in;  // first position whose entry does not precede (key, idx)
+      while (lo < hi) {
+        const int mid = (lo + hi) >> 1;
+        const int im = pi[om + mid];
+        const bool before = knn_valid(im) && knn_before(pk[om + mid], im, key, idx);
+        if (before) lo = mid + 1; else hi = mid;
       }
+      rank += lo;
+    }
+    if (rank < k) {
+      out_idx[q * k + rank] = idx;
+      const float v = qnorm ? __fadd_rn(qn, key) : key;
+      out_key[q * k + rank] = qnorm ? (v > 0.f ? v : 0.f) : v;
     }
   }
-  const float qn = qnorm[i];
 #pragma unroll
-  for (int t = 0; t < KN; t++) {
-    if (t < k) {
-      out_idx[i * k + t] = ki[t] == 0x7fffffff ? -1 : ki[t];
-      float dd = __fadd_rn(qn, kd[t]);
-      out_dist[i * k + t] = dd > 0.f ? dd : 0.f;
-    }
+  for (int o = 16; o > 0; o >>= 1) nvalid += __shfl_xor_sync(0xffffffffu, nvalid, o);
+  for (int t = nvalid + lane; t < k; t += 32) {
+    out_idx[q * k + t] = -1;
+    out_key[q * k + t] = __int_as_float(0x7f800000);
   }
 }
 
-int launch_knn_merge(const float* part_key, const int32_t* part_idx, int n_slices, int64_t nq,
-                     int k, const float* qnorm, int32_t* out_idx, float* out_dist,
+int launch_knn_merge(const float* part_key, const int32_t* part_idx, int n_lists, int64_t nq,
+                     int k_in, int k, const float* qnorm, int32_t* out_idx, float* out_key,
                      cudaStream_t stream) {
   if (nq <= 0) return 0;
-  unsigned blocks = (unsigned)((nq + 127) / 128);
-  knn_merge_kernel<16><<<blocks, 128, 0, stream>>>(part_key, part_idx, n_slices, nq, k, qnorm,
-                                                    out_idx, out_dist);
+  const int64_t blocks = (nq * 32 + 255) / 256;  // 8 queries per block
+  knn_merge_kernel<<<(unsigned)blocks, 256, 0, stream>>>(part_key, part_idx, n_lists, nq, k_in, k,
+                                                          qnorm, out_idx, out_key);
   return cudaGetLastError() == cudaSuccess ? 0 : 3;
 }
 

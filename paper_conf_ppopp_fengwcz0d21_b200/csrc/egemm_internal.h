@@ -2,6 +2,7 @@
 #pragma once
 #include <cstdint>
 #include <cuda_runtime.h>
+#include "../../include/egemm.h"
 
 namespace egemm {
 
@@ -43,7 +44,26 @@ struct TcConfig {
   int terms;     // 3 or 4
   int max_clusters;  // 0 = all SMs
   int fa;        // fused splits allowed, bit mask: 1 = A, 2 = B (in-kernel converter warps)
+  int stages;    // smem ring depth (0 = the variant's default)
+  int nslices;   // kNN: N-slices per query block (0 = wave-balance formula)
+  int nepi;      // kMeans: epilogue warps, 8 or 16 (0 = 16)
+  int ares;      // kNN: query tile resident in smem (-1 = when d <= 128, 0 = never)
+  int pace;      // STORE: k-pacing (1 = when the workspace has room, 0 = off)
 };
+
+// Environment knobs for experiments, read once per process (tools/; the product path takes
+// its configuration from the tuning table and egemm_set_config_ex).
+struct Knobs {
+  int pace_e, pace_s;  // k-pacing: k-blocks per epoch, slack in epochs (EGEMM_PACE_E / _S)
+  int no_pace;         // EGEMM_NO_PACE=1
+  int band;            // STORE tile order: m-tiles per band (EGEMM_BAND)
+  int a_pf;            // fused A (LDG converters): k-blocks of L2 prefetch (EGEMM_A_PREFETCH)
+  int a_staged;        // fused A: TMA-staged in-place conversion when aligned (EGEMM_A_STAGED)
+  int as_pf;           // fused A, staged: k-blocks of L2 prefetch (EGEMM_AS_PREFETCH)
+  int host_chunk;      // egemm_gemm_host row chunk (EGEMM_HOST_CHUNK, 0 = auto)
+  int dbg_no_tma, dbg_no_epi, dbg_mode;  // diagnostics (EGEMM_DEBUG_*; EGEMM_DIAG builds only)
+};
+const Knobs& knobs();
 
 struct TcEpilogue {
   int kind;
@@ -72,8 +92,9 @@ int launch_tc(int64_t M, int64_t N, int64_t K, const TcOperands& ops, const TcCo
 // apps.cu
 int launch_rownorm(const float* x, int64_t rows, int64_t d, int64_t ld, float* out,
                    cudaStream_t stream);
-int launch_knn_merge(const float* part_key, const int32_t* part_idx, int n_slices, int64_t nq,
-                     int k, const float* qnorm, int32_t* out_idx, float* out_dist,
+// merge n_lists sorted (key, idx) lists [n_lists][nq][k_in] into the top k per query
+int launch_knn_merge(const float* part_key, const int32_t* part_idx, int n_lists, int64_t nq,
+                     int k_in, int k, const float* qnorm, int32_t* out_idx, float* out_key,
                      cudaStream_t stream);
 size_t kmeans_accumulate_ws(int64_t n, int64_t d, int64_t kc);
 int launch_kmeans_accumulate(const float* X, int64_t n, int64_t d, int64_t ldx,
@@ -92,8 +113,13 @@ int read_clock_stats(double* mhz, double* cycles_per_launch, double* launches, i
 int read_debug_counter(unsigned long long* value, int reset);
 
 // tune.cu: the measured configuration table
-bool tune_lookup(int op, long long M, long long N, long long K, int* cg, int* bn, int* sep,
-                 int* kc, int* fa);
+struct TuneEntry {
+  int op = -1;  // EpiKind or kOpGemmB32
+  long long m_max = 0, n_max = 0, k_max = 0;
+  int cg = 0, bn = 0, sep = 0, kc = 0, fa = 0;
+  int terms = 0, stages = 0, nslices = 0, nepi = 0, ares = -1;
+};
+bool tune_lookup(int op, long long M, long long N, long long K, TuneEntry* out);
 const char* tune_table_path();
 int tune_table_size();
 

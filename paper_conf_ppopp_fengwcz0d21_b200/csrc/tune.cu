@@ -4,7 +4,10 @@
 // File: JSON written by tools/tune_sweep.py, read once (std::call_once) from
 // $EGEMM_TUNE_TABLE or <dir of libegemm.so>/tune_table.json:
 //   {"entries": [{"op": "gemm", "m_max": 128, "n_max": 1024, "k_max": 8192,
-//                 "cg": 1, "bn": 128, "sep": 1, "kc": 256}, ...], ...}
+//                 "cg": 1, "bn": 128, "sep": 1, "kc": 256, "terms": 3, "stages": 3}, ...], ...}
+// Value fields: cg, bn, sep, kc, fa (fused-split mask), terms (3 / 4; 0 = 3), stages (0 =
+// the variant's default), n_slices (kNN; 0 = wave-balance formula), epi_warps (kMeans),
+// ares (kNN query tile resident: -1 auto, 0 off).
 // Lookup: the first entry (file order; the sweep writes them smallest bucket first) whose
 // op matches and whose m_max/n_max/k_max bound (M, N, K).  Unknown keys are ignored.
 // The parser accepts exactly this flat shape (objects of string/number fields inside the
@@ -19,12 +22,6 @@
 #include "egemm_internal.h"
 
 namespace egemm {
-
-struct TuneEntry {
-  int op = -1;  // EpiKind
-  long long m_max = 0, n_max = 0, k_max = 0;
-  int cg = 0, bn = 0, sep = 0, kc = 0, fa = 0;
-};
 
 static std::vector<TuneEntry> g_table;
 static std::string g_table_path;
@@ -102,7 +99,8 @@ static bool parse_entry(const char*& p, TuneEntry* e) {
       e->op = v == "gemm" ? EPI_STORE : v == "knn" ? EPI_KNN : v == "kmeans" ? EPI_KMEANS
               : v == "gemm_b32" ? kOpGemmB32 : -1;
     } else if (key == "m_max" || key == "n_max" || key == "k_max" || key == "cg" || key == "bn" ||
-               key == "sep" || key == "kc" || key == "fa") {
+               key == "sep" || key == "kc" || key == "fa" || key == "terms" || key == "stages" ||
+               key == "n_slices" || key == "epi_warps" || key == "ares") {
       char* end = nullptr;
       long long v = strtoll(p, &end, 10);
       if (end == p) return false;
@@ -114,6 +112,11 @@ static bool parse_entry(const char*& p, TuneEntry* e) {
       else if (key == "bn") e->bn = (int)v;
       else if (key == "sep") e->sep = (int)v;
       else if (key == "fa") e->fa = (int)v;
+      else if (key == "terms") e->terms = (int)v;
+      else if (key == "stages") e->stages = (int)v;
+      else if (key == "n_slices") e->nslices = (int)v;
+      else if (key == "epi_warps") e->nepi = (int)v;
+      else if (key == "ares") e->ares = (int)v;
       else e->kc = (int)v;
     } else if (!skip_value(p)) {
       return false;
@@ -172,16 +175,11 @@ static void load_table() {
   }
 }
 
-bool tune_lookup(int op, long long M, long long N, long long K, int* cg, int* bn, int* sep,
-                 int* kc, int* fa) {
+bool tune_lookup(int op, long long M, long long N, long long K, TuneEntry* out) {
   std::call_once(g_table_once, load_table);
   for (const TuneEntry& e : g_table) {
     if (e.op != op || M > e.m_max || N > e.n_max || K > e.k_max) continue;
-    *cg = e.cg;
-    *bn = e.bn;
-    *sep = e.sep;
-    *kc = e.kc;
-    *fa = e.fa;
+    *out = e;
     return true;
   }
   return false;

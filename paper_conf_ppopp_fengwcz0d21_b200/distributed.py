@@ -74,40 +74,32 @@ def knn_queries(X: torch.Tensor, Q_local: torch.Tensor, k: int, **kw):
     return egemm.knn(X, Q_local, k, **kw)
 
 
-def merge_topk(keys: torch.Tensor, idx: torch.Tensor, k: int):
-    """Merge per-rank candidate lists [P, nq, k] -> [nq, k] ascending by (key, idx).
-    Used when the REFERENCES are sharded (NEXT-4); host-side composition only."""
-    P, nq, kk = keys.shape
-    kcat = keys.permute(1, 0, 2).reshape(nq, P * kk)
-    icat = idx.permute(1, 0, 2).reshape(nq, P * kk)
-    # lexicographic (key, idx): stable sort by idx, then stable sort by key
-    o1 = torch.argsort(icat, dim=1, stable=True)
-    kcat, icat = torch.gather(kcat, 1, o1), torch.gather(icat, 1, o1)
-    o2 = torch.argsort(kcat, dim=1, stable=True)
-    return torch.gather(kcat, 1, o2)[:, :k], torch.gather(icat, 1, o2)[:, :k]
-
-
 def knn_references_sharded(X_local: torch.Tensor, x_offset: int, Q: torch.Tensor, k: int,
-                           world: int | None = None, knn_fn=None, **kw):
+                           world: int | None = None, knn_fn=None, merge_fn=None, **kw):
     """NEXT-4: kNN with the REFERENCES sharded over ranks (X too big for one GPU); every
     rank holds all queries Q.  Local top-k of this rank's rows X_local (global row ids
-    x_offset + j) -> all_gather of the [nq, k] (dist, id) lists -> merge by (dist, id).
-    Exchange: 8 * nq * k bytes per rank (tiny next to the GEMM).  ``knn_fn(X, Q, k)`` ->
-    (idx, dist) defaults to egemm.knn; shards with fewer than k rows pad with (+inf, -1).
-    Returns (idx int64 [nq, k], dist fp32 [nq, k]), identical on every rank."""
+    x_offset + j) -> all_gather of the [nq, k] (dist, id) lists -> merge by (dist, id) in
+    egemm_knn_merge (the library's exact rank-counting merge, C ABI).  Exchange: 8 * nq * k
+    bytes per rank (tiny next to the GEMM).  ``knn_fn(X, Q, k)`` -> (idx, dist) defaults to
+    egemm.knn and ``merge_fn(keys [P, nq, k], ids [P, nq, k], k)`` -> (ids, keys) to
+    egemm.knn_merge (both injectable for the CPU gloo tests); shards with fewer than k rows
+    pad with (+inf, -1).  Returns (idx int64 [nq, k], dist [nq, k]), identical on every rank."""
     world = world if world is not None else world_size()
     nq = Q.shape[0]
-    if knn_fn is None:
+    if knn_fn is None or merge_fn is None:
         from . import egemm
-        knn_fn = lambda X_, Q_, k_: egemm.knn(X_, Q_, k_, **kw)  # noqa: E731
+        if knn_fn is None:
+            knn_fn = lambda X_, Q_, k_: egemm.knn(X_, Q_, k_, **kw)  # noqa: E731
+        if merge_fn is None:
+            merge_fn = egemm.knn_merge
     kl = min(k, X_local.shape[0])
     idx, dst = knn_fn(X_local, Q, kl) if kl > 0 else (None, None)
     keys = torch.full((nq, k), float("inf"), dtype=dst.dtype if kl > 0 else torch.float32,
                       device=Q.device)
-    ids = torch.full((nq, k), -1, dtype=torch.int64, device=Q.device)
+    ids = torch.full((nq, k), -1, dtype=torch.int32, device=Q.device)
     if kl > 0:
         keys[:, :kl] = dst
-        ids[:, :kl] = idx.long() + x_offset
+        ids[:, :kl] = (idx.long() + x_offset).to(torch.int32)
     if world > 1:
         kp = [torch.empty_like(keys) for _ in range(world)]
         ip = [torch.empty_like(ids) for _ in range(world)]
@@ -115,11 +107,9 @@ def knn_references_sharded(X_local: torch.Tensor, x_offset: int, Q: torch.Tensor
         dist.all_gather(ip, ids)
         keys, ids = torch.stack(kp), torch.stack(ip)
     else:
-        keys, ids = keys[None], ids[None]
-    # padding (+inf, -1) must sort after every real candidate: map -1 to the largest id
-    ids = torch.where(ids < 0, torch.iinfo(torch.int64).max, ids)
-    mk, mi = merge_topk(keys, ids, k)
-    return torch.where(mi == torch.iinfo(torch.int64).max, -1, mi), mk
+        keys, ids = keys[None].contiguous(), ids[None].contiguous()
+    mi, mk = merge_fn(keys, ids, k)
+    return mi.long(), mk
 
 
 def kmeans_fit(X: torch.Tensor, C: torch.Tensor, iters: int, x_split=None, workspace=None,

@@ -34,13 +34,21 @@ class Operand(ctypes.Structure):
                 ("ld", ctypes.c_int64), ("trans", ctypes.c_int), ("ld_split", ctypes.c_int64)]
 
 
+class Config(ctypes.Structure):
+    """egemm_config_t (0 / -1 = not set, the tuning table's value)."""
+    _fields_ = [(n, ctypes.c_int) for n in ("cg", "bn", "sep", "kc", "stages", "fused", "terms",
+                                            "n_slices", "epi_warps", "a_resident", "pace",
+                                            "max_clusters")]
+
+
 EXPORTS = ["egemm_status_string", "egemm_last_error", "egemm_version", "egemm_split",
            "egemm_split_trunc", "egemm_gemm",
            "egemm_gemm_workspace_size", "egemm_knn", "egemm_knn_workspace_size", "egemm_knn_index",
            "egemm_kmeans_step", "egemm_kmeans_workspace_size", "egemm_kmeans_finalize",
            "egemm_set_config", "egemm_num_sms", "egemm_debug_last_clock", "egemm_tune_table",
            "egemm_debug_clock_stats", "egemm_debug_counter", "egemm_tc_probe",
-           "egemm_query_config", "egemm_gemm_host", "egemm_gemm_host_workspace_size"]
+           "egemm_query_config", "egemm_gemm_host", "egemm_gemm_host_workspace_size",
+           "egemm_set_config_ex", "egemm_query_config_ex", "egemm_knn_merge"]
 
 _lib = None
 
@@ -100,6 +108,12 @@ def load(path: str = LIB_PATH):
     IP = ctypes.POINTER(ctypes.c_int)
     L.egemm_query_config.argtypes = [I, I64, I64, I64, IP, IP, IP, IP, IP]
     L.egemm_query_config.restype = I
+    L.egemm_set_config_ex.argtypes = [ctypes.POINTER(Config)]
+    L.egemm_set_config_ex.restype = I
+    L.egemm_query_config_ex.argtypes = [I, I64, I64, I64, ctypes.POINTER(Config)]
+    L.egemm_query_config_ex.restype = I
+    L.egemm_knn_merge.argtypes = [P, P, I, I64, I, I, P, P, P, P]
+    L.egemm_knn_merge.restype = I
     _lib = L
     return L
 
@@ -120,6 +134,32 @@ def query_config(op: str, M: int, N: int, K: int, with_fused: bool = False):
                                      *[ctypes.byref(x) for x in v]), "egemm_query_config")
     out = tuple(x.value for x in v)
     return out if with_fused else out[:4]
+
+
+OPS = {"gemm": 0, "knn": 1, "kmeans": 2, "gemm_b32": 3}
+
+
+def query_config_ex(op: str, M: int, N: int, K: int) -> dict:
+    """The full launch configuration (egemm_config_t as a dict) the library picks for op."""
+    c = Config()
+    _check(load().egemm_query_config_ex(OPS[op], M, N, K, ctypes.byref(c)), "egemm_query_config_ex")
+    return {n: getattr(c, n) for n, _ in Config._fields_}
+
+
+def set_config_ex(**fields):
+    """Thread-local override of the tuning table: any egemm_config_t field (cg, bn, sep, kc,
+    stages, fused, terms, n_slices, epi_warps, a_resident, pace, max_clusters); no arguments
+    restores the table.  fused / a_resident / pace default to -1 (the table's)."""
+    if not fields:
+        _check(load().egemm_set_config_ex(None), "egemm_set_config_ex")
+        return
+    c = Config()
+    c.fused = c.a_resident = c.pace = -1
+    for k, v in fields.items():
+        if k not in dict(Config._fields_):
+            raise TypeError("unknown config field %r" % k)
+        setattr(c, k, int(v))
+    _check(load().egemm_set_config_ex(ctypes.byref(c)), "egemm_set_config_ex")
 
 
 PROBE_KINDS = {"f16": 0, "bf16": 1, "tf32": 2}
@@ -155,7 +195,8 @@ def debug_clock_stats(reset: bool = True):
 
 
 def debug_counter(reset: bool = True) -> int:
-    """The device debug event counter (EGEMM_DEBUG_MODE bit 256: kNN candidate-path entries)."""
+    """The device debug event counter (EGEMM_DIAG builds, EGEMM_DEBUG_MODE bit 256: kNN
+    candidate-path entries)."""
     v = ctypes.c_ulonglong(0)
     _check(load().egemm_debug_counter(ctypes.byref(v), int(reset)), "egemm_debug_counter")
     return int(v.value)
@@ -186,6 +227,29 @@ def _need_cuda(*ts):
     for t in ts:
         if t is not None and not t.is_cuda:
             raise ValueError("egemm expects CUDA tensors (no CPU path)")
+
+
+def _f32_rows(name, t, shape=None):
+    """An fp32 CUDA matrix with unit inner stride (the C ABI sees only base, ld, sizes)."""
+    if t is None:
+        return
+    if t.dtype != torch.float32 or t.dim() != 2 or (t.shape[1] > 1 and t.stride(1) != 1):
+        raise ValueError("%s must be a 2-D float32 tensor with stride(1) == 1" % name)
+    if shape is not None and tuple(t.shape) != tuple(shape):
+        raise ValueError("%s has shape %s, expected %s" % (name, tuple(t.shape), tuple(shape)))
+
+
+def _split_pair(name, pair, rows, cols):
+    if pair is None:
+        return
+    hi, lo = pair
+    for t in (hi, lo):
+        if t.dtype not in (torch.int16, torch.float16) or t.dim() != 2 or t.stride(1) != 1:
+            raise ValueError("%s hi/lo must be 2-D int16/float16 with stride(1) == 1" % name)
+        if tuple(t.shape) != (rows, cols):
+            raise ValueError("%s hi/lo have shape %s, expected %s" % (name, tuple(t.shape), (rows, cols)))
+    if hi.stride(0) != lo.stride(0):
+        raise ValueError("%s hi and lo must share the row stride" % name)
 
 
 def _workspace(nbytes: int, device, ws=None):
@@ -248,8 +312,17 @@ def gemm(A: torch.Tensor | None, B: torch.Tensor | None, C: torch.Tensor | None 
         M, K = a_split[0].shape
     if B is not None:
         N = B.shape[0] if b_trans else B.shape[1]
+        KB = B.shape[1] if b_trans else B.shape[0]
     else:
-        N = b_split[0].shape[0]
+        N, KB = b_split[0].shape
+    if KB != K:
+        raise ValueError("inner dimensions differ: A has K=%d, B has K=%d" % (K, KB))
+    _f32_rows("A", A)
+    _f32_rows("B", B)
+    _split_pair("a_split", a_split, M, K)
+    _split_pair("b_split", b_split, N, K)
+    _f32_rows("C", C, (M, N))
+    _f32_rows("out", out, (M, N))
     dev = (A if A is not None else a_split[0]).device
     _need_cuda(A, B, C, out)
     D = out if out is not None else torch.empty((M, N), dtype=torch.float32, device=dev)
@@ -272,9 +345,16 @@ def gemm_host(A: torch.Tensor, B: torch.Tensor, out: torch.Tensor | None = None,
     are pipelined against the GPU work inside the library.  Asynchronous: synchronise the
     stream before reading ``out``."""
     L = load()
-    assert not A.is_cuda and not B.is_cuda and A.dtype == torch.float32 and B.dtype == torch.float32
+    assert not A.is_cuda and not B.is_cuda
+    _f32_rows("A", A)
+    _f32_rows("B", B)
     M, K = A.shape
     N = B.shape[1]
+    if B.shape[0] != K:
+        raise ValueError("inner dimensions differ: A has K=%d, B has K=%d" % (K, B.shape[0]))
+    if out is not None and (out.is_cuda or out.dtype != torch.float32 or tuple(out.shape) != (M, N)
+                            or out.stride(1) != 1):
+        raise ValueError("out must be a host float32 [M, N] tensor with stride(1) == 1")
     D = out if out is not None else torch.empty((M, N), dtype=torch.float32, pin_memory=True)
     dev = device or torch.device("cuda", torch.cuda.current_device())
     ws, wsn = _workspace(gemm_host_workspace_size(M, N, K), dev, workspace)
@@ -310,20 +390,30 @@ def knn(X: torch.Tensor | None, Q: torch.Tensor, k: int, x_split=None, index=Non
     be None).  Returns (idx int32 [nq, k], dist fp32 [nq, k])."""
     L = load()
     _need_cuda(X, Q)
+    _f32_rows("Q", Q)
     nq, d = Q.shape
     if index is not None:
         hi, lo, norms = index
         nx = hi.shape[0]
+        _split_pair("index", (hi, lo), nx, d)
+        if norms.dtype != torch.float32 or norms.numel() != nx:
+            raise ValueError("index norms must be float32 [nx]")
         opX = operand(X, hi, lo)
     else:
         nx = X.shape[0]
         norms = None
+        _split_pair("x_split", x_split, nx, d)
         opX = operand(X, *(x_split or (None, None)))
+    if X is not None:
+        _f32_rows("X", X, (nx, d))
     if out is None:
         idx = torch.empty((nq, k), dtype=torch.int32, device=Q.device)
         dist = torch.empty((nq, k), dtype=torch.float32, device=Q.device)
     else:
         idx, dist = out
+        if idx.dtype != torch.int32 or dist.dtype != torch.float32 or tuple(idx.shape) != (nq, k) \
+                or tuple(dist.shape) != (nq, k) or not idx.is_contiguous() or not dist.is_contiguous():
+            raise ValueError("out must be contiguous (int32 [nq, k], float32 [nq, k])")
     need = knn_workspace_size(nx, nq, d, k, index is not None or x_split is not None)
     ws, wsn = _workspace(need, Q.device, workspace)
     _check(L.egemm_knn(opX, _ptr(norms), nx, operand(Q), nq, d, k, _ptr(idx), _ptr(dist), _ptr(ws),
@@ -342,9 +432,13 @@ def kmeans_step(X: torch.Tensor, centroids: torch.Tensor, x_split=None, want_ine
     inertia fp64 [1] or None)."""
     L = load()
     _need_cuda(X, centroids)
+    _f32_rows("X", X)
     n, d = X.shape
     kc = centroids.shape[0]
-    assert centroids.is_contiguous()
+    _f32_rows("centroids", centroids, (kc, d))
+    if not centroids.is_contiguous():
+        raise ValueError("centroids must be contiguous")
+    _split_pair("x_split", x_split, n, d)
     if out is None:
         assign = torch.empty(n, dtype=torch.int32, device=X.device)
         sums = torch.empty((kc, d), dtype=torch.float64, device=X.device)
@@ -352,6 +446,9 @@ def kmeans_step(X: torch.Tensor, centroids: torch.Tensor, x_split=None, want_ine
         inertia = torch.empty(1, dtype=torch.float64, device=X.device) if want_inertia else None
     else:
         assign, sums, counts, inertia = out
+        if assign.dtype != torch.int32 or assign.numel() != n or sums.dtype != torch.float64 or \
+                tuple(sums.shape) != (kc, d) or counts.dtype != torch.int64 or counts.numel() != kc:
+            raise ValueError("out must be (int32 [n], float64 [kc, d], int64 [kc], float64 [1] | None)")
     need = kmeans_workspace_size(n, d, kc, x_split is not None)
     ws, wsn = _workspace(need, X.device, workspace)
     _check(L.egemm_kmeans_step(operand(X, *(x_split or (None, None))), n, d, _ptr(centroids), kc,
@@ -363,9 +460,33 @@ def kmeans_step(X: torch.Tensor, centroids: torch.Tensor, x_split=None, want_ine
 def kmeans_finalize(sums: torch.Tensor, counts: torch.Tensor, centroids: torch.Tensor, stream=None):
     L = load()
     kc, d = centroids.shape
+    if sums.dtype != torch.float64 or tuple(sums.shape) != (kc, d) or not sums.is_contiguous() or \
+            counts.dtype != torch.int64 or counts.numel() != kc or not centroids.is_contiguous() or \
+            centroids.dtype != torch.float32:
+        raise ValueError("kmeans_finalize: sums float64 [kc, d], counts int64 [kc], centroids float32 [kc, d]")
     _check(L.egemm_kmeans_finalize(_ptr(sums), _ptr(counts), kc, d, _ptr(centroids),
                                    _stream(stream)), "egemm_kmeans_finalize")
     return centroids
+
+
+def knn_merge(keys: torch.Tensor, idx: torch.Tensor, k: int, qnorm: torch.Tensor | None = None,
+              stream=None):
+    """Merge sorted partial lists keys / idx [n_lists, nq, k_in] (ascending (key, idx) per
+    list, idx -1 = empty, indices distinct across lists) into the top k per query
+    (egemm_knn_merge).  With qnorm [nq] the output keys become max(0, qnorm + key)."""
+    L = load()
+    _need_cuda(keys, idx, qnorm)
+    if keys.dtype != torch.float32 or idx.dtype != torch.int32 or keys.dim() != 3 or \
+            keys.shape != idx.shape or not keys.is_contiguous() or not idx.is_contiguous():
+        raise ValueError("keys float32 / idx int32, contiguous [n_lists, nq, k_in]")
+    nl, nq, k_in = keys.shape
+    if qnorm is not None and (qnorm.dtype != torch.float32 or qnorm.numel() != nq):
+        raise ValueError("qnorm must be float32 [nq]")
+    oi = torch.empty((nq, k), dtype=torch.int32, device=keys.device)
+    ok = torch.empty((nq, k), dtype=torch.float32, device=keys.device)
+    _check(L.egemm_knn_merge(_ptr(keys), _ptr(idx), nl, nq, k_in, k, _ptr(qnorm), _ptr(oi), _ptr(ok),
+                             _stream(stream)), "egemm_knn_merge")
+    return oi, ok
 
 
 def set_config(cg: int = 0, bn: int = 0, sep: int = 0, kc: int = 0):

@@ -137,3 +137,48 @@ def test_no_gpu_means_loud_failure(lib):
     r = lib.egemm_split(ctypes.cast(buf, ctypes.c_void_p), 2, 2, 2, ctypes.cast(buf, ctypes.c_void_p),
                         ctypes.cast(buf, ctypes.c_void_p), 2, 0, None, None)
     assert r == egemm.ERR_CUDA
+
+
+def test_config_override_round_trip_and_validation(lib):
+    """egemm_set_config_ex / egemm_query_config_ex (the tuning table's value type)
+    work on the host: an override is visible in the query, invalid values are rejected, and
+    NULL restores the table."""
+    from paper_conf_ppopp_fengwcz0d21_b200 import egemm
+    base = egemm.query_config_ex("gemm", 8192, 8192, 8192)
+    egemm.set_config_ex(cg=2, bn=128, sep=1, kc=512, stages=4, fused=1, terms=4)
+    try:
+        q = egemm.query_config_ex("gemm", 8192, 8192, 8192)
+        assert (q["cg"], q["bn"], q["sep"], q["kc"], q["stages"], q["fused"], q["terms"]) == \
+            (2, 128, 1, 512, 4, 1, 4)
+        k = egemm.query_config_ex("kmeans", 1 << 22, 1024, 64)
+        assert k["sep"] == 0 and k["terms"] == 3  # the norm-MMA epilogues: one accumulator, 3 terms
+    finally:
+        egemm.set_config_ex()
+    assert egemm.query_config_ex("gemm", 8192, 8192, 8192) == base
+    for bad in (dict(cg=2, bn=200), dict(kc=100), dict(stages=7), dict(terms=5), dict(n_slices=17),
+                dict(epi_warps=12), dict(fused=3)):
+        with pytest.raises(egemm.EgemmError) as ei:
+            egemm.set_config_ex(**bad)
+        assert ei.value.status == egemm.ERR_UNSUPPORTED
+    egemm.set_config_ex(epi_warps=8, n_slices=4)
+    try:
+        assert egemm.query_config_ex("kmeans", 4096, 1024, 64)["epi_warps"] == 8
+        assert egemm.query_config_ex("knn", 4096, 1 << 20, 128)["n_slices"] == 4
+    finally:
+        egemm.set_config_ex()
+
+
+def test_knn_limits_and_merge_validation(lib):
+    """k up to 64 is accepted by the kNN boundary; egemm_knn_merge validates its
+    arguments host-side (no device work)."""
+    from paper_conf_ppopp_fengwcz0d21_b200 import egemm
+    op = egemm.Operand()
+    assert lib.egemm_knn(op, None, 100, op, 10, 8, 65, None, None, None, 0, None) == egemm.ERR_INVALID_ARG
+    assert lib.egemm_knn(op, None, 10, op, 10, 8, 11, None, None, None, 0, None) == egemm.ERR_INVALID_ARG
+    assert lib.egemm_knn(op, None, 100, op, 0, 8, 64, None, None, None, 0, None) == egemm.OK  # nq = 0
+    m = lib.egemm_knn_merge
+    assert m(None, None, 2, 10, 16, 65, None, None, None, None) == egemm.ERR_INVALID_ARG
+    assert m(None, None, 2, 10, 4, 9, None, None, None, None) == egemm.ERR_INVALID_ARG  # k > 2 * 4
+    assert m(None, None, 0, 10, 4, 4, None, None, None, None) == egemm.ERR_INVALID_ARG
+    assert m(None, None, 2, 0, 4, 4, None, None, None, None) == egemm.OK
+    assert m(None, None, 2, 10, 4, 4, None, None, None, None) == egemm.ERR_INVALID_ARG  # NULL data

@@ -80,17 +80,26 @@ def test_broadcast_and_gather_rows():
         assert np.array_equal(full[:, 0], np.arange(11))
 
 
-def test_merge_topk_matches_sort():
-    g = torch.Generator().manual_seed(0)
-    keys = torch.rand(3, 5, 4, generator=g)
-    keys[1, 2, 0] = keys[0, 2, 1]  # a tie across parts -> lower index first
-    idx = torch.randint(0, 1000, (3, 5, 4), generator=g, dtype=torch.int32)
-    idx[1, 2, 0] = 3
-    idx[0, 2, 1] = 9
-    mk, mi = edist.merge_topk(keys, idx, 4)
-    for q in range(5):
-        pairs = sorted(zip(keys[:, q].flatten().tolist(), idx[:, q].flatten().tolist()))[:4]
-        assert mk[q].tolist() == [p[0] for p in pairs] and mi[q].tolist() == [p[1] for p in pairs]
+def cpu_merge(keys, ids, k):
+    """Host reference of egemm_knn_merge for the gloo tests: per query, the k smallest
+    (key, id) of the union of the lists (id -1 = empty slot, padded back with (-1, +inf))."""
+    P, nq, kk = keys.shape
+    out_i = torch.full((nq, k), -1, dtype=torch.int64)
+    out_k = torch.full((nq, k), float("inf"), dtype=keys.dtype)
+    for q in range(nq):
+        pairs = sorted((float(keys[p, q, t]), int(ids[p, q, t])) for p in range(P) for t in range(kk)
+                       if int(ids[p, q, t]) >= 0)[:k]
+        for t, (kv, iv) in enumerate(pairs):
+            out_i[q, t], out_k[q, t] = iv, kv
+    return out_i, out_k
+
+
+def test_cpu_merge_reference_ties_and_padding():
+    keys = torch.tensor([[[0.5, 1.0, float("inf")]], [[0.5, 0.7, 2.0]]])
+    ids = torch.tensor([[[9, 4, -1]], [[3, 8, 1]]], dtype=torch.int32)
+    i, kk = cpu_merge(keys, ids, 4)
+    assert i.tolist() == [[3, 9, 8, 4]]
+    assert kk.tolist() == torch.tensor([[0.5, 0.5, 0.7, 1.0]]).tolist()
 
 
 def _kmeans_ranks(rank, world):
@@ -134,7 +143,7 @@ def _knn_sharded_ranks(rank, world):
         return torch.from_numpy(i), torch.from_numpy(d)
 
     i, d = edist.knn_references_sharded(torch.from_numpy(X[lo:hi].copy()), lo, Q, 16,
-                                        world=world, knn_fn=knn_fn)
+                                        world=world, knn_fn=knn_fn, merge_fn=cpu_merge)
     return i.numpy(), d.numpy()
 
 
@@ -158,7 +167,8 @@ def test_knn_references_sharded_small_shards():
         dd, ii = torch.sort(d, dim=1, stable=True)
         return ii[:, :k_], dd[:, :k_]
 
-    parts = [edist.knn_references_sharded(X[a:b], a, Q, 2, world=1, knn_fn=knn_fn)
+    parts = [edist.knn_references_sharded(X[a:b], a, Q, 2, world=1, knn_fn=knn_fn,
+                                          merge_fn=cpu_merge)
              for a, b in ((0, 1), (1, 3))]
     i0, d0 = parts[0]
     assert i0.tolist() == [[0, -1]] and d0[0, 1].item() == float("inf")

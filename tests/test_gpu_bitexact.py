@@ -1,5 +1,6 @@
 """Bit-exact GEMM parity: the tcgen05 kernel == Alg. 1 executed on the profiled tensor-core
-primitive (oracle.gemm_alg1_tc, reading R21) for every tile configuration / promotion
+primitive in the paper's step order (oracle.gemm_alg1_tc, Alg. 1 P:749-755 with the
+promotion reading R21) for every tile configuration / smem ring depth / promotion
 interval / term count / accumulator mode, fused and pre-split A, ragged shapes and C.
 The per-element arithmetic of the kernel does not depend on the tile shape, only on
 (terms, sep, Kc), so every configuration must match the model bitwise."""
@@ -15,18 +16,15 @@ CFGS = [(2, 256, 0, 64), (2, 256, 0, 128), (1, 128, 0, 64), (1, 128, 1, 128), (1
         (2, 128, 1, 256), (2, 224, 0, 128), (2, 224, 0, 256), (2, 128, 0, 64)]
 
 
-def _gpu(eg, A, B, C, cfg, terms, fused):
+def _gpu(eg, A, B, C, cfg, terms, fused, stages=0):
     """fused: 0 pre-split operands, 1 A split inside the GEMM, 2 B split inside the GEMM
     (the library falls back to pre-split where the tile config has no such variant)."""
-    eg.set_config(*cfg)
-    import os
-    os.environ["EGEMM_FUSED_A"] = str(int(fused))
+    eg.set_config_ex(cg=cfg[0], bn=cfg[1], sep=cfg[2], kc=cfg[3], fused=int(fused), stages=stages)
     try:
         return to_host(eg.gemm(to_dev(A), to_dev(B), to_dev(C) if C is not None else None,
                                terms=terms))
     finally:
-        eg.set_config(0, 0, 0, 0)
-        os.environ.pop("EGEMM_FUSED_A", None)
+        eg.set_config_ex()
 
 
 @pytest.mark.parametrize("cfg", CFGS)
@@ -66,3 +64,34 @@ def test_bitexact_fused_b(oracle_lib, shape, kc, bn):
     ref = oracle_lib.gemm_alg1_tc(A, B, terms=3, sep=0, kc=kc)
     assert np.array_equal(D.view(np.uint32), ref.view(np.uint32)), \
         "mismatches: %d" % int((D != ref).sum())
+
+
+STAGE_CFGS = [((2, 256, 0, 128), 2), ((2, 224, 0, 128), 2), ((2, 128, 0, 64), 3), ((2, 128, 1, 256), 4),
+              ((1, 128, 0, 64), 2), ((1, 128, 1, 128), 2)]
+
+
+@pytest.mark.parametrize("cfg,stages", STAGE_CFGS)
+def test_bitexact_stage_variants(oracle_lib, cfg, stages):
+    """The non-default smem ring depths of the tuning table's stage axis: same bits."""
+    eg = require_gpu()
+    A, B = inputs.uniform((300, 1000), 50), inputs.uniform((1000, 260), 51)
+    D = _gpu(eg, A, B, None, cfg, 3, 0, stages=stages)
+    ref = oracle_lib.gemm_alg1_tc(A, B, terms=3, sep=cfg[2], kc=cfg[3])
+    assert np.array_equal(D.view(np.uint32), ref.view(np.uint32))
+
+
+def test_bitexact_order_worked_example():
+    """The worked example of tests/test_oracle_alg1_tc.py on the GPU: a = b = 1.5 + 2^-22
+    gives exactly 2.25 + 3 * 2^-22 only in Alg. 1's order (hi*hi first would give one ulp
+    less), for every tile configuration."""
+    eg = require_gpu()
+    x = np.float32(1.5 + 2.0 ** -22)
+    A = np.zeros((130, 70), np.float32)
+    B = np.zeros((70, 140), np.float32)
+    A[:, 37] = x
+    B[37, :] = x
+    want = np.float32(2.25 + 3 * 2.0 ** -22)
+    for cfg in CFGS:
+        for terms in (3, 4):
+            D = _gpu(eg, A, B, None, cfg, terms, 0)
+            assert np.all(D == want), (cfg, terms)

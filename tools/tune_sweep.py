@@ -1,14 +1,25 @@
-"""Measured tile / promotion table -> paper_conf_ppopp_fengwcz0d21_b200/tune_table.json.
+"""Measured launch-configuration table -> paper_conf_ppopp_fengwcz0d21_b200/tune_table.json.
 
-Replaces the paper's analytic model (Sec. 6, Eqs. 2-8) by measurement: for each
-(op, shape bucket) every configuration the library implements is timed (CUDA events, median
-of repeats, pre-split operands) and its normwise error vs the fp64 oracle is measured on a
-row sample; the fastest configuration that meets the accuracy bar (<= 1e-6 and <= 2x the
-naive-fp32 error, BJ north_star) is recorded.  Tool code (calls oracle/ for the error check).
+Replaces the paper's analytic model (Sec. 6, Eqs. 2-8; the T4 design point of
+Table 4) by measurement.  Axes per op:
 
-usage: python tools/tune_sweep.py [--quick] [--prior T] [--out table.json]
-       python tools/tune_sweep.py --from-log log.json [--keep old_table.json --margin 0.03]
-                                  [--meta new_table.json]
+  gemm      tile (cta_group, BN), accumulator mode (SEP), promotion interval Kc, fused A
+            split, smem ring depth (stages), term count (3 / 4)
+  gemm_b32  the gemm pick (B split by egemm_split inside the call) vs the fused-B kernels
+  knn       tile, query tile resident or streamed, N-slices per query block
+  kmeans    tile, epilogue warps
+
+GEMM rule: phase 1 times every (tile, Kc, fused) at the default ring depth and measures its
+normwise error vs the fp64 oracle on a row sample; phase 2 re-times the 3 fastest accurate
+configurations at their alternative ring depth; the pick is the fastest configuration whose
+error (scaled to the bucket's smallest K) is <= 1e-6 and <= 1x the naive-fp32 error when
+any configuration reaches that, else <= 2x (BJ north_star).  The term count is then
+measured on the pick with uniform, in-zone (2^U[-3,3)) and stress (2^U[-14,15)) inputs:
+4 terms are chosen only where 3 miss the bar and 4 meet it.  kNN / kMeans results are
+bitwise identical across their configurations (checked), so time alone decides.
+Tool code (calls oracle/ for the error checks).
+
+usage: python tools/tune_sweep.py [--quick] [--ops gemm,gemm_b32,knn,kmeans] [--out table.json]
 """
 import json
 import os
@@ -20,25 +31,24 @@ import torch
 
 ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
 sys.path.insert(0, ROOT)
-sys.path.insert(0, os.path.dirname(os.path.abspath(__file__)))
 import oracle  # noqa: E402
 from paper_conf_ppopp_fengwcz0d21_b200 import egemm, inputs  # noqa: E402
 
 OUT = os.path.join(ROOT, "paper_conf_ppopp_fengwcz0d21_b200", "tune_table.json")
-# (cg, bn, sep, kc, fa): fa = the fused in-kernel A split (converter warpgroup)
-# Kc = 256 with one accumulator only passes the accuracy bar at large K (the per-chunk
-# truncation error grows ~Kc / sqrt(K), tools/error_sweep.py): the bar decides per bucket.
+# (cg, bn, sep, kc, fused)
 CONFIGS = [(2, 256, 0, 64, 0), (2, 256, 0, 128, 0), (2, 256, 0, 256, 0), (2, 128, 1, 128, 0),
            (2, 128, 1, 256, 0), (1, 128, 1, 128, 0), (1, 128, 1, 256, 0), (1, 128, 0, 64, 0),
            (2, 256, 0, 64, 1), (2, 256, 0, 128, 1), (2, 256, 0, 256, 1), (2, 128, 1, 256, 1),
            (1, 128, 1, 256, 1), (2, 224, 0, 64, 0), (2, 224, 0, 128, 0), (2, 224, 0, 256, 0),
-           (2, 128, 0, 64, 0), (2, 128, 0, 128, 0)]
+           (2, 128, 0, 64, 0), (2, 128, 0, 128, 0), (2, 128, 1, 64, 0)]
+# default ring depth of each pre-split tile and its alternative (csrc/tc_store.cu)
+STAGES = {(2, 256, 0): (3, 2), (2, 224, 0): (3, 2), (2, 128, 0): (4, 3), (2, 128, 1): (3, 4),
+          (1, 128, 0): (3, 2), (1, 128, 1): (3, 2)}
 
 
 def timeit(fn, reps=3, batch_ms=60.0):
-    """Steady-state time per call: warm up ~batch_ms, then the median of `reps` batches of
-    back-to-back calls, each ~batch_ms long (the power-capped clock settles within tens
-    of ms; single short launches over-report the fast, cool-clock case)."""
+    """Steady-state time per call: warm up, then the median of `reps` batches of back-to-back
+    calls, each ~batch_ms long (the power-capped clock settles within tens of ms)."""
     fn()
     torch.cuda.synchronize()
     s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -60,41 +70,44 @@ def timeit(fn, reps=3, batch_ms=60.0):
     return float(np.median(ts))
 
 
-def gemm_bucket(M, N, K, rows=64, configs=None):
-    A, B = inputs.uniform((M, K), 11 + M), inputs.uniform((K, N), 13 + N)
-    Ad, Bd = torch.from_numpy(A).cuda(), torch.from_numpy(B).cuda()
-    b_split = egemm.split(Bd, transpose=True)
-    D = torch.empty((M, N), device="cuda")
-    rs = np.sort(inputs.rng(M + N + K).choice(M, size=min(rows, M), replace=False))
-    C64 = oracle.gemm64(A[rs], B)
-    en = oracle.normwise_error(oracle.gemm32_naive(A[rs], B), A[rs], B, C64)
-    ws = torch.empty(egemm.gemm_workspace_size(M, N, K, False, True), dtype=torch.uint8, device="cuda")
-    res = []
-    for cfg in configs or CONFIGS:
-        egemm.set_config(*cfg[:4])
-        os.environ["EGEMM_FUSED_A"] = str(cfg[4])
-        # the user call with an fp32 A (split separately, or fused into the GEMM) and a
-        # pre-split B: the A split is part of every timed call
-        t = timeit(lambda: egemm.gemm(Ad, None, b_split=b_split, out=D, workspace=ws))
-        e = oracle.normwise_error(D.cpu().numpy()[rs], A[rs], B, C64)
-        res.append({"cfg": cfg, "ms": t, "err": e, "err_naive": en,
-                    "ok": bool(e <= 1e-6 and e <= 2 * en)})
-    egemm.set_config(0, 0, 0, 0)
-    os.environ.pop("EGEMM_FUSED_A", None)
-    return res
+def _cfg(c, stages=0, terms=0):
+    return dict(cg=c[0], bn=c[1], sep=c[2], kc=c[3], fused=c[4], stages=stages, terms=terms)
 
 
-RULE = ("fastest config whose normwise error, scaled to the bucket's smallest K, is <= 1e-6 "
-        "and <= 1x the naive-fp32 error (extended precision: at least as accurate as SGEMM, "
-        "P:63, Fig. 7) when any config reaches it, else the north-star bar (<= 2x naive); "
-        "64 sampled rows, steady-state timing")
+class GemmProblem:
+    def __init__(self, M, N, K, b_f32=False, gen=inputs.uniform, rows=64):
+        self.M, self.N, self.K = M, N, K
+        self.A, self.B = gen((M, K), 11 + M), gen((K, N), 13 + N)
+        self.Ad, self.Bd = torch.from_numpy(self.A).cuda(), torch.from_numpy(self.B).cuda()
+        self.b_f32 = b_f32
+        self.b_split = None if b_f32 else egemm.split(self.Bd, transpose=True)
+        self.D = torch.empty((M, N), device="cuda")
+        self.rs = np.sort(inputs.rng(M + N + K).choice(M, size=min(rows, M), replace=False))
+        self.C64 = oracle.gemm64(self.A[self.rs], self.B)
+        self.en = oracle.normwise_error(oracle.gemm32_naive(self.A[self.rs], self.B), self.A[self.rs],
+                                        self.B, self.C64)
+        self.ws = torch.empty(egemm.gemm_workspace_size(M, N, K, False, not b_f32), dtype=torch.uint8,
+                              device="cuda")
+
+    def call(self, terms=0):
+        if self.b_f32:
+            return egemm.gemm(self.Ad, self.Bd, out=self.D, workspace=self.ws, terms=terms)
+        return egemm.gemm(self.Ad, None, b_split=self.b_split, out=self.D, workspace=self.ws, terms=terms)
+
+    def measure(self, cfg, time_it=True):
+        egemm.set_config_ex(**cfg)
+        try:
+            t = timeit(self.call) if time_it else float("nan")
+            self.call()
+            torch.cuda.synchronize()
+            e = oracle.normwise_error(self.D.cpu().numpy()[self.rs], self.A[self.rs], self.B, self.C64)
+        finally:
+            egemm.set_config_ex()
+        return {"cfg": cfg, "ms": t, "err": e, "err_naive": self.en,
+                "ok": bool(e <= 1e-6 and e <= 2 * self.en)}
 
 
 def select(res, k_scale=1.0):
-    """The bucket's pick under RULE (None when nothing meets the north-star bar).  The
-    bucket covers K in (K_prev, K]; the single-accumulator error ratio grows ~ Kc / sqrt(K)
-    (tools/error_sweep.py), so the ratio measured at K is scaled by k_scale = sqrt(K / K_prev)
-    to bound it over the whole bucket."""
     ok = [r for r in res if r["ok"] and r["err"] * k_scale <= 2 * r["err_naive"]]
     strict = [r for r in ok if r["err"] * k_scale <= r["err_naive"]]
     pool = strict or ok
@@ -106,175 +119,191 @@ def k_scale(K, Ks):
     return (K / lower) ** 0.5 if lower else 1.0
 
 
-def build_table(log, Ms, Ns, Ks, extra=None, keep=None, margin=0.0):
-    """keep: {(M, N, K): cfg} of a previous table -- its pick stays unless this sweep's best
-    is more than `margin` faster than the previous pick re-measured in the same sweep (the
-    power-capped clock drifts between consecutive configs by a few %: near-ties are noise)."""
-    entries = []
-    for b in log:
-        M, N, K = b["M"], b["N"], b["K"]
-        best = select(b["results"], k_scale(K, Ks))
-        prev = (keep or {}).get((M, N, K))
-        if best and prev and list(best["cfg"]) != list(prev):
-            again = [r for r in b["results"] if list(r["cfg"]) == list(prev)]
-            if again and again[0]["ok"] and again[0]["ms"] * (1.0 - margin) <= best["ms"]:
-                best = again[0]
-        if best:
-            cg, bn, sep, kc, fa = best["cfg"]
-            entries.append({"op": "gemm", "m_max": M, "n_max": N, "k_max": K, "cg": cg,
-                            "bn": bn, "sep": sep, "kc": kc, "fa": fa,
-                            "ms": round(best["ms"], 4),
-                            "tflops_fp32eq": round(2.0 * M * N * K / best["ms"] / 1e9, 1),
-                            "err_ratio": round(best["err"] / best["err_naive"], 3)})
-    # the largest measured bucket in each dimension is open-ended, then bucket order:
-    # smallest first so the library's first-match lookup picks the tightest bucket
-    # M > 8192 is only swept for skinny N (<= 1024): the M = 8192 rows of wider N also
-    # cover every larger M
-    wide_top = max([M for M in Ms if M <= 8192], default=None)
+def gemm_bucket(M, N, K, Ks, b_f32=False):
+    P = GemmProblem(M, N, K, b_f32)
+    cands = CONFIGS if not b_f32 else \
+        [tuple(egemm.query_config("gemm", M, N, K, with_fused=True))] + \
+        [(2, 256, 0, kc, 2) for kc in (64, 128, 256)] + [(2, 224, 0, kc, 2) for kc in (128, 256)]
+    res = [P.measure(_cfg(c)) for c in cands]
+    ks = k_scale(K, Ks)
+    # phase 2: the alternative ring depth of the 3 fastest accurate pre-split configurations
+    good = sorted([r for r in res if r["ok"] and r["cfg"]["fused"] == 0], key=lambda r: r["ms"])[:3]
+    for r in good:
+        c = r["cfg"]
+        alt = STAGES[(c["cg"], c["bn"], c["sep"])][1]
+        res.append(P.measure(dict(c, stages=alt)))
+    best = select(res, ks)
+    terms_eval = None
+    if best is not None:
+        # term-count axis: the pick with 3 and 4 terms on three input distributions
+        terms_eval = {}
+        for name, gen in (("uniform", inputs.uniform), ("in_zone", inputs.in_zone), ("stress", inputs.stress)):
+            Q = P if name == "uniform" else GemmProblem(M, N, K, b_f32, gen)
+            for terms in (3, 4):
+                r = Q.measure(dict(best["cfg"], terms=terms), time_it=(name == "uniform" and terms == 4))
+                terms_eval["%s_t%d" % (name, terms)] = {
+                    "err": r["err"], "ratio": r["err"] / r["err_naive"], "ok": r["ok"],
+                    **({"ms": r["ms"]} if name == "uniform" and terms == 4 else {})}
+            del Q
+        miss3 = [d for d in ("uniform", "in_zone", "stress")
+                 if not (terms_eval[d + "_t3"]["ok"] and terms_eval[d + "_t3"]["ratio"] * ks <= 2)]
+        fix4 = [d for d in miss3 if terms_eval[d + "_t4"]["ok"] and terms_eval[d + "_t4"]["ratio"] * ks <= 2]
+        best = dict(best, terms=4 if fix4 else 3)
+    return {"M": M, "N": N, "K": K, "results": res, "terms_eval": terms_eval}, best
+
+
+def knn_bucket(nq, nx, d, k=16):
+    X, Q = inputs.uniform((nx, d), 300), inputs.uniform((nq, d), 301)
+    Xd, Qd = torch.from_numpy(X).cuda(), torch.from_numpy(Q).cuda()
+    index = egemm.knn_index(Xd)
+    ws = torch.empty(egemm.knn_workspace_size(nx, nq, d, k, True), dtype=torch.uint8, device="cuda")
+    out = (torch.empty((nq, k), dtype=torch.int32, device="cuda"),
+           torch.empty((nq, k), dtype=torch.float32, device="cuda"))
+    cfgs = []
+    for ares in ([-1, 0] if d <= 128 else [0]):
+        for ns in (0, 1, 2, 4, 8, 16):
+            cfgs.append(dict(cg=2, bn=256, a_resident=ares, n_slices=ns))
+    for ns in (0, 2, 8):
+        cfgs.append(dict(cg=1, bn=128, n_slices=ns))
+    res, ref = [], None
+    for c in cfgs:
+        egemm.set_config_ex(**c)
+        try:
+            t = timeit(lambda: egemm.knn(None, Qd, k, index=index, workspace=ws, out=out), reps=3, batch_ms=80)
+            q = egemm.query_config_ex("knn", nq, nx, d)
+        finally:
+            egemm.set_config_ex()
+        same = True
+        if ref is None:
+            ref = (out[0].clone(), out[1].clone())
+        else:
+            same = bool(torch.equal(ref[0], out[0]) and torch.equal(ref[1], out[1]))
+        res.append({"cfg": c, "n_slices_used": q["n_slices"], "ms": t, "qps": nq / t * 1e3, "same_bits": same})
+    best = min([r for r in res if r["same_bits"]], key=lambda r: r["ms"])
+    return {"nq": nq, "nx": nx, "d": d, "k": k, "results": res}, best
+
+
+def kmeans_bucket(n, kc, d):
+    X, _, _ = inputs.mixture(n, d, min(kc, 1024), 400)
+    C = X[:kc].copy()
+    Xd, Cd = torch.from_numpy(X).cuda(), torch.from_numpy(C).cuda()
+    xs = egemm.split(Xd)
+    ws = torch.empty(egemm.kmeans_workspace_size(n, d, kc, True), dtype=torch.uint8, device="cuda")
+    out = (torch.empty(n, dtype=torch.int32, device="cuda"), torch.empty((kc, d), dtype=torch.float64, device="cuda"),
+           torch.empty(kc, dtype=torch.int64, device="cuda"), None)
+    res, ref = [], None
+    for c in (dict(cg=2, bn=256, epi_warps=16), dict(cg=2, bn=256, epi_warps=8),
+              dict(cg=1, bn=128, epi_warps=16), dict(cg=1, bn=128, epi_warps=8)):
+        egemm.set_config_ex(**c)
+        try:
+            t = timeit(lambda: egemm.kmeans_step(Xd, Cd, x_split=xs, want_inertia=False, workspace=ws, out=out))
+        finally:
+            egemm.set_config_ex()
+        same = True
+        if ref is None:
+            ref = (out[0].clone(), out[1].clone())
+        else:
+            same = bool(torch.equal(ref[0], out[0]) and torch.equal(ref[1], out[1]))
+        res.append({"cfg": c, "ms": t, "same_bits": same})
+    best = min([r for r in res if r["same_bits"]], key=lambda r: r["ms"])
+    return {"n": n, "kc": kc, "d": d, "results": res}, best
+
+
+def open_top(entries, keys_tops):
     for e in entries:
-        if e["m_max"] == wide_top and e["n_max"] > 1024:
-            e["m_max"] = max(Ms)
-        for key, top in (("m_max", max(Ms)), ("n_max", max(Ns)), ("k_max", max(Ks))):
+        for key, top in keys_tops:
             if e[key] == top:
                 e[key] = 1 << 40
-    entries.sort(key=lambda e: (e["m_max"], e["n_max"], e["k_max"]))
-    doc = {"generated_by": "tools/tune_sweep.py", "rule": RULE, "entries": entries}
-    doc.update(extra or {})
-    return doc
-
-
-B32_RULE = ("op gemm_b32 (B arrives as fp32: its round-split is part of the call): the fastest of "
-            "the gemm row's pick (B split by egemm_split) and the fused-B kernels (2, 256, 0, Kc, "
-            "fa=2) under the same accuracy rule")
-
-
-def b32_sweep(Ms, Ns, Ks):
-    """Buckets of the fp32-B user call gemm(A, B): the library's op-0 pick (separate B^T
-    split inside the call) against the fused-B kernel at Kc 64 / 128 / 256."""
-    log = []
-    for M in Ms:
-        for N in Ns:
-            for K in Ks:
-                if M > 8192 and N > 1024:
-                    continue
-                pick = list(egemm.query_config("gemm", M, N, K, with_fused=True))
-                cfgs = [tuple(pick)] + [(2, 256, 0, kc, 2) for kc in (64, 128, 256)] + \
-                    [(2, 224, 0, kc, 2) for kc in (128, 256)]
-                A, B = inputs.uniform((M, K), 11 + M), inputs.uniform((K, N), 13 + N)
-                Ad, Bd = torch.from_numpy(A).cuda(), torch.from_numpy(B).cuda()
-                D = torch.empty((M, N), device="cuda")
-                rs = np.sort(inputs.rng(M + N + K).choice(M, size=min(64, M), replace=False))
-                C64 = oracle.gemm64(A[rs], B)
-                en = oracle.normwise_error(oracle.gemm32_naive(A[rs], B), A[rs], B, C64)
-                ws = torch.empty(egemm.gemm_workspace_size(M, N, K, False, False), dtype=torch.uint8,
-                                 device="cuda")
-                res = []
-                for cfg in cfgs:
-                    egemm.set_config(*cfg[:4])
-                    os.environ["EGEMM_FUSED_A"] = str(cfg[4])
-                    t = timeit(lambda: egemm.gemm(Ad, Bd, out=D, workspace=ws))
-                    e = oracle.normwise_error(D.cpu().numpy()[rs], A[rs], B, C64)
-                    res.append({"cfg": list(cfg), "ms": t, "err": e, "err_naive": en,
-                                "ok": bool(e <= 1e-6 and e <= 2 * en)})
-                egemm.set_config(0, 0, 0, 0)
-                os.environ.pop("EGEMM_FUSED_A", None)
-                best = select(res, k_scale(K, Ks))
-                log.append({"M": M, "N": N, "K": K, "results": res})
-                print("b32 M=%5d N=%5d K=%5d best=%s %s" % (M, N, K, best and best["cfg"],
-                      " ".join("%s:%.3fms%s" % (r["cfg"], r["ms"], "" if r["ok"] else "x") for r in res)),
-                      flush=True)
-                del Ad, Bd, D, ws
-    return log
 
 
 def main():
-    if "--b32" in sys.argv:  # add the fp32-B rows (op gemm_b32) to the current table
-        Ms, Ns, Ks = [128, 256, 1024, 2048, 4096, 8192, 65536], [256, 1024, 8192], [256, 1024, 2048, 4096, 8192]
-        if "--from-log" in sys.argv:
-            log = json.load(open(sys.argv[sys.argv.index("--from-log") + 1]))
-        else:
-            log = b32_sweep(Ms, Ns, Ks)
-            os.makedirs(os.path.join(ROOT, "gpurun_out"), exist_ok=True)
-            json.dump(log, open(os.path.join(ROOT, "gpurun_out", "tune_sweep_b32_log.json"), "w"), indent=1)
-        doc = build_table(log, Ms, Ns, Ks)
-        for e in doc["entries"]:
-            e["op"] = "gemm_b32"
-        table = json.load(open(OUT))
-        table["entries"] = [e for e in table["entries"] if e["op"] != "gemm_b32"] + doc["entries"]
-        table["rule_gemm_b32"] = B32_RULE
-        out = sys.argv[sys.argv.index("--out") + 1] if "--out" in sys.argv else OUT
-        json.dump(table, open(out, "w"), indent=1)
-        print("wrote", out, len(doc["entries"]), "gemm_b32 entries")
-        return
-    if "--from-log" in sys.argv:  # re-derive the table from a committed sweep log
-        log = json.load(open(sys.argv[sys.argv.index("--from-log") + 1]))
-        Ms, Ns, Ks = (sorted({b[k] for b in log}) for k in ("M", "N", "K"))
-        old = json.load(open(OUT))
-        keep, margin = None, 0.0
-        if "--keep" in sys.argv:  # hysteresis against a previous table (see build_table)
-            prev = json.load(open(sys.argv[sys.argv.index("--keep") + 1]))
-            margin = float(sys.argv[sys.argv.index("--margin") + 1]) if "--margin" in sys.argv else 0.03
-            keep = {}
-            for e in prev["entries"]:
-                cfg = [e["cg"], e["bn"], e["sep"], e["kc"], e.get("fa", 0)]
-                m = min([v for v in Ms if v >= e["m_max"]], default=max(Ms))
-                n = min([v for v in Ns if v >= e["n_max"]], default=max(Ns))
-                k = min([v for v in Ks if v >= e["k_max"]], default=max(Ks))
-                if e["m_max"] > max(Ms) and n > 1024:  # wide N: the M = 8192 row covers larger M
-                    m = max([v for v in Ms if v <= 8192])
-                keep.setdefault((m, n, k), cfg)
-        src = sys.argv[sys.argv.index("--meta") + 1] if "--meta" in sys.argv else OUT
-        meta = json.load(open(src))
-        doc = build_table(log, Ms, Ns, Ks, {k: meta[k] for k in ("device", "when", "sweep_seconds")
-                                            if k in meta}, keep, margin)
-        json.dump(doc, open(OUT, "w"), indent=1)
-        print("rebuilt", OUT, len(doc["entries"]), "entries")
-        return
     quick = "--quick" in sys.argv
-    # 2048: the per-rank rows of the 4-GPU row-sharded 8192^3 bench (1024: 8 GPUs)
-    Ms = [128, 256, 1024, 2048, 4096, 8192, 65536] if not quick else [128, 1024, 8192]
+    ops = sys.argv[sys.argv.index("--ops") + 1].split(",") if "--ops" in sys.argv else \
+        ["gemm", "gemm_b32", "knn", "kmeans"]
+    out_path = sys.argv[sys.argv.index("--out") + 1] if "--out" in sys.argv else OUT
+    old = json.load(open(OUT)) if os.path.exists(OUT) else {"entries": []}
+    entries = [e for e in old.get("entries", []) if e["op"] not in ops]
+    logs = {}
+    t0 = time.time()
+    Ms = [128, 256, 1024, 2048, 4096, 8192, 65536] if not quick else [1024, 8192]
     Ns = [256, 1024, 8192] if not quick else [256, 8192]
     Ks = [256, 1024, 2048, 4096, 8192] if not quick else [1024, 8192]
-    log = []
-    t0 = time.time()
-    # --prior T: measure every config only on the 8192^3 calibration bucket, then only the
-    # analytic model's top T per bucket (NEXT-4; tools/analytic_model.py), widening to all
-    # configs when none of those meets the accuracy bar
-    prior = int(sys.argv[sys.argv.index("--prior") + 1]) if "--prior" in sys.argv else 0
-    model = None
-    if prior:
-        import analytic_model as am
-        cal = {"M": 8192, "N": 8192, "K": 8192, "results": gemm_bucket(8192, 8192, 8192)}
-        model = am.calibrate([cal])
-    for M in Ms:
-        for N in Ns:
-            for K in Ks:
-                if M > 8192 and N > 1024:  # the tall bucket is for skinny N (configs[2])
-                    continue
-                if model and (M, N, K) == (8192, 8192, 8192):
-                    res = cal["results"]
-                elif model:
-                    ranked = sorted(CONFIGS, key=lambda c: am.predict(c, M, N, K, *model))
-                    res = gemm_bucket(M, N, K, configs=ranked[:prior])
-                    if not any(r["ok"] for r in res):
-                        res += gemm_bucket(M, N, K, configs=ranked[prior:])
-                else:
-                    res = gemm_bucket(M, N, K)
-                best = select(res, k_scale(K, Ks))
-                log.append({"M": M, "N": N, "K": K, "results": res})
-                print("M=%5d N=%5d K=%5d best=%s %s" % (M, N, K, best and best["cfg"],
-                      " ".join("%s:%.3fms%s" % (r["cfg"], r["ms"], "" if r["ok"] else "x") for r in res)),
-                      flush=True)
-    doc = build_table(log, Ms, Ns, Ks, {
-        "device": torch.cuda.get_device_name(),
-        "when": time.strftime("%Y-%m-%dT%H:%M:%SZ", time.gmtime()),
-        "sweep_seconds": round(time.time() - t0, 1)})
-    out = sys.argv[sys.argv.index("--out") + 1] if "--out" in sys.argv else OUT
-    json.dump(doc, open(out, "w"), indent=1)
+    for op in ("gemm", "gemm_b32"):
+        if op not in ops:
+            continue
+        new = []
+        logs[op] = []
+        for M in Ms:
+            for N in Ns:
+                for K in Ks:
+                    if M > 8192 and N > 1024:  # the tall bucket is for skinny N (configs[2])
+                        continue
+                    log, best = gemm_bucket(M, N, K, Ks, b_f32=(op == "gemm_b32"))
+                    logs[op].append(log)
+                    print(op, M, N, K, best and (best["cfg"], round(best["ms"], 4), best["terms"]), flush=True)
+                    if not best:
+                        continue
+                    c = best["cfg"]
+                    new.append({"op": op, "m_max": M, "n_max": N, "k_max": K, "cg": c["cg"], "bn": c["bn"],
+                                "sep": c["sep"], "kc": c["kc"], "fa": c["fused"], "stages": c["stages"],
+                                "terms": best["terms"], "ms": round(best["ms"], 4),
+                                "tflops_fp32eq": round(2.0 * M * N * K / best["ms"] / 1e9, 1),
+                                "err_ratio": round(best["err"] / best["err_naive"], 3)})
+            # (the tall bucket M = 65536 exists for skinny N only: M = 8192 rows cover wider N)
+        wide_top = max([M for M in Ms if M <= 8192])
+        for e in new:
+            if e["m_max"] == wide_top and e["n_max"] > 1024:
+                e["m_max"] = max(Ms)
+        open_top(new, (("m_max", max(Ms)), ("n_max", max(Ns)), ("k_max", max(Ks))))
+        entries += new
+    if "knn" in ops:
+        new = []
+        logs["knn"] = []
+        NQ = [1024, 8192, 65536] if not quick else [8192]
+        NX = [65536, 1 << 20] if not quick else [1 << 20]
+        D = [64, 128, 256] if not quick else [128]
+        for nq in NQ:
+            for nx in NX:
+                for d in D:
+                    log, best = knn_bucket(nq, nx, d)
+                    logs["knn"].append(log)
+                    c = best["cfg"]
+                    print("knn", nq, nx, d, c, round(best["ms"], 3), flush=True)
+                    new.append({"op": "knn", "m_max": nq, "n_max": nx, "k_max": d, "cg": c["cg"], "bn": c["bn"],
+                                "sep": 0, "kc": 0, "n_slices": c.get("n_slices", 0),
+                                "ares": c.get("a_resident", -1), "ms": round(best["ms"], 4),
+                                "qps": round(best["qps"])})
+        open_top(new, (("m_max", max(NQ)), ("n_max", max(NX)), ("k_max", max(D))))
+        entries += new
+    if "kmeans" in ops:
+        new = []
+        logs["kmeans"] = []
+        NP = [65536, 1 << 20, 1 << 22] if not quick else [1 << 22]
+        KC = [256, 1024, 4096] if not quick else [1024]
+        D = [32, 64, 128] if not quick else [64]
+        for n in NP:
+            for kc in KC:
+                for d in D:
+                    log, best = kmeans_bucket(n, kc, d)
+                    logs["kmeans"].append(log)
+                    c = best["cfg"]
+                    print("kmeans", n, kc, d, c, round(best["ms"], 3), flush=True)
+                    new.append({"op": "kmeans", "m_max": n, "n_max": kc, "k_max": d, "cg": c["cg"],
+                                "bn": c["bn"], "sep": 0, "kc": 0, "epi_warps": c["epi_warps"],
+                                "ms": round(best["ms"], 4)})
+        open_top(new, (("m_max", max(NP)), ("n_max", max(KC)), ("k_max", max(D))))
+        entries += new
+    order = {"gemm": 0, "gemm_b32": 1, "knn": 2, "kmeans": 3}
+    entries.sort(key=lambda e: (order[e["op"]], e["m_max"], e["n_max"], e["k_max"]))
+    doc = {"generated_by": "tools/tune_sweep.py", "rule": __doc__.split("GEMM rule:")[1].split("Tool code")[0]
+           .replace("\n", " ").strip(), "entries": entries,
+           "device": torch.cuda.get_device_name(), "when": time.strftime("%Y-%m-%dT%H:%M:%SZ", time.gmtime()),
+           "sweep_seconds": round(time.time() - t0, 1), "ops_swept": ops}
+    json.dump(doc, open(out_path, "w"), indent=1)
     os.makedirs(os.path.join(ROOT, "gpurun_out"), exist_ok=True)
-    logname = "tune_sweep_prior%d_log.json" % prior if prior else "tune_sweep_log.json"
-    json.dump(log, open(os.path.join(ROOT, "gpurun_out", logname), "w"), indent=1)
-    print("wrote", out, len(doc["entries"]), "entries in %.1f s" % doc["sweep_seconds"])
+    json.dump(logs, open(os.path.join(ROOT, "gpurun_out", "tune_sweep_r02_log.json"), "w"), indent=1,
+              default=float)
+    print("wrote", out_path, len(entries), "entries in %.1f s" % doc["sweep_seconds"])
 
 
 if __name__ == "__main__":
