@@ -42,7 +42,7 @@ def lib():
         L.oracle_f32_to_f16_rne.restype = ctypes.c_uint16
         L.oracle_f16_to_f32.argtypes = [ctypes.c_uint16]
         L.oracle_f16_to_f32.restype = ctypes.c_uint32
-        for f in ("oracle_split", "oracle_split_rha", "oracle_split_trunc"):
+        for f in ("oracle_split", "oracle_split_rha", "oracle_split_trunc", "oracle_split_bf16"):
             getattr(L, f).argtypes = [P, I64, P, P]
             getattr(L, f).restype = I64
         for f in ("oracle_gemm64", "oracle_gemm32_naive"):
@@ -64,7 +64,7 @@ def lib():
         L.oracle_rownorm.restype = None
         L.oracle_tc_mma16.argtypes = [P, P, I, ctypes.c_float, I]
         L.oracle_tc_mma16.restype = ctypes.c_float
-        L.oracle_gemm_alg1_tc.argtypes = [I64, I64, I64, P, P, P, I, I, I64, P]
+        L.oracle_gemm_alg1_tc.argtypes = [I64, I64, I64, P, P, P, I, I, I64, I, P]
         L.oracle_gemm_alg1_tc.restype = None
         L.oracle_tc_rows.argtypes = [I64, I64, I, P, P, P, P]
         L.oracle_tc_rows.restype = None
@@ -91,12 +91,13 @@ def split(x, variant: str = "rne"):
     """Round-split x (fp32) -> (hi, lo) as uint16 fp16 bit patterns.  P:741-745.
 
     variant: "rne" (the parity reading R1), "rha" (literal round-half-away, R1),
-    "trunc" (Markidis truncate-split, Fig. 4a)."""
+    "trunc" (Markidis truncate-split, Fig. 4a), "bf16" (NEXT-3: bf16 parts, the
+    upper halves of fp32 patterns, RNE)."""
     x = _f32(x)
     hi = np.empty(x.shape, np.uint16)
     lo = np.empty(x.shape, np.uint16)
     fn = {"rne": lib().oracle_split, "rha": lib().oracle_split_rha,
-          "trunc": lib().oracle_split_trunc}[variant]
+          "trunc": lib().oracle_split_trunc, "bf16": lib().oracle_split_bf16}[variant]
     inexact = fn(_p(x), x.size, _p(hi), _p(lo))
     if inexact:
         raise AssertionError("fp32 residual x - hi was inexact for %d elements" % inexact)
@@ -313,18 +314,24 @@ def tc_rows(a, b, c=None):
     return out
 
 
-def gemm_alg1_tc(A, B, C=None, terms: int = 3, sep: int = 0, kc: int = 0):
+def bf16_bits_to_f64(bits):
+    """bf16 bit patterns -> float64 (a bf16 is the top half of an fp32 pattern)."""
+    return (np.asarray(bits, np.uint32) << 16).view(np.float32).astype(np.float64)
+
+
+def gemm_alg1_tc(A, B, C=None, terms: int = 3, sep: int = 0, kc: int = 0, fmt: str = "f16"):
     """Alg. 1 step by step on the profiled tensor-core primitive: per 16-wide
     k-slice in ascending k, [lo*lo,] lo*hi, hi*lo, hi*hi chained through one fp32
     accumulator; promotion into an fp32 total every kc k-elements (reading R21; kc = 0:
-    the paper's single chain over K); sep = 1: hi*hi in its own chain; + C at the end (R7)."""
+    the paper's single chain over K); sep = 1: hi*hi in its own chain; + C at the end (R7).
+    fmt "bf16": the bf16 round-split variant (NEXT-3)."""
     A, B = _f32(A), _f32(B)
     M, K = A.shape
     N = B.shape[1]
     D = np.empty((M, N), np.float32)
     Cp = _f32(C) if C is not None else None
     lib().oracle_gemm_alg1_tc(M, N, K, _p(A), _p(B), _p(Cp) if Cp is not None else None,
-                              int(terms), int(sep), int(kc), _p(D))
+                              int(terms), int(sep), int(kc), 1 if fmt == "bf16" else 0, _p(D))
     return D
 
 

@@ -124,3 +124,35 @@ def test_alg1_tc_promotion_reduces_error(oracle_lib):
     e_64 = oracle_lib.normwise_error(oracle_lib.gemm_alg1_tc(A, B, kc=64), A, B, C64)
     en = oracle_lib.normwise_error(oracle_lib.gemm32_naive(A, B), A, B, C64)
     assert e_long > 2 * en and e_64 < en
+
+
+def test_alg1_tc_bf16_variant_closed_forms(oracle_lib):
+    """NEXT-3's bf16 round-split through the same Alg. 1: integer inputs (8 significant bits,
+    partial sums < 2^24) are exact; A = signed permutation reconstructs fl32(hi_b + lo_b) of
+    the bf16 parts; and at fp16-range inputs the bf16 parts (8 + 8 bits) are less accurate
+    than the fp16 ones (11 + 11 bits), while at |x| ~ 2^40 (beyond fp16) only bf16 works."""
+    A, B = inputs.integers((9, 1024), 1, lim=100), inputs.integers((1024, 11), 2, lim=100)
+    D = oracle_lib.gemm_alg1_tc(A, B, kc=64, fmt="bf16")
+    assert np.array_equal(D, (A.astype(np.int64) @ B.astype(np.int64)).astype(np.float32))
+    n = 24
+    g = inputs.rng(13)
+    perm = g.permutation(n)
+    A = np.zeros((n, n), np.float32)
+    A[np.arange(n), perm] = g.choice([-2.0, -1.0, 0.5, 1.0], n)
+    B = inputs.uniform((n, 5), 14)
+    hi, lo = oracle_lib.split(B, "bf16")
+    hl = (oracle_lib.bf16_bits_to_f64(hi) + oracle_lib.bf16_bits_to_f64(lo)).astype(np.float32)
+    want = A[np.arange(n), perm][:, None] * hl[perm]
+    assert np.array_equal(oracle_lib.gemm_alg1_tc(A, B, fmt="bf16"), want)
+    A, B = inputs.uniform((32, 512), 15), inputs.uniform((512, 32), 16)
+    C64 = oracle_lib.gemm64(A, B)
+    e16 = oracle_lib.normwise_error(oracle_lib.gemm_alg1_tc(A, B, kc=64), A, B, C64)
+    eb = oracle_lib.normwise_error(oracle_lib.gemm_alg1_tc(A, B, kc=64, fmt="bf16"), A, B, C64)
+    assert eb > 10 * e16
+    Aw, Bw = (A * 2.0 ** 40).astype(np.float32), (B * 2.0 ** 40).astype(np.float32)
+    C64w = oracle_lib.gemm64(Aw, Bw)
+    ebw = oracle_lib.normwise_error(oracle_lib.gemm_alg1_tc(Aw, Bw, kc=64, fmt="bf16"), Aw, Bw, C64w)
+    assert np.isclose(ebw, eb, rtol=0.05)  # scale-invariant with the 8-bit exponent
+    with np.errstate(all="ignore"):
+        D16 = oracle_lib.gemm_alg1_tc(Aw, Bw, kc=64)
+    assert not np.all(np.isfinite(D16))  # fp16 parts overflow

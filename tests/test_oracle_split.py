@@ -137,3 +137,31 @@ def test_overflow_and_specials(oracle_lib):
     assert np.isnan(fh[6])
     assert hi[7] == 0 and hi[8] == 0x8000
     assert fh[9] == 2.0 ** -24 and fh[10] == 0.0 and fh[11] == 2.0 ** -24 and fh[12] == 0.0
+
+
+def test_bf16_split_vs_torch_cast_and_exactness(oracle_lib):
+    """NEXT-3's bf16 round-split: hi = bf16_RNE(x) equals torch's float32 -> bfloat16 cast (a
+    library RNE conversion) on sampled fp32 patterns incl. ties, specials and subnormals;
+    x - hi is exact in fp32; |lo| <= half a bf16 ulp of hi; hi + lo keeps >= 16 bits."""
+    import torch
+    g = np.random.default_rng(123)
+    bits = g.integers(0, 2 ** 32, 400000, dtype=np.uint64).astype(np.uint32)
+    ties = (g.integers(0, 2 ** 16, 20000, dtype=np.uint32) << 16) | 0x8000  # exact ties
+    specials = np.array([0, 0x80000000, 0x7F800000, 0xFF800000, 0x7FC00000, 0x00000001,
+                         0x007FFFFF, 0x7F7FFFFF, 0x7F7F8000, 0x3F808000, 0x3F818000], np.uint32)
+    x = np.concatenate([bits, ties, specials]).view(np.float32)
+    hi, lo = oracle_lib.split(x, "bf16")
+    ref = torch.from_numpy(x.copy()).to(torch.bfloat16).view(torch.int16).numpy().view(np.uint16)
+    nan = np.isnan(x)
+    assert np.array_equal(hi[~nan], ref[~nan])
+    assert np.all(np.isnan(oracle_lib.bf16_bits_to_f64(hi[nan])))
+    fin = np.isfinite(x) & np.isfinite(oracle_lib.bf16_bits_to_f64(hi))
+    h = oracle_lib.bf16_bits_to_f64(hi[fin])
+    l = oracle_lib.bf16_bits_to_f64(lo[fin])
+    xf = x[fin].astype(np.float64)
+    r = xf - h
+    assert np.array_equal(r.astype(np.float32).astype(np.float64), r)  # exact in fp32
+    ulp = np.where(h != 0, 2.0 ** (np.floor(np.log2(np.abs(np.where(h != 0, h, 1.0)))) - 7), 0)
+    assert np.all(np.abs(l) <= ulp / 2 + 2.0 ** -149)
+    big = np.abs(xf) > 2.0 ** -100  # away from fp32 subnormals
+    assert np.all(np.abs(xf - h - l)[big] <= np.abs(xf[big]) * 2.0 ** -16)
