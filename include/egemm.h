@@ -84,6 +84,14 @@ int egemm_split_trunc(const float* x, int64_t rows, int64_t cols, int64_t ldx, u
                       uint16_t* lo, int64_t ldo, int transpose, uint32_t* range_flags,
                       void* stream);
 
+/* The bf16 variant of the round-split (the paper's workflow, Sec. 3.1
+ * P:596-649, on the bf16 operands of tcgen05 kind::f16): hi = bf16_RN(x), lo = bf16_RN(x - hi),
+ * bf16 bit patterns (the top halves of fp32 patterns).  8 + 8 significant bits over the full
+ * fp32 exponent range (fp16 parts: 11 + 11 bits within |x| < 65520).  Same arguments as
+ * egemm_split without range_flags.  Use with egemm_gemm under operand_format = 1. */
+int egemm_split_bf16(const float* x, int64_t rows, int64_t cols, int64_t ldx, uint16_t* hi,
+                     uint16_t* lo, int64_t ldo, int transpose, void* stream);
+
 /*
  * Extended-precision GEMM (Alg. 1 "Emulation(D, A, B, C)"):
  *   D[M x N] = A[M x K] * B[K x N] (+ C[M x N] if C != NULL)
@@ -202,9 +210,13 @@ int egemm_kmeans_finalize(const double* sums, const int64_t* counts, int64_t kc,
  *  a_resident  : kNN query tile resident in smem (-1 = when d <= 128, 0 = never).
  *  pace        : k-pacing of STORE GEMMs (-1 = table / on, 0 = off).
  *  max_clusters: persistent clusters launched (0 = one per SM pair / SM).
+ *  operand_format: 0 = fp16 parts (the paper's round-split), 1 = bf16 parts (NEXT-3: the
+ *                fp32 exponent range, 8 + 8 bits; egemm_gemm only, pre-split path; pre-split
+ *                operands must come from egemm_split_bf16).
  */
 typedef struct {
-  int cg, bn, sep, kc, stages, fused, terms, n_slices, epi_warps, a_resident, pace, max_clusters;
+  int cg, bn, sep, kc, stages, fused, terms, n_slices, epi_warps, a_resident, pace, max_clusters,
+      operand_format;
 } egemm_config_t;
 
 /* Thread-local override of the tuning table for the next calls of this thread: fields set

@@ -141,6 +141,10 @@ static TcConfig choose_config(int epi_kind, int64_t M, int64_t N, int64_t K, int
     if (o.a_resident >= 0) c.ares = o.a_resident;
     if (o.pace >= 0) c.pace = o.pace;
     if (o.max_clusters) c.max_clusters = o.max_clusters;
+    if (o.operand_format == 1 && epi_kind == EPI_STORE) {
+      c.fmt = 1;
+      c.fa = 0;  // the fused converters produce fp16 parts only
+    }
   }
   if (c.kc < 64) c.kc = 64;
   c.kc = (c.kc / 64) * 64;
@@ -170,7 +174,7 @@ struct Carver {
 // rows x K logical (K-major).  f32 layout: trans==0 -> rows x K (ld), trans==1 -> K x rows.
 static int stage_operand(const egemm_operand_t& op, int64_t rows, int64_t K, Carver& cv,
                          const uint16_t** hi, const uint16_t** lo, int64_t* ld,
-                         cudaStream_t s) {
+                         cudaStream_t s, int mode = 0) {
   if (op.hi && op.lo) {
     *hi = op.hi;
     *lo = op.lo;
@@ -180,8 +184,8 @@ static int stage_operand(const egemm_operand_t& op, int64_t rows, int64_t K, Car
   const int64_t ldk = ldk_of(K);
   uint16_t* h = cv.take<uint16_t>((size_t)(rows * ldk));
   uint16_t* l = cv.take<uint16_t>((size_t)(rows * ldk));
-  int r = op.trans ? launch_split(op.f32, K, rows, op.ld, h, l, ldk, 1, nullptr, s)
-                   : launch_split(op.f32, rows, K, op.ld, h, l, ldk, 0, nullptr, s);
+  int r = op.trans ? launch_split(op.f32, K, rows, op.ld, h, l, ldk, 1, nullptr, s, mode)
+                   : launch_split(op.f32, rows, K, op.ld, h, l, ldk, 0, nullptr, s, mode);
   if (r) {
     set_last_error("split launch failed");
     return EGEMM_ERR_CUDA;
@@ -265,6 +269,7 @@ static void to_public(const TcConfig& c, int op, egemm_config_t* o) {
   o->a_resident = c.ares;
   o->pace = c.pace;
   o->max_clusters = c.max_clusters;
+  o->operand_format = c.fmt;
 }
 
 int egemm_query_config(int op, int64_t M, int64_t N, int64_t K, int* cg, int* bn, int* sep,
@@ -350,7 +355,8 @@ int egemm_set_config_ex(const egemm_config_t* cfg) {
       o.fused < -1 || o.fused > 2 || o.stages < 0 || o.stages > 4 ||
       !(o.terms == 0 || o.terms == 3 || o.terms == 4) || o.n_slices < 0 || o.n_slices > 16 ||
       !(o.epi_warps == 0 || o.epi_warps == 8 || o.epi_warps == 16) || o.a_resident < -1 ||
-      o.a_resident > 1 || o.pace < -1 || o.pace > 1 || o.max_clusters < 0) {
+      o.a_resident > 1 || o.pace < -1 || o.pace > 1 || o.max_clusters < 0 ||
+      o.operand_format < 0 || o.operand_format > 1) {
     set_last_error("unsupported config cg=%d bn=%d sep=%d kc=%d fused=%d stages=%d terms=%d "
                    "n_slices=%d epi_warps=%d", o.cg, o.bn, o.sep, o.kc, o.fused, o.stages, o.terms,
                    o.n_slices, o.epi_warps);
@@ -374,6 +380,11 @@ int egemm_split_trunc(const float* x, int64_t rows, int64_t cols, int64_t ldx, u
                       uint16_t* lo, int64_t ldo, int transpose, uint32_t* range_flags,
                       void* stream) {
   return split_entry(x, rows, cols, ldx, hi, lo, ldo, transpose, range_flags, stream, 1);
+}
+
+int egemm_split_bf16(const float* x, int64_t rows, int64_t cols, int64_t ldx, uint16_t* hi,
+                     uint16_t* lo, int64_t ldo, int transpose, void* stream) {
+  return split_entry(x, rows, cols, ldx, hi, lo, ldo, transpose, nullptr, stream, 2);
 }
 
 static int split_entry(const float* x, int64_t rows, int64_t cols, int64_t ldx, uint16_t* hi,
@@ -468,7 +479,7 @@ int egemm_gemm(int64_t M, int64_t N, int64_t K, egemm_operand_t A, egemm_operand
     ops.lda_f32 = A.ld;
     cv.take<uint16_t>((size_t)(M * ldk_of(K)));  // keep B's workspace offset unchanged
     cv.take<uint16_t>((size_t)(M * ldk_of(K)));
-  } else if ((r = stage_operand(A, M, K, cv, &ops.a_hi, &ops.a_lo, &ops.lda, s))) {
+  } else if ((r = stage_operand(A, M, K, cv, &ops.a_hi, &ops.a_lo, &ops.lda, s, cfg.fmt == 1 ? 2 : 0))) {
     return r;
   }
   // B logical K x N: as an operand it is N rows x K; f32 trans==0 means stored K x N.
@@ -479,7 +490,7 @@ int egemm_gemm(int64_t M, int64_t N, int64_t K, egemm_operand_t A, egemm_operand
     ops.ldb_f32 = B.ld;
     cv.take<uint16_t>((size_t)(N * ldk_of(K)));  // keep the workspace layout unchanged
     cv.take<uint16_t>((size_t)(N * ldk_of(K)));
-  } else if ((r = stage_operand(Bt, N, K, cv, &ops.b_hi, &ops.b_lo, &ops.ldb, s))) {
+  } else if ((r = stage_operand(Bt, N, K, cv, &ops.b_hi, &ops.b_lo, &ops.ldb, s, cfg.fmt == 1 ? 2 : 0))) {
     return r;
   }
   TcEpilogue epi = {};
@@ -894,6 +905,30 @@ int egemm_kmeans_finalize(const double* sums, const int64_t* counts, int64_t kc,
     return EGEMM_ERR_CUDA;
   }
   return launch_kmeans_finalize(sums, counts, kc, d, centroids, (cudaStream_t)stream)
+             ? EGEMM_ERR_CUDA
+             : EGEMM_OK;
+}
+
+int egemm_kmeans_allreduce_finalize(const double* const* peer_sums,
+                                    const int64_t* const* peer_counts, int nranks, int64_t kc,
+                                    int64_t d, double* sums_out, int64_t* counts_out,
+                                    float* centroids, void* stream) {
+  if (nranks < 1 || nranks > kMaxPeers || kc < 0 || d < 0 || !peer_sums || !peer_counts ||
+      (kc * d > 0 && !centroids)) {
+    set_last_error("need 1 <= nranks <= %d, host arrays of peer pointers, centroids", kMaxPeers);
+    return EGEMM_ERR_INVALID_ARG;
+  }
+  for (int r = 0; r < nranks; r++)
+    if (!peer_sums[r] || !peer_counts[r]) {
+      set_last_error("peer %d: NULL buffer", r);
+      return EGEMM_ERR_INVALID_ARG;
+    }
+  if (!device_ok()) {
+    set_last_error("no sm_100 device");
+    return EGEMM_ERR_CUDA;
+  }
+  return launch_kmeans_peer_reduce_finalize(peer_sums, peer_counts, nranks, kc, d, sums_out,
+                                            counts_out, centroids, (cudaStream_t)stream)
              ? EGEMM_ERR_CUDA
              : EGEMM_OK;
 }

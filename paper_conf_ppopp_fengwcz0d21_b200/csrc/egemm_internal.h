@@ -8,7 +8,8 @@ namespace egemm {
 
 int num_sms();
 
-// mode 0: round-split (Alg. 1), mode 1: truncate-split (Markidis, NEXT-1 variant)
+// mode 0: round-split (Alg. 1), mode 1: truncate-split (Markidis, NEXT-1 variant),
+// mode 2: round-split into bf16 parts (NEXT-3 variant; range_flags not produced)
 int launch_split(const float* x, int64_t rows, int64_t cols, int64_t ldx, uint16_t* hi,
                  uint16_t* lo, int64_t ldo, int transpose, uint32_t* range_flags,
                  cudaStream_t stream, int mode = 0);
@@ -49,6 +50,7 @@ struct TcConfig {
   int nepi;      // kMeans: epilogue warps, 8 or 16 (0 = 16)
   int ares;      // kNN: query tile resident in smem (-1 = when d <= 128, 0 = never)
   int pace;      // STORE: k-pacing (1 = when the workspace has room, 0 = off)
+  int fmt;       // operand parts: 0 = fp16 (the paper's round-split), 1 = bf16 (NEXT-3)
 };
 
 // Environment knobs for experiments, read once per process (tools/; the product path takes
@@ -102,6 +104,11 @@ int launch_kmeans_accumulate(const float* X, int64_t n, int64_t d, int64_t ldx,
                              int64_t* counts, double* inertia, void* ws, cudaStream_t stream);
 int launch_kmeans_finalize(const double* sums, const int64_t* counts, int64_t kc, int64_t d,
                            float* centroids, cudaStream_t stream);
+constexpr int kMaxPeers = 16;
+int launch_kmeans_peer_reduce_finalize(const double* const* peer_sums,
+                                       const int64_t* const* peer_counts, int nranks, int64_t kc,
+                                       int64_t d, double* sums_out, int64_t* counts_out,
+                                       float* centroids, cudaStream_t stream);
 int launch_fill_c(int64_t M, int64_t N, const float* C, int64_t ldc, float* D, int64_t ldd,
                   cudaStream_t stream);
 

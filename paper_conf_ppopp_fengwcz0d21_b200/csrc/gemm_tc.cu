@@ -124,6 +124,11 @@ int launch_tc(int64_t M, int64_t N, int64_t K, const TcOperands& ops, const TcCo
   KParams kp = {};
   kp.K = (int)K;
   kp.fb = fb ? 1 : 0;
+  kp.bf16 = cfg.fmt == 1 ? 1 : 0;
+  if (kp.bf16 && (fa || fb || epi.kind != EPI_STORE)) {
+    set_last_error("bf16 operand parts: pre-split STORE GEMMs only");
+    return 2;
+  }
   const Knobs& kn = knobs();
   kp.debug_no_tma = kn.dbg_no_tma;
   kp.debug_no_epi = kn.dbg_no_epi;

@@ -505,6 +505,51 @@ __global__ void kmeans_finalize_kernel(const double* __restrict__ sums,
   if (c > 0) centroids[e] = (float)__ddiv_rn(sums[e], (double)c);  // fp64 divide, one rounding
 }
 
+// The kMeans exchange step fused with the update (SURVEY 8e follow-up, the "fused NVLS /
+// symmetric-memory reduction in the step's tail"): every rank reads the partial sums and
+// counts of ALL ranks straight from their (peer-mapped, e.g. torch SymmetricMemory) buffers,
+// adds them in rank order 0, 1, ..., P-1 -- the same fixed order on every rank, so the
+// reduced sums and hence the centroids are bitwise identical across ranks without a
+// collective library call -- writes the reduced sums / counts locally and finalizes.
+// One thread per (j, t): reads P fp64 + P int64 over NVLink (P2P loads), no atomics.
+struct PeerPtrs {
+  const double* sums[kMaxPeers];
+  const int64_t* counts[kMaxPeers];
+};
+
+__global__ void kmeans_peer_reduce_finalize_kernel(PeerPtrs pp, int nranks, int64_t kc, int64_t d,
+                                                   double* __restrict__ sums_out,
+                                                   int64_t* __restrict__ counts_out,
+                                                   float* __restrict__ centroids) {
+  const int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (e >= kc * d) return;
+  const int64_t j = e / d, t = e - j * d;
+  double s = 0.0;
+  int64_t c = 0;
+  for (int r = 0; r < nranks; r++) {  // fixed rank order: identical bits on every rank
+    s = __dadd_rn(s, pp.sums[r][e]);
+    c += pp.counts[r][j];
+  }
+  if (sums_out) sums_out[e] = s;
+  if (counts_out && t == 0) counts_out[j] = c;
+  if (c > 0) centroids[e] = (float)__ddiv_rn(s, (double)c);
+}
+
+int launch_kmeans_peer_reduce_finalize(const double* const* peer_sums,
+                                       const int64_t* const* peer_counts, int nranks, int64_t kc,
+                                       int64_t d, double* sums_out, int64_t* counts_out,
+                                       float* centroids, cudaStream_t stream) {
+  if (kc * d <= 0) return 0;
+  PeerPtrs pp = {};
+  for (int r = 0; r < nranks; r++) {
+    pp.sums[r] = peer_sums[r];
+    pp.counts[r] = peer_counts[r];
+  }
+  kmeans_peer_reduce_finalize_kernel<<<(unsigned)((kc * d + 255) / 256), 256, 0, stream>>>(
+      pp, nranks, kc, d, sums_out, counts_out, centroids);
+  return cudaGetLastError() == cudaSuccess ? 0 : 3;
+}
+
 int launch_kmeans_finalize(const double* sums, const int64_t* counts, int64_t kc, int64_t d,
                            float* centroids, cudaStream_t stream) {
   if (kc * d <= 0) return 0;

@@ -249,16 +249,23 @@ __device__ __forceinline__ void tmem_ld16(uint32_t taddr, float* v) {
 }
 
 // ------------------------------------------------------------------ round-split helpers
+// r = x - hi for the two halves of a packed fp16x2 hi, exact in fp32: one mixed-precision
+// FMA per value, hi * (-1) + x (FHFMA: fp16 multiplicands, fp32 addend; the exact result is
+// representable, so the single rounding is exact) instead of an f16 -> f32 unpack and a
+// subtract.
+__device__ __forceinline__ void residual2(uint32_t h, float a, float b, float& ra, float& rb) {
+  asm("{\n\t.reg .f16 x, y, m;\n\tmov.b32 {x, y}, %2;\n\tmov.b16 m, 0xBC00;\n\t"
+      "fma.rn.f32.f16 %0, x, m, %3;\n\tfma.rn.f32.f16 %1, y, m, %4;\n\t}"
+      : "=f"(ra), "=f"(rb)
+      : "r"(h), "f"(a), "f"(b));
+}
 // Alg. 1 l.2 on two values: hi = fp16_RN(x) (cvt.rn.f16x2.f32, ties to even),
 // lo = fp16_RN(x - hi) with the residual exact in fp32.  Packed fp16x2 bit patterns out.
 __device__ __forceinline__ void split2(float a, float b, uint32_t& hi, uint32_t& lo) {
   uint32_t h, l;
   asm("cvt.rn.f16x2.f32 %0, %1, %2;" : "=r"(h) : "f"(b), "f"(a));  // hi half <- b, lo half <- a
-  float ha, hb;
-  asm("{\n\t.reg .f16 x, y;\n\tmov.b32 {x, y}, %2;\n\tcvt.f32.f16 %0, x;\n\tcvt.f32.f16 %1, y;\n\t}"
-      : "=f"(ha), "=f"(hb)
-      : "r"(h));
-  const float ra = __fsub_rn(a, ha), rb = __fsub_rn(b, hb);
+  float ra, rb;
+  residual2(h, a, b, ra, rb);
   asm("cvt.rn.f16x2.f32 %0, %1, %2;" : "=r"(l) : "f"(rb), "f"(ra));
   hi = h;
   lo = l;

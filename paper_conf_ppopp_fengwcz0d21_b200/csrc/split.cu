@@ -16,6 +16,7 @@
 #include <cuda_fp16.h>
 #include <cstdint>
 #include "egemm_internal.h"
+#include "ptx.cuh"
 
 namespace egemm {
 
@@ -26,11 +27,17 @@ struct SplitPair {
 template <int MODE, bool FLAGS = true>
 __device__ __forceinline__ SplitPair split2(float a, float b, uint32_t& flags) {
   uint32_t h, l;
+  if constexpr (MODE == 2) {  // bf16 parts (NEXT-3): a bf16 is the top half of an fp32 pattern
+    asm("cvt.rn.bf16x2.f32 %0, %1, %2;" : "=r"(h) : "f"(b), "f"(a));
+    const float ra = __fsub_rn(a, __uint_as_float(h << 16));
+    const float rb = __fsub_rn(b, __uint_as_float(h & 0xffff0000u));  // exact in fp32
+    asm("cvt.rn.bf16x2.f32 %0, %1, %2;" : "=r"(l) : "f"(rb), "f"(ra));
+    return SplitPair{h, l};
+  }
   if (MODE == 0) asm("cvt.rn.f16x2.f32 %0, %1, %2;" : "=r"(h) : "f"(b), "f"(a));
   else asm("cvt.rz.f16x2.f32 %0, %1, %2;" : "=r"(h) : "f"(b), "f"(a));
-  const __half2 hh = *reinterpret_cast<const __half2*>(&h);
-  const float2 hf = __half22float2(hh);
-  const float ra = __fsub_rn(a, hf.x), rb = __fsub_rn(b, hf.y);  // exact in fp32
+  float ra, rb;
+  ptx::residual2(h, a, b, ra, rb);  // x - hi, exact in fp32
   if (MODE == 0) asm("cvt.rn.f16x2.f32 %0, %1, %2;" : "=r"(l) : "f"(rb), "f"(ra));
   else asm("cvt.rz.f16x2.f32 %0, %1, %2;" : "=r"(l) : "f"(rb), "f"(ra));
   if constexpr (FLAGS) {  // only when the caller asked for range_flags
@@ -244,6 +251,7 @@ int launch_split(const float* x, int64_t rows, int64_t cols, int64_t ldx, uint16
                  cudaStream_t stream, int mode) {
   if (rows == 0 || cols == 0) return 0;
   if (mode == 1) launch_mode<1>(x, rows, cols, ldx, hi, lo, ldo, transpose, range_flags, stream);
+  else if (mode == 2) launch_mode<2>(x, rows, cols, ldx, hi, lo, ldo, transpose, range_flags, stream);
   else launch_mode<0>(x, rows, cols, ldx, hi, lo, ldo, transpose, range_flags, stream);
   return cudaGetLastError() == cudaSuccess ? 0 : -1;
 }

@@ -109,6 +109,7 @@ struct KParams {
   int pace_e, pace_s;  // k-blocks per epoch, slack in epochs
   int band_m;          // STORE tile order: m-tiles per band
   int fb;            // fused B split (host-side dispatch flag; tm_bhi maps the fp32 B)
+  int bf16;          // operands are bf16 hi / lo parts (NEXT-3 variant), not fp16
   unsigned long long* probe;  // device clock probe: [0..3] last launch, [4..6] running sums, [7] counter
   int debug_mode;    // EGEMM_DEBUG_MODE bits (diagnostics): 1 extra commit per k-block;
                      // with NO_TMA: 2 MMA warp ignores the full barriers (producer idle),
@@ -728,7 +729,8 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
     // The whole warp runs the loop (so stage / descriptor arithmetic stays in uniform
     // registers); one elected lane -- always the same one -- issues MMAs and commits.
     if (leader) {
-      constexpr uint32_t idesc = ptx::idesc_f16_f32(kBM * CG, BN);
+      // operand format: fp16 parts (the paper's round-split) or bf16 parts (NEXT-3 variant)
+      const uint32_t idesc = ptx::idesc_f16_f32(kBM * CG, BN) | (p.bf16 ? ((1u << 7) | (1u << 10)) : 0u);
       const uint32_t sbase = ptx::smem_u32(stage_base);
       int stage = 0;
       uint32_t phase = 0;

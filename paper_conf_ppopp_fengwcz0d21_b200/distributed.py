@@ -112,10 +112,43 @@ def knn_references_sharded(X_local: torch.Tensor, x_offset: int, Q: torch.Tensor
     return mi.long(), mk
 
 
+class SymmPeers:
+    """Per-rank kMeans partial buffers in torch SymmetricMemory (NVLink peer-mapped): rank r
+    writes its partial sums / counts into its own buffer; every rank can then read all of
+    them (``sums[r]`` / ``counts[r]`` are this device's views of rank r's buffer).  Used by
+    kmeans_fit(reduce="peer") with egemm_kmeans_allreduce_finalize."""
+
+    def __init__(self, kc: int, d: int, device, group=None):
+        import torch.distributed._symmetric_memory as symm_mem
+        grp = group or dist.group.WORLD
+        self.world, self.rank = dist.get_world_size(grp), dist.get_rank(grp)
+        nb = kc * d * 8 + kc * 8
+        self.buf = symm_mem.empty(nb, dtype=torch.uint8, device=device)
+        self.handle = symm_mem.rendezvous(self.buf, grp.group_name)
+        self.sums, self.counts = [], []
+        for r in range(self.world):
+            b = self.handle.get_buffer(r, (nb,), torch.uint8)
+            self.sums.append(b[: kc * d * 8].view(torch.float64).view(kc, d))
+            self.counts.append(b[kc * d * 8:].view(torch.int64))
+
+    def local(self):
+        return self.sums[self.rank], self.counts[self.rank]
+
+    def barrier(self):
+        self.handle.barrier()
+
+
 def kmeans_fit(X: torch.Tensor, C: torch.Tensor, iters: int, x_split=None, workspace=None,
-               bufs=None, world: int | None = None, step=None, finalize=None):
+               bufs=None, world: int | None = None, step=None, finalize=None, reduce: str = "nccl",
+               peers=None, peer_finalize=None):
     """Lloyd iterations on this rank's points X with replicated centroids C (updated in
-    place): local egemm_kmeans_step -> all_reduce(sums, counts) -> egemm_kmeans_finalize.
+    place).  reduce="nccl": local egemm_kmeans_step -> all_reduce(sums, counts) ->
+    egemm_kmeans_finalize.  reduce="peer": the step writes its partials into this rank's
+    SymmetricMemory buffer (``peers``, a SymmPeers), a symmetric barrier, then
+    egemm_kmeans_allreduce_finalize reads every rank's partials over NVLink, reduces them in
+    rank order and updates C (bitwise identical on every rank), and a second barrier keeps
+    the next step from overwriting partials a peer is still reading.  The step / finalize
+    hooks let the gloo tests drive the same host composition on CPU.
     Returns the last iteration's local assignment."""
     from . import egemm
     world = world if world is not None else world_size()
@@ -124,6 +157,18 @@ def kmeans_fit(X: torch.Tensor, C: torch.Tensor, iters: int, x_split=None, works
     finalize = finalize or egemm.kmeans_finalize
     assign = None
     packed = None
+    if reduce == "peer":
+        if peers is None:
+            raise ValueError("reduce='peer' needs the SymmPeers buffers")
+        peer_finalize = peer_finalize or (lambda P, C_: egemm.kmeans_allreduce_finalize(P.sums, P.counts, C_))
+        ls, lc = peers.local()
+        abuf = bufs[0] if bufs else torch.empty(X.shape[0], dtype=torch.int32, device=X.device)
+        for _ in range(iters):
+            assign, _, _, _ = step(X, C, (abuf, ls, lc, None))  # partials into the own buffer
+            peers.barrier()          # every rank's partials are written
+            peer_finalize(peers, C)  # reduce over peer memory (rank order) + update
+            peers.barrier()          # every rank has read them: the next step may overwrite
+        return assign
     for _ in range(iters):
         assign, sums, counts, _ = step(X, C, bufs)
         if world > 1:

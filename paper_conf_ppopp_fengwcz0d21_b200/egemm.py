@@ -38,7 +38,7 @@ class Config(ctypes.Structure):
     """egemm_config_t (0 / -1 = not set, the tuning table's value)."""
     _fields_ = [(n, ctypes.c_int) for n in ("cg", "bn", "sep", "kc", "stages", "fused", "terms",
                                             "n_slices", "epi_warps", "a_resident", "pace",
-                                            "max_clusters")]
+                                            "max_clusters", "operand_format")]
 
 
 EXPORTS = ["egemm_status_string", "egemm_last_error", "egemm_version", "egemm_split",
@@ -48,7 +48,8 @@ EXPORTS = ["egemm_status_string", "egemm_last_error", "egemm_version", "egemm_sp
            "egemm_set_config", "egemm_num_sms", "egemm_debug_last_clock", "egemm_tune_table",
            "egemm_debug_clock_stats", "egemm_debug_counter", "egemm_tc_probe",
            "egemm_query_config", "egemm_gemm_host", "egemm_gemm_host_workspace_size",
-           "egemm_set_config_ex", "egemm_query_config_ex", "egemm_knn_merge"]
+           "egemm_set_config_ex", "egemm_query_config_ex", "egemm_knn_merge", "egemm_split_bf16",
+           "egemm_kmeans_allreduce_finalize"]
 
 _lib = None
 
@@ -71,6 +72,8 @@ def load(path: str = LIB_PATH):
     L.egemm_split.restype = I
     L.egemm_split_trunc.argtypes = [P, I64, I64, I64, P, P, I64, I, P, P]
     L.egemm_split_trunc.restype = I
+    L.egemm_split_bf16.argtypes = [P, I64, I64, I64, P, P, I64, I, P]
+    L.egemm_split_bf16.restype = I
     L.egemm_gemm.argtypes = [I64, I64, I64, Operand, Operand, P, I64, P, I64, I, P, SZ, P]
     L.egemm_gemm.restype = I
     L.egemm_gemm_workspace_size.argtypes = [I64, I64, I64, I, I]
@@ -114,6 +117,10 @@ def load(path: str = LIB_PATH):
     L.egemm_query_config_ex.restype = I
     L.egemm_knn_merge.argtypes = [P, P, I, I64, I, I, P, P, P, P]
     L.egemm_knn_merge.restype = I
+    L.egemm_kmeans_allreduce_finalize.argtypes = [ctypes.POINTER(ctypes.c_void_p),
+                                                  ctypes.POINTER(ctypes.c_void_p), I, I64, I64, P,
+                                                  P, P, P]
+    L.egemm_kmeans_allreduce_finalize.restype = I
     _lib = L
     return L
 
@@ -155,6 +162,7 @@ def set_config_ex(**fields):
         return
     c = Config()
     c.fused = c.a_resident = c.pace = -1
+    c.operand_format = 0
     for k, v in fields.items():
         if k not in dict(Config._fields_):
             raise TypeError("unknown config field %r" % k)
@@ -265,7 +273,8 @@ def split(x: torch.Tensor, transpose: bool = False, range_flags: torch.Tensor | 
           out: tuple | None = None, stream=None, mode: str = "round"):
     """Round-split fp32 x [rows, cols] -> (hi, lo) fp16 bit patterns as int16 tensors
     (viewable as torch.float16).  transpose=True returns the [cols, rows] transpose.
-    mode="trunc": the Markidis truncate-split (egemm_split_trunc)."""
+    mode="trunc": the Markidis truncate-split (egemm_split_trunc); mode="bf16": bf16 parts
+    (egemm_split_bf16, NEXT-3)."""
     L = load()
     _need_cuda(x)
     assert x.dtype == torch.float32 and x.dim() == 2 and x.stride(1) == 1
@@ -276,6 +285,11 @@ def split(x: torch.Tensor, transpose: bool = False, range_flags: torch.Tensor | 
         lo = torch.empty(oshape, dtype=torch.int16, device=x.device)
     else:
         hi, lo = out
+    if mode == "bf16":
+        assert range_flags is None
+        _check(L.egemm_split_bf16(_ptr(x), rows, cols, x.stride(0), _ptr(hi), _ptr(lo), hi.stride(0),
+                                  1 if transpose else 0, _stream(stream)), "egemm_split_bf16")
+        return hi, lo
     fn = {"round": L.egemm_split, "trunc": L.egemm_split_trunc}[mode]
     _check(fn(_ptr(x), rows, cols, x.stride(0), _ptr(hi), _ptr(lo), hi.stride(0),
               1 if transpose else 0, _ptr(range_flags), _stream(stream)), "egemm_split")
@@ -487,6 +501,28 @@ def knn_merge(keys: torch.Tensor, idx: torch.Tensor, k: int, qnorm: torch.Tensor
     _check(L.egemm_knn_merge(_ptr(keys), _ptr(idx), nl, nq, k_in, k, _ptr(qnorm), _ptr(oi), _ptr(ok),
                              _stream(stream)), "egemm_knn_merge")
     return oi, ok
+
+
+def kmeans_allreduce_finalize(peer_sums, peer_counts, centroids: torch.Tensor, sums_out=None,
+                              counts_out=None, stream=None):
+    """The kMeans exchange step fused with the update over peer memory
+    (egemm_kmeans_allreduce_finalize): peer_sums / peer_counts are lists of the ranks' partial
+    (kc x d fp64, kc int64) tensors readable from this device (e.g. torch SymmetricMemory peer
+    buffers); reduced in rank order (bitwise identical on every rank), then finalized."""
+    L = load()
+    kc, d = centroids.shape
+    n = len(peer_sums)
+    for t in list(peer_sums) + list(peer_counts):
+        _need_cuda(t)
+    if n != len(peer_counts) or any(t.dtype != torch.float64 or t.numel() != kc * d for t in peer_sums) or \
+            any(t.dtype != torch.int64 or t.numel() != kc for t in peer_counts):
+        raise ValueError("peer_sums: float64 [kc, d] each; peer_counts: int64 [kc] each")
+    ps = (ctypes.c_void_p * n)(*[t.data_ptr() for t in peer_sums])
+    pc = (ctypes.c_void_p * n)(*[t.data_ptr() for t in peer_counts])
+    _check(L.egemm_kmeans_allreduce_finalize(ps, pc, n, kc, d, _ptr(sums_out), _ptr(counts_out),
+                                             _ptr(centroids), _stream(stream)),
+           "egemm_kmeans_allreduce_finalize")
+    return centroids
 
 
 def set_config(cg: int = 0, bn: int = 0, sep: int = 0, kc: int = 0):

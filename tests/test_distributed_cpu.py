@@ -174,3 +174,68 @@ def test_knn_references_sharded_small_shards():
     assert i0.tolist() == [[0, -1]] and d0[0, 1].item() == float("inf")
     i1, _ = parts[1]
     assert i1.tolist() == [[1, 2]]
+
+
+class _GlooPeers:
+    """CPU stand-in for distributed.SymmPeers: this rank's partial buffers, and the other
+    ranks' gathered at barrier() (gloo all_gather emulates the peer reads)."""
+
+    def __init__(self, kc, d, world, rank):
+        self.world, self.rank = world, rank
+        self.sums = [torch.zeros(kc, d, dtype=torch.float64) for _ in range(world)]
+        self.counts = [torch.zeros(kc, dtype=torch.int64) for _ in range(world)]
+        self.phase = 0
+
+    def local(self):
+        return self.sums[self.rank], self.counts[self.rank]
+
+    def barrier(self):
+        if self.phase == 0:  # first barrier of an iteration: publish the own partials
+            gs = [torch.empty_like(self.sums[0]) for _ in range(self.world)]
+            gc = [torch.empty_like(self.counts[0]) for _ in range(self.world)]
+            dist.all_gather(gs, self.sums[self.rank])
+            dist.all_gather(gc, self.counts[self.rank])
+            for r in range(self.world):
+                if r != self.rank:
+                    self.sums[r].copy_(gs[r])
+                    self.counts[r].copy_(gc[r])
+        else:
+            dist.barrier()
+        self.phase ^= 1
+
+
+def _kmeans_peer_ranks(rank, world):
+    import oracle
+    X, _, _ = inputs.mixture(6000, 8, 16, 3, sigma=0.1)
+    C = torch.from_numpy(X[:16].copy())
+    lo, hi = edist.shard_bounds(6000, world, rank)
+    Xl = torch.from_numpy(X[lo:hi].copy())
+
+    def step(X_, C_, out):
+        a, s, c, _, _ = oracle.kmeans_step(X_.numpy(), C_.numpy())
+        out[1].copy_(torch.from_numpy(s))
+        out[2].copy_(torch.from_numpy(c))
+        return torch.from_numpy(a), out[1], out[2], None
+
+    def peer_finalize(P, C_):  # rank-order reduction, as egemm_kmeans_allreduce_finalize
+        s = P.sums[0].clone()
+        c = P.counts[0].clone()
+        for r in range(1, P.world):
+            s += P.sums[r]
+            c += P.counts[r]
+        C_.copy_(torch.from_numpy(oracle.kmeans_finalize(s.numpy(), c.numpy(), C_.numpy())))
+
+    peers = _GlooPeers(16, 8, world, rank)
+    edist.kmeans_fit(Xl, C, 3, world=world, step=step, reduce="peer", peers=peers,
+                     peer_finalize=peer_finalize)
+    return C.numpy()
+
+
+def test_kmeans_fit_peer_reduce_composition(oracle_lib):
+    """reduce='peer' (partials in per-rank buffers, barrier, rank-order reduction + update,
+    barrier): identical centroids on every rank, equal to the NCCL-style path's within 1 ulp
+    (another fp64 summation order) and to the single process."""
+    out = _run(_kmeans_peer_ranks)
+    assert np.array_equal(out[0], out[1])
+    ref = _run(_kmeans_ranks)[0]
+    assert np.allclose(out[0], ref, rtol=2.0 ** -23, atol=2.0 ** -30)

@@ -326,3 +326,37 @@ def test_knn_merge_call_vs_sort():
     oi3, ok3 = eg.knn_merge(to_dev(np.full((1, 2, 4), np.inf, np.float32)),
                             to_dev(np.full((1, 2, 4), -1, np.int32)), 3)
     assert np.all(to_host(oi3) == -1) and np.all(np.isinf(to_host(ok3)))
+
+
+def test_kmeans_allreduce_finalize_peer_buffers(oracle_lib):
+    """egemm_kmeans_allreduce_finalize (the exchange step fused with the update over peer
+    memory): 3 "ranks" (shards of the points, their partials in separate device buffers, as
+    SymmetricMemory peers would be) reduced in rank order == the fp64 rank-order sum of the
+    partials + finalize, bitwise; counts exact; sums within SURVEY c-20's bound of the
+    oracle's plain sums over all points."""
+    eg = require_gpu()
+    X, _, _ = inputs.mixture(9000, 32, 40, 65, sigma=0.3)
+    C = X[:40].copy()
+    Xd, Cd = to_dev(X), to_dev(C)
+    cuts = [0, 2500, 6100, 9000]
+    ps, pc = [], []
+    assign = []
+    for a, b in zip(cuts[:-1], cuts[1:]):
+        ga, s, c, _ = eg.kmeans_step(Xd[a:b].contiguous(), Cd)
+        ps.append(s.clone())
+        pc.append(c.clone())
+        assign.append(to_host(ga))
+    sums_out = torch.empty_like(ps[0])
+    cnt_out = torch.empty_like(pc[0])
+    newc = Cd.clone()
+    eg.kmeans_allreduce_finalize(ps, pc, newc, sums_out, cnt_out)
+    ref_s = to_host(ps[0]).copy()
+    for t in ps[1:]:
+        ref_s = ref_s + to_host(t)  # fp64, rank order
+    ref_c = sum(to_host(t) for t in pc)
+    assert np.array_equal(to_host(sums_out), ref_s) and np.array_equal(to_host(cnt_out), ref_c)
+    assert np.array_equal(to_host(newc), oracle_lib.kmeans_finalize(ref_s, ref_c, C))
+    ga = np.concatenate(assign)
+    os_, oc = oracle_lib.kmeans_sums(X, ga, 40)
+    assert np.array_equal(ref_c, oc)
+    assert np.all(np.abs(ref_s - os_) <= oracle_lib.kmeans_sums_bound(X, ga, 40))

@@ -95,3 +95,23 @@ def test_bitexact_order_worked_example():
         for terms in (3, 4):
             D = _gpu(eg, A, B, None, cfg, terms, 0)
             assert np.all(D == want), (cfg, terms)
+
+
+@pytest.mark.parametrize("cfg", [(2, 256, 0, 64), (2, 128, 1, 256), (1, 128, 0, 128)])
+@pytest.mark.parametrize("terms", [3, 4])
+def test_bitexact_bf16_variant(oracle_lib, cfg, terms):
+    """NEXT-3: operand_format = 1 (bf16 hi / lo parts, egemm_split_bf16) == the oracle's Alg. 1
+    on bf16 parts bitwise, with a wide exponent range (|x| ~ 2^U[-40, 40]) that fp16 parts
+    could not represent."""
+    eg = require_gpu()
+    g = inputs.rng(60)
+    A = (g.uniform(-1, 1, (200, 300)) * 2.0 ** g.integers(-40, 40, (200, 300))).astype(np.float32)
+    B = (g.uniform(-1, 1, (300, 260)) * 2.0 ** g.integers(-40, 40, (300, 260))).astype(np.float32)
+    eg.set_config_ex(cg=cfg[0], bn=cfg[1], sep=cfg[2], kc=cfg[3], operand_format=1)
+    try:
+        assert eg.query_config_ex("gemm", 200, 260, 300)["operand_format"] == 1
+        D = to_host(eg.gemm(to_dev(A), to_dev(B), terms=terms))
+    finally:
+        eg.set_config_ex()
+    ref = oracle_lib.gemm_alg1_tc(A, B, terms=terms, sep=cfg[2], kc=cfg[3], fmt="bf16")
+    assert np.array_equal(D.view(np.uint32), ref.view(np.uint32))

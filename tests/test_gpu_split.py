@@ -128,3 +128,26 @@ def test_fig7_direction(oracle_lib):
         # the paper's own run-to-run spread is ~3x (R14): a loose ceiling of 2x its series
         assert err["round"] < 2 * paper[n], err
         assert err["round"] < err["trunc"] < err["half"], err
+
+
+def test_split_bf16_matches_oracle(oracle_lib):
+    """NEXT-3 bf16 round-split (egemm_split_bf16) bit-exact against the oracle's bit-level
+    bf16 split on 2^26 sampled fp32 patterns (flat and transposing kernels, ragged edges)."""
+    eg = require_gpu()
+    x = inputs.all_f32_patterns(0x3A000000, 1 << 26)  # spans many binades incl. ties
+    g = np.random.default_rng(7)
+    x = np.concatenate([x, g.integers(0, 2 ** 32, 1 << 20, dtype=np.uint64).astype(np.uint32).view(np.float32)])
+    ohi, olo = oracle_lib.split(x, "bf16")
+    xd = to_dev(x).view(-1, 1 << 10)
+    hi, lo = eg.split(xd, mode="bf16")
+    ghi, glo = u16(hi).ravel(), u16(lo).ravel()
+    isnan16 = lambda h: ((h & 0x7F80) == 0x7F80) & ((h & 0x7F) != 0)
+    nan = np.isnan(x)
+    ok = (ghi == ohi) & (glo == olo)
+    ok |= nan & isnan16(ghi) & isnan16(ohi)
+    ok |= (ghi == ohi) & isnan16(glo) & isnan16(olo)
+    assert ok.all(), "mismatch at %d" % int(np.argmin(ok))
+    y = inputs.uniform((300, 257), 9)
+    th, tl = eg.split(to_dev(y), transpose=True, mode="bf16")
+    yh, yl = oracle_lib.split(y, "bf16")
+    assert np.array_equal(u16(th), yh.T) and np.array_equal(u16(tl), yl.T)

@@ -91,8 +91,31 @@ def launch_list(path, first=None):
             for k, v in sorted(agg.items(), key=lambda kv: -kv[1][1])]
 
 
+def bench_summary(out, cfg, shape, gemm_rep, split_rep, label):
+    """profiles/ncu_summary.json for bench.py: the DRAM bytes of the bench's own GEMM launch
+    (identified by its configuration and shape: bench.py uses the number only when both
+    match its launch) and of its split launches."""
+    g = [k for k in summarize(gemm_rep) if "egemm_tc_kernel" in k["kernel"]][0]
+    sp = [k for k in summarize(split_rep) if "split" in k["kernel"]] if split_rep != "-" else []
+    doc = {"source": "%s (ncu --set full --clock-control none, one launch; tools/prof_all.sh)" % label,
+           "gemm_kernel": g["kernel"], "gemm_config": cfg, "gemm_shape": shape,
+           "gemm_dram_bytes_per_launch": g.get("dram_bytes_total"),
+           "gemm_profiled": {k: g.get(k) for k in ("gpu__time_duration.sum", "gpc__cycles_elapsed.avg.per_second",
+                                                    "sm__pipe_tensor_cycles_active_realtime.avg.pct_of_peak_sustained_elapsed",
+                                                    "lts__t_sector_hit_rate.pct")},
+           "split_dram_bytes_per_step": sum(k.get("dram_bytes_total") or 0 for k in sp) if sp else None,
+           "split_kernels": [k["kernel"][:60] for k in sp]}
+    json.dump(doc, open(out, "w"), indent=1)
+    print("wrote", out)
+
+
 def main():
     args = sys.argv[1:]
+    if args and args[0] == "--bench-summary":
+        # --bench-summary OUT.json "cg bn sep kc fused" "M N K" gemm.ncu-rep split.ncu-rep|- LABEL
+        _, out, cfg, shape, grep, srep, label = args[:7]
+        bench_summary(out, [int(v) for v in cfg.split()], [int(v) for v in shape.split()], grep, srep, label)
+        return
     prefix = args.pop(0)
     launch, head = None, None
     if "--launch" in args:

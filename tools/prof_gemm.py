@@ -10,7 +10,8 @@ from paper_conf_ppopp_fengwcz0d21_b200 import egemm  # noqa: E402
 
 n = int(sys.argv[1]) if len(sys.argv) > 1 else 8192
 if len(sys.argv) > 5:
-    egemm.set_config(*[int(v) for v in sys.argv[2:6]])
+    cg, bn, sep, kc = [int(v) for v in sys.argv[2:6]]
+    egemm.set_config_ex(cg=cg, bn=bn, sep=sep, kc=kc, fused=0)
 reps = int(sys.argv[6]) if len(sys.argv) > 6 else 3
 A = torch.rand(n, n, device="cuda") * 2 - 1
 B = torch.rand(n, n, device="cuda") * 2 - 1
