@@ -213,10 +213,14 @@ int egemm_kmeans_finalize(const double* sums, const int64_t* counts, int64_t kc,
  *  operand_format: 0 = fp16 parts (the paper's round-split), 1 = bf16 parts (NEXT-3: the
  *                fp32 exponent range, 8 + 8 bits; egemm_gemm only, pre-split path; pre-split
  *                operands must come from egemm_split_bf16).
+ *  tail_peel   : STORE GEMMs with one n-tile of CTA-pair tiles: the rows of a last wave at
+ *                most 60 % full run as a second, programmatically dependent launch of
+ *                128 x 128 tiles on the SMs the main grid frees (-1 = table / on, 0 = off).
+ *                Same results bit for bit.
  */
 typedef struct {
   int cg, bn, sep, kc, stages, fused, terms, n_slices, epi_warps, a_resident, pace, max_clusters,
-      operand_format;
+      operand_format, tail_peel;
 } egemm_config_t;
 
 /* Thread-local override of the tuning table for the next calls of this thread: fields set

@@ -102,6 +102,7 @@ static TcConfig choose_config(int epi_kind, int64_t M, int64_t N, int64_t K, int
   c.kc = 64;  // promotion every 64 k: the most accurate single-accumulator setting
   c.ares = -1;
   c.pace = 1;
+  c.peel = -1;
   if (epi_kind == EPI_STORE && M <= 128) { c.cg = 1; c.bn = 128; c.sep = 1; }
   {
     TuneEntry t;
@@ -119,6 +120,7 @@ static TcConfig choose_config(int epi_kind, int64_t M, int64_t N, int64_t K, int
       c.nslices = t.nslices;
       c.nepi = t.nepi;
       if (t.ares >= 0) c.ares = t.ares;
+      if (t.peel >= 0) c.peel = t.peel;
     }
   }
   if (terms == 3 || terms == 4) c.terms = terms;  // the call's explicit term count wins
@@ -141,6 +143,7 @@ static TcConfig choose_config(int epi_kind, int64_t M, int64_t N, int64_t K, int
     if (o.a_resident >= 0) c.ares = o.a_resident;
     if (o.pace >= 0) c.pace = o.pace;
     if (o.max_clusters) c.max_clusters = o.max_clusters;
+    if (o.tail_peel >= 0) c.peel = o.tail_peel;
     if (o.operand_format == 1 && epi_kind == EPI_STORE) {
       c.fmt = 1;
       c.fa = 0;  // the fused converters produce fp16 parts only
@@ -270,6 +273,7 @@ static void to_public(const TcConfig& c, int op, egemm_config_t* o) {
   o->pace = c.pace;
   o->max_clusters = c.max_clusters;
   o->operand_format = c.fmt;
+  o->tail_peel = c.peel;
 }
 
 int egemm_query_config(int op, int64_t M, int64_t N, int64_t K, int* cg, int* bn, int* sep,
@@ -341,6 +345,7 @@ int egemm_set_config(int cg, int bn, int sep, int kc) {
   o.fused = -1;
   o.a_resident = -1;
   o.pace = -1;
+  o.tail_peel = -1;
   return egemm_set_config_ex(&o);
 }
 
@@ -356,7 +361,7 @@ int egemm_set_config_ex(const egemm_config_t* cfg) {
       !(o.terms == 0 || o.terms == 3 || o.terms == 4) || o.n_slices < 0 || o.n_slices > 16 ||
       !(o.epi_warps == 0 || o.epi_warps == 8 || o.epi_warps == 16) || o.a_resident < -1 ||
       o.a_resident > 1 || o.pace < -1 || o.pace > 1 || o.max_clusters < 0 ||
-      o.operand_format < 0 || o.operand_format > 1) {
+      o.operand_format < 0 || o.operand_format > 1 || o.tail_peel < -1 || o.tail_peel > 1) {
     set_last_error("unsupported config cg=%d bn=%d sep=%d kc=%d fused=%d stages=%d terms=%d "
                    "n_slices=%d epi_warps=%d", o.cg, o.bn, o.sep, o.kc, o.fused, o.stages, o.terms,
                    o.n_slices, o.epi_warps);

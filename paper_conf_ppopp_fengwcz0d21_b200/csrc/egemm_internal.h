@@ -51,6 +51,7 @@ struct TcConfig {
   int ares;      // kNN: query tile resident in smem (-1 = when d <= 128, 0 = never)
   int pace;      // STORE: k-pacing (1 = when the workspace has room, 0 = off)
   int fmt;       // operand parts: 0 = fp16 (the paper's round-split), 1 = bf16 (NEXT-3)
+  int peel;      // STORE: peel a mostly-empty last wave into a 128 x 128 tail launch (-1 auto, 0 off)
 };
 
 // Environment knobs for experiments, read once per process (tools/; the product path takes
@@ -124,7 +125,7 @@ struct TuneEntry {
   int op = -1;  // EpiKind or kOpGemmB32
   long long m_max = 0, n_max = 0, k_max = 0;
   int cg = 0, bn = 0, sep = 0, kc = 0, fa = 0;
-  int terms = 0, stages = 0, nslices = 0, nepi = 0, ares = -1;
+  int terms = 0, stages = 0, nslices = 0, nepi = 0, ares = -1, peel = -1;
 };
 bool tune_lookup(int op, long long M, long long N, long long K, TuneEntry* out);
 const char* tune_table_path();

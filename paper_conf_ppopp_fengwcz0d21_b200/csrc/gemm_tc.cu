@@ -97,8 +97,8 @@ static bool make_tmap_f32(CUtensorMap* m, const void* base, int64_t rows, int64_
   return r == CUDA_SUCCESS;
 }
 
-int launch_tc(int64_t M, int64_t N, int64_t K, const TcOperands& ops, const TcConfig& cfg,
-              const TcEpilogue& epi, cudaStream_t stream) {
+static int launch_tc_one(int64_t M, int64_t N, int64_t K, const TcOperands& ops, const TcConfig& cfg,
+                         const TcEpilogue& epi, cudaStream_t stream, bool pdl_tail) {
   if (M <= 0 || N <= 0) return 0;
   if (M > INT32_MAX / 2 || N > INT32_MAX / 2) {
     set_last_error("M, N must be < 2^30");
@@ -125,6 +125,7 @@ int launch_tc(int64_t M, int64_t N, int64_t K, const TcOperands& ops, const TcCo
   kp.K = (int)K;
   kp.fb = fb ? 1 : 0;
   kp.bf16 = cfg.fmt == 1 ? 1 : 0;
+  kp.pdl_wait = pdl_tail ? 1 : 0;
   if (kp.bf16 && (fa || fb || epi.kind != EPI_STORE)) {
     set_last_error("bf16 operand parts: pre-split STORE GEMMs only");
     return 2;
@@ -199,6 +200,47 @@ int launch_tc(int64_t M, int64_t N, int64_t K, const TcOperands& ops, const TcCo
   }
   kp.num_units = kp.m_tiles;
   return dispatch_kmeans(maps, kp, cfg, stream);
+}
+
+// Tail peel (STORE, one n-tile of CTA-pair tiles): when the persistent grid's last wave of
+// 256-row units would be at most 60 % full, the rows of that wave go to a second launch of
+// 128 x 128 single-CTA tiles (the same per-element arithmetic: same Kc, terms, accumulator
+// mode, so the results are bitwise those of one launch).  The second launch is a
+// programmatic dependent launch: its CTAs start on the SMs the main grid frees as it
+// drains, instead of the freed SMs idling until the main grid's slowest cluster ends; it
+// waits for the main grid before it completes, so stream order is kept for later work.
+int launch_tc(int64_t M, int64_t N, int64_t K, const TcOperands& ops, const TcConfig& cfg,
+              const TcEpilogue& epi, cudaStream_t stream) {
+  const bool fb = ops.b_f32 != nullptr && ops.a_f32 == nullptr;
+  if (epi.kind == EPI_STORE && cfg.peel != 0 && cfg.cg == 2 && (cfg.bn == 256 || cfg.bn == 224) &&
+      !fb && N <= cfg.bn && M > 0) {
+    int clusters = num_sms() / 2;
+    if (cfg.max_clusters > 0 && cfg.max_clusters < clusters) clusters = cfg.max_clusters;
+    const int64_t units = (M + 255) / 256;
+    const int64_t full = units / (clusters > 0 ? clusters : 1), rem = units % (clusters > 0 ? clusters : 1);
+    if (clusters > 0 && full >= 1 && rem > 0 && rem * 10 <= (int64_t)clusters * 6) {
+      const int64_t M1 = full * clusters * 256;
+      int r = launch_tc_one(M1, N, K, ops, cfg, epi, stream, false);
+      if (r) return r;
+      TcOperands t = ops;
+      if (ops.a_f32) t.a_f32 = ops.a_f32 + M1 * ops.lda_f32;
+      if (ops.a_hi) {
+        t.a_hi = ops.a_hi + M1 * ops.lda;
+        t.a_lo = ops.a_lo + M1 * ops.lda;
+      }
+      TcConfig c2 = cfg;
+      c2.cg = 1;
+      c2.bn = 128;
+      c2.stages = 0;
+      c2.max_clusters = 0;
+      TcEpilogue e2 = epi;
+      e2.D = epi.D + M1 * epi.ldd;
+      if (epi.C) e2.C = epi.C + M1 * epi.ldc;
+      e2.sync = nullptr;
+      return launch_tc_one(M - M1, N, K, t, c2, e2, stream, true);
+    }
+  }
+  return launch_tc_one(M, N, K, ops, cfg, epi, stream, false);
 }
 
 }  // namespace egemm

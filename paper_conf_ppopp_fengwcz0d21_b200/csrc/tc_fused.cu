@@ -27,6 +27,8 @@ int dispatch_fused(const CUtensorMap* m, const KParams& kp, const TcConfig& c, c
     return launch_variant<2, 128, false, EPI_STORE, 3, true>(m, kp, mc, s);
   if (c.cg == 1 && c.bn == 128 && c.sep)
     return launch_variant<1, 128, true, EPI_STORE, 3, true>(m, kp, mc, s);
+  if (c.cg == 1 && c.bn == 128 && !c.sep)  // (the peeled tail of a (2, 256, 0) fused-A call)
+    return launch_variant<1, 128, false, EPI_STORE, 3, true>(m, kp, mc, s);
   set_last_error("fused A split: unsupported tile config cg=%d bn=%d sep=%d", c.cg, c.bn, c.sep);
   return 2;
 }

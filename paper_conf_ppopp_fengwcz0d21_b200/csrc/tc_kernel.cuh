@@ -110,6 +110,7 @@ struct KParams {
   int band_m;          // STORE tile order: m-tiles per band
   int fb;            // fused B split (host-side dispatch flag; tm_bhi maps the fp32 B)
   int bf16;          // operands are bf16 hi / lo parts (NEXT-3 variant), not fp16
+  int pdl_wait;      // a peeled tail launch (programmatic dependent launch of the main grid)
   unsigned long long* probe;  // device clock probe: [0..3] last launch, [4..6] running sums, [7] counter
   int debug_mode;    // EGEMM_DEBUG_MODE bits (diagnostics): 1 extra commit per k-block;
                      // with NO_TMA: 2 MMA warp ignores the full barriers (producer idle),
@@ -406,7 +407,10 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
   if constexpr (CG == 2) { ptx::cluster_sync(); __syncthreads(); } else __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
-  if (blockIdx.x == 0 && threadIdx.x == 0) {  // SM-clock probe (egemm_debug_last_clock)
+  // STORE: a tail launch of the same call (the peeled last wave, launched with programmatic
+  // stream serialisation) may start on the SMs this grid frees as its CTAs finish
+  if (EPI == EPI_STORE && threadIdx.x == 0) asm volatile("griddepcontrol.launch_dependents;");
+  if (blockIdx.x == 0 && threadIdx.x == 0 && !p.pdl_wait) {  // SM-clock probe (egemm_debug_last_clock)
     p.probe[0] = clock64();
     p.probe[1] = globaltimer_ns();
   }
@@ -1197,7 +1201,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
     ptx::tc_fence_after();
     ptx::tmem_dealloc<CG>(tmem_base, TMEM_COLS);
   }
-  if (blockIdx.x == 0 && threadIdx.x == 0) {
+  if (blockIdx.x == 0 && threadIdx.x == 0 && !p.pdl_wait) {
     const unsigned long long c1 = clock64(), t1 = globaltimer_ns();
     p.probe[2] = c1;
     p.probe[3] = t1;
@@ -1205,6 +1209,9 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
     p.probe[5] += t1 - p.probe[1];
     p.probe[6] += 1;
   }
+  // a peeled tail launch completes only after the grid it overlapped (its stream successors
+  // may overwrite that grid's operands)
+  if (p.pdl_wait) asm volatile("griddepcontrol.wait;" ::: "memory");
 }
 
 // ------------------------------------------------------------------ launch of one variant
@@ -1257,13 +1264,15 @@ static int launch_variant(const CUtensorMap* maps, const KParams& kp, int max_cl
   cfg.blockDim = dim3(EpiGeo<NEPI, FA || FB>::THREADS, 1, 1);
   cfg.dynamicSmemBytes = smem;
   cfg.stream = stream;
-  cudaLaunchAttribute attr[1];
+  cudaLaunchAttribute attr[2];
   attr[0].id = cudaLaunchAttributeClusterDimension;
   attr[0].val.clusterDim.x = CG;
   attr[0].val.clusterDim.y = 1;
   attr[0].val.clusterDim.z = 1;
+  attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  attr[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
-  cfg.numAttrs = 1;
+  cfg.numAttrs = kp.pdl_wait ? 2 : 1;
   cudaError_t e = cudaLaunchKernelEx(&cfg, kern, maps[0], maps[1], maps[2], maps[3], kp);
   if (e != cudaSuccess) {
     set_last_error("cudaLaunchKernelEx: %s", cudaGetErrorString(e));

@@ -115,3 +115,26 @@ def test_bitexact_bf16_variant(oracle_lib, cfg, terms):
         eg.set_config_ex()
     ref = oracle_lib.gemm_alg1_tc(A, B, terms=terms, sep=cfg[2], kc=cfg[3], fmt="bf16")
     assert np.array_equal(D.view(np.uint32), ref.view(np.uint32))
+
+
+@pytest.mark.parametrize("fused", [0, 1])
+@pytest.mark.parametrize("M", [65536, 74 * 256 + 20 * 256 + 37])
+def test_tail_peel_same_bits(oracle_lib, fused, M):
+    """The peeled last wave (a programmatic dependent launch of 128 x 128 tiles) gives the
+    same bits as one launch, and as the oracle's Alg. 1 on sampled rows of the tail."""
+    import torch
+    eg = require_gpu()
+    N, K = 256, 1024
+    A, B, C = inputs.uniform((M, K), 70), inputs.uniform((K, N), 71), inputs.uniform((M, N), 72)
+    Ad, Bd, Cd = to_dev(A), to_dev(B), to_dev(C)
+    out = {}
+    for peel in (0, 1):
+        eg.set_config_ex(cg=2, bn=256, sep=0, kc=128, fused=fused, tail_peel=peel)
+        try:
+            out[peel] = to_host(eg.gemm(Ad, Bd, Cd))
+        finally:
+            eg.set_config_ex()
+    assert np.array_equal(out[0].view(np.uint32), out[1].view(np.uint32))
+    rows = np.array([0, M // 2, M - 300, M - 1])
+    ref = oracle_lib.gemm_alg1_tc(A[rows], B, C[rows], terms=3, sep=0, kc=128)
+    assert np.array_equal(out[1][rows].view(np.uint32), ref.view(np.uint32))

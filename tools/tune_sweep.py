@@ -256,6 +256,7 @@ def main():
                 e["m_max"] = max(Ms)
         open_top(new, (("m_max", max(Ms)), ("n_max", max(Ns)), ("k_max", max(Ks))))
         entries += new
+        write(entries, logs, ops, t0, out_path)  # partial results survive a time limit
     if "knn" in ops:
         new = []
         logs["knn"] = []
@@ -275,6 +276,7 @@ def main():
                                 "qps": round(best["qps"])})
         open_top(new, (("m_max", max(NQ)), ("n_max", max(NX)), ("k_max", max(D))))
         entries += new
+        write(entries, logs, ops, t0, out_path)  # partial results survive a time limit
     if "kmeans" in ops:
         new = []
         logs["kmeans"] = []
@@ -293,8 +295,13 @@ def main():
                                 "ms": round(best["ms"], 4)})
         open_top(new, (("m_max", max(NP)), ("n_max", max(KC)), ("k_max", max(D))))
         entries += new
+        write(entries, logs, ops, t0, out_path)  # partial results survive a time limit
+    write(entries, logs, ops, t0, out_path)
+
+
+def write(entries, logs, ops, t0, out_path):
     order = {"gemm": 0, "gemm_b32": 1, "knn": 2, "kmeans": 3}
-    entries.sort(key=lambda e: (order[e["op"]], e["m_max"], e["n_max"], e["k_max"]))
+    entries = sorted(entries, key=lambda e: (order[e["op"]], e["m_max"], e["n_max"], e["k_max"]))
     doc = {"generated_by": "tools/tune_sweep.py", "rule": __doc__.split("GEMM rule:")[1].split("Tool code")[0]
            .replace("\n", " ").strip(), "entries": entries,
            "device": torch.cuda.get_device_name(), "when": time.strftime("%Y-%m-%dT%H:%M:%SZ", time.gmtime()),
