@@ -494,6 +494,46 @@ def main():
     except Exception as ex:  # pragma: no cover
         e2e = {"value": None, "unit": UNIT, "error": str(ex)[:200]}
 
+    # ---- B reused: B broadcast once and round-split once per rank (outside the timed loop,
+    # timed separately), each step splits only this rank's A rows (or fuses that split) and
+    # runs the GEMM on the pre-split B -- north_star's "B broadcast once" for a B that stays
+    # fixed across steps (e.g. reused weights); the headline above re-splits a fresh B per step
+    b_once = None
+    try:
+        _barrier(world)
+        s3, t3 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        s3.record(stream)
+        edist.broadcast_(B, world)
+        egemm.split(B, transpose=True, out=b_split)
+        t3.record(stream)
+        _barrier(world)
+        prep_ms = _allmax(s3.elapsed_time(t3), world)
+        fa_once = bool(egemm.query_config("gemm", m_loc, N, K, with_fused=True)[4] & 1)
+        ws_o = ws_a if fa_once else ws_p
+
+        def step_once():
+            if fa_once:
+                egemm.gemm(A, None, b_split=b_split, out=D, workspace=ws_o)
+            else:
+                egemm.split(A, out=a_split)
+                egemm.gemm(None, None, a_split=a_split, b_split=b_split, out=D, workspace=ws_o)
+        for _ in range(args.warmup):
+            step_once()
+        _barrier(world)
+        s3.record(stream)
+        for _ in range(args.steps):
+            step_once()
+        t3.record(stream)
+        _barrier(world)
+        o_ms = _allmax(s3.elapsed_time(t3), world) / args.steps
+        b_once = {"value": round(flop_total / (o_ms * 1e-3) / 1e12, 2), "unit": UNIT,
+                  "ms_per_step": round(o_ms, 4), "b_prepare_ms": round(prep_ms, 4),
+                  "config": list(egemm.query_config("gemm", m_loc, N, K, with_fused=True)),
+                  "note": "B broadcast + round-split once per rank (b_prepare_ms, untimed in the "
+                          "loop); per step: A-row split (or fused) + GEMM on the pre-split B"}
+    except Exception as ex:  # pragma: no cover
+        b_once = {"error": str(ex)[:200]}
+
     apps = {}
     if not args.no_apps:
         apps = _apps(world, rank, dev, args)
@@ -569,6 +609,7 @@ def main():
             "cpu_baseline": cpu, "clocks": dict(clocks, sm_mhz_in_kernel=round(kernel_mhz, 1)
                                                 if kernel_mhz else None),
             "split_ms_per_step": round(split_ms, 4),
+            "b_split_once": b_once,
             "paper_context": {"t4_speedup_vs_cublas_fp32": 3.13, "t4_speedup_vs_sdk": 11.18,
                               "note": "paper's numbers on Tesla T4 (P:63, P:2251, P:2325), context only"},
             "b200_context": context,
