@@ -578,7 +578,8 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
       // carries only B, A is loaded once per unit into a_res
       constexpr uint32_t TX = (FA || AR) ? 2 * G::B_BYTES : FB ? 2 * G::A_BYTES : G::STAGE_BYTES;
       uint32_t uctr = 0;
-      bool pace = (EPI == EPI_STORE) && p.sync != nullptr && !DIAG_NO_TMA;
+      const bool pace = (EPI == EPI_STORE) && p.sync != nullptr && !DIAG_NO_TMA;
+      bool pace_wait = pace;
       uint32_t gkb = 0;  // k-blocks this CTA has started loading, over all its units
       const bool idle = DIAG_NO_TMA && DIAG_MODE(2);  // diagnostics only
       for (int u = idle ? p.num_units : cluster; u < p.num_units; u += nclusters, uctr++) {
@@ -604,8 +605,10 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
             if (pace && (gkb % (uint32_t)p.pace_e) == 0) {
               const uint32_t e = gkb / (uint32_t)p.pace_e;
               sync_arrive(p.sync, e);
-              if (e >= (uint32_t)p.pace_s && !sync_wait(p.sync, e - p.pace_s, gridDim.x))
-                pace = false;  // not all CTAs resident: run unpaced (others time out too)
+              // a wait that times out (not all CTAs resident) stops this CTA's waiting but not
+              // its arrivals, so the CTAs that do pace are never held up by it
+              if (pace_wait && e >= (uint32_t)p.pace_s && !sync_wait(p.sync, e - p.pace_s, gridDim.x))
+                pace_wait = false;
             }
             gkb++;
             if (FA && p.a_pf && ns == 0) {
