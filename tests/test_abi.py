@@ -182,3 +182,23 @@ def test_knn_limits_and_merge_validation(lib):
     assert m(None, None, 0, 10, 4, 4, None, None, None, None) == egemm.ERR_INVALID_ARG
     assert m(None, None, 2, 0, 4, 4, None, None, None, None) == egemm.OK
     assert m(None, None, 2, 10, 4, 4, None, None, None, None) == egemm.ERR_INVALID_ARG  # NULL data
+
+
+def test_peer_reduce_and_bf16_split_validation(lib):
+    """egemm_kmeans_allreduce_finalize / egemm_split_bf16 validate host-side (no device work)."""
+    import ctypes
+    from paper_conf_ppopp_fengwcz0d21_b200 import egemm
+    arr = (ctypes.c_void_p * 2)(None, None)
+    f = lib.egemm_kmeans_allreduce_finalize
+    assert f(arr, arr, 0, 4, 4, None, None, None, None) == egemm.ERR_INVALID_ARG   # no ranks
+    assert f(arr, arr, 17, 4, 4, None, None, None, None) == egemm.ERR_INVALID_ARG  # > 16 peers
+    assert f(arr, arr, 2, 4, 4, None, None, None, None) == egemm.ERR_INVALID_ARG   # NULL peers
+    assert lib.egemm_split_bf16(None, -1, 4, 4, None, None, 4, 0, None) == egemm.ERR_INVALID_ARG
+    assert lib.egemm_split_bf16(None, 0, 4, 4, None, None, 4, 0, None) == egemm.OK
+    egemm.set_config_ex(operand_format=1)
+    try:
+        q = egemm.query_config_ex("gemm", 4096, 4096, 4096)
+        assert q["operand_format"] == 1 and q["fused"] == 0  # the converters make fp16 parts only
+        assert egemm.query_config_ex("knn", 4096, 4096, 128)["operand_format"] == 0
+    finally:
+        egemm.set_config_ex()
