@@ -6,10 +6,9 @@ set -x
 R=${1:-r02}
 O=gpurun_out
 NCU="ncu --set full --clock-control none --import-source on"
-cfg=$(python -c "from paper_conf_ppopp_fengwcz0d21_b200 import egemm; print(*egemm.query_config('gemm', 8192, 8192, 8192))")
 cfg5=$(python -c "from paper_conf_ppopp_fengwcz0d21_b200 import egemm; print(*egemm.query_config('gemm', 8192, 8192, 8192, with_fused=True))")
-timeout 600 $NCU -k regex:egemm_tc_kernel -c 1 -f -o $O/${R}_gemm8192 python tools/prof_gemm.py 8192 $cfg 2 > $O/ncu_gemm.log 2>&1
-timeout 300 $NCU -k regex:split -c 2 -f -o $O/${R}_split python tools/prof_gemm.py 8192 $cfg 1 > $O/ncu_split.log 2>&1
+timeout 600 $NCU -k regex:egemm_tc_kernel -c 1 -f -o $O/${R}_gemm8192 python tools/prof_gemm.py 8192 2 > $O/ncu_gemm.log 2>&1
+timeout 300 $NCU -k regex:split -c 2 -f -o $O/${R}_split python tools/prof_gemm.py 8192 1 > $O/ncu_split.log 2>&1
 timeout 600 $NCU -k regex:egemm_tc_kernel -c 1 -f -o $O/${R}_knn python tools/prof_apps.py knn > $O/ncu_knn.log 2>&1
 timeout 600 $NCU -k regex:"egemm_tc_kernel|km_" -c 10 -f -o $O/${R}_kmeans python tools/prof_apps.py kmeans > $O/ncu_kmeans.log 2>&1
 timeout 600 $NCU -k regex:egemm_tc_kernel -c 1 -f -o $O/${R}_skinny python tools/prof_skinny.py > $O/ncu_skinny.log 2>&1
