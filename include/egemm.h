@@ -215,7 +215,8 @@ int egemm_kmeans_finalize(const double* sums, const int64_t* counts, int64_t kc,
  *                operands must come from egemm_split_bf16).
  *  tail_peel   : STORE GEMMs with one n-tile of CTA-pair tiles: the rows of a last wave at
  *                most 60 % full run as a second, programmatically dependent launch of
- *                128 x 128 tiles on the SMs the main grid frees (-1 = table / on, 0 = off).
+ *                128 x 128 tiles on the SMs the main grid frees (-1 = table, default off;
+ *                0 = off, 1 = on).
  *                Same results bit for bit.
  */
 typedef struct {

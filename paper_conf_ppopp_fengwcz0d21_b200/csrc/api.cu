@@ -102,7 +102,7 @@ static TcConfig choose_config(int epi_kind, int64_t M, int64_t N, int64_t K, int
   c.kc = 64;  // promotion every 64 k: the most accurate single-accumulator setting
   c.ares = -1;
   c.pace = 1;
-  c.peel = -1;
+  c.peel = 0;  // measured slower on configs[2] (profiles/r02_skinny_peel.txt): table / override only
   if (epi_kind == EPI_STORE && M <= 128) { c.cg = 1; c.bn = 128; c.sep = 1; }
   {
     TuneEntry t;
