@@ -132,3 +132,21 @@ def test_elem_bound_holds_for_emu(oracle_lib):
     err = np.abs(oracle_lib.gemm_emu64(A, B, 3) - oracle_lib.gemm64(A, B))
     assert np.all(err <= oracle_lib.elem_bound(A, B, mma_ulps=0.0))
     assert math.isfinite(float(oracle_lib.elem_bound(A, B).max()))
+
+
+def test_gemm32_naive_closed_forms(oracle_lib):
+    """Reading R10 pinned by hand-derived values, not by re-running the formula:
+    * order: a = (2^24, 1, 1), b = (1, 1, 1): k ascending gives 2^24 + 1 -> 2^24 (an fp32 tie,
+      to even) twice, so 2^24; the exact sum 2^24 + 2 (what any other order would give).
+    * no FMA: a = (-1, 1 + 2^-12), b = (1, 1 + 2^-12): the product 1 + 2^-11 + 2^-24 rounds to
+      1 + 2^-11 (a tie, to even) before the add, so -1 + that = 2^-11 exactly; a fused
+      multiply-add would keep 2^-11 + 2^-24."""
+    A = np.array([[2.0 ** 24, 1.0, 1.0]], np.float32)
+    B = np.ones((3, 1), np.float32)
+    assert oracle_lib.gemm32_naive(A, B)[0, 0] == np.float32(2.0 ** 24)
+    assert oracle_lib.gemm64(A, B)[0, 0] == 2.0 ** 24 + 2
+    t = np.float32(1.0 + 2.0 ** -12)
+    A = np.array([[-1.0, t]], np.float32)
+    B = np.array([[1.0], [t]], np.float32)
+    assert oracle_lib.gemm32_naive(A, B)[0, 0] == np.float32(2.0 ** -11)
+    assert oracle_lib.gemm64(A, B)[0, 0] == 2.0 ** -11 + 2.0 ** -24
