@@ -56,6 +56,7 @@ const Knobs& knobs() {
     k.as_pf = env_int("EGEMM_AS_PREFETCH", 0);
     if (k.as_pf < 0) k.as_pf = 0;
     k.host_chunk = env_int("EGEMM_HOST_CHUNK", 0);
+    k.no_tma_store = env_int("EGEMM_NO_TMA_STORE", 0) == 1;
 #if EGEMM_DIAG
     k.dbg_no_tma = env_int("EGEMM_DEBUG_NO_TMA", 0) == 1;
     k.dbg_no_epi = env_int("EGEMM_DEBUG_NO_EPI", 0) == 1;

@@ -64,6 +64,7 @@ struct Knobs {
   int a_staged;        // fused A: TMA-staged in-place conversion when aligned (EGEMM_A_STAGED)
   int as_pf;           // fused A, staged: k-blocks of L2 prefetch (EGEMM_AS_PREFETCH)
   int host_chunk;      // egemm_gemm_host row chunk (EGEMM_HOST_CHUNK, 0 = auto)
+  int no_tma_store;    // EGEMM_NO_TMA_STORE=1: STORE epilogue with per-lane row stores (A/B runs)
   int dbg_no_tma, dbg_no_epi, dbg_mode;  // diagnostics (EGEMM_DEBUG_*; EGEMM_DIAG builds only)
 };
 const Knobs& knobs();

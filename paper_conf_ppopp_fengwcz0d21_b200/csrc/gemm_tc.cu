@@ -104,7 +104,7 @@ static int launch_tc_one(int64_t M, int64_t N, int64_t K, const TcOperands& ops,
     set_last_error("M, N must be < 2^30");
     return 2;
   }
-  CUtensorMap maps[4];
+  CUtensorMap maps[5];
   const int bnc = cfg.bn / cfg.cg;
   const bool fa = ops.a_f32 != nullptr && epi.kind == EPI_STORE;
   const bool fb = ops.b_f32 != nullptr && epi.kind == EPI_STORE && !fa;
@@ -121,6 +121,7 @@ static int launch_tc_one(int64_t M, int64_t N, int64_t K, const TcOperands& ops,
     maps[1] = maps[3];
   }
   if (fb) maps[3] = maps[2];  // fp32 B (row-major K x N) in unswizzled 64 x BNC boxes
+  maps[4] = maps[2];  // tm_d placeholder unless the STORE epilogue uses TMA stores (below)
   KParams kp = {};
   kp.K = (int)K;
   kp.fb = fb ? 1 : 0;
@@ -173,6 +174,13 @@ static int launch_tc_one(int64_t M, int64_t N, int64_t K, const TcOperands& ops,
   }
   kp.C = epi.C;
   kp.ldc = epi.ldc;
+  // D through TMA stores: STORE without C, 16-B aligned D and row stride (32 x 32 fp32 boxes,
+  // 128-B swizzle; the variants with 32-column epilogue groups use it, the others ignore it)
+  kp.tma_store = (epi.kind == EPI_STORE && !epi.C && epi.D && (epi.ldd % 4) == 0 &&
+                  ((uintptr_t)epi.D % 16) == 0 && !knobs().no_tma_store &&
+                  make_tmap_f32(&maps[4], epi.D, M, N, epi.ldd, 32, 32, true))
+                     ? 1
+                     : 0;
   kp.vec_ok = (epi.D && (epi.ldd % 4 == 0) && ((uintptr_t)epi.D % 16 == 0) &&
                (!epi.C || ((epi.ldc % 4 == 0) && ((uintptr_t)epi.C % 16 == 0))))
                   ? 1

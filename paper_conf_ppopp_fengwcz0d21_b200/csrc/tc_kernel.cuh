@@ -111,6 +111,7 @@ struct KParams {
   int fb;            // fused B split (host-side dispatch flag; tm_bhi maps the fp32 B)
   int bf16;          // operands are bf16 hi / lo parts (NEXT-3 variant), not fp16
   int pdl_wait;      // a peeled tail launch (programmatic dependent launch of the main grid)
+  int tma_store;     // STORE: D through TMA stores (tm_d; no C, aligned D); else per-lane stores
   unsigned long long* probe;  // device clock probe: [0..3] last launch, [4..6] running sums, [7] counter
   int debug_mode;    // EGEMM_DEBUG_MODE bits (diagnostics): 1 extra commit per k-block;
                      // with NO_TMA: 2 MMA warp ignores the full barriers (producer idle),
@@ -265,7 +266,8 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
     egemm_tc_kernel(const __grid_constant__ CUtensorMap tm_ahi,
                     const __grid_constant__ CUtensorMap tm_alo,
                     const __grid_constant__ CUtensorMap tm_bhi,
-                    const __grid_constant__ CUtensorMap tm_blo, const KParams p) {
+                    const __grid_constant__ CUtensorMap tm_blo,
+                    const __grid_constant__ CUtensorMap tm_d, const KParams p) {
   using G = Geo<CG, BN>;
   // FB (fused B split): the converter warpgroup builds B_hi / B_lo from TMA-staged fp32 B
   // tiles (row-major K x N, transposed to K-major on the way) while A comes pre-split by TMA
@@ -333,6 +335,12 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
   uint64_t* sempty = sfull + NSTG;           // AS: consumed by the 4 converter warps
   uint64_t* afull = sempty + NSTG;           // AS: a stage's fp32 A tile landed (TMA bytes)
   uint8_t* scratch = reinterpret_cast<uint8_t*>(bars + 2 * STAGES + 8 + 2 * NSTG + (AS ? STAGES : 0));  // merges
+  // TS (STORE): the result leaves through TMA stores -- each epilogue warp stages a 32 x 32
+  // fp32 block (128-B rows, 128-B swizzle) in its own 4 KiB buffer and one lane issues a
+  // bulk tensor store: coalesced full-line writes, the LSU free for the next unit's drains
+  // (the per-lane row stores wrote 32 rows x 16 B per instruction)
+  constexpr bool TS = (EPI == EPI_STORE) && !FB && (COLS % 32 == 0);
+  const uint32_t ts_base = (ptx::smem_u32(scratch) + 1023u) & ~1023u;
 
   const int warp = threadIdx.x >> 5;
   const int lane = threadIdx.x & 31;
@@ -901,6 +909,29 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
 #pragma unroll
             for (int j = 0; j < COLS; j++) tot[j] = __fadd_rn(tot[j], totx[j]);
           }
+          if constexpr (TS) {
+            if (p.tma_store) {
+              const uint32_t buf = ts_base + (uint32_t)ew * 4096u;
+              const int row0 = ui.m_tile * (kBM * CG) + (int)rank * kBM + q * 32;
+#pragma unroll
+              for (int c = 0; c < COLS / 32; c++) {
+                if (lane == 0) ptx::tma_store_wait_read0();  // the previous store read the buffer
+                __syncwarp();
+#pragma unroll
+                for (int k = 0; k < 8; k++)
+                  ptx::sts128(buf + lane * 128 + ((k ^ (lane & 7)) << 4), __float_as_uint(tot[c * 32 + 4 * k]),
+                              __float_as_uint(tot[c * 32 + 4 * k + 1]), __float_as_uint(tot[c * 32 + 4 * k + 2]),
+                              __float_as_uint(tot[c * 32 + 4 * k + 3]));
+                ptx::fence_proxy_async_smem();  // generic-proxy writes -> visible to the TMA unit
+                __syncwarp();
+                if (lane == 0) {  // rows >= M and columns >= N of the box are clipped by TMA
+                  ptx::tma_store_2d_u32(&tm_d, buf, col_base + c * 32, row0);
+                  ptx::tma_store_commit();
+                }
+              }
+              continue;
+            }
+          }
           if (row < p.M) {
             float* drow = p.D + row * p.ldd;
             const float* crow = p.C ? p.C + row * p.ldc : nullptr;
@@ -1197,6 +1228,9 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
   }
 
   // ============================ teardown ============================
+  if constexpr (TS) {
+    if (p.tma_store && warp >= EG::EPI0 && lane == 0) ptx::tma_store_wait0();  // stores complete
+  }
   __syncwarp();
   ptx::tc_fence_before();
   if constexpr (CG == 2) ptx::cluster_sync(); else __syncthreads();
@@ -1230,8 +1264,12 @@ constexpr size_t variant_smem() {
                              : EPI == EPI_KMEANS ? 2 * 2 * 4 * kBM * 4 : 0;
   constexpr bool NORM = (EPI != EPI_STORE);  // norm slot per stage + the A' ones tile
   constexpr size_t sb = (AR ? 2 * G::B_BYTES : G::STAGE_BYTES) + (NORM ? G::BNC * 32 : 0);
-  return 1024 + (size_t)STAGES * sb + (AR ? 4 * G::A_BYTES : 0) + (NORM ? kBM * 32 : 0) +
-         (FB ? 3 * kBM * kBK * 4 + 8 * 6 : 0) + (AS ? 8 * STAGES : 0) + 8 * (2 * STAGES + 8) + scratch;
+  constexpr size_t base = 1024 + (size_t)STAGES * sb + (AR ? 4 * G::A_BYTES : 0) + (NORM ? kBM * 32 : 0) +
+                          (FB ? 3 * kBM * kBK * 4 + 8 * 6 : 0) + (AS ? 8 * STAGES : 0) +
+                          8 * (2 * STAGES + 8) + scratch;
+  // TS: one 4 KiB TMA-store staging buffer per epilogue warp, 1 KiB aligned (128-B swizzle)
+  constexpr bool TS = (EPI == EPI_STORE) && !FB && ((BN / (NEPI / 4)) % 32 == 0);
+  return TS ? ((base + 1023) / 1024) * 1024 + (size_t)NEPI * 4096 : base;
 }
 
 template <int CG, int BN, bool SEP, int EPI, int STAGES, bool FA = false, bool AR = false,
@@ -1276,7 +1314,7 @@ static int launch_variant(const CUtensorMap* maps, const KParams& kp, int max_cl
   attr[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
   cfg.numAttrs = kp.pdl_wait ? 2 : 1;
-  cudaError_t e = cudaLaunchKernelEx(&cfg, kern, maps[0], maps[1], maps[2], maps[3], kp);
+  cudaError_t e = cudaLaunchKernelEx(&cfg, kern, maps[0], maps[1], maps[2], maps[3], maps[4], kp);
   if (e != cudaSuccess) {
     set_last_error("cudaLaunchKernelEx: %s", cudaGetErrorString(e));
     return 3;

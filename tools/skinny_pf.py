@@ -21,8 +21,8 @@ def main():
     B = torch.from_numpy(inputs.uniform((K, N), 201)).cuda()
     ws = torch.empty(egemm.gemm_workspace_size(M, N, K), dtype=torch.uint8, device="cuda")
     D = torch.empty((M, N), device="cuda")
-    cfgs = [None] + [dict(cg=2, bn=256, sep=0, kc=kc, fused=1, tail_peel=peel)
-                     for kc in (64, 128, 256) for peel in (0, 1)]
+    cfgs = [None] + [dict(cg=2, bn=256, sep=0, kc=kc, fused=1, stages=st)
+                     for kc in (64, 256) for st in (2, 3)]
     for c in cfgs:
         if c:
             egemm.set_config_ex(**c)
