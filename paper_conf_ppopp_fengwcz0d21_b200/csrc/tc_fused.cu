@@ -18,9 +18,8 @@ int dispatch_fused(const CUtensorMap* m, const KParams& kp, const TcConfig& c, c
   // fused A: aligned fp32 A is TMA-staged into the stage's A region and split in place;
   // otherwise the LDG converters
   if (c.cg == 2 && c.bn == 256 && !c.sep && kp.a_staged) {
-    // staged fused A: 4 (default) or 3 fp32-A slots + 2 B slots (decoupled rings)
-    if (c.stages == 3) return launch_variant<2, 256, false, EPI_STORE, 3, true, false, true>(m, kp, mc, s);
-    return launch_variant<2, 256, false, EPI_STORE, 4, true, false, true>(m, kp, mc, s);
+    if (c.stages == 2) return launch_variant<2, 256, false, EPI_STORE, 2, true, false, true>(m, kp, mc, s);
+    return launch_variant<2, 256, false, EPI_STORE, 3, true, false, true>(m, kp, mc, s);
   }
   if (c.cg == 2 && c.bn == 256 && !c.sep)
     return launch_variant<2, 256, false, EPI_STORE, 3, true>(m, kp, mc, s);

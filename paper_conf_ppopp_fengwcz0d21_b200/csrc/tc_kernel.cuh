@@ -315,20 +315,12 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
   // region and the converters split it in place; FB keeps a 3-slot fp32 staging ring.
   constexpr int NSTG = FB ? 3 : 0;
   constexpr int STG_BYTES = kBM * kBK * 4;
-  // AS rings (decoupled): the fp32 A tiles stream from DRAM through a STAGES-deep ring of
-  // 32 KiB slots (converted in place), the L2-resident B hi / lo through a 2-deep ring of its
-  // own -- more of the smem goes to the operand whose latency is long.  full / empty[] are the
-  // A ring's (converter arrivals / MMA commits), bfull / bempty[] the B ring's.
-  constexpr int AS_A2 = 2 * G::A_BYTES;  // one A slot: hi + lo (= the fp32 tile)
-  constexpr int AS_B2 = 2 * G::B_BYTES;  // one B slot: hi + lo
-  constexpr int AS_BR = 2;               // B ring depth
-  constexpr int RING_BYTES = AS ? STAGES * AS_A2 + AS_BR * AS_B2 : STAGES * SB;
   static_assert(!AS || FA, "AS is a fused-A mode");
   static_assert(!(FA && FB), "one fused operand at a time");
   static_assert(!FB || (CG == 2 && (BN == 256 || BN == 224) && EPI == EPI_STORE && !SEP),
                 "FB: 256 x 256 or 256 x 224 pair tiles");
   uint8_t* stage_base = smem;
-  uint8_t* a_res = smem + RING_BYTES;
+  uint8_t* a_res = smem + STAGES * SB;
   uint8_t* a_stg = a_res + AR_BYTES;
   uint8_t* ones_tile = a_stg + NSTG * STG_BYTES;
   uint64_t* bars = reinterpret_cast<uint64_t*>(ones_tile + ONES_BYTES);
@@ -341,10 +333,8 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * STAGES + 6);
   uint64_t* sfull = bars + 2 * STAGES + 8;   // AS: fp32 A tile landed (TMA bytes)
   uint64_t* sempty = sfull + NSTG;           // AS: consumed by the 4 converter warps
-  uint64_t* afull = sempty + NSTG;           // AS: a slot's fp32 A tile landed (TMA bytes)
-  uint64_t* bfull = afull + (AS ? STAGES : 0);  // AS: B ring slot landed (TMA bytes)
-  uint64_t* bempty = bfull + (AS ? AS_BR : 0);  // AS: B ring slot consumed (MMA commit)
-  uint8_t* scratch = reinterpret_cast<uint8_t*>(bars + 2 * STAGES + 8 + 2 * NSTG + (AS ? STAGES + 2 * AS_BR : 0));  // merges
+  uint64_t* afull = sempty + NSTG;           // AS: a stage's fp32 A tile landed (TMA bytes)
+  uint8_t* scratch = reinterpret_cast<uint8_t*>(bars + 2 * STAGES + 8 + 2 * NSTG + (AS ? STAGES : 0));  // merges
   // TS (STORE): the result leaves through TMA stores -- each epilogue warp stages a 32 x 32
   // fp32 block (128-B rows, 128-B swizzle) in its own 4 KiB buffer and one lane issues a
   // bulk tensor store: coalesced full-line writes, the LSU free for the next unit's drains
@@ -369,8 +359,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
     for (int s = 0; s < STAGES; s++) {
       // FA: the producer's expect_tx arrive plus one arrive per converter warp of the pair;
       // NORM: plus one arrive per norm warp of the pair
-      // (AS: the A ring's full[] only counts the converter warps; the B bytes go to bfull[])
-      ptx::mbar_init(&full[s], (AS ? 0 : 1) + (CONV ? 4 * CG : 0) + (NORM ? CG : 0));
+      ptx::mbar_init(&full[s], 1 + (CONV ? 4 * CG : 0) + (NORM ? CG : 0));
       ptx::mbar_init(&empty[s], 1);
     }
     for (int b = 0; b < 2; b++) {
@@ -379,13 +368,8 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
     }
     ptx::mbar_init(a_full, 1);
     ptx::mbar_init(a_empty, 1);
-    if constexpr (AS) {
+    if constexpr (AS)
       for (int s = 0; s < STAGES; s++) ptx::mbar_init(&afull[s], 1);
-      for (int s = 0; s < AS_BR; s++) {
-        ptx::mbar_init(&bfull[s], 1);
-        ptx::mbar_init(&bempty[s], 1);
-      }
-    }
     for (int i = 0; i < NSTG; i++) {
       ptx::mbar_init(&sfull[i], 1);
       ptx::mbar_init(&sempty[i], 4);
@@ -513,12 +497,10 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
             if constexpr (AS) {
               // the stage's A region holds the fp32 tile (2 boxes of 32 columns, SW128): row r,
               // 8 values k = 8c..8c+7 are fp32 16-B chunks 2(c%4), 2(c%4)+1 of box c/4 at chunk
-              // position j ^ (r & 7).  Each converter warp reads its 32 rows' values, then
-              // overwrites them with the hi / lo K-major tiles: the hi rows of warp w land on
-              // box 0's rows of warp w, the lo rows on box 1's -- a warp only overwrites what it
-              // has itself read (in order within the warp), so the warps need no barrier.
-              ptx::mbar_wait(&afull[stage], phase);  // (the producer waited for the free slot)
-              const uint32_t sb = ptx::smem_u32(stage_base + stage * AS_A2);
+              // position j ^ (r & 7).  All 4 converter warps read their 64 values first, meet
+              // at a named barrier, then overwrite the region with the hi / lo K-major tiles.
+              ptx::mbar_wait(&afull[stage], phase);  // (the producer waited for the free stage)
+              const uint32_t sb = ptx::smem_u32(stage_base + stage * G::STAGE_BYTES);
               const uint32_t xb = sb + (c >> 2) * (STG_BYTES / 2);
               const int j0 = (c & 3) * 2;
               float4 u[16];
@@ -529,7 +511,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
                 u[2 * it] = ptx::lds128f(rb + ((j0 ^ (r & 7)) << 4));
                 u[2 * it + 1] = ptx::lds128f(rb + (((j0 + 1) ^ (r & 7)) << 4));
               }
-              __syncwarp();  // this warp's fp32 values are in registers
+              named_bar_sync(9, 128);  // every fp32 value of the tile is in registers
 #pragma unroll
               for (int it = 0; it < 8; it++) {
                 const int r = warp * 32 + it * 4 + rsub;
@@ -603,8 +585,6 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
       // FA: only B comes through TMA (A is written by the converter warps); AR: the ring
       // carries only B, A is loaded once per unit into a_res
       constexpr uint32_t TX = (FA || AR) ? 2 * G::B_BYTES : FB ? 2 * G::A_BYTES : G::STAGE_BYTES;
-      int bst = 0;  // AS: B ring slot / parity
-      uint32_t bph = 0;
       uint32_t uctr = 0;
       const bool pace = (EPI == EPI_STORE) && p.sync != nullptr && !DIAG_NO_TMA;
       bool pace_wait = pace;
@@ -657,28 +637,6 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
                 pf(kf - p.num_kb, nu.m_tile * (kBM * CG) + (int)rank * kBM);
               }
             }
-            if constexpr (AS) {
-              // A slot: this CTA's fp32 A tile (two 32-column SW128 boxes) for the converters
-              ptx::mbar_wait(&empty[stage], phase ^ 1u);
-              uint8_t* as_ = stage_base + stage * AS_A2;
-              ptx::mbar_arrive_expect_tx(&afull[stage], STG_BYTES);
-              ptx::tma_load_2d(&tm_ahi, &afull[stage], as_, kb * kBK, arow);
-              ptx::tma_load_2d(&tm_ahi, &afull[stage], as_ + STG_BYTES / 2, kb * kBK + 32, arow);
-              if (++stage == STAGES) { stage = 0; phase ^= 1u; }
-              // B slot: this CTA's half of the B hi / lo tile (pair loads signal the leader)
-              ptx::mbar_wait(&bempty[bst], bph ^ 1u);
-              uint8_t* bs_ = stage_base + STAGES * AS_A2 + bst * AS_B2;
-              if (leader) ptx::mbar_arrive_expect_tx(&bfull[bst], AS_B2 * CG);
-              if constexpr (CG == 1) {
-                ptx::tma_load_2d(&tm_bhi, &bfull[bst], bs_, kb * kBK, brow);
-                ptx::tma_load_2d(&tm_blo, &bfull[bst], bs_ + G::B_BYTES, kb * kBK, brow);
-              } else {
-                ptx::tma_load_2d_pair(&tm_bhi, &bfull[bst], bs_, kb * kBK, brow);
-                ptx::tma_load_2d_pair(&tm_blo, &bfull[bst], bs_ + G::B_BYTES, kb * kBK, brow);
-              }
-              if (++bst == AS_BR) { bst = 0; bph ^= 1u; }
-              continue;
-            }
             ptx::mbar_wait(&empty[stage], phase ^ 1u);
             uint8_t* sb = stage_base + stage * SB;
             if (DIAG_NO_TMA) {  // diagnostics only: MMA-issue ceiling without operand traffic
@@ -688,6 +646,11 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
             }
             if (leader) ptx::mbar_arrive_expect_tx(&full[stage], TX * CG);
             const int k0 = kb * kBK;
+            if constexpr (AS) {  // this CTA's fp32 A tile into the stage's A region
+              ptx::mbar_arrive_expect_tx(&afull[stage], STG_BYTES);
+              ptx::tma_load_2d(&tm_ahi, &afull[stage], sb, k0, arow);
+              ptx::tma_load_2d(&tm_ahi, &afull[stage], sb + STG_BYTES / 2, k0 + 32, arow);
+            }
             if constexpr (CG == 1) {
               if (!FA && !AR) {
                 ptx::tma_load_2d(&tm_ahi, &full[stage], sb, k0, arow);
@@ -786,8 +749,6 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
       const uint32_t sbase = ptx::smem_u32(stage_base);
       int stage = 0;
       uint32_t phase = 0;
-      int bst = 0;  // AS: B ring slot / parity
-      uint32_t bph = 0;
       uint32_t chunk_ctr = 0;
       uint32_t uctr = 0;
       const uint32_t abase = ptx::smem_u32(a_res);
@@ -809,15 +770,13 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
             const int kb1 = min(p.num_kb, kb0 + p.kb_per_chunk);
             for (int kb = kb0; kb < kb1; kb++) {
               if (!(DIAG_NO_TMA && DIAG_MODE(2))) ptx::mbar_wait(&full[stage], phase);
-              if constexpr (AS) ptx::mbar_wait(&bfull[bst], bph);
               ptx::tc_fence_after();
-              const uint32_t sa = sbase + stage * (AS ? AS_A2 : SB);
+              const uint32_t sa = sbase + stage * SB;
               const uint32_t aa = AR ? abase + kb * 2 * G::A_BYTES : sa;
-              const uint32_t bb = AS ? sbase + STAGES * AS_A2 + bst * AS_B2 : sa + B_OFF;
               const uint64_t d_ahi = ptx::sdesc_kmajor_sw128(aa);
               const uint64_t d_alo = ptx::sdesc_kmajor_sw128(aa + G::A_BYTES);
-              const uint64_t d_bhi = ptx::sdesc_kmajor_sw128(bb);
-              const uint64_t d_blo = ptx::sdesc_kmajor_sw128(bb + G::B_BYTES);
+              const uint64_t d_bhi = ptx::sdesc_kmajor_sw128(sa + B_OFF);
+              const uint64_t d_blo = ptx::sdesc_kmajor_sw128(sa + B_OFF + G::B_BYTES);
               // Alg. 1 on every 16-wide k-slice, in the paper's order:
               // [lo*lo,] lo*hi, hi*lo, hi*hi chained through the accumulator (SEP: hi*hi in
               // its own).  The first MMA of a promotion chunk starts it from zero.
@@ -854,14 +813,10 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
                                       ptx::idesc_tf32_f32(kBM * CG, BN), 1u);
                 }
                 if (!(DIAG_NO_TMA && DIAG_MODE(4))) ptx::mma_commit<CG>(&empty[stage]);
-                if constexpr (AS) ptx::mma_commit<CG>(&bempty[bst]);
                 if (DIAG_MODE(1)) ptx::mma_commit<CG>(a_empty);  // diagnostics only
               }
               __syncwarp();
               if (++stage == STAGES) { stage = 0; phase ^= 1u; }
-              if constexpr (AS) {
-                if (++bst == AS_BR) { bst = 0; bph ^= 1u; }
-              }
             }
             if (ptx::elect_one()) ptx::mma_commit<CG>(&acc_full[buf]);
             __syncwarp();
@@ -1309,10 +1264,8 @@ constexpr size_t variant_smem() {
                              : EPI == EPI_KMEANS ? 2 * 2 * 4 * kBM * 4 : 0;
   constexpr bool NORM = (EPI != EPI_STORE);  // norm slot per stage + the A' ones tile
   constexpr size_t sb = (AR ? 2 * G::B_BYTES : G::STAGE_BYTES) + (NORM ? G::BNC * 32 : 0);
-  // AS: decoupled rings -- STAGES fp32-A slots (= A hi + lo bytes) and 2 B hi / lo slots
-  constexpr size_t ring = AS ? (size_t)STAGES * 2 * G::A_BYTES + 2 * 2 * G::B_BYTES : (size_t)STAGES * sb;
-  constexpr size_t base = 1024 + ring + (AR ? 4 * G::A_BYTES : 0) + (NORM ? kBM * 32 : 0) +
-                          (FB ? 3 * kBM * kBK * 4 + 8 * 6 : 0) + (AS ? 8 * (STAGES + 4) : 0) +
+  constexpr size_t base = 1024 + (size_t)STAGES * sb + (AR ? 4 * G::A_BYTES : 0) + (NORM ? kBM * 32 : 0) +
+                          (FB ? 3 * kBM * kBK * 4 + 8 * 6 : 0) + (AS ? 8 * STAGES : 0) +
                           8 * (2 * STAGES + 8) + scratch;
   // TS: one 4 KiB TMA-store staging buffer per epilogue warp, 1 KiB aligned (128-B swizzle)
   constexpr bool TS = (EPI == EPI_STORE) && !FB && ((BN / (NEPI / 4)) % 32 == 0);
