@@ -497,8 +497,10 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
             if constexpr (AS) {
               // the stage's A region holds the fp32 tile (2 boxes of 32 columns, SW128): row r,
               // 8 values k = 8c..8c+7 are fp32 16-B chunks 2(c%4), 2(c%4)+1 of box c/4 at chunk
-              // position j ^ (r & 7).  All 4 converter warps read their 64 values first, meet
-              // at a named barrier, then overwrite the region with the hi / lo K-major tiles.
+              // position j ^ (r & 7).  Each converter warp reads its 32 rows' values, then
+              // overwrites them with the hi / lo K-major tiles: the hi rows of warp w land on
+              // box 0's rows of warp w, the lo rows on box 1's -- a warp only overwrites what it
+              // has itself read (in order within the warp), so the warps need no barrier.
               ptx::mbar_wait(&afull[stage], phase);  // (the producer waited for the free stage)
               const uint32_t sb = ptx::smem_u32(stage_base + stage * G::STAGE_BYTES);
               const uint32_t xb = sb + (c >> 2) * (STG_BYTES / 2);
@@ -511,7 +513,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
                 u[2 * it] = ptx::lds128f(rb + ((j0 ^ (r & 7)) << 4));
                 u[2 * it + 1] = ptx::lds128f(rb + (((j0 + 1) ^ (r & 7)) << 4));
               }
-              named_bar_sync(9, 128);  // every fp32 value of the tile is in registers
+              __syncwarp();  // this warp's fp32 values are in registers
 #pragma unroll
               for (int it = 0; it < 8; it++) {
                 const int r = warp * 32 + it * 4 + rsub;
