@@ -237,12 +237,20 @@ def main():
         ["gemm", "gemm_b32", "knn", "kmeans"]
     out_path = sys.argv[sys.argv.index("--out") + 1] if "--out" in sys.argv else OUT
     old = json.load(open(OUT)) if os.path.exists(OUT) else {"entries": []}
-    entries = [e for e in old.get("entries", []) if e["op"] not in ops]
+    entries = [e for e in old.get("entries", []) if e["op"] not in ops]  # (--merge: all kept, below)
     logs = {}
     t0 = time.time()
     Ms = [128, 256, 1024, 2048, 4096, 8192, 65536] if not quick else [1024, 8192]
     Ns = [256, 1024, 8192] if not quick else [256, 8192]
     Ks = [256, 1024, 2048, 4096, 8192] if not quick else [1024, 8192]
+    # --merge --ns 2048,4096: add buckets between the existing ones (e.g. the square sweep's
+    # 2048^3 / 4096^3 shapes) and keep every other entry of the op
+    merge = "--merge" in sys.argv
+    grid_n = [int(v) for v in sys.argv[sys.argv.index("--ns") + 1].split(",")] if "--ns" in sys.argv else None
+    if merge:
+        entries = list(old.get("entries", []))
+    if grid_n:
+        Ns = grid_n
     for op in ("gemm", "gemm_b32"):
         if op not in ops:
             continue
@@ -269,7 +277,10 @@ def main():
         for e in new:
             if e["m_max"] == wide_top and e["n_max"] > 1024:
                 e["m_max"] = max(Ms)
-        open_top(new, (("m_max", max(Ms)), ("n_max", max(Ns)), ("k_max", max(Ks))))
+        open_top(new, (("m_max", max(Ms)), ("k_max", max(Ks))) + ((("n_max", max(Ns)),) if not merge else ()))
+        if merge:  # replace only the re-swept buckets
+            keys = {(e["op"], e["m_max"], e["n_max"], e["k_max"]) for e in new}
+            entries = [e for e in entries if (e["op"], e["m_max"], e["n_max"], e["k_max"]) not in keys]
         entries += new
         write(entries, logs, ops, t0, out_path)  # partial results survive a time limit
     if "knn" in ops:
