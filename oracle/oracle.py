@@ -64,7 +64,7 @@ def lib():
         L.oracle_rownorm.restype = None
         L.oracle_tc_mma16.argtypes = [P, P, I, ctypes.c_float, I]
         L.oracle_tc_mma16.restype = ctypes.c_float
-        L.oracle_gemm_alg1_tc.argtypes = [I64, I64, I64, P, P, P, I, I, I64, I, P]
+        L.oracle_gemm_alg1_tc.argtypes = [I64, I64, I64, P, P, P, I, I, I64, I, I64, P]
         L.oracle_gemm_alg1_tc.restype = None
         L.oracle_tc_rows.argtypes = [I64, I64, I, P, P, P, P]
         L.oracle_tc_rows.restype = None
@@ -319,19 +319,23 @@ def bf16_bits_to_f64(bits):
     return (np.asarray(bits, np.uint32) << 16).view(np.float32).astype(np.float64)
 
 
-def gemm_alg1_tc(A, B, C=None, terms: int = 3, sep: int = 0, kc: int = 0, fmt: str = "f16"):
+def gemm_alg1_tc(A, B, C=None, terms: int = 3, sep: int = 0, kc: int = 0, fmt: str = "f16",
+                 kpart: int = 0):
     """Alg. 1 step by step on the profiled tensor-core primitive: per 16-wide
     k-slice in ascending k, [lo*lo,] lo*hi, hi*lo, hi*hi chained through one fp32
     accumulator; promotion into an fp32 total every kc k-elements (reading R21; kc = 0:
     the paper's single chain over K); sep = 1: hi*hi in its own chain; + C at the end (R7).
-    fmt "bf16": the bf16 round-split variant (NEXT-3)."""
+    fmt "bf16": the bf16 round-split variant (NEXT-3).  kpart > 0: split-K reading -- K in
+    contiguous parts of kpart elements, each chained and promoted on its own, the part totals
+    added in k order (then + C)."""
     A, B = _f32(A), _f32(B)
     M, K = A.shape
     N = B.shape[1]
     D = np.empty((M, N), np.float32)
     Cp = _f32(C) if C is not None else None
     lib().oracle_gemm_alg1_tc(M, N, K, _p(A), _p(B), _p(Cp) if Cp is not None else None,
-                              int(terms), int(sep), int(kc), 1 if fmt == "bf16" else 0, _p(D))
+                              int(terms), int(sep), int(kc), 1 if fmt == "bf16" else 0, int(kpart),
+                              _p(D))
     return D
 
 

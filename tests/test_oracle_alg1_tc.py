@@ -156,3 +156,23 @@ def test_alg1_tc_bf16_variant_closed_forms(oracle_lib):
     with np.errstate(all="ignore"):
         D16 = oracle_lib.gemm_alg1_tc(Aw, Bw, kc=64)
     assert not np.all(np.isfinite(D16))  # fp16 parts overflow
+
+
+def test_alg1_tc_kparts_split_k_reading(oracle_lib):
+    """Split-K reading (R21): kpart >= K is the single part; integer inputs stay exact for any
+    split; and the parts compose as their own Alg. 1 runs: D(kpart) = RN(D(A[:, :p], B[:p]) +
+    D(A[:, p:], B[p:])) with C added last -- checked against two independent oracle calls."""
+    A, B = inputs.uniform((20, 500), 31), inputs.uniform((500, 17), 32)
+    C = inputs.uniform((20, 17), 33)
+    one = oracle_lib.gemm_alg1_tc(A, B, C, kc=128)
+    assert np.array_equal(oracle_lib.gemm_alg1_tc(A, B, C, kc=128, kpart=500), one)
+    assert np.array_equal(oracle_lib.gemm_alg1_tc(A, B, C, kc=128, kpart=1024), one)
+    for sep in (0, 1):
+        two = oracle_lib.gemm_alg1_tc(A, B, C, sep=sep, kc=128, kpart=256)
+        lo = oracle_lib.gemm_alg1_tc(A[:, :256], B[:256], sep=sep, kc=128)
+        hi = oracle_lib.gemm_alg1_tc(A[:, 256:], B[256:], sep=sep, kc=128)
+        assert np.array_equal(two, ((lo + hi).astype(np.float32) + C).astype(np.float32))
+    Ai, Bi = inputs.integers((9, 700), 34), inputs.integers((700, 5), 35)
+    ref = (Ai.astype(np.int64) @ Bi.astype(np.int64)).astype(np.float32)
+    for kp in (64, 192, 448):
+        assert np.array_equal(oracle_lib.gemm_alg1_tc(Ai, Bi, kc=64, kpart=kp), ref)
