@@ -103,8 +103,9 @@ int egemm_split_bf16(const float* x, int64_t rows, int64_t cols, int64_t ldx, ui
  *      alias A or B; D may equal C only if ldd == ldc.
  *  terms : 0 (tuning-table default, 3), 3, or 4.
  *  workspace : device scratch of >= egemm_gemm_workspace_size(...) bytes (256-B aligned),
- *      used for the on-the-fly split of operands given only in fp32 and, in its last
- *      256 B, for the k-pacing counters that keep the persistent clusters within a few
+ *      used for the on-the-fly split of operands given only in fp32, for the split-K parts
+ *      buffer when the configuration splits K (EGEMM_ERR_WORKSPACE if it does not fit), and,
+ *      in its last 256 B, for the k-pacing counters that keep the persistent clusters within a few
  *      k-blocks of each other (L2 reuse of shared tiles).  The pacing is
  *      optional: a workspace that only covers the splits (NULL when both operands are
  *      pre-split) is accepted and the kernel runs unpaced; results are identical.
@@ -218,10 +219,13 @@ int egemm_kmeans_finalize(const double* sums, const int64_t* counts, int64_t kc,
  *                128 x 128 tiles on the SMs the main grid frees (-1 = table, default off;
  *                0 = off, 1 = on).
  *                Same results bit for bit.
+ *  ksplit      : STORE split-K (R21's k-parts): K in up to ksplit contiguous parts, each tile's
+ *                parts run as separate units, their fp32 results are added in k order (then
+ *                + C) by a reduce pass; needs the larger egemm_gemm_workspace_size (0/1 = none).
  */
 typedef struct {
   int cg, bn, sep, kc, stages, fused, terms, n_slices, epi_warps, a_resident, pace, max_clusters,
-      operand_format, tail_peel;
+      operand_format, tail_peel, ksplit;
 } egemm_config_t;
 
 /* Thread-local override of the tuning table for the next calls of this thread: fields set

@@ -122,6 +122,7 @@ static TcConfig choose_config(int epi_kind, int64_t M, int64_t N, int64_t K, int
       c.nepi = t.nepi;
       if (t.ares >= 0) c.ares = t.ares;
       if (t.peel >= 0) c.peel = t.peel;
+      if (t.ksplit > 1) c.ksplit = t.ksplit;
     }
   }
   if (terms == 3 || terms == 4) c.terms = terms;  // the call's explicit term count wins
@@ -145,6 +146,7 @@ static TcConfig choose_config(int epi_kind, int64_t M, int64_t N, int64_t K, int
     if (o.pace >= 0) c.pace = o.pace;
     if (o.max_clusters) c.max_clusters = o.max_clusters;
     if (o.tail_peel >= 0) c.peel = o.tail_peel;
+    if (o.ksplit) c.ksplit = o.ksplit;
     if (o.operand_format == 1 && epi_kind == EPI_STORE) {
       c.fmt = 1;
       c.fa = 0;  // the fused converters produce fp16 parts only
@@ -153,6 +155,7 @@ static TcConfig choose_config(int epi_kind, int64_t M, int64_t N, int64_t K, int
   if (c.kc < 64) c.kc = 64;
   c.kc = (c.kc / 64) * 64;
   if (epi_kind != EPI_STORE) {  // kNN / kMeans: one accumulator (the norm MMA adds into it)
+    c.ksplit = 0;
     c.sep = 0;
     c.terms = 3;
     if (!((c.cg == 2 && c.bn == 256) || (c.cg == 1 && c.bn == 128))) { c.cg = 2; c.bn = 256; }
@@ -275,6 +278,7 @@ static void to_public(const TcConfig& c, int op, egemm_config_t* o) {
   o->max_clusters = c.max_clusters;
   o->operand_format = c.fmt;
   o->tail_peel = c.peel;
+  o->ksplit = c.ksplit > 1 ? c.ksplit : 1;
 }
 
 int egemm_query_config(int op, int64_t M, int64_t N, int64_t K, int* cg, int* bn, int* sep,
@@ -362,7 +366,8 @@ int egemm_set_config_ex(const egemm_config_t* cfg) {
       !(o.terms == 0 || o.terms == 3 || o.terms == 4) || o.n_slices < 0 || o.n_slices > 16 ||
       !(o.epi_warps == 0 || o.epi_warps == 8 || o.epi_warps == 16) || o.a_resident < -1 ||
       o.a_resident > 1 || o.pace < -1 || o.pace > 1 || o.max_clusters < 0 ||
-      o.operand_format < 0 || o.operand_format > 1 || o.tail_peel < -1 || o.tail_peel > 1) {
+      o.operand_format < 0 || o.operand_format > 1 || o.tail_peel < -1 || o.tail_peel > 1 ||
+      o.ksplit < 0 || o.ksplit > 16) {
     set_last_error("unsupported config cg=%d bn=%d sep=%d kc=%d fused=%d stages=%d terms=%d "
                    "n_slices=%d epi_warps=%d", o.cg, o.bn, o.sep, o.kc, o.fused, o.stages, o.terms,
                    o.n_slices, o.epi_warps);
@@ -436,7 +441,10 @@ static size_t gemm_operand_ws(int64_t M, int64_t N, int64_t K, int a_presplit, i
 size_t egemm_gemm_workspace_size(int64_t M, int64_t N, int64_t K, int a_presplit,
                                  int b_presplit) {
   if (M <= 0 || N <= 0 || K <= 0) return 0;
-  return gemm_operand_ws(M, N, K, a_presplit, b_presplit) + kPaceBytes;
+  // (+ the split-K parts buffer when the table / this thread's override picks split-K)
+  const TcConfig cfg = choose_config(EPI_STORE, M, N, K, 0, !b_presplit);
+  return gemm_operand_ws(M, N, K, a_presplit, b_presplit) +
+         ((ksplit_ws_bytes(M, N, K, cfg) + 255) & ~size_t(255)) + kPaceBytes;
 }
 
 int egemm_gemm(int64_t M, int64_t N, int64_t K, egemm_operand_t A, egemm_operand_t B,
@@ -505,6 +513,14 @@ int egemm_gemm(int64_t M, int64_t N, int64_t K, egemm_operand_t A, egemm_operand
   epi.ldd = ldd;
   epi.C = C;
   epi.ldc = ldc;
+  if (const size_t pb = ksplit_ws_bytes(M, N, K, cfg)) {  // split-K parts buffer
+    if (!workspace || workspace_bytes < cv.off + pb) {
+      set_last_error("workspace %zu < %zu (split-K parts buffer; see egemm_gemm_workspace_size)",
+                     workspace_bytes, cv.off + pb);
+      return EGEMM_ERR_WORKSPACE;
+    }
+    epi.partial = cv.take<float>(pb / sizeof(float));
+  }
   if (workspace && workspace_bytes >= cv.off + kPaceBytes) epi.sync = cv.take<uint32_t>(64);
   r = launch_tc(M, N, K, ops, cfg, epi, s);
   return r == 0 ? EGEMM_OK : (r == 2 ? EGEMM_ERR_UNSUPPORTED : EGEMM_ERR_CUDA);
@@ -626,6 +642,7 @@ int egemm_gemm_host(int64_t M, int64_t N, int64_t K, const float* A_host, int64_
     Dd[b] = cv.take<float>((size_t)(mc * N));
   }
   TcConfig cfg = choose_config(EPI_STORE, mc, N, K, terms);
+  cfg.ksplit = 0;  // (no parts buffer in the host pipeline's workspace)
   bool ok = true;
   auto chk = [&](cudaError_t e) { ok = ok && (e == cudaSuccess); };
   chk(cudaStreamWaitEvent(s, hp->ev_done, 0));  // the previous call's pipeline has drained

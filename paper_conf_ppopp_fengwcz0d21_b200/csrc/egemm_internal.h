@@ -52,7 +52,17 @@ struct TcConfig {
   int pace;      // STORE: k-pacing (1 = when the workspace has room, 0 = off)
   int fmt;       // operand parts: 0 = fp16 (the paper's round-split), 1 = bf16 (NEXT-3)
   int peel;      // STORE: peel a mostly-empty last wave into a 128 x 128 tail launch (-1 auto, 0 off)
+  int ksplit;    // STORE: split-K parts (<= 1: none)
 };
+
+// Split-K geometry of a STORE launch: k-blocks per part, parts actually used (no empty part),
+// rows per part block (the tile height multiple) and the parts buffer's row stride.
+struct KSplit {
+  int parts, kb_per_part;
+  int64_t m_pad, ld;
+};
+KSplit ksplit_geometry(int64_t M, int64_t N, int64_t K, const TcConfig& cfg);
+size_t ksplit_ws_bytes(int64_t M, int64_t N, int64_t K, const TcConfig& cfg);
 
 // Environment knobs for experiments, read once per process (tools/; the product path takes
 // its configuration from the tuning table and egemm_set_config_ex).
@@ -77,6 +87,7 @@ struct TcEpilogue {
   const float* C;
   int64_t ldc;
   uint32_t* sync;      // nullable: 256 B of workspace for the k-pacing counters
+  float* partial;      // split-K (cfg.ksplit > 1): the parts' results, ksplit_ws_bytes() of workspace
   // EPI_KNN / EPI_KMEANS: per-B-row squared norms (||x_j||^2 or ||c_j||^2)
   const float* bnorm;
   // EPI_KNN
@@ -126,7 +137,7 @@ struct TuneEntry {
   int op = -1;  // EpiKind or kOpGemmB32
   long long m_max = 0, n_max = 0, k_max = 0;
   int cg = 0, bn = 0, sep = 0, kc = 0, fa = 0;
-  int terms = 0, stages = 0, nslices = 0, nepi = 0, ares = -1, peel = -1;
+  int terms = 0, stages = 0, nslices = 0, nepi = 0, ares = -1, peel = -1, ksplit = 0;
 };
 bool tune_lookup(int op, long long M, long long N, long long K, TuneEntry* out);
 const char* tune_table_path();

@@ -157,6 +157,13 @@ static int launch_tc_one(int64_t M, int64_t N, int64_t K, const TcOperands& ops,
   kp.num_kb = (int)((K + kBK - 1) / kBK);
   kp.kb_per_chunk = cfg.kc / kBK;
   if (kp.kb_per_chunk < 1) kp.kb_per_chunk = 1;
+  {
+    const KSplit ks = ksplit_geometry(M, N, K, cfg);
+    kp.ksplit = epi.kind == EPI_STORE ? ks.parts : 1;
+    kp.kb_per_part = ks.kb_per_part;
+    kp.m_pad = (int)ks.m_pad;
+    if (kp.ksplit > 1) kp.a_pf = 0;  // (the L2 prefetch follows one k-range per unit)
+  }
   kp.terms = cfg.terms;
   kp.m_tiles = (int)((M + kBM * cfg.cg - 1) / (kBM * cfg.cg));
   kp.n_tiles = (int)((N + cfg.bn - 1) / cfg.bn);
@@ -180,7 +187,8 @@ static int launch_tc_one(int64_t M, int64_t N, int64_t K, const TcOperands& ops,
   // 128-B swizzle; the variants with 32-column epilogue groups use it, the others ignore it)
   kp.tma_store = (epi.kind == EPI_STORE && !epi.C && epi.D && (epi.ldd % 4) == 0 &&
                   ((uintptr_t)epi.D % 16) == 0 && !knobs().no_tma_store &&
-                  make_tmap_f32(&maps[4], epi.D, M, N, epi.ldd, 32, 32, true))
+                  make_tmap_f32(&maps[4], epi.D, cfg.ksplit > 1 ? ksplit_geometry(M, N, K, cfg).parts *
+                                ksplit_geometry(M, N, K, cfg).m_pad : M, N, epi.ldd, 32, 32, true))
                      ? 1
                      : 0;
   kp.vec_ok = (epi.D && (epi.ldd % 4 == 0) && ((uintptr_t)epi.D % 16 == 0) &&
@@ -195,7 +203,7 @@ static int launch_tc_one(int64_t M, int64_t N, int64_t K, const TcOperands& ops,
   kp.assign = epi.assign;
   kp.best_key = epi.best_key;
   if (epi.kind == EPI_STORE) {
-    kp.num_units = kp.m_tiles * kp.n_tiles;
+    kp.num_units = kp.m_tiles * kp.n_tiles * kp.ksplit;
     return (fa || fb) ? dispatch_fused(maps, kp, cfg, stream) : dispatch_store(maps, kp, cfg, stream);
   }
   if (kp.num_kb > kp.kb_per_chunk) {
@@ -219,10 +227,68 @@ static int launch_tc_one(int64_t M, int64_t N, int64_t K, const TcOperands& ops,
 // programmatic dependent launch: its CTAs start on the SMs the main grid frees as it
 // drains, instead of the freed SMs idling until the main grid's slowest cluster ends; it
 // waits for the main grid before it completes, so stream order is kept for later work.
+KSplit ksplit_geometry(int64_t M, int64_t N, int64_t K, const TcConfig& cfg) {
+  KSplit g = {1, (int)((K + kBK - 1) / kBK), M, N};
+  const int num_kb = (int)((K + kBK - 1) / kBK);
+  if (cfg.ksplit > 1 && num_kb > 1) {
+    const int q = (num_kb + cfg.ksplit - 1) / cfg.ksplit;
+    g.parts = (num_kb + q - 1) / q;
+    g.kb_per_part = q;
+    const int64_t th = (int64_t)kBM * cfg.cg;
+    g.m_pad = (M + th - 1) / th * th;
+    g.ld = (N + 3) / 4 * 4;
+  }
+  return g;
+}
+
+size_t ksplit_ws_bytes(int64_t M, int64_t N, int64_t K, const TcConfig& cfg) {
+  const KSplit g = ksplit_geometry(M, N, K, cfg);
+  return g.parts > 1 ? (size_t)g.parts * (size_t)g.m_pad * (size_t)g.ld * sizeof(float) : 0;
+}
+
+// D = fold over the parts in k order (RN) of the split-K part results (+ C last): the
+// promotion reading's combination of R21's k-parts.
+__global__ void __launch_bounds__(256) ksplit_reduce_kernel(const float* __restrict__ part, int parts,
+                                                            int64_t M, int64_t N, int64_t m_pad,
+                                                            int64_t ldp, const float* __restrict__ C,
+                                                            int64_t ldc, float* __restrict__ D,
+                                                            int64_t ldd) {
+  const int64_t total = M * N;
+  const int64_t stride = (int64_t)gridDim.x * blockDim.x;
+  for (int64_t e = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; e < total; e += stride) {
+    const int64_t i = e / N, j = e - i * N;
+    float v = part[i * ldp + j];
+    for (int s = 1; s < parts; s++) v = __fadd_rn(v, part[((int64_t)s * m_pad + i) * ldp + j]);
+    if (C) v = __fadd_rn(v, C[i * ldc + j]);
+    D[i * ldd + j] = v;
+  }
+}
+
 int launch_tc(int64_t M, int64_t N, int64_t K, const TcOperands& ops, const TcConfig& cfg,
               const TcEpilogue& epi, cudaStream_t stream) {
   const bool fb = ops.b_f32 != nullptr && ops.a_f32 == nullptr;
-  if (epi.kind == EPI_STORE && cfg.peel != 0 && cfg.cg == 2 && (cfg.bn == 256 || cfg.bn == 224) &&
+  if (epi.kind == EPI_STORE && cfg.ksplit > 1) {
+    const KSplit g = ksplit_geometry(M, N, K, cfg);
+    if (g.parts > 1) {
+      if (!epi.partial) {
+        set_last_error("split-K: no parts buffer (workspace)");
+        return 2;
+      }
+      TcEpilogue e2 = epi;
+      e2.D = epi.partial;
+      e2.ldd = g.ld;
+      e2.C = nullptr;
+      int r = launch_tc_one(M, N, K, ops, cfg, e2, stream, false);
+      if (r) return r;
+      int64_t blocks = (M * N + 255) / 256;
+      const int64_t cap = (int64_t)num_sms() * 8;
+      if (blocks > cap) blocks = cap;
+      ksplit_reduce_kernel<<<(unsigned)blocks, 256, 0, stream>>>(epi.partial, g.parts, M, N, g.m_pad, g.ld,
+                                                                 epi.C, epi.ldc, epi.D, epi.ldd);
+      return cudaGetLastError() == cudaSuccess ? 0 : 3;
+    }
+  }
+  if (epi.kind == EPI_STORE && cfg.peel > 0 && cfg.cg == 2 && (cfg.bn == 256 || cfg.bn == 224) &&
       !fb && N <= cfg.bn && M > 0) {
     int clusters = num_sms() / 2;
     if (cfg.max_clusters > 0 && cfg.max_clusters < clusters) clusters = cfg.max_clusters;

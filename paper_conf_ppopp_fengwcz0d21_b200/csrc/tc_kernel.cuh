@@ -79,6 +79,9 @@ struct KParams {
   int M, N;
   int num_kb;       // ceil(K / 64)
   int kb_per_chunk; // Kc / 64
+  int ksplit;       // STORE: k-parts per tile (1 = none); part results go to D's row block ks
+  int kb_per_part;  // k-blocks per part
+  int m_pad;        // rows per part block of D (a multiple of the tile height)
   int terms;
   int m_tiles, n_tiles;
   int num_units;
@@ -174,12 +177,23 @@ struct EpiGeo {
 
 struct UnitInfo {
   int m_tile, n_begin, n_count, slice;
+  int kb0, kb1, ks;  // the unit's k-blocks [kb0, kb1) and split-K part (STORE); else [0, num_kb)
 };
 
 template <int EPI>
 __device__ __forceinline__ UnitInfo decode_unit(const KParams& p, int u) {
   UnitInfo r;
+  r.kb0 = 0;
+  r.kb1 = p.num_kb;
+  r.ks = 0;
   if constexpr (EPI == EPI_STORE) {
+    // split-K (R21's k-parts): the parts of one tile are consecutive units
+    if (p.ksplit > 1) {
+      r.ks = u % p.ksplit;
+      u /= p.ksplit;
+      r.kb0 = r.ks * p.kb_per_part;
+      r.kb1 = min(p.num_kb, r.kb0 + p.kb_per_part);
+    }
     // bands of up to band_m (8) m-tiles, m fastest inside a band: concurrent clusters share
     // A and B k-slabs in L2.
     const int GM = p.band_m;
@@ -423,7 +437,6 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
     p.probe[1] = globaltimer_ns();
   }
 
-  const int nch = (p.num_kb + p.kb_per_chunk - 1) / p.kb_per_chunk;
 
   // FA register budget per warpgroup (512 threads share 64K registers): converters 96,
   // producer / MMA / allocator 56, the two epilogue warpgroups 176 (running totals).  Each
@@ -447,7 +460,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
       for (int u = cluster; u < p.num_units; u += nclusters) {
         UnitInfo ui = decode_unit<EPI>(p, u);
         for (int ns = 0; ns < ui.n_count; ns++) {
-          for (int kb = 0; kb < p.num_kb; kb++) {
+          for (int kb = ui.kb0; kb < ui.kb1; kb++) {
             ptx::mbar_wait(&sfull[si], sph);
             ptx::mbar_wait(&empty[stage], phase ^ 1u);
             const uint32_t sb = ptx::smem_u32(stage_base + stage * G::STAGE_BYTES) + 2 * G::A_BYTES;
@@ -493,7 +506,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
         UnitInfo ui = decode_unit<EPI>(p, u);
         const int64_t arow0 = (int64_t)ui.m_tile * (kBM * CG) + rank * kBM;
         for (int ns = 0; ns < ui.n_count; ns++) {
-          for (int kb = 0; kb < p.num_kb; kb++) {
+          for (int kb = ui.kb0; kb < ui.kb1; kb++) {
             if constexpr (AS) {
               // the stage's A region holds the fp32 tile (2 boxes of 32 columns, SW128): row r,
               // 8 values k = 8c..8c+7 are fp32 16-B chunks 2(c%4), 2(c%4)+1 of box c/4 at chunk
@@ -611,7 +624,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
         }
         for (int ns = 0; ns < ui.n_count; ns++) {
           const int brow = (ui.n_begin + ns) * BN + (int)rank * G::BNC;
-          for (int kb = 0; kb < p.num_kb; kb++) {
+          for (int kb = ui.kb0; kb < ui.kb1; kb++) {
             if (pace && (gkb % (uint32_t)p.pace_e) == 0) {
               const uint32_t e = gkb / (uint32_t)p.pace_e;
               sync_arrive(p.sync, e);
@@ -629,14 +642,15 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
                 ptx::tma_prefetch_2d_l2(&tm_ahi, kbp * kBK, row);
                 if (AS) ptx::tma_prefetch_2d_l2(&tm_ahi, kbp * kBK + kBK / 2, row);  // 32-column boxes
               };
-              if (kb == 0 && uctr == 0)
-                for (int j = 0; j < p.a_pf && j < p.num_kb; j++) pf(j, arow);
+              if (kb == ui.kb0 && uctr == 0)
+                for (int j = ui.kb0; j < ui.kb0 + p.a_pf && j < ui.kb1; j++) pf(j, arow);
               const int kf = kb + p.a_pf;
-              if (kf < p.num_kb) {
+              if (kf < ui.kb1) {
                 pf(kf, arow);
-              } else if (u + nclusters < p.num_units && kf - p.num_kb < p.num_kb) {
+              } else if (u + nclusters < p.num_units) {
                 const UnitInfo nu = decode_unit<EPI>(p, u + nclusters);
-                pf(kf - p.num_kb, nu.m_tile * (kBM * CG) + (int)rank * kBM);
+                if (nu.kb0 + kf - ui.kb1 < nu.kb1)
+                  pf(nu.kb0 + kf - ui.kb1, nu.m_tile * (kBM * CG) + (int)rank * kBM);
               }
             }
             ptx::mbar_wait(&empty[stage], phase ^ 1u);
@@ -677,7 +691,8 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
         }
       }
       if (pace) {  // out of units: arrive at every remaining epoch so nobody waits on us
-        const uint32_t per_cta = (uint32_t)((p.num_units + nclusters - 1) / nclusters) * p.num_kb;
+        const uint32_t per_cta = (uint32_t)((p.num_units + nclusters - 1) / nclusters) *
+                                 (uint32_t)(p.ksplit > 1 ? p.kb_per_part : p.num_kb);
         const uint32_t pe = (uint32_t)p.pace_e;
         const uint32_t total = (per_cta + pe - 1) / pe;
         for (uint32_t e = (gkb + pe - 1) / pe; e < total; e++) sync_arrive(p.sync, e);
@@ -693,7 +708,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
           UnitInfo ui = decode_unit<EPI>(p, u);
           for (int ns = 0; ns < ui.n_count; ns++) {
             const int n0 = (ui.n_begin + ns) * BN + (int)rank * G::BNC;
-            for (int kb = 0; kb < p.num_kb; kb++) {
+            for (int kb = ui.kb0; kb < ui.kb1; kb++) {
               ptx::mbar_wait(&sempty[si], sph ^ 1u);
               ptx::mbar_arrive_expect_tx(&sfull[si], G::BNC * kBK * 4);
               uint8_t* dst = a_stg + si * STG_BYTES;
@@ -716,7 +731,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
         UnitInfo ui = decode_unit<EPI>(p, u);
         for (int ns = 0; ns < ui.n_count; ns++) {
           const int64_t brow0 = (int64_t)(ui.n_begin + ns) * BN + (int)rank * G::BNC;
-          for (int kb = 0; kb < p.num_kb; kb++) {
+          for (int kb = ui.kb0; kb < ui.kb1; kb++) {
             ptx::mbar_wait(&empty[stage], phase ^ 1u);
             if (kb == p.num_kb - 1) {
               const uint32_t np = ptx::smem_u32(stage_base + stage * SB + NP_OFF);
@@ -761,6 +776,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
           ptx::tc_fence_after();
         }
         for (int ns = 0; ns < ui.n_count; ns++) {
+          const int nch = (ui.kb1 - ui.kb0 + p.kb_per_chunk - 1) / p.kb_per_chunk;
           for (int ch = 0; ch < nch; ch++) {
             const uint32_t buf = chunk_ctr & 1u;
             const uint32_t use = chunk_ctr >> 1;
@@ -768,8 +784,8 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
             ptx::tc_fence_after();
             const uint32_t acc_hh = tmem_base + (SEP ? 2 * buf : buf) * BN;
             const uint32_t acc_x = SEP ? acc_hh + BN : acc_hh;
-            const int kb0 = ch * p.kb_per_chunk;
-            const int kb1 = min(p.num_kb, kb0 + p.kb_per_chunk);
+            const int kb0 = ui.kb0 + ch * p.kb_per_chunk;
+            const int kb1 = min(ui.kb1, kb0 + p.kb_per_chunk);
             for (int kb = kb0; kb < kb1; kb++) {
               if (!(DIAG_NO_TMA && DIAG_MODE(2))) ptx::mbar_wait(&full[stage], phase);
               ptx::tc_fence_after();
@@ -876,6 +892,9 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
 #pragma unroll
             for (int j = 0; j < COLS; j++) totx[j] = 0.f;
           }
+          const int nch = (ui.kb1 - ui.kb0 + p.kb_per_chunk - 1) / p.kb_per_chunk;
+          // split-K: this part's result goes to row block ks of D (the host reduces the parts)
+          const int64_t drow0 = (int64_t)ui.ks * p.m_pad;
           for (int ch = 0; ch < nch; ch++) {
             const uint32_t buf = chunk_ctr & 1u;
             const uint32_t use = chunk_ctr >> 1;
@@ -914,7 +933,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
           if constexpr (TS) {
             if (p.tma_store) {
               const uint32_t buf = ts_base + (uint32_t)ew * 4096u;
-              const int row0 = ui.m_tile * (kBM * CG) + (int)rank * kBM + q * 32;
+              const int row0 = (int)drow0 + ui.m_tile * (kBM * CG) + (int)rank * kBM + q * 32;
 #pragma unroll
               for (int c = 0; c < COLS / 32; c++) {
                 if (lane == 0) ptx::tma_store_wait_read0();  // the previous store read the buffer
@@ -935,7 +954,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
             }
           }
           if (row < p.M) {
-            float* drow = p.D + row * p.ldd;
+            float* drow = p.D + (drow0 + row) * p.ldd;
             const float* crow = p.C ? p.C + row * p.ldc : nullptr;
             if (p.vec_ok && col_base + COLS <= p.N) {
 #pragma unroll

@@ -100,7 +100,8 @@ static bool parse_entry(const char*& p, TuneEntry* e) {
               : v == "gemm_b32" ? kOpGemmB32 : -1;
     } else if (key == "m_max" || key == "n_max" || key == "k_max" || key == "cg" || key == "bn" ||
                key == "sep" || key == "kc" || key == "fa" || key == "terms" || key == "stages" ||
-               key == "n_slices" || key == "epi_warps" || key == "ares" || key == "peel") {
+               key == "n_slices" || key == "epi_warps" || key == "ares" || key == "peel" ||
+               key == "ksplit") {
       char* end = nullptr;
       long long v = strtoll(p, &end, 10);
       if (end == p) return false;
@@ -118,6 +119,7 @@ static bool parse_entry(const char*& p, TuneEntry* e) {
       else if (key == "epi_warps") e->nepi = (int)v;
       else if (key == "ares") e->ares = (int)v;
       else if (key == "peel") e->peel = (int)v;
+      else if (key == "ksplit") e->ksplit = (int)v;
       else e->kc = (int)v;
     } else if (!skip_value(p)) {
       return false;

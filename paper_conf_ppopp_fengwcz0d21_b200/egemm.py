@@ -38,7 +38,7 @@ class Config(ctypes.Structure):
     """egemm_config_t (0 / -1 = not set, the tuning table's value)."""
     _fields_ = [(n, ctypes.c_int) for n in ("cg", "bn", "sep", "kc", "stages", "fused", "terms",
                                             "n_slices", "epi_warps", "a_resident", "pace",
-                                            "max_clusters", "operand_format", "tail_peel")]
+                                            "max_clusters", "operand_format", "tail_peel", "ksplit")]
 
 
 EXPORTS = ["egemm_status_string", "egemm_last_error", "egemm_version", "egemm_split",

@@ -202,3 +202,16 @@ def test_peer_reduce_and_bf16_split_validation(lib):
         assert egemm.query_config_ex("knn", 4096, 4096, 128)["operand_format"] == 0
     finally:
         egemm.set_config_ex()
+
+
+def test_split_k_workspace_size_grows(lib):
+    """egemm_gemm_workspace_size includes the split-K parts buffer under a ksplit override."""
+    from paper_conf_ppopp_fengwcz0d21_b200 import egemm
+    base = egemm.gemm_workspace_size(1024, 1024, 1024)
+    egemm.set_config_ex(cg=2, bn=256, sep=0, kc=64, ksplit=4)
+    try:
+        assert egemm.query_config_ex("gemm", 1024, 1024, 1024)["ksplit"] == 4
+        grown = egemm.gemm_workspace_size(1024, 1024, 1024)
+    finally:
+        egemm.set_config_ex()
+    assert grown >= base + 4 * 1024 * 1024 * 4

@@ -138,3 +138,44 @@ def test_tail_peel_same_bits(oracle_lib, fused, M):
     rows = np.array([0, M // 2, M - 300, M - 1])
     ref = oracle_lib.gemm_alg1_tc(A[rows], B, C[rows], terms=3, sep=0, kc=128)
     assert np.array_equal(out[1][rows].view(np.uint32), ref.view(np.uint32))
+
+
+@pytest.mark.parametrize("cfg,fused", [((2, 256, 0, 128), 0), ((1, 128, 0, 64), 0), ((2, 128, 1, 128), 0),
+                                       ((2, 256, 0, 64), 1), ((2, 224, 0, 128), 0)])
+@pytest.mark.parametrize("ksplit", [2, 3, 4])
+def test_bitexact_split_k(oracle_lib, cfg, fused, ksplit):
+    """Split-K (R21's k-parts, the table's ksplit axis): each tile's k-parts run as separate
+    units and a reduce pass adds their results in k order, then C -- bitwise the oracle's
+    Alg. 1 with kpart = 64 * ceil(ceil(K / 64) / ksplit), on ragged shapes, with C."""
+    eg = require_gpu()
+    for (M, N, K) in ((300, 200, 1000), (129, 257, 4100)):
+        A, B, C = inputs.uniform((M, K), 60 + K), inputs.uniform((K, N), 61 + N), inputs.uniform((M, N), 62)
+        nkb = -(-K // 64)
+        kpart = 64 * -(-nkb // ksplit)
+        for terms in (3, 4):
+            eg.set_config_ex(cg=cfg[0], bn=cfg[1], sep=cfg[2], kc=cfg[3], fused=fused, ksplit=ksplit)
+            try:
+                D = to_host(eg.gemm(to_dev(A), to_dev(B), to_dev(C), terms=terms))
+            finally:
+                eg.set_config_ex()
+            ref = oracle_lib.gemm_alg1_tc(A, B, C, terms=terms, sep=cfg[2], kc=cfg[3], kpart=kpart)
+            assert np.array_equal(D.view(np.uint32), ref.view(np.uint32)), (M, N, K, terms)
+
+
+def test_split_k_workspace_too_small():
+    """The split-K parts buffer lives in the caller's workspace: a workspace sized without it
+    is rejected (EGEMM_ERR_WORKSPACE), never silently run with another arithmetic."""
+    import torch
+    eg = require_gpu()
+    A, B = to_dev(inputs.uniform((256, 512), 1)), to_dev(inputs.uniform((512, 256), 2))
+    small = torch.empty(eg.gemm_workspace_size(256, 256, 512), dtype=torch.uint8, device="cuda")
+    D = torch.empty((256, 256), device="cuda")
+    eg.set_config_ex(cg=2, bn=256, sep=0, kc=64, fused=0, ksplit=4)
+    try:
+        st = eg.load().egemm_gemm(256, 256, 512, eg.operand(A), eg.operand(B), None, 0, eg._ptr(D), 256,
+                                  0, eg._ptr(small), small.numel(), eg._stream())
+        assert st == eg.ERR_WORKSPACE
+        D = eg.gemm(A, B)  # the wrapper sizes the workspace under the override
+    finally:
+        eg.set_config_ex()
+    assert torch.isfinite(D).all()
