@@ -73,7 +73,15 @@ def timeit(fn, reps=3, batch_ms=60.0):
 
 
 def _cfg(c, stages=0, terms=0):
-    return dict(cg=c[0], bn=c[1], sep=c[2], kc=c[3], fused=c[4], stages=stages, terms=terms)
+    d = dict(cg=c[0], bn=c[1], sep=c[2], kc=c[3], fused=c[4], stages=stages, terms=terms)
+    if len(c) > 5 and c[5] > 1:
+        d["ksplit"] = c[5]
+    return d
+
+
+# split-K candidates (R21's k-parts) for grids that fill under two waves of 256 x 256 units
+KSPLIT_CONFIGS = [(cg, bn, sep, kc, 0, ks) for (cg, bn, sep, kc) in
+                  ((2, 256, 0, 64), (1, 128, 0, 64), (2, 128, 1, 128), (1, 128, 1, 128)) for ks in (2, 4)]
 
 
 class GemmProblem:
@@ -128,16 +136,22 @@ def gemm_bucket(M, N, K, Ks, b_f32=False):
     # the table's current pick for this bucket (re-measured below, kept within HYSTERESIS)
     q = egemm.query_config_ex("gemm_b32" if b_f32 else "gemm", M, N, K)
     prev = dict(cg=q["cg"], bn=q["bn"], sep=q["sep"], kc=q["kc"], fused=q["fused"], stages=q["stages"], terms=0)
+    if q.get("ksplit", 1) > 1:
+        prev["ksplit"] = q["ksplit"]
     P = GemmProblem(M, N, K, b_f32)
-    cands = CONFIGS if not b_f32 else \
+    cands = list(CONFIGS) if not b_f32 else \
         [tuple(egemm.query_config("gemm", M, N, K, with_fused=True))] + \
         [(2, 256, 0, kc, 2) for kc in (64, 128, 256)] + [(2, 224, 0, kc, 2) for kc in (128, 256)]
+    if not b_f32 and (-(-M // 256)) * (-(-N // 256)) < 148 and K >= 512:
+        cands += KSPLIT_CONFIGS
     res = [P.measure(_cfg(c)) for c in cands]
     ks = k_scale(K, Ks)
     # phase 2: the alternative ring depth of the 3 fastest accurate pre-split configurations
     good = sorted([r for r in res if r["ok"] and r["cfg"]["fused"] == 0], key=lambda r: r["ms"])[:3]
     for r in good:
         c = r["cfg"]
+        if c.get("ksplit"):
+            continue
         alt = STAGES[(c["cg"], c["bn"], c["sep"])][1]
         res.append(P.measure(dict(c, stages=alt)))
     best = select(res, ks)
@@ -269,6 +283,7 @@ def main():
                     c = best["cfg"]
                     new.append({"op": op, "m_max": M, "n_max": N, "k_max": K, "cg": c["cg"], "bn": c["bn"],
                                 "sep": c["sep"], "kc": c["kc"], "fa": c["fused"], "stages": c["stages"],
+                                "ksplit": c.get("ksplit", 0),
                                 "terms": best["terms"], "ms": round(best["ms"], 4),
                                 "tflops_fp32eq": round(2.0 * M * N * K / best["ms"] / 1e9, 1),
                                 "err_ratio": round(best["err"] / best["err_naive"], 3)})
