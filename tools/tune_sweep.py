@@ -106,6 +106,10 @@ class GemmProblem:
 
     def measure(self, cfg, time_it=True):
         egemm.set_config_ex(**cfg)
+        # (a split-K config needs the larger workspace: allocate it outside the timing)
+        need = egemm.gemm_workspace_size(self.M, self.N, self.K, False, not self.b_f32)
+        if need > self.ws.numel():
+            self.ws = torch.empty(need, dtype=torch.uint8, device="cuda")
         try:
             t = timeit(self.call) if time_it else float("nan")
             self.call()
