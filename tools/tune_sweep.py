@@ -48,11 +48,33 @@ STAGES = {(2, 256, 0): (3, 2), (2, 224, 0): (3, 2), (2, 128, 0): (4, 3), (2, 128
           (1, 128, 0): (3, 2), (1, 128, 1): (3, 2)}
 
 
-def timeit(fn, reps=3, batch_ms=60.0):
+def timeit(fn, reps=3, batch_ms=60.0, graph=True):
     """Steady-state time per call: warm up, then the median of `reps` batches of back-to-back
-    calls, each ~batch_ms long (the power-capped clock settles within tens of ms)."""
+    calls, each ~batch_ms long (the power-capped clock settles within tens of ms).  Calls
+    shorter than 0.2 ms are captured once into a CUDA graph and the graph is replayed, so the
+    host cost of a Python / ctypes call does not set their rate (as in bench.py)."""
     fn()
     torch.cuda.synchronize()
+    s0, e0 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+    s0.record()
+    fn()
+    e0.record()
+    e0.synchronize()
+    if graph and s0.elapsed_time(e0) < 0.2:
+        try:
+            cs = torch.cuda.Stream()
+            cs.wait_stream(torch.cuda.current_stream())
+            with torch.cuda.stream(cs):
+                fn()
+            torch.cuda.current_stream().wait_stream(cs)
+            g = torch.cuda.CUDAGraph()
+            with torch.cuda.graph(g):
+                for _ in range(20):
+                    fn()
+            torch.cuda.synchronize()
+            return timeit(g.replay, reps, batch_ms, graph=False) / 20
+        except Exception:  # capture unsupported for this call: fall back to direct calls
+            torch.cuda.synchronize()
     s, e = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
     s.record()
     fn()
