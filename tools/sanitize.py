@@ -26,6 +26,10 @@ VARIANTS = {
     "fused_a_128_sep": ({"fused": 1}, (2, 128, 1, 64), (300, 300, 200)),
     "fused_b": ({"fused": 2}, (2, 256, 0, 64), (300, 520, 256)),
     "presplit_256_s2": ({"stages": 2}, (2, 256, 0, 64), (300, 520, 200)),
+    "presplit_256_ksplit3": ({"ksplit": 3}, (2, 256, 0, 64), (300, 520, 700)),
+    "cg1_128_ksplit2_sep": ({"ksplit": 2}, (1, 128, 1, 128), (200, 200, 600)),
+    "fused_a_tail_peel": ({"fused": 1, "tail_peel": 1}, (2, 256, 0, 64), (94 * 256 + 37, 256, 256)),
+    "bf16_parts": ({"operand_format": 1}, (2, 256, 0, 64), (300, 520, 200)),
     "presplit_128_s3": ({"stages": 3}, (2, 128, 0, 64), (300, 300, 200)),
 }
 
