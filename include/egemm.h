@@ -222,10 +222,17 @@ int egemm_kmeans_finalize(const double* sums, const int64_t* counts, int64_t kc,
  *  ksplit      : STORE split-K (R21's k-parts): K in up to ksplit contiguous parts, each tile's
  *                parts run as separate units, their fp32 results are added in k order (then
  *                + C) by a reduce pass; needs the larger egemm_gemm_workspace_size (0/1 = none).
+ *  tail_split  : STORE GEMMs whose persistent grid's last wave is at most half full: only
+ *                that wave's tiles are cut into 2..4 k-parts (R21) run side by side; each part
+ *                leaves its fp32 sums in the workspace and the part that finishes last adds
+ *                them in k order (+ C) and stores the tile -- no extra launch.  Uses
+ *                egemm_gemm_workspace_size's room (without it the wave runs unsplit)
+ *                (-1 = table, default off: fewer SM cycles but no shorter time under the
+ *                power cap, profiles/r02_tail_split_ab.json; 0 = off, 1 = on).
  */
 typedef struct {
   int cg, bn, sep, kc, stages, fused, terms, n_slices, epi_warps, a_resident, pace, max_clusters,
-      operand_format, tail_peel, ksplit;
+      operand_format, tail_peel, ksplit, tail_split;
 } egemm_config_t;
 
 /* Thread-local override of the tuning table for the next calls of this thread: fields set

@@ -104,6 +104,7 @@ static TcConfig choose_config(int epi_kind, int64_t M, int64_t N, int64_t K, int
   c.ares = -1;
   c.pace = 1;
   c.peel = 0;  // measured slower on configs[2] (profiles/r02_skinny_peel.txt): table / override only
+  c.tsplit = 0;  // tail split: fewer cycles but no faster under the power cap (profiles/r02_tail_split_ab.json)
   if (epi_kind == EPI_STORE && M <= 128) { c.cg = 1; c.bn = 128; c.sep = 1; }
   {
     TuneEntry t;
@@ -123,6 +124,7 @@ static TcConfig choose_config(int epi_kind, int64_t M, int64_t N, int64_t K, int
       if (t.ares >= 0) c.ares = t.ares;
       if (t.peel >= 0) c.peel = t.peel;
       if (t.ksplit > 1) c.ksplit = t.ksplit;
+      if (t.tsplit >= 0) c.tsplit = t.tsplit;
     }
   }
   if (terms == 3 || terms == 4) c.terms = terms;  // the call's explicit term count wins
@@ -147,6 +149,7 @@ static TcConfig choose_config(int epi_kind, int64_t M, int64_t N, int64_t K, int
     if (o.max_clusters) c.max_clusters = o.max_clusters;
     if (o.tail_peel >= 0) c.peel = o.tail_peel;
     if (o.ksplit) c.ksplit = o.ksplit;
+    if (o.tail_split >= 0) c.tsplit = o.tail_split;
     if (o.operand_format == 1 && epi_kind == EPI_STORE) {
       c.fmt = 1;
       c.fa = 0;  // the fused converters produce fp16 parts only
@@ -279,6 +282,7 @@ static void to_public(const TcConfig& c, int op, egemm_config_t* o) {
   o->operand_format = c.fmt;
   o->tail_peel = c.peel;
   o->ksplit = c.ksplit > 1 ? c.ksplit : 1;
+  o->tail_split = c.tsplit > 0 ? 1 : 0;
 }
 
 int egemm_query_config(int op, int64_t M, int64_t N, int64_t K, int* cg, int* bn, int* sep,
@@ -351,6 +355,7 @@ int egemm_set_config(int cg, int bn, int sep, int kc) {
   o.a_resident = -1;
   o.pace = -1;
   o.tail_peel = -1;
+  o.tail_split = -1;
   return egemm_set_config_ex(&o);
 }
 
@@ -367,7 +372,7 @@ int egemm_set_config_ex(const egemm_config_t* cfg) {
       !(o.epi_warps == 0 || o.epi_warps == 8 || o.epi_warps == 16) || o.a_resident < -1 ||
       o.a_resident > 1 || o.pace < -1 || o.pace > 1 || o.max_clusters < 0 ||
       o.operand_format < 0 || o.operand_format > 1 || o.tail_peel < -1 || o.tail_peel > 1 ||
-      o.ksplit < 0 || o.ksplit > 16) {
+      o.ksplit < 0 || o.ksplit > 16 || o.tail_split < -1 || o.tail_split > 1) {
     set_last_error("unsupported config cg=%d bn=%d sep=%d kc=%d fused=%d stages=%d terms=%d "
                    "n_slices=%d epi_warps=%d", o.cg, o.bn, o.sep, o.kc, o.fused, o.stages, o.terms,
                    o.n_slices, o.epi_warps);
@@ -444,7 +449,7 @@ size_t egemm_gemm_workspace_size(int64_t M, int64_t N, int64_t K, int a_presplit
   // (+ the split-K parts buffer when the table / this thread's override picks split-K)
   const TcConfig cfg = choose_config(EPI_STORE, M, N, K, 0, !b_presplit);
   return gemm_operand_ws(M, N, K, a_presplit, b_presplit) +
-         ((ksplit_ws_bytes(M, N, K, cfg) + 255) & ~size_t(255)) + kPaceBytes;
+         ((parts_ws_bytes(M, N, K, cfg) + 255) & ~size_t(255)) + kPaceBytes;
 }
 
 int egemm_gemm(int64_t M, int64_t N, int64_t K, egemm_operand_t A, egemm_operand_t B,
@@ -520,6 +525,10 @@ int egemm_gemm(int64_t M, int64_t N, int64_t K, egemm_operand_t A, egemm_operand
       return EGEMM_ERR_WORKSPACE;
     }
     epi.partial = cv.take<float>(pb / sizeof(float));
+  } else if (const size_t tb = parts_ws_bytes(M, N, K, cfg)) {
+    // tail split: optional -- without the room the last wave runs unsplit (same arithmetic
+    // class; the split tiles follow R21's k-parts)
+    if (workspace && workspace_bytes >= cv.off + tb + kPaceBytes) epi.partial = cv.take<float>(tb / sizeof(float));
   }
   if (workspace && workspace_bytes >= cv.off + kPaceBytes) epi.sync = cv.take<uint32_t>(64);
   r = launch_tc(M, N, K, ops, cfg, epi, s);
@@ -643,6 +652,7 @@ int egemm_gemm_host(int64_t M, int64_t N, int64_t K, const float* A_host, int64_
   }
   TcConfig cfg = choose_config(EPI_STORE, mc, N, K, terms);
   cfg.ksplit = 0;  // (no parts buffer in the host pipeline's workspace)
+  cfg.tsplit = 0;
   bool ok = true;
   auto chk = [&](cudaError_t e) { ok = ok && (e == cudaSuccess); };
   chk(cudaStreamWaitEvent(s, hp->ev_done, 0));  // the previous call's pipeline has drained

@@ -53,6 +53,7 @@ struct TcConfig {
   int fmt;       // operand parts: 0 = fp16 (the paper's round-split), 1 = bf16 (NEXT-3)
   int peel;      // STORE: peel a mostly-empty last wave into a 128 x 128 tail launch (-1 auto, 0 off)
   int ksplit;    // STORE: split-K parts (<= 1: none)
+  int tsplit;    // STORE: tail split -- k-parts for the tiles of a last wave at most half full (0 off, 1 on)
 };
 
 // Split-K geometry of a STORE launch: k-blocks per part, parts actually used (no empty part),
@@ -63,6 +64,17 @@ struct KSplit {
 };
 KSplit ksplit_geometry(int64_t M, int64_t N, int64_t K, const TcConfig& cfg);
 size_t ksplit_ws_bytes(int64_t M, int64_t N, int64_t K, const TcConfig& cfg);
+// Tail split of a STORE launch (cfg.tsplit, no uniform split-K): tiles [u0, u0 + tiles) of the
+// unit order -- the last, at most half-full wave of the persistent grid -- run as `parts`
+// k-parts of kbpp k-blocks each; parts = 0 when it does not apply.  The workspace holds the
+// parts' fp32 sums (parts x tile) per split tile plus a counter per epilogue-warp slab.
+struct TailSplit {
+  int u0, tiles, parts, kbpp;
+  size_t ws_floats, cnt_words;
+};
+TailSplit tail_geometry(int64_t M, int64_t N, int64_t K, const TcConfig& cfg);
+// Workspace bytes of the STORE launch's k-parts: the split-K parts buffer or the tail split's.
+size_t parts_ws_bytes(int64_t M, int64_t N, int64_t K, const TcConfig& cfg);
 
 // Environment knobs for experiments, read once per process (tools/; the product path takes
 // its configuration from the tuning table and egemm_set_config_ex).
@@ -87,7 +99,7 @@ struct TcEpilogue {
   const float* C;
   int64_t ldc;
   uint32_t* sync;      // nullable: 256 B of workspace for the k-pacing counters
-  float* partial;      // split-K (cfg.ksplit > 1): the parts' results, ksplit_ws_bytes() of workspace
+  float* partial;      // split-K / tail split: the parts' results, parts_ws_bytes() of workspace
   // EPI_KNN / EPI_KMEANS: per-B-row squared norms (||x_j||^2 or ||c_j||^2)
   const float* bnorm;
   // EPI_KNN
@@ -137,7 +149,7 @@ struct TuneEntry {
   int op = -1;  // EpiKind or kOpGemmB32
   long long m_max = 0, n_max = 0, k_max = 0;
   int cg = 0, bn = 0, sep = 0, kc = 0, fa = 0;
-  int terms = 0, stages = 0, nslices = 0, nepi = 0, ares = -1, peel = -1, ksplit = 0;
+  int terms = 0, stages = 0, nslices = 0, nepi = 0, ares = -1, peel = -1, ksplit = 0, tsplit = -1;
 };
 bool tune_lookup(int op, long long M, long long N, long long K, TuneEntry* out);
 const char* tune_table_path();

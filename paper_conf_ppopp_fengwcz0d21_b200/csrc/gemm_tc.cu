@@ -204,6 +204,19 @@ static int launch_tc_one(int64_t M, int64_t N, int64_t K, const TcOperands& ops,
   kp.best_key = epi.best_key;
   if (epi.kind == EPI_STORE) {
     kp.num_units = kp.m_tiles * kp.n_tiles * kp.ksplit;
+    const TailSplit tg = tail_geometry(M, N, K, cfg);
+    if (tg.parts > 1 && epi.partial && !pdl_tail) {
+      kp.tail_u0 = tg.u0;
+      kp.tail_parts = tg.parts;
+      kp.tail_kbpp = tg.kbpp;
+      kp.fix_ws = epi.partial;
+      kp.fix_cnt = reinterpret_cast<uint32_t*>(epi.partial + tg.ws_floats);
+      kp.num_units = tg.u0 + tg.tiles * tg.parts;
+      if (cudaMemsetAsync(kp.fix_cnt, 0, tg.cnt_words * sizeof(uint32_t), stream) != cudaSuccess) {
+        set_last_error("memset of the tail-split counters failed");
+        return 3;
+      }
+    }
     return (fa || fb) ? dispatch_fused(maps, kp, cfg, stream) : dispatch_store(maps, kp, cfg, stream);
   }
   if (kp.num_kb > kp.kb_per_chunk) {
@@ -244,6 +257,42 @@ KSplit ksplit_geometry(int64_t M, int64_t N, int64_t K, const TcConfig& cfg) {
 size_t ksplit_ws_bytes(int64_t M, int64_t N, int64_t K, const TcConfig& cfg) {
   const KSplit g = ksplit_geometry(M, N, K, cfg);
   return g.parts > 1 ? (size_t)g.parts * (size_t)g.m_pad * (size_t)g.ld * sizeof(float) : 0;
+}
+
+// The persistent grid runs `clusters` units at a time; when the last wave holds rem <= half
+// of them, its tiles' k-range is cut into parts = min(4, clusters / rem) parts run side by
+// side, so the last wave takes ~1/parts of a wave instead of a whole one.
+TailSplit tail_geometry(int64_t M, int64_t N, int64_t K, const TcConfig& cfg) {
+  TailSplit t = {0, 0, 0, 0, 0, 0};
+  if (cfg.tsplit <= 0 || cfg.ksplit > 1 || cfg.peel > 0 || M <= 0 || N <= 0 || K <= 0) return t;
+  const int num_kb = (int)((K + kBK - 1) / kBK);
+  if (num_kb < 4) return t;
+  int clusters = num_sms() / cfg.cg;
+  if (cfg.max_clusters > 0 && cfg.max_clusters < clusters) clusters = cfg.max_clusters;
+  const int64_t th = (int64_t)kBM * cfg.cg;
+  const int64_t tiles = ((M + th - 1) / th) * ((N + cfg.bn - 1) / cfg.bn);
+  if (clusters < 2 || tiles <= clusters) return t;
+  const int64_t rem = tiles % clusters;
+  if (rem == 0 || 2 * rem > clusters) return t;
+  int parts = (int)(clusters / rem);
+  if (parts > 4) parts = 4;
+  if (parts > num_kb / 2) parts = num_kb / 2;
+  const int kbpp = (num_kb + parts - 1) / parts;
+  parts = (num_kb + kbpp - 1) / kbpp;  // no empty part
+  if (parts < 2) return t;
+  t.u0 = (int)(tiles - rem);
+  t.tiles = (int)rem;
+  t.parts = parts;
+  t.kbpp = kbpp;
+  t.ws_floats = (size_t)rem * parts * (size_t)th * cfg.bn;
+  t.cnt_words = (size_t)rem * cfg.cg * 16;  // one counter per epilogue warp (<= 16 per CTA)
+  return t;
+}
+
+size_t parts_ws_bytes(int64_t M, int64_t N, int64_t K, const TcConfig& cfg) {
+  if (const size_t b = ksplit_ws_bytes(M, N, K, cfg)) return b;
+  const TailSplit t = tail_geometry(M, N, K, cfg);
+  return t.parts > 1 ? t.ws_floats * sizeof(float) + t.cnt_words * sizeof(uint32_t) : 0;
 }
 
 // D = fold over the parts in k order (RN) of the split-K part results (+ C last): the

@@ -5,8 +5,9 @@
 // Sums are fp64 and deterministic, in the fixed two-level order of reading R20:
 //   the members of group j (points with a_i == j) in ascending i are cut into chunks of
 //   kKmChunk; each chunk is summed sequentially from 0.0; the chunk sums are then added
-//   sequentially from 0.0.  The CPU oracle implements the same order, so the sums are
-//   bitwise equal to it for equal assignments.
+//   sequentially from 0.0.  tests/kernel_model.py (group_sums_chunked) models this order
+//   for the bitwise regression test; the oracle sums each group plainly in ascending i
+//   (SURVEY c-6) and the GPU sums are checked against it within the fp64 sum bound.
 // Instead of 4M x 64 fp64 atomics (measured 1.9 ms) a stable counting sort groups the
 // point indices by centroid, then one CTA per chunk (one thread per dimension) adds rows
 // gathered 32 at a time, and one CTA per centroid adds its chunk sums:

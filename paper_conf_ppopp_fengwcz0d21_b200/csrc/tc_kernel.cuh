@@ -119,6 +119,13 @@ struct KParams {
   int debug_mode;    // EGEMM_DEBUG_MODE bits (diagnostics): 1 extra commit per k-block;
                      // with NO_TMA: 2 MMA warp ignores the full barriers (producer idle),
                      // 4 no per-k-block commits
+  // STORE tail split (R21's k-parts for the last, partly filled wave only): units >= tail_u0
+  // are k-parts (tail_parts per tile, tail_kbpp k-blocks each) of the tiles tail_u0, ...;
+  // each part leaves its fp32 sum in fix_ws and the last part to finish a warp's slab (per
+  // slab counter fix_cnt, zeroed per launch) adds them in k order and stores the tile.
+  int tail_u0, tail_parts, tail_kbpp;
+  float* fix_ws;
+  uint32_t* fix_cnt;
 };
 
 // ---------------------------------------------------------------- k-pacing (STORE GEMMs)
@@ -178,6 +185,7 @@ struct EpiGeo {
 struct UnitInfo {
   int m_tile, n_begin, n_count, slice;
   int kb0, kb1, ks;  // the unit's k-blocks [kb0, kb1) and split-K part (STORE); else [0, num_kb)
+  int fx;            // STORE tail split: index of the unit's tile among the split tiles (else -1)
 };
 
 template <int EPI>
@@ -186,6 +194,7 @@ __device__ __forceinline__ UnitInfo decode_unit(const KParams& p, int u) {
   r.kb0 = 0;
   r.kb1 = p.num_kb;
   r.ks = 0;
+  r.fx = -1;
   if constexpr (EPI == EPI_STORE) {
     // split-K (R21's k-parts): the parts of one tile are consecutive units
     if (p.ksplit > 1) {
@@ -193,6 +202,14 @@ __device__ __forceinline__ UnitInfo decode_unit(const KParams& p, int u) {
       u /= p.ksplit;
       r.kb0 = r.ks * p.kb_per_part;
       r.kb1 = min(p.num_kb, r.kb0 + p.kb_per_part);
+    } else if (p.tail_parts > 1 && u >= p.tail_u0) {
+      // tail split: the k-parts of the last wave's tiles (consecutive units: concurrent)
+      const int v = u - p.tail_u0;
+      r.fx = v / p.tail_parts;
+      r.ks = v - r.fx * p.tail_parts;
+      r.kb0 = r.ks * p.tail_kbpp;
+      r.kb1 = min(p.num_kb, r.kb0 + p.tail_kbpp);
+      u = p.tail_u0 + r.fx;
     }
     // bands of up to band_m (8) m-tiles, m fastest inside a band: concurrent clusters share
     // A and B k-slabs in L2.
@@ -894,7 +911,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
           }
           const int nch = (ui.kb1 - ui.kb0 + p.kb_per_chunk - 1) / p.kb_per_chunk;
           // split-K: this part's result goes to row block ks of D (the host reduces the parts)
-          const int64_t drow0 = (int64_t)ui.ks * p.m_pad;
+          const int64_t drow0 = p.ksplit > 1 ? (int64_t)ui.ks * p.m_pad : 0;
           for (int ch = 0; ch < nch; ch++) {
             const uint32_t buf = chunk_ctr & 1u;
             const uint32_t use = chunk_ctr >> 1;
@@ -929,6 +946,41 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
           if constexpr (SEP) {
 #pragma unroll
             for (int j = 0; j < COLS; j++) tot[j] = __fadd_rn(tot[j], totx[j]);
+          }
+          if (ui.fx >= 0) {
+            // tail split: this part's sums go to the workspace (coalesced float4 slab per
+            // warp); the warp that completes a slab's last part adds the parts in k order
+            // (RN, R21 -- the split-K reduce's order) and stores the tile.  No part ever waits.
+            constexpr int SLABS = CG * NEPI;
+            constexpr int SLAB_F4 = COLS / 4 * 32;
+            const int slab = (int)rank * NEPI + ew;
+            float4* wsb = reinterpret_cast<float4*>(p.fix_ws) +
+                          ((size_t)ui.fx * p.tail_parts * SLABS + slab) * SLAB_F4;
+            float4* own = wsb + (size_t)ui.ks * SLABS * SLAB_F4;
+#pragma unroll
+            for (int j = 0; j < COLS / 4; j++)
+              own[j * 32 + lane] = make_float4(tot[4 * j], tot[4 * j + 1], tot[4 * j + 2], tot[4 * j + 3]);
+            __threadfence();
+            __syncwarp();
+            uint32_t old = 0;
+            if (lane == 0) old = atomicAdd(p.fix_cnt + (size_t)ui.fx * SLABS + slab, 1u);
+            old = __shfl_sync(0xffffffffu, old, 0);
+            if (old + 1u != (uint32_t)p.tail_parts) continue;  // another part completes it
+            __threadfence();
+            // (the own part is read back too: tot need not stay live across the hand-off)
+#pragma unroll
+            for (int j = 0; j < COLS / 4; j++) {
+              float4 a = __ldcg(wsb + j * 32 + lane);
+#pragma unroll
+              for (int s2 = 1; s2 < 4; s2++) {  // (host: tail_parts <= 4)
+                if (s2 < p.tail_parts) {
+                  const float4 b = __ldcg(wsb + (size_t)s2 * SLABS * SLAB_F4 + j * 32 + lane);
+                  a.x = __fadd_rn(a.x, b.x); a.y = __fadd_rn(a.y, b.y);
+                  a.z = __fadd_rn(a.z, b.z); a.w = __fadd_rn(a.w, b.w);
+                }
+              }
+              tot[4 * j] = a.x; tot[4 * j + 1] = a.y; tot[4 * j + 2] = a.z; tot[4 * j + 3] = a.w;
+            }
           }
           if constexpr (TS) {
             if (p.tma_store) {

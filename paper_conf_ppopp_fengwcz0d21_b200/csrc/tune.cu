@@ -101,7 +101,7 @@ static bool parse_entry(const char*& p, TuneEntry* e) {
     } else if (key == "m_max" || key == "n_max" || key == "k_max" || key == "cg" || key == "bn" ||
                key == "sep" || key == "kc" || key == "fa" || key == "terms" || key == "stages" ||
                key == "n_slices" || key == "epi_warps" || key == "ares" || key == "peel" ||
-               key == "ksplit") {
+               key == "ksplit" || key == "tsplit") {
       char* end = nullptr;
       long long v = strtoll(p, &end, 10);
       if (end == p) return false;
@@ -120,6 +120,7 @@ static bool parse_entry(const char*& p, TuneEntry* e) {
       else if (key == "ares") e->ares = (int)v;
       else if (key == "peel") e->peel = (int)v;
       else if (key == "ksplit") e->ksplit = (int)v;
+      else if (key == "tsplit") e->tsplit = (int)v;
       else e->kc = (int)v;
     } else if (!skip_value(p)) {
       return false;

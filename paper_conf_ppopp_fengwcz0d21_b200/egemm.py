@@ -38,7 +38,8 @@ class Config(ctypes.Structure):
     """egemm_config_t (0 / -1 = not set, the tuning table's value)."""
     _fields_ = [(n, ctypes.c_int) for n in ("cg", "bn", "sep", "kc", "stages", "fused", "terms",
                                             "n_slices", "epi_warps", "a_resident", "pace",
-                                            "max_clusters", "operand_format", "tail_peel", "ksplit")]
+                                            "max_clusters", "operand_format", "tail_peel", "ksplit",
+                                            "tail_split")]
 
 
 EXPORTS = ["egemm_status_string", "egemm_last_error", "egemm_version", "egemm_split",
@@ -161,7 +162,7 @@ def set_config_ex(**fields):
         _check(load().egemm_set_config_ex(None), "egemm_set_config_ex")
         return
     c = Config()
-    c.fused = c.a_resident = c.pace = c.tail_peel = -1
+    c.fused = c.a_resident = c.pace = c.tail_peel = c.tail_split = -1
     c.operand_format = 0
     for k, v in fields.items():
         if k not in dict(Config._fields_):

@@ -156,12 +156,14 @@ def test_config_override_round_trip_and_validation(lib):
         egemm.set_config_ex()
     assert egemm.query_config_ex("gemm", 8192, 8192, 8192) == base
     for bad in (dict(cg=2, bn=200), dict(kc=100), dict(stages=7), dict(terms=5), dict(n_slices=17),
-                dict(epi_warps=12), dict(fused=3)):
+                dict(epi_warps=12), dict(fused=3), dict(tail_split=2), dict(ksplit=17)):
         with pytest.raises(egemm.EgemmError) as ei:
             egemm.set_config_ex(**bad)
         assert ei.value.status == egemm.ERR_UNSUPPORTED
-    egemm.set_config_ex(epi_warps=8, n_slices=4)
+    assert base["tail_split"] == 0  # the tail split is opt-in (profiles/r02_tail_split_ab.json)
+    egemm.set_config_ex(epi_warps=8, n_slices=4, tail_split=1)
     try:
+        assert egemm.query_config_ex("gemm", 65536, 256, 1024)["tail_split"] == 1
         assert egemm.query_config_ex("kmeans", 4096, 1024, 64)["epi_warps"] == 8
         assert egemm.query_config_ex("knn", 4096, 1 << 20, 128)["n_slices"] == 4
     finally:

@@ -129,7 +129,7 @@ def test_tail_peel_same_bits(oracle_lib, fused, M):
     Ad, Bd, Cd = to_dev(A), to_dev(B), to_dev(C)
     out = {}
     for peel in (0, 1):
-        eg.set_config_ex(cg=2, bn=256, sep=0, kc=128, fused=fused, tail_peel=peel)
+        eg.set_config_ex(cg=2, bn=256, sep=0, kc=128, fused=fused, tail_peel=peel, tail_split=0)
         try:
             out[peel] = to_host(eg.gemm(Ad, Bd, Cd))
         finally:
@@ -179,3 +179,40 @@ def test_split_k_workspace_too_small():
     finally:
         eg.set_config_ex()
     assert torch.isfinite(D).all()
+
+
+@pytest.mark.parametrize("fused", [0, 1, 2])
+@pytest.mark.parametrize("shape,clusters", [((51 * 256 + 37, 300, 1000), 16),  # 104 tiles: 8 split in 2
+                                            ((5 * 256 + 37, 700, 4100), 8),     # 18 tiles: 2 split in 4
+                                            ((65536, 256, 1024), 0)])          # configs[2]: 34 in 2
+def test_tail_split_bitexact(oracle_lib, fused, shape, clusters):
+    """Tail split: the tiles of the last, at most half-full wave run as 2..4 k-parts and the
+    last part to finish adds them in k order (+ C) -- bitwise the oracle's Alg. 1 with kpart
+    (R21) on those tiles and without on the others; the other tiles equal the unsplit launch."""
+    import torch
+    from tests.gpu_util import alg1_rows_with_tail, tail_split_tiles
+    eg = require_gpu()
+    M, N, K = shape
+    A, B, C = inputs.uniform((M, K), 80 + K), inputs.uniform((K, N), 81), inputs.uniform((M, N), 82)
+    Ad, Bd, Cd = to_dev(A), to_dev(B), to_dev(C)
+    out = {}
+    for ts in (0, 1):
+        eg.set_config_ex(cg=2, bn=256, sep=0, kc=128, fused=fused, tail_split=ts, max_clusters=clusters)
+        try:
+            sched = tail_split_tiles(eg, "gemm_b32", M, N, K)
+            out[ts] = to_host(eg.gemm(Ad, Bd, Cd))
+        finally:
+            eg.set_config_ex()
+    tiles, kpart, th, bn = sched
+    assert tiles and 2 * 64 <= kpart < K  # the shape exercises the split
+    split_rows = sorted({m for m, _ in tiles})
+    rows = np.unique(np.concatenate([np.arange(m * th, min(M, m * th + th), 37) for m in split_rows] +
+                                    [np.array([m * th + th - 1 for m in split_rows if m * th + th - 1 < M]),
+                                     np.array([0, M // 3, M - 1])]))
+    ref = alg1_rows_with_tail(oracle_lib, A, B, rows, sched, C=C, kc=128)
+    assert np.array_equal(out[1][rows].view(np.uint32), ref.view(np.uint32))
+    # tiles outside the split: the unsplit launch's bits
+    mask = np.ones((M, N), dtype=bool)
+    for m, n in tiles:
+        mask[m * th:(m + 1) * th, n * bn:(n + 1) * bn] = False
+    assert np.array_equal(out[1][mask].view(np.uint32), out[0][mask].view(np.uint32))

@@ -7,7 +7,7 @@ import torch
 
 from paper_conf_ppopp_fengwcz0d21_b200 import inputs
 from tests import kernel_model as km
-from tests.gpu_util import require_gpu, to_dev, to_host
+from tests.gpu_util import alg1_rows_with_tail, require_gpu, tail_split_tiles, to_dev, to_host
 
 pytestmark = pytest.mark.gpu
 
@@ -33,8 +33,10 @@ def _gemm_sampled(oracle_lib, M, N, K, seed_a, seed_b, n_rows, presplit=False):
     cg, bn, sep, kc = eg.query_config("gemm" if presplit else "gemm_b32", M, N, K)
     bound = oracle_lib.elem_bound(As, B, kc=kc)
     assert np.all(np.abs(D[rows].astype(np.float64) - C64) <= bound)
-    br = rows[: min(len(rows), 8)]
-    ref = oracle_lib.gemm_alg1_tc(A[br], B, terms=3, sep=sep, kc=kc)
+    # (plus the last rows: with a tail-split last wave (R21 k-parts) they are split tiles')
+    sched = tail_split_tiles(eg, "gemm" if presplit else "gemm_b32", M, N, K)
+    br = np.unique(np.concatenate([rows[: min(len(rows), 8)], rows[-4:]]))
+    ref = alg1_rows_with_tail(oracle_lib, A, B, br, sched, sep=sep, kc=kc)
     assert np.array_equal(D[br].view(np.uint32), ref.view(np.uint32))
     return e, en
 

@@ -91,7 +91,9 @@ def test_gemm_transposed_and_presplit(oracle_lib):
     D2 = to_host(eg.gemm(Ad, to_dev(np.ascontiguousarray(B.T)), b_trans=True))
     a_split = eg.split(Ad)
     b_split = eg.split(Bd, transpose=True)
-    eg.set_config(*eg.query_config("gemm_b32", 256, 512, 384))  # same (sep, Kc) as D1
+    c = eg.query_config_ex("gemm_b32", 256, 512, 384)  # same (sep, Kc, k-parts) as D1
+    eg.set_config_ex(cg=c["cg"], bn=c["bn"], sep=c["sep"], kc=c["kc"], ksplit=c["ksplit"],
+                     tail_split=c["tail_split"], fused=0)
     try:
         D3 = to_host(eg.gemm(None, None, a_split=a_split, b_split=b_split))
     finally:

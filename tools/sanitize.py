@@ -30,6 +30,10 @@ VARIANTS = {
     "cg1_128_ksplit2_sep": ({"ksplit": 2}, (1, 128, 1, 128), (200, 200, 600)),
     "fused_a_tail_peel": ({"fused": 1, "tail_peel": 1}, (2, 256, 0, 64), (94 * 256 + 37, 256, 256)),
     "bf16_parts": ({"operand_format": 1}, (2, 256, 0, 64), (300, 520, 200)),
+    # 18 tiles on 8 clusters: the last 2 tiles as 4 k-parts each, last-arriver fix-up
+    "tail_split": ({"tail_split": 1, "max_clusters": 8}, (2, 256, 0, 64), (5 * 256 + 37, 700, 1100)),
+    "fused_a_tail_split": ({"fused": 1, "tail_split": 1, "max_clusters": 8}, (2, 256, 0, 64),
+                           (5 * 256 + 37, 700, 1100)),
     "presplit_128_s3": ({"stages": 3}, (2, 128, 0, 64), (300, 300, 200)),
 }
 
