@@ -25,6 +25,9 @@ def main():
     ap = argparse.ArgumentParser()
     ap.add_argument("--reps", type=int, default=5)
     ap.add_argument("--out", default=None)
+    ap.add_argument("--short", type=int, default=0,
+                    help="also time windows of this many back-to-back calls (the bench's tall-skinny "
+                         "window is 20), alternating off / on, 7 trials, median")
     args = ap.parse_args()
     rows = []
     for (M, N, K) in SHAPES:
@@ -52,6 +55,26 @@ def main():
             r["mhz_ts%d" % ts] = round(sum(x[1] for x in res[ts]) / len(res[ts]), 0)
             r["cycles_ts%d" % ts] = round(min(x[2] for x in res[ts]), 0)
         r["speedup"] = round(r["ms_ts0"] / r["ms_ts1"], 4)
+        if args.short:
+            sh = {0: [], 1: []}
+            for trial in range(7):
+                for ts in ((0, 1) if trial % 2 == 0 else (1, 0)):
+                    egemm.set_config_ex(tail_split=ts)
+                    try:
+                        for _ in range(3):
+                            egemm.gemm(A, B, out=D, workspace=ws)
+                        s0, e0 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                        s0.record()
+                        for _ in range(args.short):
+                            egemm.gemm(A, B, out=D, workspace=ws)
+                        e0.record()
+                        e0.synchronize()
+                        sh[ts].append(s0.elapsed_time(e0) / args.short)
+                    finally:
+                        egemm.set_config_ex()
+            for ts in (0, 1):
+                r["short_ms_ts%d" % ts] = round(sorted(sh[ts])[len(sh[ts]) // 2], 5)
+            r["short_speedup"] = round(r["short_ms_ts0"] / r["short_ms_ts1"], 4)
         rows.append(r)
         print(json.dumps(r), flush=True)
         del A, B, ws, D

@@ -19,6 +19,9 @@ power-capped clock is a few %).  The term count is then
 measured on the pick with uniform, in-zone (2^U[-3,3)) and stress (2^U[-14,15)) inputs:
 4 terms are chosen only where 3 miss the bar and 4 meet it.  kNN / kMeans results are
 bitwise identical across their configurations (checked), so time alone decides.
+The tail-split flag ("tsplit") is not swept here: tools/tail_split_ab.py measures it on the
+shapes whose last wave is partly filled and it is set by hand on the buckets where it wins
+(the table's tsplit_note); re-add it after a re-sweep.
 Tool code (calls oracle/ for the error checks).
 
 usage: python tools/tune_sweep.py [--quick] [--ops gemm,gemm_b32,knn,kmeans] [--out table.json]
