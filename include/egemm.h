@@ -208,7 +208,8 @@ int egemm_kmeans_finalize(const double* sums, const int64_t* counts, int64_t kc,
  *  terms       : 3 or 4 products (0 = the call's / table's).
  *  n_slices    : kNN N-slices per query block (1..16; 0 = table / wave-balance formula).
  *  epi_warps   : kMeans epilogue warps (8 or 16; 0 = table / 16).
- *  a_resident  : kNN query tile resident in smem (-1 = when d <= 128, 0 = never).
+ *  a_resident  : kNN query tile resident in smem (-1 = when d <= 128, 0 = never); kMeans
+ *                point tile resident (1 = when d <= 128; -1 / 0 = streamed, the default).
  *  pace        : k-pacing of STORE GEMMs (-1 = table / on, 0 = off).
  *  max_clusters: persistent clusters launched (0 = one per SM pair / SM).
  *  operand_format: 0 = fp16 parts (the paper's round-split), 1 = bf16 parts (NEXT-3: the

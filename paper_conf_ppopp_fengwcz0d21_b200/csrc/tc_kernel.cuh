@@ -359,13 +359,17 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
   uint64_t* empty = bars + STAGES;
   uint64_t* acc_full = bars + 2 * STAGES;
   uint64_t* acc_empty = bars + 2 * STAGES + 2;
+  // AR: resident A slots (K <= 64: two slots, the next unit's tile loads while this unit's
+  // MMAs run; K <= 128: one slot holding both k-blocks)
   uint64_t* a_full = bars + 2 * STAGES + 4;
   uint64_t* a_empty = bars + 2 * STAGES + 5;
   uint32_t* tmem_slot = reinterpret_cast<uint32_t*>(bars + 2 * STAGES + 6);
-  uint64_t* sfull = bars + 2 * STAGES + 8;   // AS: fp32 A tile landed (TMA bytes)
+  uint64_t* a_full1 = bars + 2 * STAGES + 7;
+  uint64_t* a_empty1 = bars + 2 * STAGES + 8;
+  uint64_t* sfull = bars + 2 * STAGES + 10;  // AS: fp32 A tile landed (TMA bytes)
   uint64_t* sempty = sfull + NSTG;           // AS: consumed by the 4 converter warps
   uint64_t* afull = sempty + NSTG;           // AS: a stage's fp32 A tile landed (TMA bytes)
-  uint8_t* scratch = reinterpret_cast<uint8_t*>(bars + 2 * STAGES + 8 + 2 * NSTG + (AS ? STAGES : 0));  // merges
+  uint8_t* scratch = reinterpret_cast<uint8_t*>(bars + 2 * STAGES + 10 + 2 * NSTG + (AS ? STAGES : 0));  // merges
   // TS (STORE): the result leaves through TMA stores -- each epilogue warp stages a 32 x 32
   // fp32 block (128-B rows, 128-B swizzle) in its own 4 KiB buffer and one lane issues a
   // bulk tensor store: coalesced full-line writes, the LSU free for the next unit's drains
@@ -399,6 +403,8 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
     }
     ptx::mbar_init(a_full, 1);
     ptx::mbar_init(a_empty, 1);
+    ptx::mbar_init(a_full1, 1);
+    ptx::mbar_init(a_empty1, 1);
     if constexpr (AS)
       for (int s = 0; s < STAGES; s++) ptx::mbar_init(&afull[s], 1);
     for (int i = 0; i < NSTG; i++) {
@@ -626,16 +632,18 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
         UnitInfo ui = decode_unit<EPI>(p, u);
         const int arow = ui.m_tile * (kBM * CG) + (int)rank * kBM;
         if constexpr (AR) {
-          ptx::mbar_wait(a_empty, (uctr & 1u) ^ 1u);  // the previous unit's MMAs are done
-          if (leader) ptx::mbar_arrive_expect_tx(a_full, 2 * G::A_BYTES * p.num_kb * CG);
+          const uint32_t nsl = p.num_kb == 1 ? 2u : 1u, slot = uctr % nsl, use = uctr / nsl;
+          uint64_t* af = slot ? a_full1 : a_full;
+          ptx::mbar_wait(slot ? a_empty1 : a_empty, (use & 1u) ^ 1u);  // the slot's last unit is done
+          if (leader) ptx::mbar_arrive_expect_tx(af, 2 * G::A_BYTES * p.num_kb * CG);
           for (int kb = 0; kb < p.num_kb; kb++) {
-            uint8_t* ab = a_res + kb * 2 * G::A_BYTES;
+            uint8_t* ab = a_res + (slot + kb) * 2 * G::A_BYTES;
             if constexpr (CG == 1) {
-              ptx::tma_load_2d(&tm_ahi, a_full, ab, kb * kBK, arow);
-              ptx::tma_load_2d(&tm_alo, a_full, ab + G::A_BYTES, kb * kBK, arow);
+              ptx::tma_load_2d(&tm_ahi, af, ab, kb * kBK, arow);
+              ptx::tma_load_2d(&tm_alo, af, ab + G::A_BYTES, kb * kBK, arow);
             } else {
-              ptx::tma_load_2d_pair(&tm_ahi, a_full, ab, kb * kBK, arow);
-              ptx::tma_load_2d_pair(&tm_alo, a_full, ab + G::A_BYTES, kb * kBK, arow);
+              ptx::tma_load_2d_pair(&tm_ahi, af, ab, kb * kBK, arow);
+              ptx::tma_load_2d_pair(&tm_alo, af, ab + G::A_BYTES, kb * kBK, arow);
             }
           }
         }
@@ -788,8 +796,9 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
       const uint32_t abase = ptx::smem_u32(a_res);
       for (int u = cluster; u < p.num_units; u += nclusters, uctr++) {
         UnitInfo ui = decode_unit<EPI>(p, u);
+        const uint32_t nsl = p.num_kb == 1 ? 2u : 1u, aslot = AR ? uctr % nsl : 0u;
         if constexpr (AR) {
-          ptx::mbar_wait(a_full, uctr & 1u);  // this unit's A tile is resident
+          ptx::mbar_wait(aslot ? a_full1 : a_full, (uctr / nsl) & 1u);  // this unit's A tile is resident
           ptx::tc_fence_after();
         }
         for (int ns = 0; ns < ui.n_count; ns++) {
@@ -807,7 +816,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
               if (!(DIAG_NO_TMA && DIAG_MODE(2))) ptx::mbar_wait(&full[stage], phase);
               ptx::tc_fence_after();
               const uint32_t sa = sbase + stage * SB;
-              const uint32_t aa = AR ? abase + kb * 2 * G::A_BYTES : sa;
+              const uint32_t aa = AR ? abase + (aslot + kb) * 2 * G::A_BYTES : sa;
               const uint64_t d_ahi = ptx::sdesc_kmajor_sw128(aa);
               const uint64_t d_alo = ptx::sdesc_kmajor_sw128(aa + G::A_BYTES);
               const uint64_t d_bhi = ptx::sdesc_kmajor_sw128(sa + B_OFF);
@@ -848,7 +857,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
                                       ptx::idesc_tf32_f32(kBM * CG, BN), 1u);
                 }
                 if (!(DIAG_NO_TMA && DIAG_MODE(4))) ptx::mma_commit<CG>(&empty[stage]);
-                if (DIAG_MODE(1)) ptx::mma_commit<CG>(a_empty);  // diagnostics only
+                if (!AR && DIAG_MODE(1)) ptx::mma_commit<CG>(a_empty);  // diagnostics only
               }
               __syncwarp();
               if (++stage == STAGES) { stage = 0; phase ^= 1u; }
@@ -859,7 +868,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
           }
         }
         if constexpr (AR) {  // the resident A tile is free once this unit's MMAs complete
-          if (ptx::elect_one()) ptx::mma_commit<CG>(a_empty);
+          if (ptx::elect_one()) ptx::mma_commit<CG>(aslot ? a_empty1 : a_empty);
           __syncwarp();
         }
       }
@@ -1228,15 +1237,23 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
               // the improving quarter in smem and searching once per unit measured the same.)
               // (a depth-5 tree here, or loading both groups and releasing the accumulator
               // before the search, measured slower than this chain with 16 warps)
-              float mx = __int_as_float(0xff800000);
+              // The search runs for the whole warp whenever one lane improves (nearly every
+              // group: the first groups of a row always do), so it is kept short: the half
+              // holding the maximum (the lower half on a tie) is selected first, then searched.
+              float mxa = __int_as_float(0xff800000), mxb = mxa;
 #pragma unroll
-              for (int i = 0; i < 32; i++) mx = fmaxf(mx, v[i]);
+              for (int i = 0; i < 16; i++) { mxa = fmaxf(mxa, v[i]); mxb = fmaxf(mxb, v[16 + i]); }
+              const float mx = fmaxf(mxa, mxb);
               if (mx > best) {  // strict: an equal key from a later column never wins
-                int idx = 31;
+                const bool lo = (mxa == mx);
+                float w[16];
 #pragma unroll
-                for (int i = 30; i >= 0; i--) idx = (v[i] == mx) ? i : idx;  // lowest index
+                for (int i = 0; i < 16; i++) w[i] = lo ? v[i] : v[16 + i];
+                int idx = 15;
+#pragma unroll
+                for (int i = 14; i >= 0; i--) idx = (w[i] == mx) ? i : idx;  // lowest index
                 best = mx;
-                besti = c0 + idx;
+                besti = c0 + (lo ? idx : 16 + idx);
               }
             }
           }
@@ -1339,7 +1356,7 @@ constexpr size_t variant_smem() {
   constexpr size_t sb = (AR ? 2 * G::B_BYTES : G::STAGE_BYTES) + (NORM ? G::BNC * 32 : 0);
   constexpr size_t base = 1024 + (size_t)STAGES * sb + (AR ? 4 * G::A_BYTES : 0) + (NORM ? kBM * 32 : 0) +
                           (FB ? 3 * kBM * kBK * 4 + 8 * 6 : 0) + (AS ? 8 * STAGES : 0) +
-                          8 * (2 * STAGES + 8) + scratch;
+                          8 * (2 * STAGES + 10) + scratch;
   // TS: one 4 KiB TMA-store staging buffer per epilogue warp, 1 KiB aligned (128-B swizzle)
   constexpr bool TS = (EPI == EPI_STORE) && !FB && ((BN / (NEPI / 4)) % 32 == 0);
   return TS ? ((base + 1023) / 1024) * 1024 + (size_t)NEPI * 4096 : base;

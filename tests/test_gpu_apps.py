@@ -360,3 +360,23 @@ def test_kmeans_allreduce_finalize_peer_buffers(oracle_lib):
     os_, oc = oracle_lib.kmeans_sums(X, ga, 40)
     assert np.array_equal(ref_c, oc)
     assert np.all(np.abs(ref_s - os_) <= oracle_lib.kmeans_sums_bound(X, ga, 40))
+
+
+@pytest.mark.parametrize("n,d,kc,epi", [(20000, 64, 1024, 16), (5000, 128, 300, 8), (3001, 64, 100, 16)])
+def test_kmeans_resident_points_same_bits(oracle_lib, n, d, kc, epi):
+    """The point tile resident in smem across the centroid tiles (a_resident, d <= 128) or
+    streamed with every centroid tile: the same arithmetic, so the same bits (assignment,
+    fp64 sums, counts, inertia)."""
+    eg = require_gpu()
+    X, _, _ = inputs.mixture(n, d, min(kc, 1024), 70 + d, sigma=0.2)
+    C = X[:kc].copy()
+    out = {}
+    for ar in (0, 1):
+        eg.set_config_ex(a_resident=ar, epi_warps=epi)
+        try:
+            out[ar] = [to_host(t) for t in eg.kmeans_step(to_dev(X), to_dev(C))]
+            assert eg.query_config_ex("kmeans", n, kc, d)["a_resident"] == ar
+        finally:
+            eg.set_config_ex()
+    for u, v in zip(out[0], out[1]):
+        assert np.array_equal(u.view(np.uint8), v.view(np.uint8))
