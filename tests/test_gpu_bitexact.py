@@ -216,3 +216,25 @@ def test_tail_split_bitexact(oracle_lib, fused, shape, clusters):
     for m, n in tiles:
         mask[m * th:(m + 1) * th, n * bn:(n + 1) * bn] = False
     assert np.array_equal(out[1][mask].view(np.uint32), out[0][mask].view(np.uint32))
+
+
+@pytest.mark.parametrize("cfg", [(2, 128, 1, 256), (1, 128, 1, 128), (2, 224, 0, 128), (1, 128, 0, 64)])
+def test_tail_split_other_tiles(oracle_lib, cfg):
+    """The tail split's fix-up on the other tile shapes / accumulator modes (SEP: the parts
+    carry hi*hi + cross totals; single-CTA tiles; 224-wide tiles), with C."""
+    from tests.gpu_util import alg1_rows_with_tail, tail_split_tiles
+    eg = require_gpu()
+    M, N, K = 5 * 256 + 37, 650, 4100
+    A, B, C = inputs.uniform((M, K), 83), inputs.uniform((K, N), 84), inputs.uniform((M, N), 85)
+    eg.set_config_ex(cg=cfg[0], bn=cfg[1], sep=cfg[2], kc=cfg[3], fused=0, tail_split=1, max_clusters=8)
+    try:
+        sched = tail_split_tiles(eg, "gemm", M, N, K)
+        D = to_host(eg.gemm(to_dev(A), to_dev(B), to_dev(C)))
+    finally:
+        eg.set_config_ex()
+    tiles, kpart, th, bn = sched
+    assert tiles and kpart < K
+    rows = np.unique(np.concatenate([np.arange(m * th, min(M, m * th + th), 29) for m, _ in tiles] +
+                                    [np.array([0, M - 1])]))
+    ref = alg1_rows_with_tail(oracle_lib, A, B, rows, sched, C=C, sep=cfg[2], kc=cfg[3])
+    assert np.array_equal(D[rows].view(np.uint32), ref.view(np.uint32))
