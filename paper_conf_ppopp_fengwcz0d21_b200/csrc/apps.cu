@@ -23,8 +23,8 @@ __global__ void __launch_bounds__(256) rownorm_kernel(const float* __restrict__ 
     double s = 0.0;
     for (int64_t t0 = 0; t0 < d; t0 += kNormSlab) {
       __syncwarp();
-#pragma unroll 4
-      for (int rr = 0; rr < 32; rr++) {  // row r0 + rr, columns t0 + lane
+#pragma unroll
+      for (int rr = 0; rr < 32; rr++) {  // row r0 + rr, columns t0 + lane (all 32 loads in flight)
         const int64_t r = r0 + rr, t = t0 + lane;
         slab[w][rr][lane] = (r < rows && t < d) ? __ldg(x + r * ld + t) : 0.f;
       }

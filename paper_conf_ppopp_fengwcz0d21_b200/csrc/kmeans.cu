@@ -145,6 +145,11 @@ __global__ void __launch_bounds__(32 * W) km_scatter_kernel(
   const int64_t s0 = i0 + (int64_t)w * SUB, s1 = min(i1, s0 + SUB);
   int32_t* mine = hw + (int64_t)w * kc;
   const int nbits = kc > 1 ? 32 - __clz((int)(kc - 1)) : 0;
+  // KEEP (one batch per warp, W = 8): the batch's keys and peer masks stay in registers for
+  // pass 2 instead of being loaded and recomputed (the ballots are most of the kernel's work)
+  constexpr bool KEEP = (SUB == 32 * B);
+  int kav[KEEP ? B : 1];
+  uint32_t kpeers[KEEP ? B : 1];
   for (int64_t cb = s0; cb < s1; cb += 32 * B) {
     int av[B];
 #pragma unroll
@@ -157,6 +162,7 @@ __global__ void __launch_bounds__(32 * W) km_scatter_kernel(
       const int64_t i = cb + 32 * t + lane;
       const uint32_t peers = same_key_lanes(av[t], i < s1, nbits);
       if (i < s1 && lane == __ffs(peers) - 1) mine[av[t]] += __popc(peers);
+      if constexpr (KEEP) { kav[t] = av[t]; kpeers[t] = peers; }
       __syncwarp();  // the next batch's leader of this centroid may be another lane
     }
   }
@@ -175,17 +181,19 @@ __global__ void __launch_bounds__(32 * W) km_scatter_kernel(
   __syncthreads();
   for (int64_t cb = s0; cb < s1; cb += 32 * B) {
     int av[B];
+    if constexpr (!KEEP) {
 #pragma unroll
-    for (int t = 0; t < B; t++) {
-      const int64_t i = cb + 32 * t + lane;
-      av[t] = i < s1 ? assign[i] : 0;
+      for (int t = 0; t < B; t++) {
+        const int64_t i = cb + 32 * t + lane;
+        av[t] = i < s1 ? assign[i] : 0;
+      }
     }
 #pragma unroll
     for (int t = 0; t < B; t++) {
       const int64_t i = cb + 32 * t + lane;
       const bool valid = i < s1;
-      const int a = av[t];
-      const uint32_t peers = same_key_lanes(a, valid, nbits);
+      const int a = KEEP ? kav[t] : av[t];
+      const uint32_t peers = KEEP ? kpeers[t] : same_key_lanes(a, valid, nbits);
       const int rank = __popc(peers & ((1u << lane) - 1u));
       if (valid) order[mine[a] + rank] = (int32_t)i;
       __syncwarp();
