@@ -118,7 +118,8 @@ struct KParams {
   unsigned long long* probe;  // device clock probe: [0..3] last launch, [4..6] running sums, [7] counter
   int debug_mode;    // EGEMM_DEBUG_MODE bits (diagnostics): 1 extra commit per k-block;
                      // with NO_TMA: 2 MMA warp ignores the full barriers (producer idle),
-                     // 4 no per-k-block commits
+                     // 4 no per-k-block commits; 1024 (fused-A / resident-A variants) no B
+                     // loads after the ring's first fill
   // STORE tail split (R21's k-parts for the last, partly filled wave only): units >= tail_u0
   // are k-parts (tail_parts per tile, tail_kbpp k-blocks each) of the tiles tail_u0, ...;
   // each part leaves its fp32 sum in fix_ws and the last part to finish a warp's slab (per
@@ -685,7 +686,14 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
               if (++stage == STAGES) { stage = 0; phase ^= 1u; }
               continue;
             }
-            if (leader) ptx::mbar_arrive_expect_tx(&full[stage], TX * CG);
+            // (diagnostics only, bit 1024: after the ring's first fill, skip the B loads -- the
+            // MMAs re-read real but stale B tiles; the time / clock change bounds what removing
+            // B's L2 -> smem traffic can buy)
+            const bool skip_b = DIAG_MODE(1024) && (FA || AR) && gkb > (uint32_t)STAGES;
+            if (leader) {
+              if (skip_b) ptx::mbar_arrive(&full[stage]);
+              else ptx::mbar_arrive_expect_tx(&full[stage], TX * CG);
+            }
             const int k0 = kb * kBK;
             if constexpr (AS) {  // this CTA's fp32 A tile into the stage's A region
               ptx::mbar_arrive_expect_tx(&afull[stage], STG_BYTES);
@@ -697,7 +705,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
                 ptx::tma_load_2d(&tm_ahi, &full[stage], sb, k0, arow);
                 ptx::tma_load_2d(&tm_alo, &full[stage], sb + G::A_BYTES, k0, arow);
               }
-              if (!FB) {
+              if (!FB && !skip_b) {
                 ptx::tma_load_2d(&tm_bhi, &full[stage], sb + B_OFF, k0, brow);
                 ptx::tma_load_2d(&tm_blo, &full[stage], sb + B_OFF + G::B_BYTES, k0, brow);
               }
@@ -706,7 +714,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
                 ptx::tma_load_2d_pair(&tm_ahi, &full[stage], sb, k0, arow);
                 ptx::tma_load_2d_pair(&tm_alo, &full[stage], sb + G::A_BYTES, k0, arow);
               }
-              if (!FB) {
+              if (!FB && !skip_b) {
                 ptx::tma_load_2d_pair(&tm_bhi, &full[stage], sb + B_OFF, k0, brow);
                 ptx::tma_load_2d_pair(&tm_blo, &full[stage], sb + B_OFF + G::B_BYTES, k0, brow);
               }
