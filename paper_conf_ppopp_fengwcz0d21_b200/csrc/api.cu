@@ -8,6 +8,7 @@
 #include <cstring>
 #include <mutex>
 #include <thread>
+#include <nvtx3/nvToolsExt.h>
 #include "../../include/egemm.h"
 #include "egemm_internal.h"
 
@@ -239,6 +240,15 @@ static int check_operand(const egemm_operand_t& op, int64_t rows, int64_t K, boo
 
 using namespace egemm;
 
+// NVTX range around each public compute call (header-only NVTX 3: a no-op unless a
+// profiler such as Nsight Systems is attached), so timelines show the C-ABI calls by name.
+namespace {
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
+}  // namespace
+
 extern "C" {
 
 const char* egemm_status_string(int s) {
@@ -389,17 +399,20 @@ static int split_entry(const float* x, int64_t rows, int64_t cols, int64_t ldx, 
 
 int egemm_split(const float* x, int64_t rows, int64_t cols, int64_t ldx, uint16_t* hi,
                 uint16_t* lo, int64_t ldo, int transpose, uint32_t* range_flags, void* stream) {
+  NvtxRange nvtx_range("egemm_split");
   return split_entry(x, rows, cols, ldx, hi, lo, ldo, transpose, range_flags, stream, 0);
 }
 
 int egemm_split_trunc(const float* x, int64_t rows, int64_t cols, int64_t ldx, uint16_t* hi,
                       uint16_t* lo, int64_t ldo, int transpose, uint32_t* range_flags,
                       void* stream) {
+  NvtxRange nvtx_range("egemm_split_trunc");
   return split_entry(x, rows, cols, ldx, hi, lo, ldo, transpose, range_flags, stream, 1);
 }
 
 int egemm_split_bf16(const float* x, int64_t rows, int64_t cols, int64_t ldx, uint16_t* hi,
                      uint16_t* lo, int64_t ldo, int transpose, void* stream) {
+  NvtxRange nvtx_range("egemm_split_bf16");
   return split_entry(x, rows, cols, ldx, hi, lo, ldo, transpose, nullptr, stream, 2);
 }
 
@@ -455,6 +468,7 @@ size_t egemm_gemm_workspace_size(int64_t M, int64_t N, int64_t K, int a_presplit
 int egemm_gemm(int64_t M, int64_t N, int64_t K, egemm_operand_t A, egemm_operand_t B,
                const float* C, int64_t ldc, float* D, int64_t ldd, int terms, void* workspace,
                size_t workspace_bytes, void* stream) {
+  NvtxRange nvtx_range("egemm_gemm");
   cudaStream_t s = (cudaStream_t)stream;
   if (M < 0 || N < 0 || K < 0) {
     set_last_error("negative size");
@@ -599,6 +613,7 @@ size_t egemm_gemm_host_workspace_size(int64_t M, int64_t N, int64_t K) {
 int egemm_gemm_host(int64_t M, int64_t N, int64_t K, const float* A_host, int64_t lda,
                     const float* B_host, int64_t ldb, float* D_host, int64_t ldd, int terms,
                     void* workspace, size_t workspace_bytes, void* stream) {
+  NvtxRange nvtx_range("egemm_gemm_host");
   cudaStream_t s = (cudaStream_t)stream;
   if (M < 0 || N < 0 || K < 0 || lda < K || ldb < N || ldd < N) {
     set_last_error("negative size or ld too small");
@@ -746,6 +761,7 @@ size_t egemm_knn_workspace_size(int64_t nx, int64_t nq, int64_t d, int k, int x_
 
 int egemm_knn_index(const float* X, int64_t nx, int64_t d, int64_t ldx, uint16_t* hi, uint16_t* lo,
                     int64_t ld_split, float* norms, void* stream) {
+  NvtxRange nvtx_range("egemm_knn_index");
   cudaStream_t s = (cudaStream_t)stream;
   if (nx < 0 || d <= 0 || ldx < d || ld_split < d || (ld_split % 8) != 0) {
     set_last_error("need nx >= 0, d > 0, ldx >= d, ld_split >= d and a multiple of 8");
@@ -769,6 +785,7 @@ int egemm_knn_index(const float* X, int64_t nx, int64_t d, int64_t ldx, uint16_t
 int egemm_knn(egemm_operand_t X, const float* x_norms, int64_t nx, egemm_operand_t Q, int64_t nq,
               int64_t d, int k, int32_t* out_idx, float* out_dist, void* workspace,
               size_t workspace_bytes, void* stream) {
+  NvtxRange nvtx_range("egemm_knn");
   cudaStream_t s = (cudaStream_t)stream;
   if (nx < 0 || nq < 0 || d <= 0 || k < 1 || k > 64 || k > nx) {
     set_last_error("need nx, nq >= 0, d > 0, 1 <= k <= min(64, nx)");
@@ -841,6 +858,7 @@ int egemm_knn(egemm_operand_t X, const float* x_norms, int64_t nx, egemm_operand
 
 int egemm_knn_merge(const float* keys, const int32_t* idx, int n_lists, int64_t nq, int k_in, int k,
                     const float* qnorm, int32_t* out_idx, float* out_key, void* stream) {
+  NvtxRange nvtx_range("egemm_knn_merge");
   if (nq < 0 || n_lists < 1 || n_lists > 64 || k_in < 1 || k_in > 1024 || k < 1 || k > 64 ||
       (int64_t)k > (int64_t)k_in * n_lists) {
     set_last_error("need nq >= 0, 1 <= n_lists <= 64, 1 <= k_in <= 1024, 1 <= k <= min(64, k_in * n_lists)");
@@ -877,6 +895,7 @@ size_t egemm_kmeans_workspace_size(int64_t n, int64_t d, int64_t kc, int x_presp
 int egemm_kmeans_step(egemm_operand_t X, int64_t n, int64_t d, const float* centroids, int64_t kc,
                       int32_t* assign, double* sums, int64_t* counts, double* inertia,
                       void* workspace, size_t workspace_bytes, void* stream) {
+  NvtxRange nvtx_range("egemm_kmeans_step");
   cudaStream_t s = (cudaStream_t)stream;
   if (n < 0 || d <= 0 || kc <= 0 || !centroids || !assign || !sums || !counts) {
     set_last_error("need n >= 0, d > 0, kc > 0 and non-NULL centroids/assign/sums/counts");
@@ -929,6 +948,7 @@ int egemm_kmeans_step(egemm_operand_t X, int64_t n, int64_t d, const float* cent
 
 int egemm_kmeans_finalize(const double* sums, const int64_t* counts, int64_t kc, int64_t d,
                           float* centroids, void* stream) {
+  NvtxRange nvtx_range("egemm_kmeans_finalize");
   if (kc < 0 || d < 0 || (kc * d > 0 && (!sums || !counts || !centroids))) {
     set_last_error("bad kmeans_finalize arguments");
     return EGEMM_ERR_INVALID_ARG;
@@ -946,6 +966,7 @@ int egemm_kmeans_allreduce_finalize(const double* const* peer_sums,
                                     const int64_t* const* peer_counts, int nranks, int64_t kc,
                                     int64_t d, double* sums_out, int64_t* counts_out,
                                     float* centroids, void* stream) {
+  NvtxRange nvtx_range("egemm_kmeans_allreduce_finalize");
   if (nranks < 1 || nranks > kMaxPeers || kc < 0 || d < 0 || !peer_sums || !peer_counts ||
       (kc * d > 0 && !centroids)) {
     set_last_error("need 1 <= nranks <= %d, host arrays of peer pointers, centroids", kMaxPeers);
