@@ -5,6 +5,7 @@
 // descriptor", "Instruction descriptor" for .kind::f16).
 #pragma once
 #include <cstdint>
+#include <cstdio>
 #include <cuda_runtime.h>
 
 namespace egemm {
@@ -60,6 +61,30 @@ __device__ __forceinline__ void mbar_arrive_cluster(uint64_t* bar, uint32_t cta)
 #else
 #define EGEMM_WAIT_HINT ""
 #endif
+#if defined(EGEMM_DIAG) && EGEMM_DIAG
+// Diagnostic builds: a wait that has not completed after ~10 s (1000 suspended try_waits of
+// up to 10 ms each) reports the barrier and traps, so a protocol bug surfaces as a launch
+// error naming the stuck barrier instead of a hung GPU.
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  const uint32_t addr = smem_u32(bar);
+  for (uint32_t it = 0;; it++) {
+    uint32_t ok;
+    asm volatile(
+        "{\n\t.reg .pred P;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 P, [%1], %2, 0x989680;\n\t"
+        "selp.u32 %0, 1, 0, P;\n\t}"
+        : "=r"(ok)
+        : "r"(addr), "r"(parity)
+        : "memory");
+    if (ok) return;
+    if (it == 1000) {
+      printf("egemm: mbarrier wait stuck (block %d, thread %d, smem 0x%x, parity %u)\n", (int)blockIdx.x,
+             (int)threadIdx.x, addr, parity);
+      __trap();
+    }
+  }
+}
+#else
 __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
   uint32_t addr = smem_u32(bar);
   asm volatile(
@@ -70,6 +95,7 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
       "r"(parity)
       : "memory");
 }
+#endif
 // Wait with cluster-scope acquire (for barriers completed by remote arrivals/commits).
 __device__ __forceinline__ void mbar_wait_cluster(uint64_t* bar, uint32_t parity) {
   uint32_t addr = smem_u32(bar);
