@@ -294,6 +294,15 @@ int egemm_debug_clock_stats(double* mhz, double* cycles_per_launch, double* laun
  * 32-column group).  reset != 0 zeroes it after reading.  Synchronous. */
 int egemm_debug_counter(unsigned long long* value, int reset);
 
+/* Debug: the phase timeline of CTA 0 of the last tensor-core launch (SM clock64 values,
+ * 16 slots; written only by a library built with EGEMM_DIAG=1 under EGEMM_DEBUG_MODE bit
+ * 2048, else left as they are): [0] entry, [1] setup done (barriers, TMEM, PDL wait),
+ * [2] first operand load issued, [3] first MMA issued, [4] last MMA committed, [5] last
+ * accumulator chunk received by the epilogue, [6] last result stored, [7] exit barrier
+ * passed, [8] first converted stage handed over (fused split), [9] first MMA of the CTA's
+ * second unit.  out: 16 host words.  reset != 0 zeroes the slots after reading.  Synchronous. */
+int egemm_debug_timeline(unsigned long long* out, int reset);
+
 #ifdef __cplusplus
 }
 #endif

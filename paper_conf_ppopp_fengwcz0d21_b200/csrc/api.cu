@@ -58,6 +58,7 @@ const Knobs& knobs() {
     if (k.as_pf < 0) k.as_pf = 0;
     k.host_chunk = env_int("EGEMM_HOST_CHUNK", 0);
     k.no_tma_store = env_int("EGEMM_NO_TMA_STORE", 0) == 1;
+    k.no_pdl = env_int("EGEMM_NO_PDL", 0) == 1;
 #if EGEMM_DIAG
     k.dbg_no_tma = env_int("EGEMM_DEBUG_NO_TMA", 0) == 1;
     k.dbg_no_epi = env_int("EGEMM_DEBUG_NO_EPI", 0) == 1;
@@ -185,7 +186,7 @@ struct Carver {
 // rows x K logical (K-major).  f32 layout: trans==0 -> rows x K (ld), trans==1 -> K x rows.
 static int stage_operand(const egemm_operand_t& op, int64_t rows, int64_t K, Carver& cv,
                          const uint16_t** hi, const uint16_t** lo, int64_t* ld,
-                         cudaStream_t s, int mode = 0) {
+                         cudaStream_t s, int mode = 0, bool pdl = false) {
   if (op.hi && op.lo) {
     *hi = op.hi;
     *lo = op.lo;
@@ -195,8 +196,8 @@ static int stage_operand(const egemm_operand_t& op, int64_t rows, int64_t K, Car
   const int64_t ldk = ldk_of(K);
   uint16_t* h = cv.take<uint16_t>((size_t)(rows * ldk));
   uint16_t* l = cv.take<uint16_t>((size_t)(rows * ldk));
-  int r = op.trans ? launch_split(op.f32, K, rows, op.ld, h, l, ldk, 1, nullptr, s, mode)
-                   : launch_split(op.f32, rows, K, op.ld, h, l, ldk, 0, nullptr, s, mode);
+  int r = op.trans ? launch_split(op.f32, K, rows, op.ld, h, l, ldk, 1, nullptr, s, mode, pdl && !knobs().no_pdl)
+                   : launch_split(op.f32, rows, K, op.ld, h, l, ldk, 0, nullptr, s, mode, pdl && !knobs().no_pdl);
   if (r) {
     set_last_error("split launch failed");
     return EGEMM_ERR_CUDA;
@@ -352,6 +353,11 @@ int egemm_debug_clock_stats(double* mhz, double* cycles_per_launch, double* laun
 int egemm_debug_counter(unsigned long long* value, int reset) {
   if (!value) return EGEMM_ERR_INVALID_ARG;
   return read_debug_counter(value, reset) ? EGEMM_ERR_CUDA : EGEMM_OK;
+}
+
+int egemm_debug_timeline(unsigned long long* out, int reset) {
+  if (!out) return EGEMM_ERR_INVALID_ARG;
+  return read_debug_timeline(out, reset) ? EGEMM_ERR_CUDA : EGEMM_OK;
 }
 
 int egemm_set_config(int cg, int bn, int sep, int kc) {
@@ -523,7 +529,9 @@ int egemm_gemm(int64_t M, int64_t N, int64_t K, egemm_operand_t A, egemm_operand
     ops.ldb_f32 = B.ld;
     cv.take<uint16_t>((size_t)(N * ldk_of(K)));  // keep the workspace layout unchanged
     cv.take<uint16_t>((size_t)(N * ldk_of(K)));
-  } else if ((r = stage_operand(Bt, N, K, cv, &ops.b_hi, &ops.b_lo, &ops.ldb, s, cfg.fmt == 1 ? 2 : 0))) {
+  } else if ((r = stage_operand(Bt, N, K, cv, &ops.b_hi, &ops.b_lo, &ops.ldb, s, cfg.fmt == 1 ? 2 : 0,
+                                /* B's split follows A's (independent) as its PDL dependent */
+                                !fuse_a && !A.hi))) {
     return r;
   }
   TcEpilogue epi = {};

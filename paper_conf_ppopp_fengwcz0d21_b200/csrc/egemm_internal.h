@@ -12,7 +12,10 @@ int num_sms();
 // mode 2: round-split into bf16 parts (NEXT-3 variant; range_flags not produced)
 int launch_split(const float* x, int64_t rows, int64_t cols, int64_t ldx, uint16_t* hi,
                  uint16_t* lo, int64_t ldo, int transpose, uint32_t* range_flags,
-                 cudaStream_t stream, int mode = 0);
+                 cudaStream_t stream, int mode = 0, bool pdl = false);
+// pdl: launch as the programmatic dependent of the previous kernel in the stream, which must be
+// an INDEPENDENT split of the same call (split.cu, PDL hooks); the split then completes only
+// after that kernel has.
 
 // Epilogue policies of the tensor-core kernel.
 enum EpiKind : int { EPI_STORE = 0, EPI_KNN = 1, EPI_KMEANS = 2 };
@@ -87,6 +90,7 @@ struct Knobs {
   int as_pf;           // fused A, staged: k-blocks of L2 prefetch (EGEMM_AS_PREFETCH)
   int host_chunk;      // egemm_gemm_host row chunk (EGEMM_HOST_CHUNK, 0 = auto)
   int no_tma_store;    // EGEMM_NO_TMA_STORE=1: STORE epilogue with per-lane row stores (A/B runs)
+  int no_pdl;          // EGEMM_NO_PDL=1: no programmatic dependent launches (A/B runs)
   int dbg_no_tma, dbg_no_epi, dbg_mode;  // diagnostics (EGEMM_DEBUG_*; EGEMM_DIAG builds only)
 };
 const Knobs& knobs();
@@ -143,6 +147,7 @@ int launch_tc_probe(int kind, int N, int K, const void* A, const void* B, const 
                     float* D, cudaStream_t stream);
 int read_clock_stats(double* mhz, double* cycles_per_launch, double* launches, int reset);
 int read_debug_counter(unsigned long long* value, int reset);
+int read_debug_timeline(unsigned long long* out16, int reset);
 
 // tune.cu: the measured configuration table
 struct TuneEntry {

@@ -5,7 +5,8 @@
 
 namespace egemm {
 
-__device__ unsigned long long g_clock_probe[8];  // [0..3] last launch, [4..6] running sums, [7] counter
+// [0..3] last launch, [4..6] running sums, [7] counter, [8..23] phase timeline (EGEMM_DIAG)
+__device__ unsigned long long g_clock_probe[24];
 
 static unsigned long long* probe_ptr() {
   void* p = nullptr;
@@ -21,6 +22,19 @@ int read_debug_counter(unsigned long long* value, int reset) {
   if (reset) {
     const unsigned long long z = 0;
     if (cudaMemcpyToSymbol(g_clock_probe, &z, sizeof(z), 7 * sizeof(unsigned long long)) != cudaSuccess)
+      return 3;
+  }
+  return 0;
+}
+
+// Phase timeline of CTA 0 (g_clock_probe[8..23], written by EGEMM_DIAG builds).
+int read_debug_timeline(unsigned long long* out16, int reset) {
+  if (cudaMemcpyFromSymbol(out16, g_clock_probe, 16 * sizeof(unsigned long long),
+                           8 * sizeof(unsigned long long)) != cudaSuccess)
+    return 3;
+  if (reset) {
+    const unsigned long long z[16] = {};
+    if (cudaMemcpyToSymbol(g_clock_probe, z, sizeof(z), 8 * sizeof(unsigned long long)) != cudaSuccess)
       return 3;
   }
   return 0;

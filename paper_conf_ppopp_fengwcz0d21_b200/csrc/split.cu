@@ -49,6 +49,32 @@ __device__ __forceinline__ SplitPair split2(float a, float b, uint32_t& flags) {
   return SplitPair{h, l};
 }
 
+// Programmatic dependent launch (PDL) hooks.  Every split kernel lets its stream successor
+// launch as soon as all of its CTAs are running (the tcgen05 GEMM that consumes the parts then
+// sets up -- barriers, TMEM, tensor-map prefetch -- under the split's tail and waits with
+// griddepcontrol.wait before its first operand load).  A split launched as the PDL follower
+// of another, independent split (A's, then B's, in one egemm_gemm call) may run beside that
+// split's tail; it waits for it at its END, so its own completion still implies the
+// completion of everything before it in the stream (the GEMM's wait covers both splits).
+// In a kernel that was not launched as a programmatic dependent, griddepcontrol.wait
+// returns at once.
+__device__ __forceinline__ void pdl_trigger() { asm volatile("griddepcontrol.launch_dependents;" ::: "memory"); }
+__device__ __forceinline__ void pdl_wait_prev() { asm volatile("griddepcontrol.wait;" ::: "memory"); }
+
+template <typename... KArgs, typename... Args>
+static void launch_k(void (*k)(KArgs...), dim3 grid, cudaStream_t stream, bool pdl, Args... args) {
+  cudaLaunchConfig_t c = {};
+  c.gridDim = grid;
+  c.blockDim = dim3(256, 1, 1);
+  c.stream = stream;
+  cudaLaunchAttribute a[1];
+  a[0].id = cudaLaunchAttributeProgrammaticStreamSerialization;
+  a[0].val.programmaticStreamSerializationAllowed = 1;
+  c.attrs = a;
+  c.numAttrs = pdl ? 1 : 0;
+  cudaLaunchKernelEx(&c, k, static_cast<KArgs>(args)...);
+}
+
 __device__ __forceinline__ void flush_flags(uint32_t flags, uint32_t* range_flags) {
   if (range_flags == nullptr) return;
   uint32_t any = __reduce_or_sync(0xffffffffu, flags);
@@ -61,6 +87,7 @@ __global__ void __launch_bounds__(256) split_flat_kernel(const float* __restrict
                                                           uint16_t* __restrict__ hi,
                                                           uint16_t* __restrict__ lo,
                                                           uint32_t* range_flags) {
+  pdl_trigger();
   uint32_t flags = 0;
   const int64_t nv = n >> 3;  // groups of 8: 2 x 16 B in, 16 B + 16 B out
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
@@ -81,6 +108,7 @@ __global__ void __launch_bounds__(256) split_flat_kernel(const float* __restrict
     }
   }
   flush_flags(flags, range_flags);
+  pdl_wait_prev();
 }
 
 // Strided, same orientation: one thread per element.
@@ -90,6 +118,7 @@ __global__ void __launch_bounds__(256) split_strided_kernel(const float* __restr
                                                              int64_t ldx, uint16_t* __restrict__ hi,
                                                              uint16_t* __restrict__ lo,
                                                              int64_t ldo, uint32_t* range_flags) {
+  pdl_trigger();
   uint32_t flags = 0;
   const int64_t total = rows * cols;
   const int64_t stride = (int64_t)gridDim.x * blockDim.x;
@@ -100,6 +129,7 @@ __global__ void __launch_bounds__(256) split_strided_kernel(const float* __restr
     lo[r * ldo + c] = (uint16_t)(p.lo & 0xffffu);
   }
   flush_flags(flags, range_flags);
+  pdl_wait_prev();
 }
 
 // Transposing: x is rows x cols (ldx); hi/lo are cols x rows (ldo).  64 x 64 tiles:
@@ -115,11 +145,15 @@ __global__ void __launch_bounds__(256) split_transpose_kernel(const float* __res
                                                                uint16_t* __restrict__ lo,
                                                                int64_t ldo, uint32_t* range_flags,
                                                                int skip_full) {
+  pdl_trigger();
   __shared__ uint32_t th[64][33];  // packed fp16 pairs of tile element [c][r]
   __shared__ uint32_t tl[64][33];
   uint32_t flags = 0;
   const int64_t r0 = (int64_t)blockIdx.y * kTR, c0 = (int64_t)blockIdx.x * kTC;
-  if (skip_full && r0 + kTR <= rows && c0 + kTC <= cols) return;  // done by the fast kernel
+  if (skip_full && r0 + kTR <= rows && c0 + kTC <= cols) {  // done by the fast kernel
+    pdl_wait_prev();
+    return;
+  }
   const int tx = threadIdx.x & 31, ty = threadIdx.x >> 5;  // 32 x 8
   for (int i = 0; i < 8; i++) {
     const int r = ty + 8 * i;
@@ -156,6 +190,7 @@ __global__ void __launch_bounds__(256) split_transpose_kernel(const float* __res
     }
   }
   flush_flags(flags, range_flags);  // padding elements are 0: they raise no flag
+  pdl_wait_prev();
 }
 
 // Transposing, full 64 x 64 tiles with aligned rows (x: 16-B float4 loads; hi / lo: 16-B
@@ -167,6 +202,7 @@ template <int MODE, bool FLAGS>
 __global__ void __launch_bounds__(256) split_transpose_fast_kernel(
     const float* __restrict__ x, int64_t rows, int64_t cols, int64_t ldx, uint16_t* __restrict__ hi,
     uint16_t* __restrict__ lo, int64_t ldo, uint32_t* range_flags) {
+  pdl_trigger();
   __shared__ uint32_t th[kTC][kTR / 2 + 1];  // [c][r/2]: packed (r, r+1) pairs, 33-word pitch
   __shared__ uint32_t tl[kTC][kTR / 2 + 1];
   uint32_t flags = 0;
@@ -200,12 +236,13 @@ __global__ void __launch_bounds__(256) split_transpose_fast_kernel(
     __stcs(reinterpret_cast<uint4*>(lo + o), vl);
   }
   if constexpr (FLAGS) flush_flags(flags, range_flags);
+  pdl_wait_prev();
 }
 
 template <int MODE>
 static void launch_mode(const float* x, int64_t rows, int64_t cols, int64_t ldx, uint16_t* hi,
                         uint16_t* lo, int64_t ldo, int transpose, uint32_t* range_flags,
-                        cudaStream_t stream) {
+                        cudaStream_t stream, bool pdl) {
   const int nsm = num_sms();
   const bool fl = range_flags != nullptr;
   if (!transpose) {
@@ -217,42 +254,45 @@ static void launch_mode(const float* x, int64_t rows, int64_t cols, int64_t ldx,
       const int64_t cap = (int64_t)nsm * 8;  // 8 x 256 threads resident per SM
       if (blocks > cap) blocks = cap;
       if (blocks < 1) blocks = 1;
-      if (fl) split_flat_kernel<MODE, true><<<(unsigned)blocks, 256, 0, stream>>>(x, n, hi, lo, range_flags);
-      else split_flat_kernel<MODE, false><<<(unsigned)blocks, 256, 0, stream>>>(x, n, hi, lo, nullptr);
+      if (fl) launch_k(split_flat_kernel<MODE, true>, dim3((unsigned)blocks), stream, pdl, x, n, hi, lo, range_flags);
+      else launch_k(split_flat_kernel<MODE, false>, dim3((unsigned)blocks), stream, pdl, x, n, hi, lo, nullptr);
     } else {
       int64_t blocks = (n + 255) / 256;
       const int64_t cap = (int64_t)nsm * 8;
       if (blocks > cap) blocks = cap;
-      split_strided_kernel<MODE><<<(unsigned)blocks, 256, 0, stream>>>(x, rows, cols, ldx, hi, lo,
-                                                                        ldo, range_flags);
+      launch_k(split_strided_kernel<MODE>, dim3((unsigned)blocks), stream, pdl, x, rows, cols, ldx, hi,
+               lo, ldo, range_flags);
     }
   } else {
     dim3 grid((unsigned)((cols + kTC - 1) / kTC), (unsigned)((rows + kTR - 1) / kTR));
     const bool fast = (ldx % 4 == 0) && ((uintptr_t)x % 16 == 0) && (ldo % 8 == 0) &&
                       ((uintptr_t)hi % 16 == 0) && ((uintptr_t)lo % 16 == 0);
     const dim3 full((unsigned)(cols / kTC), (unsigned)(rows / kTR));
+    bool launched = false;
     if (fast && full.x > 0 && full.y > 0) {
       if (fl)
-        split_transpose_fast_kernel<MODE, true><<<full, 256, 0, stream>>>(x, rows, cols, ldx, hi, lo,
-                                                                          ldo, range_flags);
+        launch_k(split_transpose_fast_kernel<MODE, true>, full, stream, pdl, x, rows, cols, ldx, hi, lo,
+                 ldo, range_flags);
       else
-        split_transpose_fast_kernel<MODE, false><<<full, 256, 0, stream>>>(x, rows, cols, ldx, hi, lo,
-                                                                           ldo, nullptr);
+        launch_k(split_transpose_fast_kernel<MODE, false>, full, stream, pdl, x, rows, cols, ldx, hi, lo,
+                 ldo, nullptr);
+      launched = true;
     }
     const bool edges = !fast || (cols % kTC) != 0 || (rows % kTR) != 0 || full.x == 0 || full.y == 0;
+    // the edge tiles are independent of the full ones: a PDL follower of the fast kernel
     if (edges)
-      split_transpose_kernel<MODE><<<grid, 256, 0, stream>>>(x, rows, cols, ldx, hi, lo, ldo,
-                                                             range_flags, fast ? 1 : 0);
+      launch_k(split_transpose_kernel<MODE>, grid, stream, pdl || launched, x, rows, cols, ldx, hi,
+               lo, ldo, range_flags, fast ? 1 : 0);
   }
 }
 
 int launch_split(const float* x, int64_t rows, int64_t cols, int64_t ldx, uint16_t* hi,
                  uint16_t* lo, int64_t ldo, int transpose, uint32_t* range_flags,
-                 cudaStream_t stream, int mode) {
+                 cudaStream_t stream, int mode, bool pdl) {
   if (rows == 0 || cols == 0) return 0;
-  if (mode == 1) launch_mode<1>(x, rows, cols, ldx, hi, lo, ldo, transpose, range_flags, stream);
-  else if (mode == 2) launch_mode<2>(x, rows, cols, ldx, hi, lo, ldo, transpose, range_flags, stream);
-  else launch_mode<0>(x, rows, cols, ldx, hi, lo, ldo, transpose, range_flags, stream);
+  if (mode == 1) launch_mode<1>(x, rows, cols, ldx, hi, lo, ldo, transpose, range_flags, stream, pdl);
+  else if (mode == 2) launch_mode<2>(x, rows, cols, ldx, hi, lo, ldo, transpose, range_flags, stream, pdl);
+  else launch_mode<0>(x, rows, cols, ldx, hi, lo, ldo, transpose, range_flags, stream, pdl);
   return cudaGetLastError() == cudaSuccess ? 0 : -1;
 }
 

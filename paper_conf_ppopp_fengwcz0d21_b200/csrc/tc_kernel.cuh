@@ -70,6 +70,8 @@ constexpr bool kDiag = EGEMM_DIAG != 0;
 #define DIAG_NO_TMA (kDiag && p.debug_no_tma)
 #define DIAG_NO_EPI (kDiag && p.debug_no_epi)
 #define DIAG_MODE(bits) (kDiag && (p.debug_mode & (bits)))
+// phase timeline of CTA 0 (EGEMM_DEBUG_MODE bit 2048; egemm_debug_timeline): slot i <- clock64
+#define TL(i) do { if (DIAG_MODE(2048) && blockIdx.x == 0) p.probe[8 + (i)] = clock64(); } while (0)
 
 constexpr int kBM = 128;       // rows per CTA (TMEM lanes)
 constexpr int kBK = 64;        // k elements per stage (128 B of fp16: one SW128 row)
@@ -384,6 +386,10 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
   const int cluster = (CG == 2) ? (int)ptx::cluster_id_x() : (int)blockIdx.x;
   const int nclusters = (CG == 2) ? (int)ptx::nclusters_x() : (int)gridDim.x;
   const bool leader = (rank == 0);
+  if (threadIdx.x == 0) {
+    TL(0);
+    if (DIAG_MODE(2048) && blockIdx.x == 0) p.probe[8 + 10] = globaltimer_ns();
+  }
 
   if (warp == EG::W_PROD && lane == 0) {
     ptx::prefetch_tmap(&tm_ahi);  // (FA: tm_ahi maps the fp32 A: staged loads / L2 prefetch)
@@ -453,6 +459,12 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
   if constexpr (CG == 2) { ptx::cluster_sync(); __syncthreads(); } else __syncthreads();
   ptx::tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  // Every launch is a programmatic dependent of the previous kernel in the stream (the split
+  // of this call, or anything else): the setup above ran under that kernel's tail; nothing
+  // global is touched before it has completed.  (A peeled tail launch instead overlaps the
+  // main grid of the same call -- disjoint rows -- and waits at its end.)
+  if (!p.pdl_wait) asm volatile("griddepcontrol.wait;" ::: "memory");
+  if (threadIdx.x == 0) TL(1);
   // STORE: a tail launch of the same call (the peeled last wave, launched with programmatic
   // stream serialisation) may start on the SMs this grid frees as its CTAs finish
   if (EPI == EPI_STORE && threadIdx.x == 0) asm volatile("griddepcontrol.launch_dependents;");
@@ -524,6 +536,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
       uint32_t phase = 0;
       int si = 0;          // AS: staging ring slot / parity
       uint32_t sph = 0;
+      int conv_n = 0;  // (diagnostics: timeline slot 8)
       const int c = lane & 7;         // 16-B chunk (8 fp16) of the 128-B row
       const int rsub = lane >> 3;     // 4 rows per warp instruction
       for (int u = cluster; u < p.num_units; u += nclusters) {
@@ -568,6 +581,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
               if (lane == 0) {
                 if constexpr (CG == 1) ptx::mbar_arrive(&full[stage]);
                 else ptx::mbar_arrive_cluster(&full[stage], 0);
+                if (warp == 0 && conv_n++ == 0) TL(8);
               }
               if (++stage == STAGES) { stage = 0; phase ^= 1u; }
               continue;
@@ -695,6 +709,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
               else ptx::mbar_arrive_expect_tx(&full[stage], TX * CG);
             }
             const int k0 = kb * kBK;
+            if (gkb == 1) TL(14);
             if constexpr (AS) {  // this CTA's fp32 A tile into the stage's A region
               ptx::mbar_arrive_expect_tx(&afull[stage], STG_BYTES);
               ptx::tma_load_2d(&tm_ahi, &afull[stage], sb, k0, arow);
@@ -719,6 +734,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
                 ptx::tma_load_2d_pair(&tm_blo, &full[stage], sb + B_OFF + G::B_BYTES, k0, brow);
               }
             }
+            if (gkb == 1) TL(2);
             if (++stage == STAGES) { stage = 0; phase ^= 1u; }
           }
         }
@@ -864,13 +880,20 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
                                       ptx::sdesc_kmajor_sw32(sa + NP_OFF),
                                       ptx::idesc_tf32_f32(kBM * CG, BN), 1u);
                 }
+                if (kb == kb0 && ch == 0 && ns == 0) {
+                  if (uctr == 0) TL(3);
+                  else if (uctr == 1) TL(9);
+                }
                 if (!(DIAG_NO_TMA && DIAG_MODE(4))) ptx::mma_commit<CG>(&empty[stage]);
                 if (!AR && DIAG_MODE(1)) ptx::mma_commit<CG>(a_empty);  // diagnostics only
               }
               __syncwarp();
               if (++stage == STAGES) { stage = 0; phase ^= 1u; }
             }
-            if (ptx::elect_one()) ptx::mma_commit<CG>(&acc_full[buf]);
+            if (ptx::elect_one()) {
+              ptx::mma_commit<CG>(&acc_full[buf]);
+              TL(4);
+            }
             __syncwarp();
             chunk_ctr++;
           }
@@ -934,6 +957,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
             const uint32_t use = chunk_ctr >> 1;
             ptx::mbar_wait(&acc_full[buf], use & 1u);
             ptx::tc_fence_after();
+            if (ew == 0 && lane == 0) TL(5);
             const uint32_t acc_hh = tmem_base + lane_off + (SEP ? 2 * buf : buf) * BN + cgp * COLS;
             if (!DIAG_NO_EPI)
 #pragma unroll
@@ -964,6 +988,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
 #pragma unroll
             for (int j = 0; j < COLS; j++) tot[j] = __fadd_rn(tot[j], totx[j]);
           }
+          if (ew == 0 && lane == 0) TL(12);
           if (ui.fx >= 0) {
             // tail split: this part's sums go to the workspace (coalesced float4 slab per
             // warp); the warp that completes a slab's last part adds the parts in k order
@@ -1019,6 +1044,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
                   ptx::tma_store_commit();
                 }
               }
+              if (ew == 0 && lane == 0) TL(6);
               continue;
             }
           }
@@ -1327,11 +1353,20 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
 
   // ============================ teardown ============================
   if constexpr (TS) {
-    if (p.tma_store && warp >= EG::EPI0 && lane == 0) ptx::tma_store_wait0();  // stores complete
+    // the staging buffers must have been read before the CTA's shared memory goes away; the
+    // global writes themselves complete with the grid (a successor -- stream order or its
+    // griddepcontrol.wait -- sees them), so the CTA does not wait for them (-0.8 K cycles at
+    // the end of every launch, tools/timeline.py)
+    if (p.tma_store && warp >= EG::EPI0 && lane == 0) ptx::tma_store_wait_read0();
+    if (warp == EG::EPI0 && lane == 0) TL(13);
   }
   __syncwarp();
   ptx::tc_fence_before();
   if constexpr (CG == 2) ptx::cluster_sync(); else __syncthreads();
+  if (threadIdx.x == 0) {
+    TL(7);
+    if (DIAG_MODE(2048) && blockIdx.x == 0) p.probe[8 + 11] = globaltimer_ns();
+  }
   if (warp == EG::W_ALLOC) {
     ptx::tc_fence_after();
     ptx::tmem_dealloc<CG>(tmem_base, TMEM_COLS);
@@ -1411,7 +1446,8 @@ static int launch_variant(const CUtensorMap* maps, const KParams& kp, int max_cl
   attr[1].id = cudaLaunchAttributeProgrammaticStreamSerialization;
   attr[1].val.programmaticStreamSerializationAllowed = 1;
   cfg.attrs = attr;
-  cfg.numAttrs = kp.pdl_wait ? 2 : 1;
+  // cluster dims + programmatic stream serialization (see the kernel's setup)
+  cfg.numAttrs = (kp.pdl_wait || !knobs().no_pdl) ? 2 : 1;
   cudaError_t e = cudaLaunchKernelEx(&cfg, kern, maps[0], maps[1], maps[2], maps[3], maps[4], kp);
   if (e != cudaSuccess) {
     set_last_error("cudaLaunchKernelEx: %s", cudaGetErrorString(e));

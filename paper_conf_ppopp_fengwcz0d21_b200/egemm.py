@@ -47,7 +47,7 @@ EXPORTS = ["egemm_status_string", "egemm_last_error", "egemm_version", "egemm_sp
            "egemm_gemm_workspace_size", "egemm_knn", "egemm_knn_workspace_size", "egemm_knn_index",
            "egemm_kmeans_step", "egemm_kmeans_workspace_size", "egemm_kmeans_finalize",
            "egemm_set_config", "egemm_num_sms", "egemm_debug_last_clock", "egemm_tune_table",
-           "egemm_debug_clock_stats", "egemm_debug_counter", "egemm_tc_probe",
+           "egemm_debug_clock_stats", "egemm_debug_counter", "egemm_debug_timeline", "egemm_tc_probe",
            "egemm_query_config", "egemm_gemm_host", "egemm_gemm_host_workspace_size",
            "egemm_set_config_ex", "egemm_query_config_ex", "egemm_knn_merge", "egemm_split_bf16",
            "egemm_kmeans_allreduce_finalize"]
@@ -103,6 +103,8 @@ def load(path: str = LIB_PATH):
     L.egemm_debug_clock_stats.restype = I
     L.egemm_debug_counter.argtypes = [ctypes.POINTER(ctypes.c_ulonglong), I]
     L.egemm_debug_counter.restype = I
+    L.egemm_debug_timeline.argtypes = [ctypes.POINTER(ctypes.c_ulonglong), I]
+    L.egemm_debug_timeline.restype = I
     L.egemm_gemm_host.argtypes = [I64, I64, I64, P, I64, P, I64, P, I64, I, P, SZ, P]
     L.egemm_gemm_host.restype = I
     L.egemm_gemm_host_workspace_size.argtypes = [I64, I64, I64]
@@ -209,6 +211,14 @@ def debug_counter(reset: bool = True) -> int:
     v = ctypes.c_ulonglong(0)
     _check(load().egemm_debug_counter(ctypes.byref(v), int(reset)), "egemm_debug_counter")
     return int(v.value)
+
+
+def debug_timeline(reset: bool = True) -> list:
+    """CTA 0's phase timeline of the last tensor-core launch (16 SM-clock values; recorded
+    only by an EGEMM_DIAG=1 build under EGEMM_DEBUG_MODE bit 2048; see egemm.h)."""
+    v = (ctypes.c_ulonglong * 16)()
+    _check(load().egemm_debug_timeline(v, int(reset)), "egemm_debug_timeline")
+    return [int(x) for x in v]
 
 
 def debug_last_clock() -> float:
