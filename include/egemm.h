@@ -9,6 +9,9 @@
  *  - Every pointer argument is a DEVICE pointer owned by the caller, unless stated.
  *  - Calls are asynchronous on `stream` (a cudaStream_t; NULL = legacy default stream), never
  *    synchronise the device, never allocate device memory, and are re-entrant.
+ *  - Stream order is kept exactly: the kernels are programmatic dependent launches that may
+ *    start their setup (barriers, tensor memory) under the previous kernel's tail, but touch
+ *    no global memory before that kernel has completed (griddepcontrol.wait).
  *  - Matrices are row-major with an explicit row stride `ld*` in ELEMENTS.
  *  - fp16 "hi"/"lo" buffers hold IEEE binary16 bit patterns (uint16_t).
  *  - Return value: an egemm_status_t.  Host-side validation is synchronous; EGEMM_ERR_CUDA
