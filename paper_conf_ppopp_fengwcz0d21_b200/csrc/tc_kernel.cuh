@@ -119,6 +119,8 @@ struct KParams {
   int tma_store;     // STORE: D through TMA stores (tm_d; no C, aligned D); else per-lane stores
   unsigned long long* probe;  // device clock probe: [0..3] last launch, [4..6] running sums, [7] counter
   int debug_mode;    // EGEMM_DEBUG_MODE bits (diagnostics): 1 extra commit per k-block;
+                     // 2048 phase timeline of CTA 0; 4096 staged fused-A converters skip the
+                     // conversion (wrong results; bounds its cost);
                      // with NO_TMA: 2 MMA warp ignores the full barriers (producer idle),
                      // 4 no per-k-block commits; 1024 (fused-A / resident-A variants) no B
                      // loads after the ring's first fill
@@ -555,6 +557,14 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
               const uint32_t sb = ptx::smem_u32(stage_base + stage * G::STAGE_BYTES);
               const uint32_t xb = sb + (c >> 2) * (STG_BYTES / 2);
               const int j0 = (c & 3) * 2;
+              if (DIAG_MODE(4096)) {  // diagnostics only: hand the fp32 tile over unconverted
+                if (lane == 0) {      // (results wrong by design: bounds the conversion's cost)
+                  if constexpr (CG == 1) ptx::mbar_arrive(&full[stage]);
+                  else ptx::mbar_arrive_cluster(&full[stage], 0);
+                }
+                if (++stage == STAGES) { stage = 0; phase ^= 1u; }
+                continue;
+              }
               float4 u[16];
 #pragma unroll
               for (int it = 0; it < 8; it++) {
