@@ -226,13 +226,16 @@ int egemm_kmeans_finalize(const double* sums, const int64_t* counts, int64_t kc,
  *  ksplit      : STORE split-K (R21's k-parts): K in up to ksplit contiguous parts, each tile's
  *                parts run as separate units, their fp32 results are added in k order (then
  *                + C) by a reduce pass; needs the larger egemm_gemm_workspace_size (0/1 = none).
- *  tail_split  : STORE GEMMs whose persistent grid's last wave is at most half full: only
- *                that wave's tiles are cut into 2..4 k-parts (R21) run side by side; each part
- *                leaves its fp32 sums in the workspace and the part that finishes last adds
- *                them in k order (+ C) and stores the tile -- no extra launch.  Uses
- *                egemm_gemm_workspace_size's room (without it the wave runs unsplit)
- *                (-1 = table, default off: fewer SM cycles but no shorter time under the
- *                power cap, profiles/r02_tail_split_ab.json; 0 = off, 1 = on).
+ *  tail_split  : STORE GEMMs whose persistent grid's last wave is at most half full (also a
+ *                single, partly filled wave): only that wave's tiles are cut into 2..4
+ *                k-parts (R21) run side by side; each part leaves its fp32 sums in the
+ *                workspace and the part that finishes last adds them in k order (+ C) and
+ *                stores the tile -- no extra launch.  Uses egemm_gemm_workspace_size's room
+ *                (without it the wave runs unsplit) (-1 = table: on for the buckets where it
+ *                measured faster -- single-wave K >= 4096 shapes, up to 2x; off for multi-wave
+ *                shapes, where it saves SM cycles but not time under the power cap,
+ *                profiles/r02_tail_split_ab.json, profiles/r02_tail_split_single_wave.json;
+ *                0 = off, 1 = on).  An explicit tile override (cg != 0) starts from off.
  */
 typedef struct {
   int cg, bn, sep, kc, stages, fused, terms, n_slices, epi_warps, a_resident, pace, max_clusters,

@@ -285,7 +285,9 @@ TailSplit tail_geometry(int64_t M, int64_t N, int64_t K, const TcConfig& cfg) {
   if (cfg.max_clusters > 0 && cfg.max_clusters < clusters) clusters = cfg.max_clusters;
   const int64_t th = (int64_t)kBM * cfg.cg;
   const int64_t tiles = ((M + th - 1) / th) * ((N + cfg.bn - 1) / cfg.bn);
-  if (clusters < 2 || tiles <= clusters) return t;
+  // (a single partly filled wave -- tiles < clusters -- is its own last wave: all of its tiles
+  // become k-parts, e.g. 1024^3 at 256 x 128 pair tiles: 32 tiles on 74 clusters)
+  if (clusters < 2) return t;
   const int64_t rem = tiles % clusters;
   if (rem == 0 || 2 * rem > clusters) return t;
   int parts = (int)(clusters / rem);

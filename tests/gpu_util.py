@@ -45,7 +45,7 @@ def tail_split_tiles(eg, op, M, N, K):
         clusters = c["max_clusters"]
     mt, nt = -(-M // th), -(-N // bn)
     tiles = mt * nt
-    if clusters < 2 or tiles <= clusters:
+    if clusters < 2:
         return none
     rem = tiles % clusters
     if rem == 0 or 2 * rem > clusters:

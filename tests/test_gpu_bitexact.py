@@ -238,3 +238,28 @@ def test_tail_split_other_tiles(oracle_lib, cfg):
                                     [np.array([0, M - 1])]))
     ref = alg1_rows_with_tail(oracle_lib, A, B, rows, sched, C=C, sep=cfg[2], kc=cfg[3])
     assert np.array_equal(D[rows].view(np.uint32), ref.view(np.uint32))
+
+
+@pytest.mark.parametrize("case", [((300, 700, 4100), (2, 128, 0, 128), 0),    # 2 x 6 tiles: 4 parts
+                                  ((1000, 1000, 8192), (2, 128, 0, 128), 0),  # 4 x 8 tiles: 2 parts
+                                  ((200, 300, 5000), (1, 128, 1, 128), 0),    # single CTAs, SEP
+                                  ((8192, 256, 4096), (2, 256, 0, 128), 1)])  # fused A, 32 tiles
+def test_tail_split_single_wave(oracle_lib, case):
+    """A single, partly filled wave (tiles <= clusters / 2): every tile runs as k-parts with the
+    in-kernel fix-up -- bitwise the oracle's Alg. 1 with kpart (R21), with C; the table turns
+    this on for the single-wave K >= 4096 buckets (profiles/r02_tail_split_single_wave.json)."""
+    from tests.gpu_util import alg1_rows_with_tail, tail_split_tiles
+    eg = require_gpu()
+    (M, N, K), cfg, fused = case
+    A, B, C = inputs.uniform((M, K), 86), inputs.uniform((K, N), 87), inputs.uniform((M, N), 88)
+    eg.set_config_ex(cg=cfg[0], bn=cfg[1], sep=cfg[2], kc=cfg[3], fused=fused, tail_split=1)
+    try:
+        sched = tail_split_tiles(eg, "gemm_b32", M, N, K)
+        D = to_host(eg.gemm(to_dev(A), to_dev(B), to_dev(C)))
+    finally:
+        eg.set_config_ex()
+    tiles, kpart, th, bn = sched
+    assert len(tiles) == -(-M // th) * -(-N // bn) and kpart < K  # every tile is split
+    rows = np.unique(np.concatenate([np.arange(0, M, 23), np.array([M - 1])]))
+    ref = alg1_rows_with_tail(oracle_lib, A, B, rows, sched, C=C, sep=cfg[2], kc=cfg[3])
+    assert np.array_equal(D[rows].view(np.uint32), ref.view(np.uint32))
