@@ -235,7 +235,8 @@ int egemm_kmeans_finalize(const double* sums, const int64_t* counts, int64_t kc,
  *                measured faster -- single-wave K >= 4096 shapes, up to 2x; off for multi-wave
  *                shapes, where it saves SM cycles but not time under the power cap,
  *                profiles/r02_tail_split_ab.json, profiles/r02_tail_split_single_wave.json;
- *                0 = off, 1 = on).  An explicit tile override (cg != 0) starts from off.
+ *                0 = off, 1 = on).  An explicit tile override (cg != 0) starts with both the
+ *                tail split and split-K off (the override names one launch configuration).
  */
 typedef struct {
   int cg, bn, sep, kc, stages, fused, terms, n_slices, epi_warps, a_resident, pace, max_clusters,

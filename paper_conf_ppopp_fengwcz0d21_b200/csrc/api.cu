@@ -139,7 +139,8 @@ static TcConfig choose_config(int epi_kind, int64_t M, int64_t N, int64_t K, int
       c.sep = o.sep;
       c.fa = 0;  // an explicit tile override measures the pre-split path unless `fused` says
       c.stages = 0;
-      c.tsplit = 0;  // ... and no tail split unless `tail_split` says
+      c.tsplit = 0;  // ... and no tail split / split-K unless `tail_split` / `ksplit` say
+      c.ksplit = 0;
     }
     if (o.kc && epi_kind == EPI_STORE) c.kc = o.kc;
     if (o.fused >= 0) c.fa = o.fused;

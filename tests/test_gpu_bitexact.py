@@ -168,6 +168,7 @@ def test_split_k_workspace_too_small():
     import torch
     eg = require_gpu()
     A, B = to_dev(inputs.uniform((256, 512), 1)), to_dev(inputs.uniform((512, 256), 2))
+    eg.set_config_ex(cg=2, bn=256, sep=0, kc=64, fused=0)  # (an explicit tile: no split-K)
     small = torch.empty(eg.gemm_workspace_size(256, 256, 512), dtype=torch.uint8, device="cuda")
     D = torch.empty((256, 256), device="cuda")
     eg.set_config_ex(cg=2, bn=256, sep=0, kc=64, fused=0, ksplit=4)
