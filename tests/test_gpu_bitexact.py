@@ -264,3 +264,20 @@ def test_tail_split_single_wave(oracle_lib, case):
     rows = np.unique(np.concatenate([np.arange(0, M, 23), np.array([M - 1])]))
     ref = alg1_rows_with_tail(oracle_lib, A, B, rows, sched, C=C, sep=cfg[2], kc=cfg[3])
     assert np.array_equal(D[rows].view(np.uint32), ref.view(np.uint32))
+
+
+@pytest.mark.parametrize("shape", [(128, 256, 4096), (200, 256, 8192), (256, 1000, 3000)])
+def test_table_split_k_small_shapes(oracle_lib, shape):
+    """The table's split-K picks for short-M/N, long-K calls (ksplit up to 16, post-sweep
+    passes, profiles/r02_ksplit_8_16.json) through the public call with no override: bitwise
+    the oracle's Alg. 1 with kpart = the part length the library reports (R21)."""
+    eg = require_gpu()
+    M, N, K = shape
+    c = eg.query_config_ex("gemm_b32", M, N, K)
+    assert c["ksplit"] > 1  # the shape exercises a table split-K row
+    nkb = -(-K // 64)
+    kpart = 64 * -(-nkb // c["ksplit"])
+    A, B, C = inputs.uniform((M, K), 90), inputs.uniform((K, N), 91), inputs.uniform((M, N), 92)
+    D = to_host(eg.gemm(to_dev(A), to_dev(B), to_dev(C)))
+    ref = oracle_lib.gemm_alg1_tc(A, B, C, terms=3, sep=c["sep"], kc=c["kc"], kpart=kpart)
+    assert np.array_equal(D.view(np.uint32), ref.view(np.uint32)), int((D != ref).sum())

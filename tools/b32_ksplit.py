@@ -30,6 +30,8 @@ def main(out, op="gemm_b32"):
         tiles = -(-M // (128 * cg)) * -(-N // bn)
         if 2 * tiles > nsm // cg or e.get("fa", 0) == 2:
             continue
+        if "MAXTILES" in os.environ and (tiles > int(os.environ["MAXTILES"]) or K < 2048):
+            continue
         A, B = inputs.uniform((M, K), 11 + M), inputs.uniform((K, N), 13 + N)
         Ad, Bd = torch.from_numpy(A).cuda(), torch.from_numpy(B).cuda()
         bs = egemm.split(Bd, transpose=True) if op == "gemm" else None
@@ -39,8 +41,12 @@ def main(out, op="gemm_b32"):
         C64 = oracle.gemm64(A[rs], B)
         en = oracle.normwise_error(oracle.gemm32_naive(A[rs], B), A[rs], B, C64)
         base = dict(cg=cg, bn=bn, sep=e["sep"], kc=e["kc"], fused=e.get("fa", 0), stages=e.get("stages", 0))
-        cands = {"ks1": dict(base, fused=0, tail_split=0, ksplit=1), "pick": dict(base, tail_split=e.get("tsplit", 0), ksplit=max(1, e.get("ksplit", 0))),
-                 "ks2": dict(base, fused=0, tail_split=0, ksplit=2), "ks4": dict(base, fused=0, tail_split=0, ksplit=4)}
+        kss = [int(v) for v in os.environ.get("KS", "2,4").split(",")]
+        cands = {"pick": dict(base, tail_split=e.get("tsplit", 0), ksplit=max(1, e.get("ksplit", 0)))}
+        if "KS" not in os.environ:
+            cands["ks1"] = dict(base, fused=0, tail_split=0, ksplit=1)
+        for v in kss:
+            cands["ks%d" % v] = dict(base, fused=0, tail_split=0, ksplit=v)
         row = {"op": op, "bucket": [e["m_max"], e["n_max"], e["k_max"]], "shape": [M, N, K], "pick": base,
                "ksplit": e.get("ksplit", 0),
                "tsplit": e.get("tsplit", 0), "tiles": tiles}
