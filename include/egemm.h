@@ -307,7 +307,8 @@ int egemm_debug_counter(unsigned long long* value, int reset);
  * [2] first operand load issued, [3] first MMA issued, [4] last MMA committed, [5] last
  * accumulator chunk received by the epilogue, [6] last result stored, [7] exit barrier
  * passed, [8] first converted stage handed over (fused split), [9] first MMA of the CTA's
- * second unit.  out: 16 host words.  reset != 0 zeroes the slots after reading.  Synchronous. */
+ * second unit, [12] last chunk drained, [13] stores' reads done, [14] first TMA issue about to
+ * start, [15] producer entered its loop.  out: 16 host words.  reset != 0 zeroes the slots after reading.  Synchronous. */
 int egemm_debug_timeline(unsigned long long* out, int reset);
 
 #ifdef __cplusplus

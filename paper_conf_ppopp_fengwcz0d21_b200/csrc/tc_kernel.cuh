@@ -643,6 +643,7 @@ __global__ void __launch_bounds__(EpiGeo<NEPI, FA || FB>::THREADS, 1)
    if (warp == EG::W_PROD) {
     // ============================ TMA producer ============================
     if (lane == 0) {
+      TL(15);
       int stage = 0;
       uint32_t phase = 0;
       // FA: only B comes through TMA (A is written by the converter warps); AR: the ring

@@ -13,7 +13,8 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 from paper_conf_ppopp_fengwcz0d21_b200 import egemm, inputs  # noqa: E402
 
 NAMES = ["entry", "setup", "1st load", "1st MMA", "last commit", "last chunk rx", "last store",
-         "exit bar", "1st conv", "unit2 MMA", "-", "last drained", "stores done", "pre-1st-TMA"]
+         "exit bar", "1st conv", "unit2 MMA", "-", "last drained", "stores done", "pre-1st-TMA",
+         "producer start"]
 
 
 def run(M, N, K, fused, kc, cg=2, bn=256, reps=20):
@@ -35,7 +36,7 @@ def run(M, N, K, fused, kc, cg=2, bn=256, reps=20):
         if i < 3:
             continue
         d = [(x - t[0]) if x else -1 for x in t[:10]] + [t[11] - t[10]] + \
-            [(x - t[0]) if x else -1 for x in t[12:15]]
+            [(x - t[0]) if x else -1 for x in t[12:16]]
         acc = d if acc is None else [a + b for a, b in zip(acc, d)]
     egemm.set_config_ex()
     mma = 128 * bn * K * 6 / 8192.0 * (2 if cg == 1 else 1) / (1 if cg == 2 else 2)
