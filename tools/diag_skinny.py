@@ -37,13 +37,13 @@ def main():
         egemm.set_config(*cfg)
         ms, mhz, cyc = timed(lambda: egemm.gemm(None, None, a_split=a_s, b_split=b_s, out=D))
         print("presplit GEMM", cfg, "%.4f ms  %.0f MHz  %.0f kcyc  eff %.3f" % (ms, mhz, cyc / 1e3, need / cyc))
-        os.environ["EGEMM_FUSED_A"] = "1"
+        egemm.set_config_ex(cg=cfg[0], bn=cfg[1], sep=cfg[2], kc=cfg[3], fused=1)
         try:
             ms, mhz, cyc = timed(lambda: egemm.gemm(A, None, b_split=b_s, out=D, workspace=ws))
             print("fused-A GEMM ", cfg, "%.4f ms  %.0f MHz  %.0f kcyc  eff %.3f" % (ms, mhz, cyc / 1e3, need / cyc))
         except Exception as ex:  # unsupported combination
             print("fused-A GEMM ", cfg, "n/a", str(ex)[:80])
-        os.environ.pop("EGEMM_FUSED_A", None)
+        egemm.set_config_ex()
     egemm.set_config(0, 0, 0, 0)
     ms, _, _ = timed(lambda: egemm.split(A, out=a_s))
     print("split A alone %.4f ms (%.0f GB/s)" % (ms, M * K * 8 / ms / 1e6))

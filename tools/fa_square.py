@@ -45,9 +45,10 @@ def main():
                 egemm.gemm(A, None, b_split=b_s, out=D, workspace=ws)
 
             t0 = steady(pre, reps)
-            os.environ["EGEMM_FUSED_A"] = "1"
+            q = egemm.query_config_ex("gemm", n, n, n)
+            egemm.set_config_ex(cg=q["cg"], bn=q["bn"], sep=q["sep"], kc=q["kc"], fused=1)
             t1 = steady(fused, reps)
-            os.environ.pop("EGEMM_FUSED_A", None)
+            egemm.set_config_ex()
             f = 2.0 * n ** 3 / 1e9
             print("n=%d kc=%d  pre-split step %.4f ms (%.1f TF)  fused-A step %.4f ms (%.1f TF)"
                   % (n, kc, t0, f / t0, t1, f / t1), flush=True)

@@ -13,8 +13,7 @@ A = torch.from_numpy(inputs.uniform((M, K), 101)).cuda()
 B = torch.from_numpy(inputs.uniform((K, N), 102)).cuda()
 a_s = egemm.split(A)
 D = torch.empty(M, N, device="cuda")
-os.environ["EGEMM_FUSED_A"] = "2"
-egemm.set_config(2, 256, 0, 256)
+egemm.set_config_ex(cg=2, bn=256, sep=0, kc=256, fused=2)
 for _ in range(2):
     egemm.gemm(None, B, a_split=a_s, out=D)
 torch.cuda.synchronize()

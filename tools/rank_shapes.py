@@ -36,12 +36,11 @@ def main():
                   flush=True)
         # B round-split inside the GEMM (fa bit 1): no separate B^T split pass per step
         for cfg in [(2, 256, 0, 256), (2, 224, 0, 256)]:
-            egemm.set_config(*cfg)
-            os.environ["EGEMM_FUSED_A"] = "2"
+            egemm.set_config_ex(cg=cfg[0], bn=cfg[1], sep=cfg[2], kc=cfg[3], fused=2)
             t = timeit(lambda: egemm.gemm(None, B, a_split=a_split, out=D, workspace=ws))
             t2 = timeit(lambda: egemm.gemm(None, B, a_split=egemm.split(A), out=D,
                                            workspace=ws))
-            os.environ.pop("EGEMM_FUSED_A", None)
+            egemm.set_config_ex()
             print("ranks=%d M=%5d cfg=%-18s fused-B gemm %.4f ms  %.1f TF;  step (A split + fused-B GEMM) "
                   "%.4f ms  %.1f TF per rank, x%d = %.1f" % (world, m, cfg, t, flop / t / 1e9, t2,
                                                              flop / t2 / 1e9, world, world * flop / t2 / 1e9),
