@@ -28,7 +28,8 @@ def main(out, op="gemm_b32"):
         M, N, K = e["m_max"], e["n_max"], min(e["k_max"], 8192)
         cg, bn = e["cg"], e["bn"]
         tiles = -(-M // (128 * cg)) * -(-N // bn)
-        if 2 * tiles > nsm // cg or e.get("fa", 0) == 2:
+        lo_t, hi_t = (int(v) for v in os.environ.get("TILES", "0,%d" % (nsm // cg // 2)).split(","))
+        if not (lo_t < tiles <= hi_t) or e.get("fa", 0) == 2:
             continue
         if "MAXTILES" in os.environ and (tiles > int(os.environ["MAXTILES"]) or K < 2048):
             continue
